@@ -1,0 +1,27 @@
+# Build the product library (CUDA sm_100a) and the oracle (plain C).
+NVCC      ?= nvcc
+ARCH      := -gencode arch=compute_100a,code=sm_100a
+NVFLAGS   := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -Xcompiler -O2 --expt-relaxed-constexpr
+PKG       := paper_conf_ipps_overmanpmm13_b200
+SRC       := $(PKG)/csrc
+LIB       := $(PKG)/libafmm_p2p.so
+CU_SRCS   := $(SRC)/afmm_p2p.cu $(SRC)/peak.cu $(SRC)/tree_build.cu
+CU_HDRS   := $(SRC)/p2p_kernel.cuh include/afmm_p2p.h include/afmm_tree.h
+ORACLE    := oracle/liboracle.so
+
+all: $(LIB) $(ORACLE)
+
+$(LIB): $(CU_SRCS) $(CU_HDRS)
+	$(NVCC) $(NVFLAGS) -Xptxas -v -shared -o $@ $(CU_SRCS) 2> $(PKG)/ptxas.log || (cat $(PKG)/ptxas.log; false)
+	@grep -E "registers|spill" $(PKG)/ptxas.log | grep -E "p2p_kernel|tree" -A0 | head -20 || true
+
+$(ORACLE): oracle/oracle.c
+	gcc -O2 -fopenmp -ffp-contract=off -fno-fast-math -fPIC -shared -std=c11 -o $@ $< -lm
+
+sass: $(LIB)
+	cuobjdump -sass $(LIB) > $(PKG)/sass.txt
+
+clean:
+	rm -f $(LIB) $(ORACLE) $(PKG)/ptxas.log
+
+.PHONY: all clean sass

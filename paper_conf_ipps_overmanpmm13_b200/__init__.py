@@ -1,0 +1,334 @@
+"""Thin ctypes binding of libafmm_p2p.so (include/afmm_p2p.h, include/afmm_tree.h).
+
+Argument marshalling only: every step of the near-field path (packing, tree
+construction, U-lists, the P2P kernel) runs in the CUDA library.  There is no
+CPU fallback: importing this package raises if the shared library is missing,
+and every call raises ``AfmmError`` on a non-zero status.
+
+Names follow the C ABI: ``create``, ``set_bodies``, ``set_tree``, ``eval`` ...
+of AFMM P2P (Overman et al., IPDPSW 2013, PAPER.md L12 SI.C / L16 SIII.C).
+Tensors are ``torch`` CUDA tensors (device pointers) or numpy arrays (host
+pointers) -- torch is only the device-memory / stream provider.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libafmm_p2p.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"{LIB_PATH} not built: run `make` (or __graft_entry__.build()) first; "
+                      "there is no CPU fallback for the AFMM P2P path")
+_lib = C.CDLL(LIB_PATH)
+
+AFMM_OK, AFMM_EINVAL, AFMM_ESTATE, AFMM_ENOMEM, AFMM_ECUDA, AFMM_ENCCL, AFMM_ENOTSUP = 0, -1, -2, -3, -4, -5, -6
+_STATUS = {0: "AFMM_OK", -1: "AFMM_EINVAL", -2: "AFMM_ESTATE", -3: "AFMM_ENOMEM", -4: "AFMM_ECUDA",
+           -5: "AFMM_ENCCL", -6: "AFMM_ENOTSUP"}
+N_BUCKETS = 8
+
+
+class AfmmError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"{_STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class Config(C.Structure):
+    _fields_ = [("device", C.c_int), ("rank", C.c_int), ("world", C.c_int), ("G", C.c_float),
+                ("eps2", C.c_float), ("max_leaf", C.c_int), ("stream", C.c_void_p)]
+
+
+class Stats(C.Structure):
+    _fields_ = [("kernel_ms", C.c_double), ("interactions_total", C.c_longlong),
+                ("interactions_rank", C.c_longlong), ("leaf_lo", C.c_longlong),
+                ("leaf_hi", C.c_longlong), ("body_lo", C.c_longlong), ("body_hi", C.c_longlong),
+                ("n_work_items", C.c_int), ("n_launches", C.c_int),
+                ("bucket_interactions", C.c_longlong * N_BUCKETS)]
+
+    def as_dict(self):
+        d = {f: getattr(self, f) for f, _ in self._fields_ if f != "bucket_interactions"}
+        d["bucket_interactions"] = list(self.bucket_interactions)
+        return d
+
+
+_p, _i, _ll, _d = C.c_void_p, C.c_int, C.c_longlong, C.c_double
+
+
+def _sig(name, res, *args):
+    f = getattr(_lib, name)
+    f.restype = res
+    f.argtypes = list(args)
+    return f
+
+
+_sig("afmm_p2p_config_init", _i, C.POINTER(Config))
+_sig("afmm_p2p_create", _i, C.POINTER(Config), C.POINTER(_p))
+_sig("afmm_p2p_set_bodies", _i, _p, _ll, _p, _p, _p, _p)
+_sig("afmm_p2p_set_bodies_host", _i, _p, _ll, _p, _p, _p, _p)
+_sig("afmm_p2p_bodies_buffer", _i, _p, C.POINTER(_p), C.POINTER(_ll))
+_sig("afmm_p2p_set_tree", _i, _p, _i, _p, _p, _p, _p)
+_sig("afmm_p2p_set_partition", _i, _p, _p)
+_sig("afmm_p2p_get_partition", _i, _p, _p, _p)
+_sig("afmm_p2p_rebalance", _i, _p, _p, _d, C.POINTER(_i))
+_sig("afmm_p2p_eval", _i, _p, _p, _p, _p, _p, C.POINTER(Stats))
+_sig("afmm_p2p_eval_host", _i, _p, _p, _p, _p, _p, C.POINTER(Stats))
+_sig("afmm_p2p_stats_get", _i, _p, C.POINTER(Stats))
+_sig("afmm_p2p_stream", _p, _p)
+_sig("afmm_p2p_destroy", None, _p)
+_sig("afmm_p2p_last_error", C.c_char_p, _p)
+_sig("afmm_interactions", _i, _i, _p, _p, _p, _p)
+_sig("afmm_partition_literal", _i, _i, _p, _i, _p)
+_sig("afmm_partition_weighted", _i, _i, _p, _i, _p)
+_sig("afmm_fp32_peak", _i, _i, C.POINTER(_d), C.POINTER(_d), C.POINTER(_d))
+_sig("afmm_version", C.c_char_p)
+_sig("afmm_tree_create", _i, _i, _p, C.POINTER(_p))
+_sig("afmm_tree_build", _i, _p, _ll, _p, _p, _p, _i, _i, _p, _i)
+_sig("afmm_tree_info", _i, _p, C.POINTER(_i), C.POINTER(_ll), _p, C.POINTER(_i), C.POINTER(_i),
+     C.POINTER(_ll))
+_sig("afmm_tree_copy_out", _i, _p, _p, _p, _p, _p, _p, _p, _p)
+_sig("afmm_tree_gather", _i, _p, _p, _p)
+_sig("afmm_tree_scatter", _i, _p, _p, _p)
+_sig("afmm_tree_destroy", None, _p)
+_sig("afmm_tree_last_error", C.c_char_p, _p)
+
+# every symbol include/*.h declares (checked by tests/test_abi.py)
+EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
+            "afmm_p2p_set_bodies_host", "afmm_p2p_bodies_buffer", "afmm_p2p_set_tree",
+            "afmm_p2p_set_partition", "afmm_p2p_get_partition", "afmm_p2p_rebalance",
+            "afmm_p2p_eval", "afmm_p2p_eval_host", "afmm_p2p_stats_get", "afmm_p2p_stream",
+            "afmm_p2p_destroy", "afmm_p2p_last_error", "afmm_interactions",
+            "afmm_partition_literal", "afmm_partition_weighted", "afmm_fp32_peak", "afmm_version",
+            "afmm_tree_create", "afmm_tree_build", "afmm_tree_info", "afmm_tree_copy_out",
+            "afmm_tree_gather", "afmm_tree_scatter", "afmm_tree_destroy", "afmm_tree_last_error"]
+
+
+def version() -> str:
+    return _lib.afmm_version().decode()
+
+
+def _np(a, dt):
+    return np.ascontiguousarray(a, dtype=dt)
+
+
+def _ptr(a):
+    """Raw pointer of a numpy array or a torch tensor (host or device)."""
+    if a is None:
+        return None
+    if isinstance(a, np.ndarray):
+        return a.ctypes.data
+    return a.data_ptr()
+
+
+def _is_device(a) -> bool:
+    return not isinstance(a, np.ndarray) and getattr(a, "is_cuda", False)
+
+
+# ------------------------------------------------------------------ host-only helpers
+
+def interactions(leaf_count, u_off, u_idx) -> np.ndarray:
+    """Interactions(t) = n_t * sum_{s in U(t)} n_s (PAPER L16 SIII.C)."""
+    lc, uo, ui = _np(leaf_count, np.int32), _np(u_off, np.int64), _np(u_idx, np.int32)
+    out = np.empty(lc.shape[0], np.int64)
+    st = _lib.afmm_interactions(lc.shape[0], _ptr(lc), _ptr(uo), _ptr(ui), _ptr(out))
+    if st:
+        raise AfmmError(st, "afmm_interactions")
+    return out
+
+
+def partition_literal(I, G: int) -> np.ndarray:
+    """Literal greedy split of PAPER L16 SIII.C -> leaf_split[G+1]."""
+    I = _np(I, np.int64)
+    out = np.empty(G + 1, np.int64)
+    st = _lib.afmm_partition_literal(I.shape[0], _ptr(I), int(G), _ptr(out))
+    if st:
+        raise AfmmError(st, "afmm_partition_literal")
+    return out
+
+
+def partition_weighted(w, G: int) -> np.ndarray:
+    w = _np(w, np.float64)
+    out = np.empty(G + 1, np.int64)
+    st = _lib.afmm_partition_weighted(w.shape[0], _ptr(w), int(G), _ptr(out))
+    if st:
+        raise AfmmError(st, "afmm_partition_weighted")
+    return out
+
+
+def fp32_peak(device: int = 0):
+    """Measured FP32 FFMA / FFMA2 TFLOP/s and the SM clock (MHz) on `device`."""
+    a, b, c = _d(), _d(), _d()
+    st = _lib.afmm_fp32_peak(int(device), C.byref(a), C.byref(b), C.byref(c))
+    if st:
+        raise AfmmError(st, "afmm_fp32_peak")
+    return {"ffma_tflops": a.value, "ffma2_tflops": b.value, "sm_mhz": c.value}
+
+
+# ------------------------------------------------------------------ P2P handle
+
+class P2P:
+    """One afmm_p2p handle (one per rank / GPU)."""
+
+    def __init__(self, device=0, rank=0, world=1, G=1.0, eps2=0.0, max_leaf=1024, stream=None):
+        cfg = Config()
+        _lib.afmm_p2p_config_init(C.byref(cfg))
+        cfg.device, cfg.rank, cfg.world = int(device), int(rank), int(world)
+        cfg.G, cfg.eps2, cfg.max_leaf = float(G), float(eps2), int(max_leaf)
+        cfg.stream = stream
+        h = _p()
+        st = _lib.afmm_p2p_create(C.byref(cfg), C.byref(h))
+        if st:
+            raise AfmmError(st, "afmm_p2p_create")
+        self._h = h
+        self.world, self.rank, self.device = world, rank, device
+
+    def _check(self, st, what):
+        if st:
+            raise AfmmError(st, f"{what}: {_lib.afmm_p2p_last_error(self._h).decode()}")
+
+    def close(self):
+        if getattr(self, "_h", None):
+            _lib.afmm_p2p_destroy(self._h)
+            self._h = None
+
+    __del__ = close
+
+    @property
+    def stream(self):
+        return _lib.afmm_p2p_stream(self._h)
+
+    def set_bodies(self, x, y, z, m, n=None):
+        """Bodies in tree order.  torch CUDA tensors -> afmm_p2p_set_bodies;
+        numpy arrays -> afmm_p2p_set_bodies_host; all None with n -> allocate only."""
+        if x is None:
+            self._check(_lib.afmm_p2p_set_bodies(self._h, int(n), None, None, None, None),
+                        "afmm_p2p_set_bodies")
+            return
+        n = int(x.shape[0])
+        if _is_device(x):
+            self._check(_lib.afmm_p2p_set_bodies(self._h, n, _ptr(x), _ptr(y), _ptr(z), _ptr(m)),
+                        "afmm_p2p_set_bodies")
+        else:
+            x, y, z, m = (_np(v, np.float32) for v in (x, y, z, m))
+            self._check(_lib.afmm_p2p_set_bodies_host(self._h, n, _ptr(x), _ptr(y), _ptr(z), _ptr(m)),
+                        "afmm_p2p_set_bodies_host")
+
+    def bodies_buffer(self):
+        p, b = _p(), _ll()
+        self._check(_lib.afmm_p2p_bodies_buffer(self._h, C.byref(p), C.byref(b)), "afmm_p2p_bodies_buffer")
+        return p.value, b.value
+
+    def set_tree(self, leaf_start, leaf_count, u_off, u_idx):
+        ls, lc = _np(leaf_start, np.int32), _np(leaf_count, np.int32)
+        uo, ui = _np(u_off, np.int64), _np(u_idx, np.int32)
+        self._check(_lib.afmm_p2p_set_tree(self._h, ls.shape[0], _ptr(ls), _ptr(lc), _ptr(uo), _ptr(ui)),
+                    "afmm_p2p_set_tree")
+
+    def set_partition(self, leaf_split=None):
+        ls = None if leaf_split is None else _np(leaf_split, np.int64)
+        self._check(_lib.afmm_p2p_set_partition(self._h, _ptr(ls)), "afmm_p2p_set_partition")
+
+    def get_partition(self):
+        ls = np.empty(self.world + 1, np.int64)
+        bs = np.empty(self.world + 1, np.int64)
+        self._check(_lib.afmm_p2p_get_partition(self._h, _ptr(ls), _ptr(bs)), "afmm_p2p_get_partition")
+        return ls, bs
+
+    def rebalance(self, rank_ms, threshold=0.02) -> bool:
+        r = _np(rank_ms, np.float64)
+        ch = _i()
+        self._check(_lib.afmm_p2p_rebalance(self._h, _ptr(r), float(threshold), C.byref(ch)),
+                    "afmm_p2p_rebalance")
+        return bool(ch.value)
+
+    def eval(self, ax, ay, az, phi, stats=False):
+        """Outputs: torch CUDA tensors (async; stats forces a sync) or numpy
+        arrays (blocking, afmm_p2p_eval_host)."""
+        s = Stats()
+        sp = C.byref(s) if stats else None
+        if _is_device(ax):
+            self._check(_lib.afmm_p2p_eval(self._h, _ptr(ax), _ptr(ay), _ptr(az), _ptr(phi), sp),
+                        "afmm_p2p_eval")
+        else:
+            for a in (ax, ay, az, phi):
+                if not (isinstance(a, np.ndarray) and a.dtype == np.float32 and a.flags.c_contiguous):
+                    raise TypeError("host outputs must be contiguous float32 numpy arrays")
+            sp = C.byref(s)
+            self._check(_lib.afmm_p2p_eval_host(self._h, _ptr(ax), _ptr(ay), _ptr(az), _ptr(phi), sp),
+                        "afmm_p2p_eval_host")
+        return s.as_dict() if (stats or not _is_device(ax)) else None
+
+    def stats(self):
+        s = Stats()
+        self._check(_lib.afmm_p2p_stats_get(self._h, C.byref(s)), "afmm_p2p_stats_get")
+        return s.as_dict()
+
+
+# ------------------------------------------------------------------ GPU tree builder
+
+class GpuTree:
+    """afmm_tree handle: adaptive octree + U-list built on the GPU."""
+
+    def __init__(self, device=0, stream=None):
+        h = _p()
+        st = _lib.afmm_tree_create(int(device), stream, C.byref(h))
+        if st:
+            raise AfmmError(st, "afmm_tree_create")
+        self._h = h
+
+    def _check(self, st, what):
+        if st:
+            raise AfmmError(st, f"{what}: {_lib.afmm_tree_last_error(self._h).decode()}")
+
+    def close(self):
+        if getattr(self, "_h", None):
+            _lib.afmm_tree_destroy(self._h)
+            self._h = None
+
+    __del__ = close
+
+    def build(self, x, y, z, S, domain=None):
+        """x, y, z: torch CUDA float32 tensors (input order).  domain=(lo[3], k) fixes it."""
+        lo = None
+        k = 0
+        fixed = 0
+        if domain is not None:
+            lo = _np(domain[0], np.float64)
+            k = int(domain[1])
+            fixed = 1
+        self._check(_lib.afmm_tree_build(self._h, int(x.shape[0]), _ptr(x), _ptr(y), _ptr(z), int(S),
+                                         fixed, _ptr(lo), k), "afmm_tree_build")
+        return self.info()
+
+    def info(self):
+        L, nnz, k, ml, nn = _i(), _ll(), _i(), _i(), _ll()
+        lo = np.empty(3)
+        self._check(_lib.afmm_tree_info(self._h, C.byref(L), C.byref(nnz), _ptr(lo), C.byref(k),
+                                        C.byref(ml), C.byref(nn)), "afmm_tree_info")
+        return {"n_leaves": L.value, "nnz": nnz.value, "lo": lo, "k": k.value,
+                "max_level": ml.value, "n_nodes": nn.value}
+
+    def copy_out(self, n):
+        inf = self.info()
+        L, nnz = inf["n_leaves"], inf["nnz"]
+        out = {"perm": np.empty(n, np.int32), "leaf_start": np.empty(L, np.int32),
+               "leaf_count": np.empty(L, np.int32), "leaf_level": np.empty(L, np.int32),
+               "leaf_prefix": np.empty(L, np.uint64), "u_off": np.empty(L + 1, np.int64),
+               "u_idx": np.empty(max(nnz, 1), np.int32)}
+        self._check(_lib.afmm_tree_copy_out(self._h, *[_ptr(out[k]) for k in
+                                                      ("perm", "leaf_start", "leaf_count", "leaf_level",
+                                                       "leaf_prefix", "u_off", "u_idx")]),
+                    "afmm_tree_copy_out")
+        out["u_idx"] = out["u_idx"][:nnz]
+        out.update(inf)
+        return out
+
+    def gather(self, src, dst):
+        """dst[p] = src[perm[p]] (device tensors)."""
+        self._check(_lib.afmm_tree_gather(self._h, _ptr(src), _ptr(dst)), "afmm_tree_gather")
+
+    def scatter(self, src, dst):
+        self._check(_lib.afmm_tree_scatter(self._h, _ptr(src), _ptr(dst)), "afmm_tree_scatter")

@@ -1,0 +1,729 @@
+// afmm_p2p.cu -- host side of the C ABI (include/afmm_p2p.h) and launches.
+//
+// Rows of SURVEY.md S8(a) implemented here: a1 body ingest (pack kernel),
+// a2 tree ingest (validation, Interactions(t), segment merge, chunking, LPT
+// order), a3 partition (literal greedy rule of PAPER L16 SIII.C + the
+// incremental rebalance of L18 SIV.D), a5/a6 launch of the P2P kernel, a8
+// cudaEvent timing (PAPER L20 SVII.A).  Rows a4/a7 (replication, gather) are
+// collectives issued by the caller on the buffers this library exposes.
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <numeric>
+#include <string>
+#include <vector>
+
+#include <cuda_runtime.h>
+
+#include "../../include/afmm_p2p.h"
+#include "p2p_kernel.cuh"
+
+using afmm::Chunk;
+using afmm::Item;
+using afmm::Seg;
+
+struct afmm_p2p {
+    afmm_p2p_config cfg{};
+    cudaStream_t stream = nullptr;
+    bool own_stream = false;
+    bool poisoned = false;
+    std::string err;
+    int num_sms = 148;
+    int blocks_per_sm = 1;
+
+    // bodies
+    long long n = 0;
+    float4 *d_bodies = nullptr;
+    long long bodies_cap = 0;
+    float *d_soa = nullptr;          // staging for host ingest (4n floats)
+    long long soa_cap = 0;
+    float *d_out = nullptr;          // eval_host outputs (4n floats)
+    long long out_cap = 0;
+
+    // tree (host copies)
+    bool have_tree = false;
+    int L = 0;
+    std::vector<int> leaf_start, leaf_count;
+    std::vector<long long> u_off;
+    std::vector<int> u_idx;
+    std::vector<long long> I;
+    long long I_total = 0;
+
+    // partition
+    bool user_partition = false;
+    std::vector<long long> leaf_split, body_split;
+
+    // this rank's work list
+    std::vector<Item> h_items;
+    std::vector<Chunk> h_chunks;
+    std::vector<Seg> h_segs;
+    Item *d_items = nullptr;
+    Chunk *d_chunks = nullptr;
+    Seg *d_segs = nullptr;
+    size_t items_cap = 0, chunks_cap = 0, segs_cap = 0;
+    int *d_queue = nullptr;
+    long long rank_interactions = 0;
+    long long bucket_inter[8] = {0};
+
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    bool evaluated = false;
+    afmm_p2p_stats last{};
+};
+
+namespace {
+
+afmm_status fail(afmm_p2p *h, afmm_status st, const char *fmt, ...) {
+    if (h) {
+        char buf[512];
+        va_list ap;
+        va_start(ap, fmt);
+        vsnprintf(buf, sizeof(buf), fmt, ap);
+        va_end(ap);
+        h->err = buf;
+        if (st == AFMM_ECUDA || st == AFMM_ENOMEM) h->poisoned = true;
+    }
+    return st;
+}
+
+#define CUDA_TRY(h, call)                                                                    \
+    do {                                                                                     \
+        cudaError_t e_ = (call);                                                             \
+        if (e_ != cudaSuccess)                                                               \
+            return fail((h), e_ == cudaErrorMemoryAllocation ? AFMM_ENOMEM : AFMM_ECUDA,      \
+                        "%s failed: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__,    \
+                        __LINE__);                                                           \
+    } while (0)
+
+#define CHECK_HANDLE(h)                                                                      \
+    do {                                                                                     \
+        if (!(h)) return AFMM_EINVAL;                                                        \
+        if ((h)->poisoned) return AFMM_ESTATE;                                               \
+    } while (0)
+
+int bucket_of(int nt) {
+    int b = 0;
+    int cap = 8;
+    while (nt > cap && b < 7) {
+        cap <<= 1;
+        ++b;
+    }
+    return b;
+}
+
+template <typename T>
+afmm_status ensure_device(afmm_p2p *h, T **ptr, size_t &cap, size_t count) {
+    if (count <= cap && *ptr) return AFMM_OK;
+    if (*ptr) cudaFree(*ptr);
+    *ptr = nullptr;
+    cap = 0;
+    size_t c = std::max<size_t>(count, 1);
+    CUDA_TRY(h, cudaMalloc(reinterpret_cast<void **>(ptr), c * sizeof(T)));
+    cap = c;
+    return AFMM_OK;
+}
+
+afmm_status set_device(afmm_p2p *h) {
+    CUDA_TRY(h, cudaSetDevice(h->cfg.device));
+    return AFMM_OK;
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------ host-only
+
+extern "C" afmm_status afmm_interactions(int n_leaves, const int *leaf_count,
+                                         const long long *u_off, const int *u_idx,
+                                         long long *I) {
+    if (n_leaves < 0 || (n_leaves > 0 && (!leaf_count || !u_off || !u_idx || !I)))
+        return AFMM_EINVAL;
+    for (int t = 0; t < n_leaves; ++t) {
+        long long src = 0;
+        for (long long u = u_off[t]; u < u_off[t + 1]; ++u) {
+            const int s = u_idx[u];
+            if (s < 0 || s >= n_leaves) return AFMM_EINVAL;
+            src += leaf_count[s];
+        }
+        I[t] = (long long)leaf_count[t] * src;
+    }
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_partition_literal(int n_leaves, const long long *I, int G,
+                                              long long *leaf_split) {
+    if (n_leaves < 0 || G < 1 || !leaf_split || (n_leaves > 0 && !I)) return AFMM_EINVAL;
+    __int128 total = 0;
+    for (int t = 0; t < n_leaves; ++t) {
+        if (I[t] < 0) return AFMM_EINVAL;
+        total += I[t];
+    }
+    // walk leaves; once the running count c satisfies c*G >= total the next
+    // leaf opens the next GPU (PAPER L16 SIII.C); the last GPU takes the rest
+    int g = 0;
+    __int128 c = 0;
+    leaf_split[0] = 0;
+    for (int t = 0; t < n_leaves; ++t) {
+        c += I[t];
+        if (g < G - 1 && c * G >= total) {
+            leaf_split[++g] = t + 1;
+            c = 0;
+        }
+    }
+    for (int r = g + 1; r <= G; ++r) leaf_split[r] = n_leaves;
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_partition_weighted(int n_leaves, const double *w, int G,
+                                               long long *leaf_split) {
+    if (n_leaves < 0 || G < 1 || !leaf_split || (n_leaves > 0 && !w)) return AFMM_EINVAL;
+    long double total = 0;
+    for (int t = 0; t < n_leaves; ++t) {
+        if (!(w[t] >= 0.0) || !std::isfinite(w[t])) return AFMM_EINVAL;
+        total += w[t];
+    }
+    int g = 0;
+    long double c = 0;
+    leaf_split[0] = 0;
+    for (int t = 0; t < n_leaves; ++t) {
+        c += w[t];
+        if (g < G - 1 && c * G >= total) {
+            leaf_split[++g] = t + 1;
+            c = 0;
+        }
+    }
+    for (int r = g + 1; r <= G; ++r) leaf_split[r] = n_leaves;
+    return AFMM_OK;
+}
+
+// ------------------------------------------------------------------ handle
+
+extern "C" afmm_status afmm_p2p_config_init(afmm_p2p_config *cfg) {
+    if (!cfg) return AFMM_EINVAL;
+    cfg->device = 0;
+    cfg->rank = 0;
+    cfg->world = 1;
+    cfg->G = 1.0f;
+    cfg->eps2 = 0.0f;
+    cfg->max_leaf = 1024;
+    cfg->stream = nullptr;
+    return AFMM_OK;
+}
+
+extern "C" const char *afmm_version(void) { return "afmm_p2p 0.1 sm_100a"; }
+
+extern "C" afmm_status afmm_p2p_create(const afmm_p2p_config *cfg, afmm_p2p **out) {
+    if (!out) return AFMM_EINVAL;
+    *out = nullptr;
+    if (!cfg) return AFMM_EINVAL;
+    if (cfg->max_leaf > 1024) return AFMM_ENOTSUP;
+    if (cfg->max_leaf < 1 || cfg->world < 1 || cfg->rank < 0 || cfg->rank >= cfg->world ||
+        !std::isfinite(cfg->G) || !std::isfinite(cfg->eps2) || !(cfg->eps2 >= 0.0f) ||
+        cfg->device < 0)
+        return AFMM_EINVAL;
+    afmm_p2p *h = new (std::nothrow) afmm_p2p();
+    if (!h) return AFMM_ENOMEM;
+    h->cfg = *cfg;
+    afmm_status st = set_device(h);
+    if (st == AFMM_OK) {
+        cudaError_t e = cudaSuccess;
+        if (cfg->stream) {
+            h->stream = static_cast<cudaStream_t>(cfg->stream);
+        } else {
+            e = cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking);
+            h->own_stream = (e == cudaSuccess);
+        }
+        if (e == cudaSuccess) e = cudaEventCreate(&h->ev0);
+        if (e == cudaSuccess) e = cudaEventCreate(&h->ev1);
+        if (e == cudaSuccess) e = cudaMalloc(&h->d_queue, sizeof(int));
+        if (e == cudaSuccess) e = cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, cfg->device);
+        if (e == cudaSuccess)
+            e = cudaFuncSetAttribute(afmm::p2p_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     afmm::kDynSmem);
+        if (e == cudaSuccess)
+            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&h->blocks_per_sm, afmm::p2p_kernel,
+                                                              afmm::kThreads, afmm::kDynSmem);
+        if (e != cudaSuccess) st = fail(h, AFMM_ECUDA, "create: %s", cudaGetErrorString(e));
+        if (h->blocks_per_sm < 1) h->blocks_per_sm = 1;
+    }
+    if (st != AFMM_OK) {
+        afmm_p2p_destroy(h);
+        return st;
+    }
+    *out = h;
+    return AFMM_OK;
+}
+
+extern "C" void afmm_p2p_destroy(afmm_p2p *h) {
+    if (!h) return;
+    cudaSetDevice(h->cfg.device);
+    if (h->stream) cudaStreamSynchronize(h->stream);
+    cudaFree(h->d_bodies);
+    cudaFree(h->d_soa);
+    cudaFree(h->d_out);
+    cudaFree(h->d_items);
+    cudaFree(h->d_chunks);
+    cudaFree(h->d_segs);
+    cudaFree(h->d_queue);
+    if (h->ev0) cudaEventDestroy(h->ev0);
+    if (h->ev1) cudaEventDestroy(h->ev1);
+    if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
+    delete h;
+}
+
+extern "C" const char *afmm_p2p_last_error(const afmm_p2p *h) {
+    if (!h) return "null handle";
+    return h->err.c_str();
+}
+
+extern "C" void *afmm_p2p_stream(const afmm_p2p *h) { return h ? (void *)h->stream : nullptr; }
+
+// ------------------------------------------------------------------ bodies
+
+static afmm_status alloc_bodies(afmm_p2p *h, long long n) {
+    if (n > h->bodies_cap) {
+        cudaFree(h->d_bodies);
+        h->d_bodies = nullptr;
+        h->bodies_cap = 0;
+        CUDA_TRY(h, cudaMalloc(&h->d_bodies, (size_t)n * sizeof(float4)));
+        h->bodies_cap = n;
+    }
+    if (h->n != n) h->have_tree = false;   // a tree for another n is stale
+    h->n = n;
+    h->evaluated = false;
+    return AFMM_OK;
+}
+
+static afmm_status pack(afmm_p2p *h, const float *x, const float *y, const float *z,
+                        const float *m) {
+    const int threads = 256;
+    long long blocks = std::min<long long>((h->n + threads - 1) / threads, (long long)h->num_sms * 16);
+    afmm::pack_bodies_kernel<<<(int)blocks, threads, 0, h->stream>>>(h->n, x, y, z, m, h->d_bodies);
+    CUDA_TRY(h, cudaGetLastError());
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_p2p_set_bodies(afmm_p2p *h, long long n, const float *x,
+                                           const float *y, const float *z, const float *m) {
+    CHECK_HANDLE(h);
+    if (n < 1 || n >= (1LL << 31)) return fail(h, AFMM_EINVAL, "set_bodies: n=%lld out of [1, 2^31)", n);
+    const int nn = (x != nullptr) + (y != nullptr) + (z != nullptr) + (m != nullptr);
+    if (nn != 0 && nn != 4) return fail(h, AFMM_EINVAL, "set_bodies: pass all four pointers or none");
+    afmm_status st = set_device(h);
+    if (st) return st;
+    if ((st = alloc_bodies(h, n))) return st;
+    if (nn == 4) return pack(h, x, y, z, m);
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_p2p_set_bodies_host(afmm_p2p *h, long long n, const float *x,
+                                                const float *y, const float *z, const float *m) {
+    CHECK_HANDLE(h);
+    if (n < 1 || n >= (1LL << 31)) return fail(h, AFMM_EINVAL, "set_bodies_host: n=%lld out of [1, 2^31)", n);
+    if (!x || !y || !z || !m) return fail(h, AFMM_EINVAL, "set_bodies_host: null pointer");
+    afmm_status st = set_device(h);
+    if (st) return st;
+    if ((st = alloc_bodies(h, n))) return st;
+    if (4 * n > h->soa_cap) {
+        cudaFree(h->d_soa);
+        h->d_soa = nullptr;
+        h->soa_cap = 0;
+        CUDA_TRY(h, cudaMalloc(&h->d_soa, (size_t)(4 * n) * sizeof(float)));
+        h->soa_cap = 4 * n;
+    }
+    const size_t b = (size_t)n * sizeof(float);
+    CUDA_TRY(h, cudaMemcpyAsync(h->d_soa + 0 * n, x, b, cudaMemcpyHostToDevice, h->stream));
+    CUDA_TRY(h, cudaMemcpyAsync(h->d_soa + 1 * n, y, b, cudaMemcpyHostToDevice, h->stream));
+    CUDA_TRY(h, cudaMemcpyAsync(h->d_soa + 2 * n, z, b, cudaMemcpyHostToDevice, h->stream));
+    CUDA_TRY(h, cudaMemcpyAsync(h->d_soa + 3 * n, m, b, cudaMemcpyHostToDevice, h->stream));
+    if ((st = pack(h, h->d_soa, h->d_soa + n, h->d_soa + 2 * n, h->d_soa + 3 * n))) return st;
+    CUDA_TRY(h, cudaStreamSynchronize(h->stream));
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_p2p_bodies_buffer(afmm_p2p *h, void **dev_ptr, long long *bytes) {
+    CHECK_HANDLE(h);
+    if (!h->d_bodies || h->n < 1) return fail(h, AFMM_ESTATE, "bodies_buffer: no bodies set");
+    if (dev_ptr) *dev_ptr = h->d_bodies;
+    if (bytes) *bytes = h->n * (long long)sizeof(float4);
+    return AFMM_OK;
+}
+
+// ------------------------------------------------------------------ tree / work list
+
+static void compute_body_split(afmm_p2p *h) {
+    const int W = h->cfg.world;
+    h->body_split.assign(W + 1, 0);
+    for (int r = 0; r <= W; ++r) {
+        const long long ls = h->leaf_split[r];
+        h->body_split[r] = (ls >= h->L) ? h->n : h->leaf_start[ls];
+    }
+}
+
+// Build this rank's work list on the host and upload it.
+static afmm_status build_worklist(afmm_p2p *h) {
+    const int r = h->cfg.rank;
+    const long long lo = h->leaf_split[r], hi = h->leaf_split[r + 1];
+    h->h_items.clear();
+    h->h_chunks.clear();
+    h->h_segs.clear();
+    h->rank_interactions = 0;
+    std::fill(h->bucket_inter, h->bucket_inter + 8, 0LL);
+    std::vector<long long> cost;
+    std::vector<Seg> segs;   // staged list of one leaf: self first, then merged neighbours
+    for (long long t = lo; t < hi; ++t) {
+        const int ts = h->leaf_start[t], tn = h->leaf_count[t];
+        segs.clear();
+        bool has_self = false;
+        for (long long u = h->u_off[t]; u < h->u_off[t + 1]; ++u)
+            if (h->u_idx[u] == t) has_self = true;
+        if (has_self) segs.push_back(Seg{ts, tn, 0, 0});
+        // merge runs of leaves whose body ranges are contiguous (consecutive leaf ids)
+        const size_t first_other = segs.size();
+        for (long long u = h->u_off[t]; u < h->u_off[t + 1]; ++u) {
+            const int s = h->u_idx[u];
+            if (s == t) continue;
+            const int bs = h->leaf_start[s], bn = h->leaf_count[s];
+            if (segs.size() > first_other && segs.back().gstart + segs.back().len == bs) {
+                segs.back().len += bn;
+            } else {
+                segs.push_back(Seg{bs, bn, 0, 0});
+            }
+        }
+        // cut the staged list into chunks of <= kCap bodies (self stays in chunk 0)
+        const int chunk_begin = (int)h->h_chunks.size();
+        int cur_bodies = 0;
+        Chunk cur{(int)h->h_segs.size(), 0, 0, 0};
+        long long nsrc = 0;
+        for (const Seg &sg0 : segs) {
+            Seg sg = sg0;
+            nsrc += sg.len;
+            while (sg.len > 0) {
+                if (cur_bodies == afmm::kCap) {
+                    h->h_chunks.push_back(cur);
+                    cur = Chunk{(int)h->h_segs.size(), 0, 0, 0};
+                    cur_bodies = 0;
+                }
+                const int take = std::min(sg.len, afmm::kCap - cur_bodies);
+                h->h_segs.push_back(Seg{sg.gstart, take, cur_bodies, 0});
+                cur.seg_count++;
+                cur.nbodies += take;
+                cur_bodies += take;
+                sg.gstart += take;
+                sg.len -= take;
+            }
+        }
+        if (cur.seg_count > 0 || h->h_chunks.size() == (size_t)chunk_begin) h->h_chunks.push_back(cur);
+        const int chunk_count = (int)h->h_chunks.size() - chunk_begin;
+        for (int a = 0; a < tn; a += afmm::kMaxTargets) {
+            const int cnt = std::min(afmm::kMaxTargets, tn - a);
+            h->h_items.push_back(Item{ts + a, cnt, ts, has_self ? tn : 0, chunk_begin, chunk_count, 0, 0});
+            cost.push_back((long long)(((cnt + 1) / 2) * 2) * std::max<long long>(nsrc, 1));
+        }
+        h->rank_interactions += h->I[t];
+        h->bucket_inter[bucket_of(tn)] += h->I[t];
+    }
+    // largest-cost-first order (stable for determinism of scheduling inputs)
+    std::vector<int> order(h->h_items.size());
+    std::iota(order.begin(), order.end(), 0);
+    std::stable_sort(order.begin(), order.end(), [&](int a, int b) { return cost[a] > cost[b]; });
+    std::vector<Item> sorted(order.size());
+    for (size_t i = 0; i < order.size(); ++i) sorted[i] = h->h_items[order[i]];
+    h->h_items.swap(sorted);
+
+    afmm_status st;
+    if ((st = ensure_device(h, &h->d_items, h->items_cap, h->h_items.size()))) return st;
+    if ((st = ensure_device(h, &h->d_chunks, h->chunks_cap, h->h_chunks.size()))) return st;
+    if ((st = ensure_device(h, &h->d_segs, h->segs_cap, h->h_segs.size()))) return st;
+    if (!h->h_items.empty())
+        CUDA_TRY(h, cudaMemcpyAsync(h->d_items, h->h_items.data(), h->h_items.size() * sizeof(Item),
+                                    cudaMemcpyHostToDevice, h->stream));
+    if (!h->h_chunks.empty())
+        CUDA_TRY(h, cudaMemcpyAsync(h->d_chunks, h->h_chunks.data(), h->h_chunks.size() * sizeof(Chunk),
+                                    cudaMemcpyHostToDevice, h->stream));
+    if (!h->h_segs.empty())
+        CUDA_TRY(h, cudaMemcpyAsync(h->d_segs, h->h_segs.data(), h->h_segs.size() * sizeof(Seg),
+                                    cudaMemcpyHostToDevice, h->stream));
+    CUDA_TRY(h, cudaStreamSynchronize(h->stream));
+    h->evaluated = false;
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_p2p_set_tree(afmm_p2p *h, int n_leaves, const int *leaf_start,
+                                         const int *leaf_count, const long long *u_off,
+                                         const int *u_idx) {
+    CHECK_HANDLE(h);
+    if (h->n < 1 || !h->d_bodies) return fail(h, AFMM_ESTATE, "set_tree: call set_bodies first");
+    if (n_leaves < 1 || !leaf_start || !leaf_count || !u_off)
+        return fail(h, AFMM_EINVAL, "set_tree: n_leaves=%d / null pointer", n_leaves);
+    // leaves must tile [0, n) exactly, 1 <= count <= max_leaf
+    long long expect = 0;
+    for (int t = 0; t < n_leaves; ++t) {
+        if (leaf_start[t] != expect)
+            return fail(h, AFMM_EINVAL, "set_tree: leaf %d starts at %d, expected %lld", t, leaf_start[t], expect);
+        if (leaf_count[t] < 1 || leaf_count[t] > h->cfg.max_leaf)
+            return fail(h, AFMM_EINVAL, "set_tree: leaf %d count %d outside [1, max_leaf=%d]", t,
+                        leaf_count[t], h->cfg.max_leaf);
+        expect += leaf_count[t];
+    }
+    if (expect != h->n) return fail(h, AFMM_EINVAL, "set_tree: leaves cover %lld bodies, n=%lld", expect, h->n);
+    if (u_off[0] != 0) return fail(h, AFMM_EINVAL, "set_tree: u_off[0]=%lld != 0", u_off[0]);
+    for (int t = 0; t < n_leaves; ++t)
+        if (u_off[t + 1] < u_off[t]) return fail(h, AFMM_EINVAL, "set_tree: u_off not monotone at %d", t);
+    const long long nnz = u_off[n_leaves];
+    if (nnz > 0 && !u_idx) return fail(h, AFMM_EINVAL, "set_tree: u_idx is null");
+    for (int t = 0; t < n_leaves; ++t) {
+        for (long long u = u_off[t]; u < u_off[t + 1]; ++u) {
+            if (u_idx[u] < 0 || u_idx[u] >= n_leaves)
+                return fail(h, AFMM_EINVAL, "set_tree: u_idx[%lld]=%d outside [0,%d)", u, u_idx[u], n_leaves);
+            if (u > u_off[t] && u_idx[u] <= u_idx[u - 1])
+                return fail(h, AFMM_EINVAL, "set_tree: row %d of u_idx not strictly ascending", t);
+        }
+    }
+    afmm_status st = set_device(h);
+    if (st) return st;
+    h->L = n_leaves;
+    h->leaf_start.assign(leaf_start, leaf_start + n_leaves);
+    h->leaf_count.assign(leaf_count, leaf_count + n_leaves);
+    h->u_off.assign(u_off, u_off + n_leaves + 1);
+    h->u_idx.assign(u_idx, u_idx + nnz);
+    h->I.assign(n_leaves, 0);
+    afmm_interactions(n_leaves, leaf_count, u_off, u_idx, h->I.data());
+    h->I_total = 0;
+    for (long long v : h->I) h->I_total += v;
+    const int W = h->cfg.world;
+    if (!h->user_partition || (long long)h->leaf_split.size() != W + 1 || h->leaf_split[W] != n_leaves) {
+        h->user_partition = false;
+        h->leaf_split.assign(W + 1, 0);
+        afmm_partition_literal(n_leaves, h->I.data(), W, h->leaf_split.data());
+    }
+    compute_body_split(h);
+    h->have_tree = true;
+    return build_worklist(h);
+}
+
+extern "C" afmm_status afmm_p2p_set_partition(afmm_p2p *h, const long long *leaf_split) {
+    CHECK_HANDLE(h);
+    const int W = h->cfg.world;
+    if (!leaf_split) {
+        h->user_partition = false;
+        if (!h->have_tree) return AFMM_OK;
+        afmm_partition_literal(h->L, h->I.data(), W, h->leaf_split.data());
+    } else {
+        if (leaf_split[0] != 0) return fail(h, AFMM_EINVAL, "set_partition: leaf_split[0] != 0");
+        for (int r = 0; r < W; ++r)
+            if (leaf_split[r + 1] < leaf_split[r]) return fail(h, AFMM_EINVAL, "set_partition: not monotone");
+        if (h->have_tree && leaf_split[W] != h->L)
+            return fail(h, AFMM_EINVAL, "set_partition: leaf_split[world]=%lld != n_leaves=%d", leaf_split[W], h->L);
+        h->leaf_split.assign(leaf_split, leaf_split + W + 1);
+        h->user_partition = true;
+        if (!h->have_tree) return AFMM_OK;
+    }
+    afmm_status st = set_device(h);
+    if (st) return st;
+    compute_body_split(h);
+    return build_worklist(h);
+}
+
+extern "C" afmm_status afmm_p2p_get_partition(const afmm_p2p *h, long long *leaf_split,
+                                              long long *body_split) {
+    if (!h) return AFMM_EINVAL;
+    if (!h->have_tree) return AFMM_ESTATE;
+    const int W = h->cfg.world;
+    if (leaf_split) std::copy(h->leaf_split.begin(), h->leaf_split.end(), leaf_split);
+    if (body_split) std::copy(h->body_split.begin(), h->body_split.end(), body_split);
+    (void)W;
+    return AFMM_OK;
+}
+
+// Solve the small SPD system M c = b (Gaussian elimination with partial pivoting).
+static bool solve_small(std::vector<double> M, std::vector<double> b, int k, std::vector<double> &x) {
+    for (int col = 0; col < k; ++col) {
+        int piv = col;
+        for (int r = col + 1; r < k; ++r)
+            if (std::fabs(M[r * k + col]) > std::fabs(M[piv * k + col])) piv = r;
+        if (std::fabs(M[piv * k + col]) < 1e-300) return false;
+        if (piv != col) {
+            for (int cc = 0; cc < k; ++cc) std::swap(M[col * k + cc], M[piv * k + cc]);
+            std::swap(b[col], b[piv]);
+        }
+        for (int r = col + 1; r < k; ++r) {
+            const double f = M[r * k + col] / M[col * k + col];
+            for (int cc = col; cc < k; ++cc) M[r * k + cc] -= f * M[col * k + cc];
+            b[r] -= f * b[col];
+        }
+    }
+    x.assign(k, 0.0);
+    for (int r = k - 1; r >= 0; --r) {
+        double s = b[r];
+        for (int cc = r + 1; cc < k; ++cc) s -= M[r * k + cc] * x[cc];
+        x[r] = s / M[r * k + r];
+    }
+    return true;
+}
+
+extern "C" afmm_status afmm_p2p_rebalance(afmm_p2p *h, const double *rank_ms, double threshold,
+                                          int *changed) {
+    CHECK_HANDLE(h);
+    if (changed) *changed = 0;
+    if (!h->have_tree) return fail(h, AFMM_ESTATE, "rebalance: no tree");
+    if (!rank_ms) return fail(h, AFMM_EINVAL, "rebalance: rank_ms is null");
+    const int W = h->cfg.world;
+    if (W == 1) return AFMM_OK;
+    for (int r = 0; r < W; ++r)
+        if (!(rank_ms[r] >= 0.0) || !std::isfinite(rank_ms[r]))
+            return fail(h, AFMM_EINVAL, "rebalance: rank_ms[%d] invalid", r);
+    // per-rank bucket interaction counts for the CURRENT partition (all ranks)
+    std::vector<double> B((size_t)W * 8, 0.0);
+    double Isum = 0, Tsum = 0;
+    for (int r = 0; r < W; ++r) {
+        for (long long t = h->leaf_split[r]; t < h->leaf_split[r + 1]; ++t)
+            B[r * 8 + bucket_of(h->leaf_count[t])] += (double)h->I[t];
+        Tsum += rank_ms[r];
+    }
+    for (double v : B) Isum += v;
+    if (Isum <= 0 || Tsum <= 0) return AFMM_OK;
+    const double k0 = Tsum / Isum;     // the paper's GPU coefficient, all ranks (L18 SIV.D)
+    // ridge-regularised least squares for per-bucket coefficients around k0:
+    // min sum_r (sum_b B_rb c_b - T_r)^2 + lam * sum_b (Bsum_b/W)^2 (c_b - k0)^2
+    std::vector<double> M(64, 0.0), rhs(8, 0.0), Bs(8, 0.0);
+    for (int r = 0; r < W; ++r)
+        for (int b = 0; b < 8; ++b) Bs[b] += B[r * 8 + b];
+    const double lam = 0.1;
+    for (int r = 0; r < W; ++r)
+        for (int a = 0; a < 8; ++a) {
+            for (int b = 0; b < 8; ++b) M[a * 8 + b] += B[r * 8 + a] * B[r * 8 + b];
+            rhs[a] += B[r * 8 + a] * rank_ms[r];
+        }
+    for (int b = 0; b < 8; ++b) {
+        const double wgt = lam * (Bs[b] / W) * (Bs[b] / W) + 1e-30;
+        M[b * 8 + b] += wgt;
+        rhs[b] += wgt * k0;
+    }
+    std::vector<double> coef;
+    if (!solve_small(M, rhs, 8, coef)) coef.assign(8, k0);
+    for (double &c : coef)
+        if (!(c > 0.05 * k0)) c = 0.05 * k0;      // keep weights positive
+    std::vector<double> w(h->L);
+    for (int t = 0; t < h->L; ++t) w[t] = (double)h->I[t] * coef[bucket_of(h->leaf_count[t])];
+    std::vector<long long> split(W + 1);
+    afmm_partition_weighted(h->L, w.data(), W, split.data());
+    // predicted imbalance of the new cut vs the measured one
+    double tmax = 0, pmax = 0, psum = 0;
+    for (int r = 0; r < W; ++r) tmax = std::max(tmax, rank_ms[r]);
+    for (int r = 0; r < W; ++r) {
+        double p = 0;
+        for (long long t = split[r]; t < split[r + 1]; ++t) p += w[t];
+        pmax = std::max(pmax, p);
+        psum += p;
+    }
+    const double cur_imb = tmax / (Tsum / W);
+    const double new_imb = psum > 0 ? pmax / (psum / W) : 1.0;
+    if (cur_imb - new_imb > threshold && split != h->leaf_split) {
+        h->leaf_split = split;
+        h->user_partition = true;
+        compute_body_split(h);
+        afmm_status st = set_device(h);
+        if (st) return st;
+        if ((st = build_worklist(h))) return st;
+        if (changed) *changed = 1;
+    }
+    return AFMM_OK;
+}
+
+// ------------------------------------------------------------------ eval
+
+static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, float *phi) {
+    afmm::P2PParams p;
+    p.bodies = h->d_bodies;
+    p.items = h->d_items;
+    p.chunks = h->d_chunks;
+    p.segs = h->d_segs;
+    p.n_items = (int)h->h_items.size();
+    p.queue = h->d_queue;
+    p.ax = ax;
+    p.ay = ay;
+    p.az = az;
+    p.phi = phi;
+    p.eps2 = h->cfg.eps2;
+    p.G = (double)h->cfg.G;
+    CUDA_TRY(h, cudaMemsetAsync(h->d_queue, 0, sizeof(int), h->stream));
+    CUDA_TRY(h, cudaEventRecord(h->ev0, h->stream));
+    int nlaunch = 0;
+    if (p.n_items > 0) {
+        const int grid = std::max(1, std::min(p.n_items, h->num_sms * h->blocks_per_sm));
+        afmm::p2p_kernel<<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(p);
+        CUDA_TRY(h, cudaGetLastError());
+        nlaunch = 1;
+    }
+    CUDA_TRY(h, cudaEventRecord(h->ev1, h->stream));
+    h->evaluated = true;
+    h->last.n_launches = nlaunch;
+    return AFMM_OK;
+}
+
+static afmm_status fill_stats(afmm_p2p *h, afmm_p2p_stats *s) {
+    CUDA_TRY(h, cudaStreamSynchronize(h->stream));
+    float ms = 0.f;
+    CUDA_TRY(h, cudaEventElapsedTime(&ms, h->ev0, h->ev1));
+    afmm_p2p_stats o{};
+    o.kernel_ms = ms;
+    o.interactions_total = h->I_total;
+    o.interactions_rank = h->rank_interactions;
+    o.leaf_lo = h->leaf_split[h->cfg.rank];
+    o.leaf_hi = h->leaf_split[h->cfg.rank + 1];
+    o.body_lo = h->body_split[h->cfg.rank];
+    o.body_hi = h->body_split[h->cfg.rank + 1];
+    o.n_work_items = (int)h->h_items.size();
+    o.n_launches = h->last.n_launches;
+    for (int b = 0; b < 8; ++b) o.bucket_interactions[b] = h->bucket_inter[b];
+    h->last = o;
+    if (s) *s = o;
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_p2p_eval(afmm_p2p *h, float *ax, float *ay, float *az, float *phi,
+                                     afmm_p2p_stats *stats) {
+    CHECK_HANDLE(h);
+    if (!h->d_bodies || !h->have_tree) return fail(h, AFMM_ESTATE, "eval: set_bodies and set_tree first");
+    if (!ax || !ay || !az || !phi) return fail(h, AFMM_EINVAL, "eval: null output pointer");
+    afmm_status st = set_device(h);
+    if (st) return st;
+    if ((st = launch_eval(h, ax, ay, az, phi))) return st;
+    if (stats) return fill_stats(h, stats);
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_p2p_eval_host(afmm_p2p *h, float *ax, float *ay, float *az, float *phi,
+                                          afmm_p2p_stats *stats) {
+    CHECK_HANDLE(h);
+    if (!h->d_bodies || !h->have_tree) return fail(h, AFMM_ESTATE, "eval_host: set_bodies and set_tree first");
+    if (!ax || !ay || !az || !phi) return fail(h, AFMM_EINVAL, "eval_host: null output pointer");
+    afmm_status st = set_device(h);
+    if (st) return st;
+    const long long n = h->n;
+    if (4 * n > h->out_cap) {
+        cudaFree(h->d_out);
+        h->d_out = nullptr;
+        h->out_cap = 0;
+        CUDA_TRY(h, cudaMalloc(&h->d_out, (size_t)(4 * n) * sizeof(float)));
+        h->out_cap = 4 * n;
+    }
+    float *d[4] = {h->d_out, h->d_out + n, h->d_out + 2 * n, h->d_out + 3 * n};
+    if ((st = launch_eval(h, d[0], d[1], d[2], d[3]))) return st;
+    const long long lo = h->body_split[h->cfg.rank], hi = h->body_split[h->cfg.rank + 1];
+    float *hp[4] = {ax, ay, az, phi};
+    if (hi > lo)
+        for (int a = 0; a < 4; ++a)
+            CUDA_TRY(h, cudaMemcpyAsync(hp[a] + lo, d[a] + lo, (size_t)(hi - lo) * sizeof(float),
+                                        cudaMemcpyDeviceToHost, h->stream));
+    return fill_stats(h, stats);
+}
+
+extern "C" afmm_status afmm_p2p_stats_get(afmm_p2p *h, afmm_p2p_stats *stats) {
+    CHECK_HANDLE(h);
+    if (!h->evaluated) return fail(h, AFMM_ESTATE, "stats_get: no eval yet");
+    afmm_status st = set_device(h);
+    if (st) return st;
+    return fill_stats(h, stats);
+}

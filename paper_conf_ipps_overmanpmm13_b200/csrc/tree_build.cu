@@ -1,0 +1,626 @@
+// tree_build.cu -- GPU adaptive octree + U-list builder (include/afmm_tree.h).
+//
+// PAPER.md L10 SI.B: "a node is subdivided into eight children if it holds more
+// than [S] bodies"; L16 SIII.B builds the tree by "recursive parallel partition
+// of the body locations into the child trees on the way down".  The B200 form
+// of that partition: fp64 quantisation + 63-bit Morton keys (one kernel), a
+// stable radix sort (CUB), then a level-synchronous split where each open node
+// finds its octant ranges by binary search in the sorted keys and children are
+// placed by an exclusive scan (deterministic, no atomics).  Leaves are numbered
+// by a scan over their first-body flags, which is Morton (DFS) order.  U-lists
+// come from a per-leaf descent over the node arrays (count, scan, fill).
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <string>
+#include <vector>
+
+#include <cub/cub.cuh>
+#include <cuda_runtime.h>
+
+#include "../../include/afmm_tree.h"
+
+namespace {
+
+constexpr int kMaxLevel = 21;
+
+__device__ __forceinline__ unsigned long long spread3(unsigned long long v) {
+    v &= 0x1fffffull;
+    v = (v | (v << 32)) & 0x1f00000000ffffull;
+    v = (v | (v << 16)) & 0x1f0000ff0000ffull;
+    v = (v | (v << 8)) & 0x100f00f00f00f00full;
+    v = (v | (v << 4)) & 0x10c30c30c30c30c3ull;
+    v = (v | (v << 2)) & 0x1249249249249249ull;
+    return v;
+}
+__device__ __forceinline__ unsigned long long compact3(unsigned long long v) {
+    v &= 0x1249249249249249ull;
+    v = (v ^ (v >> 2)) & 0x10c30c30c30c30c3ull;
+    v = (v ^ (v >> 4)) & 0x100f00f00f00f00full;
+    v = (v ^ (v >> 8)) & 0x1f0000ff0000ffull;
+    v = (v ^ (v >> 16)) & 0x1f00000000ffffull;
+    v = (v ^ (v >> 32)) & 0x1fffffull;
+    return v;
+}
+
+// q = clamp(floor((v - lo) * 2^(21-k)), 0, 2^21 - 1); fp64, explicit RN ops (no FMA)
+__device__ __forceinline__ unsigned long long quantize(float v, double lo, double scale) {
+    const double t = __dmul_rn(__dsub_rn((double)v, lo), scale);
+    const double f = floor(t);
+    if (!(f >= 0.0)) return 0ull;
+    if (f > 2097151.0) return 2097151ull;
+    return (unsigned long long)f;
+}
+
+__global__ void minmax_kernel(long long n, const float *__restrict__ x, const float *__restrict__ y,
+                              const float *__restrict__ z, float *__restrict__ part) {
+    float mn[3] = {INFINITY, INFINITY, INFINITY}, mx[3] = {-INFINITY, -INFINITY, -INFINITY};
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n;
+         i += (long long)gridDim.x * blockDim.x) {
+        const float v[3] = {x[i], y[i], z[i]};
+#pragma unroll
+        for (int a = 0; a < 3; ++a) {
+            mn[a] = fminf(mn[a], v[a]);
+            mx[a] = fmaxf(mx[a], v[a]);
+        }
+    }
+    __shared__ float s[6][256];
+#pragma unroll
+    for (int a = 0; a < 3; ++a) {
+        s[a][threadIdx.x] = mn[a];
+        s[3 + a][threadIdx.x] = mx[a];
+    }
+    __syncthreads();
+    for (int w = blockDim.x / 2; w > 0; w >>= 1) {
+        if (threadIdx.x < w) {
+#pragma unroll
+            for (int a = 0; a < 3; ++a) {
+                s[a][threadIdx.x] = fminf(s[a][threadIdx.x], s[a][threadIdx.x + w]);
+                s[3 + a][threadIdx.x] = fmaxf(s[3 + a][threadIdx.x], s[3 + a][threadIdx.x + w]);
+            }
+        }
+        __syncthreads();
+    }
+    if (threadIdx.x < 6) part[blockIdx.x * 6 + threadIdx.x] = s[threadIdx.x][0];
+}
+
+__global__ void keys_kernel(long long n, const float *__restrict__ x, const float *__restrict__ y,
+                            const float *__restrict__ z, double lx, double ly, double lz,
+                            double scale, unsigned long long *__restrict__ keys,
+                            int *__restrict__ idx) {
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n;
+         i += (long long)gridDim.x * blockDim.x) {
+        const unsigned long long qx = quantize(x[i], lx, scale);
+        const unsigned long long qy = quantize(y[i], ly, scale);
+        const unsigned long long qz = quantize(z[i], lz, scale);
+        keys[i] = spread3(qx) | (spread3(qy) << 1) | (spread3(qz) << 2);
+        idx[i] = (int)i;
+    }
+}
+
+struct Nodes {
+    int *b, *e, *first_child, *nchild, *level;
+    unsigned long long *prefix;
+};
+
+// For each node of the current level: split if > S bodies and level < 21.
+// Child ranges by binary search on the octant digit inside [b, e).
+__global__ void split_count_kernel(int m, int base, Nodes nd, const unsigned long long *__restrict__ keys,
+                                   int S, int *__restrict__ cb, int *__restrict__ nc) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= m) return;
+    const int id = base + i;
+    const int b = nd.b[id], e = nd.e[id], lev = nd.level[id];
+    int cnt = 0;
+    if (e - b > S && lev < kMaxLevel) {
+        const int shift = 3 * (kMaxLevel - 1 - lev);
+        int bound[9];
+        bound[0] = b;
+        bound[8] = e;
+        for (int o = 1; o < 8; ++o) {
+            int lo = bound[o - 1], hi = e;            // first position with digit >= o
+            while (lo < hi) {
+                const int mid = lo + ((hi - lo) >> 1);
+                if ((int)((keys[mid] >> shift) & 7ull) < o) lo = mid + 1;
+                else hi = mid;
+            }
+            bound[o] = lo;
+        }
+        for (int o = 0; o < 8; ++o) {
+            cb[i * 9 + o] = bound[o];
+            cnt += bound[o + 1] > bound[o];
+        }
+        cb[i * 9 + 8] = e;
+    }
+    nc[i] = cnt;
+}
+
+__global__ void split_write_kernel(int m, int base, int next_base, Nodes nd, const int *__restrict__ cb,
+                                   const int *__restrict__ nc, const int *__restrict__ off) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= m) return;
+    const int id = base + i;
+    const int cnt = nc[i];
+    nd.nchild[id] = cnt;
+    nd.first_child[id] = cnt ? next_base + off[i] : -1;
+    if (!cnt) return;
+    int w = next_base + off[i];
+    const unsigned long long pre = nd.prefix[id];
+    const int lev = nd.level[id];
+    for (int o = 0; o < 8; ++o) {
+        const int b = cb[i * 9 + o], e = cb[i * 9 + o + 1];
+        if (e > b) {
+            nd.b[w] = b;
+            nd.e[w] = e;
+            nd.level[w] = lev + 1;
+            nd.prefix[w] = (pre << 3) | (unsigned long long)o;
+            nd.first_child[w] = -1;
+            nd.nchild[w] = 0;
+            ++w;
+        }
+    }
+}
+
+__global__ void leaf_flag_kernel(int nn, Nodes nd, int *__restrict__ flag) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= nn) return;
+    if (nd.nchild[i] == 0) flag[nd.b[i]] = 1;
+}
+
+__global__ void leaf_write_kernel(int nn, Nodes nd, const int *__restrict__ leaf_at,
+                                  int *__restrict__ node_leaf, int *__restrict__ ls,
+                                  int *__restrict__ lc, int *__restrict__ ll,
+                                  unsigned long long *__restrict__ lp) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= nn) return;
+    if (nd.nchild[i] != 0) {
+        node_leaf[i] = -1;
+        return;
+    }
+    const int id = leaf_at[nd.b[i]];
+    node_leaf[i] = id;
+    ls[id] = nd.b[i];
+    lc[id] = nd.e[i] - nd.b[i];
+    ll[id] = nd.level[i];
+    lp[id] = nd.prefix[i];
+}
+
+__device__ __forceinline__ void box_of(int level, unsigned long long prefix, long long A[3], long long &w) {
+    const int sh = kMaxLevel - level;
+    A[0] = (long long)compact3(prefix) << sh;
+    A[1] = (long long)compact3(prefix >> 1) << sh;
+    A[2] = (long long)compact3(prefix >> 2) << sh;
+    w = 1LL << sh;
+}
+
+// Per-leaf descent: count (out == nullptr) or fill the U-list row.
+__global__ void ulist_kernel(int L, Nodes nd, const int *__restrict__ node_leaf,
+                             const int *__restrict__ leaf_node, const long long *__restrict__ u_off,
+                             int *__restrict__ u_idx, long long *__restrict__ counts) {
+    const int t = blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= L) return;
+    const int tn = leaf_node[t];
+    long long At[3], wt;
+    box_of(nd.level[tn], nd.prefix[tn], At, wt);
+    int stack[8 * (kMaxLevel + 2)];
+    int sp = 0;
+    stack[sp++] = 0;
+    long long cnt = 0;
+    long long w0 = u_idx ? u_off[t] : 0;
+    while (sp > 0) {
+        const int ni = stack[--sp];
+        long long As[3], ws;
+        box_of(nd.level[ni], nd.prefix[ni], As, ws);
+        bool touch = true;
+#pragma unroll
+        for (int a = 0; a < 3; ++a) touch &= (At[a] <= As[a] + ws) && (As[a] <= At[a] + wt);
+        if (!touch) continue;
+        const int nc = nd.nchild[ni];
+        if (nc == 0) {
+            if (u_idx) u_idx[w0 + cnt] = node_leaf[ni];
+            ++cnt;
+        } else {
+            const int fc = nd.first_child[ni];
+            for (int c = nc - 1; c >= 0; --c) stack[sp++] = fc + c;
+        }
+    }
+    if (counts) counts[t] = cnt;
+}
+
+__global__ void leaf_node_kernel(int nn, const int *__restrict__ node_leaf, int *__restrict__ leaf_node) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= nn) return;
+    const int l = node_leaf[i];
+    if (l >= 0) leaf_node[l] = i;
+}
+
+__global__ void gather_kernel(long long n, const int *__restrict__ perm, const float *__restrict__ in,
+                              float *__restrict__ out) {
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n;
+         i += (long long)gridDim.x * blockDim.x)
+        out[i] = in[perm[i]];
+}
+__global__ void scatter_kernel(long long n, const int *__restrict__ perm, const float *__restrict__ in,
+                               float *__restrict__ out) {
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n;
+         i += (long long)gridDim.x * blockDim.x)
+        out[perm[i]] = in[i];
+}
+
+int grid_for(long long n, int threads) {
+    long long g = (n + threads - 1) / threads;
+    return (int)std::max<long long>(1, std::min<long long>(g, 1 << 20));
+}
+
+}  // namespace
+
+struct afmm_tree {
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    bool own_stream = false;
+    bool poisoned = false;
+    bool built = false;
+    std::string err;
+    long long n = 0;
+    int L = 0;
+    long long nnz = 0, n_nodes = 0;
+    double lo[3] = {0, 0, 0};
+    int k = 0, max_level = 0;
+    // device arrays
+    int *perm = nullptr;
+    unsigned long long *keys_sorted = nullptr;
+    int *ls = nullptr, *lc = nullptr, *ll = nullptr;
+    unsigned long long *lp = nullptr;
+    long long *u_off = nullptr;
+    int *u_idx = nullptr;
+    std::vector<void *> owned;
+};
+
+namespace {
+
+afmm_status tfail(afmm_tree *t, afmm_status st, const char *fmt, ...) {
+    if (t) {
+        char buf[512];
+        va_list ap;
+        va_start(ap, fmt);
+        vsnprintf(buf, sizeof(buf), fmt, ap);
+        va_end(ap);
+        t->err = buf;
+        if (st == AFMM_ECUDA || st == AFMM_ENOMEM) t->poisoned = true;
+    }
+    return st;
+}
+
+#define TCU(t, call)                                                                          \
+    do {                                                                                      \
+        cudaError_t e_ = (call);                                                              \
+        if (e_ != cudaSuccess)                                                                \
+            return tfail((t), e_ == cudaErrorMemoryAllocation ? AFMM_ENOMEM : AFMM_ECUDA,      \
+                         "%s failed: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__,     \
+                         __LINE__);                                                           \
+    } while (0)
+
+void free_all(afmm_tree *t) {
+    for (void *p : t->owned) cudaFree(p);
+    t->owned.clear();
+    t->perm = nullptr;
+    t->keys_sorted = nullptr;
+    t->ls = t->lc = t->ll = nullptr;
+    t->lp = nullptr;
+    t->u_off = nullptr;
+    t->u_idx = nullptr;
+}
+
+template <typename T>
+afmm_status dalloc(afmm_tree *t, T **p, size_t count) {
+    void *q = nullptr;
+    TCU(t, cudaMalloc(&q, std::max<size_t>(count, 1) * sizeof(T)));
+    t->owned.push_back(q);
+    *p = static_cast<T *>(q);
+    return AFMM_OK;
+}
+
+// scoped temporaries
+struct Tmp {
+    std::vector<void *> v;
+    ~Tmp() {
+        for (void *p : v) cudaFree(p);
+    }
+};
+template <typename T>
+afmm_status talloc(afmm_tree *t, Tmp &tmp, T **p, size_t count) {
+    void *q = nullptr;
+    TCU(t, cudaMalloc(&q, std::max<size_t>(count, 1) * sizeof(T)));
+    tmp.v.push_back(q);
+    *p = static_cast<T *>(q);
+    return AFMM_OK;
+}
+
+}  // namespace
+
+extern "C" afmm_status afmm_tree_create(int device, void *stream, afmm_tree **out) {
+    if (!out) return AFMM_EINVAL;
+    *out = nullptr;
+    if (device < 0) return AFMM_EINVAL;
+    afmm_tree *t = new (std::nothrow) afmm_tree();
+    if (!t) return AFMM_ENOMEM;
+    t->device = device;
+    cudaError_t e = cudaSetDevice(device);
+    if (e == cudaSuccess) {
+        if (stream) {
+            t->stream = static_cast<cudaStream_t>(stream);
+        } else {
+            e = cudaStreamCreateWithFlags(&t->stream, cudaStreamNonBlocking);
+            t->own_stream = (e == cudaSuccess);
+        }
+    }
+    if (e != cudaSuccess) {
+        delete t;
+        return AFMM_ECUDA;
+    }
+    *out = t;
+    return AFMM_OK;
+}
+
+extern "C" void afmm_tree_destroy(afmm_tree *t) {
+    if (!t) return;
+    cudaSetDevice(t->device);
+    if (t->stream) cudaStreamSynchronize(t->stream);
+    free_all(t);
+    if (t->own_stream && t->stream) cudaStreamDestroy(t->stream);
+    delete t;
+}
+
+extern "C" const char *afmm_tree_last_error(const afmm_tree *t) { return t ? t->err.c_str() : "null handle"; }
+
+extern "C" afmm_status afmm_tree_build(afmm_tree *t, long long n, const float *x, const float *y,
+                                       const float *z, int S, int fixed_domain, const double *lo_in,
+                                       int k_in) {
+    if (!t) return AFMM_EINVAL;
+    if (t->poisoned) return AFMM_ESTATE;
+    if (n < 1 || n >= (1LL << 31)) return tfail(t, AFMM_EINVAL, "tree_build: n=%lld out of range", n);
+    if (S < 1) return tfail(t, AFMM_EINVAL, "tree_build: S=%d < 1", S);
+    if (!x || !y || !z) return tfail(t, AFMM_EINVAL, "tree_build: null coordinate pointer");
+    if (fixed_domain && (!lo_in || !std::isfinite(lo_in[0]) || !std::isfinite(lo_in[1]) ||
+                         !std::isfinite(lo_in[2]) || k_in < -1000 || k_in > 1000))
+        return tfail(t, AFMM_EINVAL, "tree_build: bad fixed domain");
+    TCU(t, cudaSetDevice(t->device));
+    free_all(t);
+    t->built = false;
+    cudaStream_t st = t->stream;
+    Tmp tmp;
+    const int TH = 256;
+
+    // 1. domain (reading R6): lo = min, side = smallest power of two > max extent
+    if (fixed_domain) {
+        for (int a = 0; a < 3; ++a) t->lo[a] = lo_in[a];
+        t->k = k_in;
+    } else {
+        const int g = 296;
+        float *part;
+        if (afmm_status s = talloc(t, tmp, &part, (size_t)g * 6)) return s;
+        minmax_kernel<<<g, TH, 0, st>>>(n, x, y, z, part);
+        TCU(t, cudaGetLastError());
+        std::vector<float> h(g * 6);
+        TCU(t, cudaMemcpyAsync(h.data(), part, h.size() * sizeof(float), cudaMemcpyDeviceToHost, st));
+        TCU(t, cudaStreamSynchronize(st));
+        double ext = 0.0;
+        for (int a = 0; a < 3; ++a) {
+            float mn = h[a], mx = h[3 + a];
+            for (int b = 1; b < g; ++b) {
+                mn = std::min(mn, h[b * 6 + a]);
+                mx = std::max(mx, h[b * 6 + 3 + a]);
+            }
+            t->lo[a] = (double)mn;
+            ext = std::max(ext, (double)mx - (double)mn);
+        }
+        int e = 0;
+        if (ext > 0.0) std::frexp(ext, &e);
+        t->k = e;
+    }
+    const double scale = std::ldexp(1.0, kMaxLevel - t->k);
+
+    // 2. keys; 3. stable radix sort by (key, index)
+    unsigned long long *keys;
+    int *idx;
+    if (afmm_status s = talloc(t, tmp, &keys, n)) return s;
+    if (afmm_status s = talloc(t, tmp, &idx, n)) return s;
+    if (afmm_status s = dalloc(t, &t->keys_sorted, n)) return s;
+    if (afmm_status s = dalloc(t, &t->perm, n)) return s;
+    keys_kernel<<<grid_for(n, TH), TH, 0, st>>>(n, x, y, z, t->lo[0], t->lo[1], t->lo[2], scale, keys, idx);
+    TCU(t, cudaGetLastError());
+    {
+        size_t tb = 0;
+        TCU(t, cub::DeviceRadixSort::SortPairs(nullptr, tb, keys, t->keys_sorted, idx, t->perm, (int)n, 0,
+                                               3 * kMaxLevel, st));
+        void *tbuf;
+        if (afmm_status s = talloc(t, tmp, reinterpret_cast<char **>(&tbuf), tb)) return s;
+        TCU(t, cub::DeviceRadixSort::SortPairs(tbuf, tb, keys, t->keys_sorted, idx, t->perm, (int)n, 0,
+                                               3 * kMaxLevel, st));
+    }
+
+    // 4. level-synchronous split into one node array (level-major)
+    size_t cap = 1024;
+    std::vector<void *> node_bufs;
+    Nodes nd{};
+    auto alloc_nodes = [&](size_t c, Nodes &o) -> afmm_status {
+        if (afmm_status s = talloc(t, tmp, &o.b, c)) return s;
+        if (afmm_status s = talloc(t, tmp, &o.e, c)) return s;
+        if (afmm_status s = talloc(t, tmp, &o.first_child, c)) return s;
+        if (afmm_status s = talloc(t, tmp, &o.nchild, c)) return s;
+        if (afmm_status s = talloc(t, tmp, &o.level, c)) return s;
+        if (afmm_status s = talloc(t, tmp, &o.prefix, c)) return s;
+        return AFMM_OK;
+    };
+    if (afmm_status s = alloc_nodes(cap, nd)) return s;
+    {
+        const int zero = 0, nn = (int)n, lv = 0, m1 = -1;
+        const unsigned long long p0 = 0;
+        TCU(t, cudaMemcpyAsync(nd.b, &zero, sizeof(int), cudaMemcpyHostToDevice, st));
+        TCU(t, cudaMemcpyAsync(nd.e, &nn, sizeof(int), cudaMemcpyHostToDevice, st));
+        TCU(t, cudaMemcpyAsync(nd.first_child, &m1, sizeof(int), cudaMemcpyHostToDevice, st));
+        TCU(t, cudaMemcpyAsync(nd.nchild, &zero, sizeof(int), cudaMemcpyHostToDevice, st));
+        TCU(t, cudaMemcpyAsync(nd.level, &lv, sizeof(int), cudaMemcpyHostToDevice, st));
+        TCU(t, cudaMemcpyAsync(nd.prefix, &p0, sizeof(p0), cudaMemcpyHostToDevice, st));
+        TCU(t, cudaStreamSynchronize(st));
+    }
+    long long base = 0, m = 1;     // current level occupies [base, base+m)
+    int level = 0;
+    int *cb = nullptr, *nc = nullptr, *off = nullptr;
+    size_t lvl_cap = 0;
+    void *scan_tmp = nullptr;
+    size_t scan_tmp_bytes = 0;
+    Tmp lvl_tmp_holder;
+    while (m > 0) {
+        if ((size_t)m + 1 > lvl_cap) {
+            lvl_cap = std::max<size_t>((size_t)m + 1, 2 * lvl_cap);
+            if (afmm_status s = talloc(t, tmp, &cb, lvl_cap * 9)) return s;
+            if (afmm_status s = talloc(t, tmp, &nc, lvl_cap)) return s;
+            if (afmm_status s = talloc(t, tmp, &off, lvl_cap)) return s;
+            size_t need = 0;
+            TCU(t, cub::DeviceScan::ExclusiveSum(nullptr, need, nc, off, (int)lvl_cap, st));
+            if (need > scan_tmp_bytes) {
+                if (afmm_status s = talloc(t, tmp, reinterpret_cast<char **>(&scan_tmp), need)) return s;
+                scan_tmp_bytes = need;
+            }
+        }
+        split_count_kernel<<<grid_for(m, TH), TH, 0, st>>>((int)m, (int)base, nd, t->keys_sorted, S, cb, nc);
+        TCU(t, cudaGetLastError());
+        TCU(t, cudaMemsetAsync(nc + m, 0, sizeof(int), st));
+        size_t sb = scan_tmp_bytes;
+        TCU(t, cub::DeviceScan::ExclusiveSum(scan_tmp, sb, nc, off, (int)(m + 1), st));
+        int total = 0;
+        TCU(t, cudaMemcpyAsync(&total, off + m, sizeof(int), cudaMemcpyDeviceToHost, st));
+        TCU(t, cudaStreamSynchronize(st));
+        const long long next_base = base + m;
+        if ((size_t)(next_base + total) > cap) {
+            size_t ncap = std::max<size_t>(2 * cap, (size_t)(next_base + total));
+            Nodes n2{};
+            if (afmm_status s = alloc_nodes(ncap, n2)) return s;
+            TCU(t, cudaMemcpyAsync(n2.b, nd.b, next_base * sizeof(int), cudaMemcpyDeviceToDevice, st));
+            TCU(t, cudaMemcpyAsync(n2.e, nd.e, next_base * sizeof(int), cudaMemcpyDeviceToDevice, st));
+            TCU(t, cudaMemcpyAsync(n2.first_child, nd.first_child, next_base * sizeof(int), cudaMemcpyDeviceToDevice, st));
+            TCU(t, cudaMemcpyAsync(n2.nchild, nd.nchild, next_base * sizeof(int), cudaMemcpyDeviceToDevice, st));
+            TCU(t, cudaMemcpyAsync(n2.level, nd.level, next_base * sizeof(int), cudaMemcpyDeviceToDevice, st));
+            TCU(t, cudaMemcpyAsync(n2.prefix, nd.prefix, next_base * sizeof(unsigned long long), cudaMemcpyDeviceToDevice, st));
+            nd = n2;
+            cap = ncap;
+        }
+        split_write_kernel<<<grid_for(m, TH), TH, 0, st>>>((int)m, (int)base, (int)next_base, nd, cb, nc, off);
+        TCU(t, cudaGetLastError());
+        t->max_level = level;
+        base = next_base;
+        m = total;
+        ++level;
+    }
+    const long long nn = base;     // total nodes
+    t->n_nodes = nn;
+
+    // 5. leaves in Morton order: flag first bodies, scan
+    int *flag, *leaf_at, *node_leaf;
+    if (afmm_status s = talloc(t, tmp, &flag, n + 1)) return s;
+    if (afmm_status s = talloc(t, tmp, &leaf_at, n + 1)) return s;
+    if (afmm_status s = talloc(t, tmp, &node_leaf, nn)) return s;
+    TCU(t, cudaMemsetAsync(flag, 0, (n + 1) * sizeof(int), st));
+    leaf_flag_kernel<<<grid_for(nn, TH), TH, 0, st>>>((int)nn, nd, flag);
+    TCU(t, cudaGetLastError());
+    {
+        size_t sb = 0;
+        TCU(t, cub::DeviceScan::ExclusiveSum(nullptr, sb, flag, leaf_at, (int)(n + 1), st));
+        char *sbuf;
+        if (afmm_status s = talloc(t, tmp, &sbuf, sb)) return s;
+        TCU(t, cub::DeviceScan::ExclusiveSum(sbuf, sb, flag, leaf_at, (int)(n + 1), st));
+    }
+    int L = 0;
+    TCU(t, cudaMemcpyAsync(&L, leaf_at + n, sizeof(int), cudaMemcpyDeviceToHost, st));
+    TCU(t, cudaStreamSynchronize(st));
+    t->L = L;
+    if (afmm_status s = dalloc(t, &t->ls, L)) return s;
+    if (afmm_status s = dalloc(t, &t->lc, L)) return s;
+    if (afmm_status s = dalloc(t, &t->ll, L)) return s;
+    if (afmm_status s = dalloc(t, &t->lp, L)) return s;
+    leaf_write_kernel<<<grid_for(nn, TH), TH, 0, st>>>((int)nn, nd, leaf_at, node_leaf, t->ls, t->lc, t->ll, t->lp);
+    TCU(t, cudaGetLastError());
+    int *leaf_node;
+    if (afmm_status s = talloc(t, tmp, &leaf_node, L)) return s;
+    leaf_node_kernel<<<grid_for(nn, TH), TH, 0, st>>>((int)nn, node_leaf, leaf_node);
+    TCU(t, cudaGetLastError());
+
+    // 6. U-lists: count, scan, fill
+    long long *counts;
+    if (afmm_status s = talloc(t, tmp, &counts, (size_t)L + 1)) return s;
+    if (afmm_status s = dalloc(t, &t->u_off, (size_t)L + 1)) return s;
+    TCU(t, cudaMemsetAsync(counts + L, 0, sizeof(long long), st));
+    ulist_kernel<<<grid_for(L, 128), 128, 0, st>>>(L, nd, node_leaf, leaf_node, nullptr, nullptr, counts);
+    TCU(t, cudaGetLastError());
+    {
+        size_t sb = 0;
+        TCU(t, cub::DeviceScan::ExclusiveSum(nullptr, sb, counts, t->u_off, L + 1, st));
+        char *sbuf;
+        if (afmm_status s = talloc(t, tmp, &sbuf, sb)) return s;
+        TCU(t, cub::DeviceScan::ExclusiveSum(sbuf, sb, counts, t->u_off, L + 1, st));
+    }
+    TCU(t, cudaMemcpyAsync(&t->nnz, t->u_off + L, sizeof(long long), cudaMemcpyDeviceToHost, st));
+    TCU(t, cudaStreamSynchronize(st));
+    if (afmm_status s = dalloc(t, &t->u_idx, (size_t)t->nnz)) return s;
+    ulist_kernel<<<grid_for(L, 128), 128, 0, st>>>(L, nd, node_leaf, leaf_node, t->u_off, t->u_idx, nullptr);
+    TCU(t, cudaGetLastError());
+    TCU(t, cudaStreamSynchronize(st));
+    t->n = n;
+    t->built = true;
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_tree_info(const afmm_tree *t, int *n_leaves, long long *nnz, double *lo,
+                                      int *k, int *max_level, long long *n_nodes) {
+    if (!t) return AFMM_EINVAL;
+    if (!t->built) return AFMM_ESTATE;
+    if (n_leaves) *n_leaves = t->L;
+    if (nnz) *nnz = t->nnz;
+    if (lo)
+        for (int a = 0; a < 3; ++a) lo[a] = t->lo[a];
+    if (k) *k = t->k;
+    if (max_level) *max_level = t->max_level;
+    if (n_nodes) *n_nodes = t->n_nodes;
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_tree_copy_out(const afmm_tree *tc, int *perm, int *leaf_start, int *leaf_count,
+                                          int *leaf_level, unsigned long long *leaf_prefix,
+                                          long long *u_off, int *u_idx) {
+    afmm_tree *t = const_cast<afmm_tree *>(tc);
+    if (!t) return AFMM_EINVAL;
+    if (!t->built) return AFMM_ESTATE;
+    TCU(t, cudaSetDevice(t->device));
+    cudaStream_t st = t->stream;
+    if (perm) TCU(t, cudaMemcpyAsync(perm, t->perm, t->n * sizeof(int), cudaMemcpyDeviceToHost, st));
+    if (leaf_start) TCU(t, cudaMemcpyAsync(leaf_start, t->ls, t->L * sizeof(int), cudaMemcpyDeviceToHost, st));
+    if (leaf_count) TCU(t, cudaMemcpyAsync(leaf_count, t->lc, t->L * sizeof(int), cudaMemcpyDeviceToHost, st));
+    if (leaf_level) TCU(t, cudaMemcpyAsync(leaf_level, t->ll, t->L * sizeof(int), cudaMemcpyDeviceToHost, st));
+    if (leaf_prefix)
+        TCU(t, cudaMemcpyAsync(leaf_prefix, t->lp, t->L * sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
+    if (u_off) TCU(t, cudaMemcpyAsync(u_off, t->u_off, (t->L + 1) * sizeof(long long), cudaMemcpyDeviceToHost, st));
+    if (u_idx && t->nnz > 0)
+        TCU(t, cudaMemcpyAsync(u_idx, t->u_idx, t->nnz * sizeof(int), cudaMemcpyDeviceToHost, st));
+    TCU(t, cudaStreamSynchronize(st));
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_tree_gather(afmm_tree *t, const float *in, float *out) {
+    if (!t || !in || !out) return AFMM_EINVAL;
+    if (!t->built) return AFMM_ESTATE;
+    TCU(t, cudaSetDevice(t->device));
+    gather_kernel<<<grid_for(t->n, 256), 256, 0, t->stream>>>(t->n, t->perm, in, out);
+    TCU(t, cudaGetLastError());
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_tree_scatter(afmm_tree *t, const float *in, float *out) {
+    if (!t || !in || !out) return AFMM_EINVAL;
+    if (!t->built) return AFMM_ESTATE;
+    TCU(t, cudaSetDevice(t->device));
+    scatter_kernel<<<grid_for(t->n, 256), 256, 0, t->stream>>>(t->n, t->perm, in, out);
+    TCU(t, cudaGetLastError());
+    return AFMM_OK;
+}

@@ -1,0 +1,275 @@
+"""GPU parity of the CUDA P2P path (through the C ABI) against the fp64 oracle.
+
+Tolerance: DESIGN.md reading R16 (tests/_tol.py).  Integer tree inputs come
+from the oracle here; tests/test_gpu_tree.py checks the GPU tree builder
+bit-exactly against it and runs the full-size configs end to end."""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from tests import _tol
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+
+def _afmm():
+    import paper_conf_ipps_overmanpmm13_b200 as afmm
+    return afmm
+
+
+def _dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a, np.float32)).cuda()
+
+
+def gpu_eval(xs, ys, zs, ms, T, eps2, G=1.0, world=1, max_leaf=1024, leaf_split=None):
+    """Run the library for every rank of `world` on this one GPU and merge the
+    disjoint output slices (ranks write only their own bodies)."""
+    afmm = _afmm()
+    n = xs.shape[0]
+    out = [torch.full((n,), float("nan"), device="cuda") for _ in range(4)]
+    bodies = [_dev(v) for v in (xs, ys, zs, ms)]
+    stats = []
+    for r in range(world):
+        h = afmm.P2P(device=0, rank=r, world=world, G=G, eps2=eps2, max_leaf=max_leaf)
+        h.set_bodies(*bodies)
+        if leaf_split is not None:
+            h.set_partition(leaf_split)
+        h.set_tree(T["leaf_start"], T["leaf_count"], T["u_off"], T["u_idx"])
+        stats.append(h.eval(*out, stats=True))
+        h.close()
+    torch.cuda.synchronize()
+    ax, ay, az, phi = (o.cpu().numpy() for o in out)
+    return (phi, ax, ay, az), stats                 # the oracle's order
+
+
+def _tree(x, y, z, S):
+    T = oracle.Tree(x, y, z, S)
+    return T, {"leaf_start": T.leaf_start, "leaf_count": T.leaf_count, "u_off": T.u_off,
+               "u_idx": T.u_idx}
+
+
+def _parity(x, y, z, m, S, eps2, G=1.0, targets=None, world=1):
+    T, d = _tree(x, y, z, S)
+    xs, ys, zs, ms = T.sorted_bodies(x, y, z, m)
+    got, stats = gpu_eval(xs, ys, zs, ms, d, eps2, G, world=world)
+    ref = oracle.p2p(xs, ys, zs, ms, T.leaf_start, T.leaf_count, T.u_off, T.u_idx, G, eps2,
+                     targets=targets, with_scale=True)
+    sel = np.ones(xs.shape[0], bool)
+    if targets is not None:
+        sel[:] = False
+        for t in targets:
+            sel[T.leaf_start[t]:T.leaf_start[t] + T.leaf_count[t]] = True
+    e = _tol.check([g[sel] for g in got], [r[sel] for r in ref[:4]], ref[4][sel])
+    I = oracle.interactions(T.leaf_count, T.u_off, T.u_idx)
+    assert sum(s["interactions_rank"] for s in stats) == int(I.sum())
+    assert stats[0]["interactions_total"] == int(I.sum())
+    return e, got, T
+
+
+def test_c1_parity():
+    x, y, z, m = synth.make("C1")
+    e, _, _ = _parity(x, y, z, m, 64, 1e-6)
+    assert e["phi_max_rel"] < 2e-6
+
+
+@pytest.mark.parametrize("S", [32, 128, 512])
+def test_c2_plummer_parity_full(S):
+    """C2 (1M Plummer) at three points of the S sweep, every body checked."""
+    x, y, z, m = synth.make("C2")
+    _parity(x, y, z, m, S, 1e-6)
+
+
+def test_c3_colliding_parity_full():
+    x, y, z, m = synth.make("C3")
+    _parity(x, y, z, m, 128, 1e-6)
+
+
+@pytest.mark.parametrize("dist,n,S,eps2", [("uniform", 20000, 1, 1e-6), ("uniform", 20000, 7, 0.0),
+                                           ("plummer", 50000, 300, 1e-4), ("colliding", 30000, 33, 1e-6),
+                                           ("plummer", 1000, 5000, 1e-6)])
+def test_ragged_leaf_sizes(dist, n, S, eps2):
+    """Leaves of every size 1..S (ragged tails of the lane mapping), eps2 = 0,
+    one-leaf trees (N <= S), sources spanning several 1024-body stages."""
+    x, y, z, m = synth.make(dist, n, 17)
+    _parity(x, y, z, m, S, eps2)
+
+
+def test_single_body_and_two_bodies():
+    afmm = _afmm()
+    x = np.array([0.25], np.float32)
+    T, d = _tree(x, x, x, 1)
+    got, _ = gpu_eval(x, x, x, np.ones(1, np.float32), d, 0.0)
+    assert all(g[0] == 0.0 for g in got)          # self entry only, n_t = 1 -> exactly 0
+    x = np.array([0.25, 0.75], np.float32)
+    y = np.array([0.5, 0.125], np.float32)
+    z = np.array([0.0, 0.5], np.float32)
+    m = np.array([0.5, 0.25], np.float32)
+    for S in (1, 2):
+        T, d = _tree(x, y, z, S)
+        xs, ys, zs, ms = T.sorted_bodies(x, y, z, m)
+        got, _ = gpu_eval(xs, ys, zs, ms, d, 1e-2, G=2.0)
+        for i in range(2):
+            j = 1 - i
+            dd = np.array([xs[j] - xs[i], ys[j] - ys[i], zs[j] - zs[i]], float)
+            r2 = dd @ dd + 1e-2
+            assert got[0][i] == pytest.approx(-2.0 * ms[j] / np.sqrt(r2), rel=1e-6)
+            assert np.allclose([got[1][i], got[2][i], got[3][i]], 2.0 * ms[j] * dd / r2 ** 1.5, rtol=1e-6)
+
+
+def test_big_leaves_target_chunking():
+    """Level-21 leaves larger than 512 targets (split into target chunks) and
+    larger than one 1024-body stage."""
+    rng = np.random.default_rng(3)
+    base = np.array([0.5, 0.5, 0.5])
+    cl = base + rng.random((1000, 3)) * 1e-7             # one quantisation cell
+    far = rng.random((3000, 3))
+    P = np.concatenate([cl, far, [[0, 0, 0], [0.999, 0.999, 0.999]]]).astype(np.float32)
+    m = np.full(P.shape[0], 1.0 / P.shape[0], np.float32)
+    x, y, z = P[:, 0].copy(), P[:, 1].copy(), P[:, 2].copy()
+    T = oracle.Tree(x, y, z, 16)
+    assert T.leaf_count.max() >= 900 and T.leaf_level[T.leaf_count.argmax()] == 21
+    e, _, _ = _parity(x, y, z, m, 16, 1e-12)
+
+
+def test_deterministic_and_world_invariant():
+    """Bit-identical results across repeated evals and world sizes 1/2/3/8."""
+    x, y, z, m = synth.make("plummer", 200000, 9)
+    T, d = _tree(x, y, z, 64)
+    xs, ys, zs, ms = T.sorted_bodies(x, y, z, m)
+    ref, _ = gpu_eval(xs, ys, zs, ms, d, 1e-6)
+    again, _ = gpu_eval(xs, ys, zs, ms, d, 1e-6)
+    for a, b in zip(ref, again):
+        assert np.array_equal(a, b)
+    for W in (2, 3, 8):
+        got, stats = gpu_eval(xs, ys, zs, ms, d, 1e-6, world=W)
+        for a, b in zip(ref, got):
+            assert np.array_equal(a, b)
+        # ranks own disjoint contiguous slices covering every body
+        lo = [s["body_lo"] for s in stats]
+        hi = [s["body_hi"] for s in stats]
+        assert lo[0] == 0 and hi[-1] == xs.shape[0] and all(hi[i] == lo[i + 1] for i in range(W - 1))
+
+
+def test_mass_scaling_bit_exact():
+    x, y, z, m = synth.make("plummer", 50000, 4)
+    T, d = _tree(x, y, z, 48)
+    xs, ys, zs, ms = T.sorted_bodies(x, y, z, m)
+    a, _ = gpu_eval(xs, ys, zs, ms, d, 1e-6)
+    b, _ = gpu_eval(xs, ys, zs, (ms * np.float32(8)).astype(np.float32), d, 1e-6)
+    for u, v in zip(a, b):
+        assert np.array_equal(v, u * np.float32(8))
+
+
+def test_momentum_conservation():
+    """Newton's third law on the GPU result (symmetric U): |sum m a| small vs sum m A."""
+    x, y, z, m = synth.make("plummer", 100000, 6)
+    T, d = _tree(x, y, z, 64)
+    xs, ys, zs, ms = T.sorted_bodies(x, y, z, m)
+    got, _ = gpu_eval(xs, ys, zs, ms, d, 1e-6)
+    ref = oracle.p2p(xs, ys, zs, ms, T.leaf_start, T.leaf_count, T.u_off, T.u_idx, 1.0, 1e-6,
+                     with_scale=True)
+    mm = ms.astype(np.float64)
+    scale = (mm * ref[4]).sum()
+    for c in range(3):
+        assert abs((mm * got[1 + c].astype(np.float64)).sum()) <= 1e-6 * scale
+
+
+def test_host_pointer_api_matches_device_api():
+    afmm = _afmm()
+    x, y, z, m = synth.make("C1")
+    T, d = _tree(x, y, z, 64)
+    xs, ys, zs, ms = T.sorted_bodies(x, y, z, m)
+    ref, _ = gpu_eval(xs, ys, zs, ms, d, 1e-6)
+    h = afmm.P2P(eps2=1e-6)
+    h.set_bodies(xs, ys, zs, ms)                     # numpy -> afmm_p2p_set_bodies_host
+    h.set_tree(d["leaf_start"], d["leaf_count"], d["u_off"], d["u_idx"])
+    out = [np.zeros(xs.shape[0], np.float32) for _ in range(4)]
+    st = h.eval(*out)                                # numpy -> afmm_p2p_eval_host (blocking)
+    for a, b in zip(ref, [out[3], out[0], out[1], out[2]]):
+        assert np.array_equal(a, b)
+    assert st["n_launches"] == 1 and st["kernel_ms"] > 0
+    h.close()
+
+
+def test_error_statuses():
+    afmm = _afmm()
+    with pytest.raises(afmm.AfmmError) as e:
+        afmm.P2P(max_leaf=2048)
+    assert e.value.status == afmm.AFMM_ENOTSUP
+    for kw in ({"eps2": -1.0}, {"G": float("inf")}, {"world": 0}, {"rank": 2, "world": 2}):
+        with pytest.raises(afmm.AfmmError) as e:
+            afmm.P2P(**kw)
+        assert e.value.status == afmm.AFMM_EINVAL
+    h = afmm.P2P(max_leaf=64)
+    out = [torch.zeros(8, device="cuda") for _ in range(4)]
+    with pytest.raises(afmm.AfmmError) as e:
+        h.eval(*out)
+    assert e.value.status == afmm.AFMM_ESTATE
+    with pytest.raises(afmm.AfmmError) as e:
+        h.set_tree([0], [8], [0, 1], [0])
+    assert e.value.status == afmm.AFMM_ESTATE
+    xs = torch.rand(8, device="cuda")
+    h.set_bodies(xs, xs, xs, xs)
+    bad = [
+        ([0, 4], [4, 3], [0, 1, 2], [0, 1]),          # leaves do not cover n
+        ([0, 5], [4, 4], [0, 1, 2], [0, 1]),          # gap between leaves
+        ([0, 4], [4, 4], [0, 2, 3], [1, 0, 1]),       # row not ascending
+        ([0, 4], [4, 4], [0, 1, 3], [0, 1, 1]),       # duplicate entry in a row
+        ([0, 4], [4, 4], [0, 1, 2], [0, 2]),          # index out of range
+        ([0, 4], [4, 4], [1, 1, 2], [0, 1]),          # u_off[0] != 0
+        ([0, 4], [4, 4], [0, 2, 1], [0, 1]),          # u_off not monotone
+    ]
+    for ls, lc, uo, ui in bad:
+        with pytest.raises(afmm.AfmmError) as e:
+            h.set_tree(ls, lc, uo, ui)
+        assert e.value.status == afmm.AFMM_EINVAL
+    h2 = afmm.P2P(max_leaf=4)
+    h2.set_bodies(xs, xs, xs, xs)
+    with pytest.raises(afmm.AfmmError) as e:
+        h2.set_tree([0, 2], [2, 6], [0, 1, 2], [0, 1])          # 6 > max_leaf
+    assert e.value.status == afmm.AFMM_EINVAL
+    h2.close()
+    # the handle stays usable after EINVAL
+    h.set_tree([0, 4], [4, 4], [0, 2, 4], [0, 1, 0, 1])
+    h.eval(*out, stats=True)
+    with pytest.raises(afmm.AfmmError) as e:
+        h.set_bodies(None, None, None, None, n=0)
+    assert e.value.status == afmm.AFMM_EINVAL
+    h.close()
+
+
+def test_rebalance_keeps_results_and_valid_split():
+    afmm = _afmm()
+    x, y, z, m = synth.make("plummer", 100000, 8)
+    T, d = _tree(x, y, z, 64)
+    xs, ys, zs, ms = T.sorted_bodies(x, y, z, m)
+    ref, _ = gpu_eval(xs, ys, zs, ms, d, 1e-6)
+    W = 4
+    hs = [afmm.P2P(rank=r, world=W, eps2=1e-6) for r in range(W)]
+    bodies = [_dev(v) for v in (xs, ys, zs, ms)]
+    for h in hs:
+        h.set_bodies(*bodies)
+        h.set_tree(d["leaf_start"], d["leaf_count"], d["u_off"], d["u_idx"])
+    fake_ms = np.array([1.0, 2.0, 1.0, 1.0])              # rank 1 "slow"
+    changed = [h.rebalance(fake_ms, 0.02) for h in hs]
+    assert len(set(changed)) == 1 and changed[0]
+    splits = [h.get_partition()[0] for h in hs]
+    assert all(np.array_equal(splits[0], s) for s in splits)
+    sp = splits[0]
+    assert sp[0] == 0 and sp[-1] == T.L and (np.diff(sp) >= 0).all()
+    out = [torch.full((xs.shape[0],), float("nan"), device="cuda") for _ in range(4)]
+    for h in hs:
+        h.eval(*out)
+    torch.cuda.synchronize()
+    for a, b in zip(ref, [out[3], out[0], out[1], out[2]]):
+        assert np.array_equal(a, b.cpu().numpy())
+    for h in hs:
+        h.close()
+
+
+def test_fp32_peak_sane():
+    afmm = _afmm()
+    p = afmm.fp32_peak(0)
+    assert 30 < p["ffma_tflops"] < 90 and 20 < p["ffma2_tflops"] < 180

@@ -1,0 +1,127 @@
+"""GPU octree + U-list builder (include/afmm_tree.h) vs the oracle: bit-exact
+integer indexing (perm, leaves, levels, prefixes, CSR U-lists), plus the
+full-size configs end to end (GPU tree -> GPU P2P) checked on sampled leaves."""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from tests import _tol
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+
+def _afmm():
+    import paper_conf_ipps_overmanpmm13_b200 as afmm
+    return afmm
+
+
+def _dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a, np.float32)).cuda()
+
+
+def gpu_tree(x, y, z, S, domain=None):
+    afmm = _afmm()
+    t = afmm.GpuTree(0)
+    t.build(_dev(x), _dev(y), _dev(z), S, domain=domain)
+    out = t.copy_out(x.shape[0])
+    t.close()
+    return out
+
+
+def assert_same_tree(G, T):
+    assert G["n_leaves"] == T.L
+    assert G["k"] == T.k and np.array_equal(G["lo"], T.lo)
+    assert np.array_equal(G["perm"], T.perm)
+    assert np.array_equal(G["leaf_start"], T.leaf_start)
+    assert np.array_equal(G["leaf_count"], T.leaf_count)
+    assert np.array_equal(G["leaf_level"], T.leaf_level)
+    assert np.array_equal(G["leaf_prefix"], T.leaf_prefix)
+    assert np.array_equal(G["u_off"], T.u_off)
+    assert np.array_equal(G["u_idx"], T.u_idx)
+
+
+@pytest.mark.parametrize("dist,n,S,seed", [("uniform", 4096, 64, 1), ("plummer", 100000, 32, 2),
+                                           ("colliding", 100000, 100, 3), ("plummer", 50000, 1, 4),
+                                           ("uniform", 1, 4, 5), ("uniform", 300, 500, 6),
+                                           ("plummer", 1 << 20, 128, 2)])
+def test_tree_bit_exact(dist, n, S, seed):
+    x, y, z, m = synth.make(dist, n, seed)
+    assert_same_tree(gpu_tree(x, y, z, S), oracle.Tree(x, y, z, S))
+
+
+def test_tree_lattice_and_duplicates_bit_exact():
+    x, y, z, m = synth.lattice(16)
+    assert_same_tree(gpu_tree(x, y, z, 1), oracle.Tree(x, y, z, 1))
+    x, y, z, m = synth.make("uniform", 600, 3)
+    idx = np.arange(600) % 40
+    x, y, z = x[idx], y[idx], z[idx]
+    assert_same_tree(gpu_tree(x, y, z, 4), oracle.Tree(x, y, z, 4))
+
+
+def test_tree_fixed_domain_bit_exact():
+    x, y, z, m = synth.make("colliding", 50000, 7)
+    dom = (np.array([-40.0, -40.0, -40.0]), 7)          # side 128, some bodies clamp nowhere
+    assert_same_tree(gpu_tree(x, y, z, 64, domain=dom), oracle.Tree(x, y, z, 64, domain=dom))
+    dom = (np.array([-2.0, -2.0, -2.0]), 2)             # bodies outside are clamped to the edge cells
+    assert_same_tree(gpu_tree(x, y, z, 64, domain=dom), oracle.Tree(x, y, z, 64, domain=dom))
+
+
+def test_gather_scatter_roundtrip():
+    afmm = _afmm()
+    x, y, z, m = synth.make("plummer", 10000, 1)
+    t = afmm.GpuTree(0)
+    X = _dev(x)
+    t.build(X, _dev(y), _dev(z), 16)
+    perm = t.copy_out(10000)["perm"]
+    out = torch.empty_like(X)
+    t.gather(X, out)
+    torch.cuda.synchronize()
+    assert np.array_equal(out.cpu().numpy(), x[perm])
+    back = torch.empty_like(X)
+    t.scatter(out, back)
+    torch.cuda.synchronize()
+    assert np.array_equal(back.cpu().numpy(), x)
+    t.close()
+
+
+def _end_to_end(cfg, n_sample_leaves, seed=0):
+    """GPU tree + GPU P2P (the bench's launch configuration) at full size;
+    tree checked bit-exact, P2P checked on a seeded sample of target leaves."""
+    afmm = _afmm()
+    c = synth.CONFIGS[cfg]
+    x, y, z, m = synth.make(cfg)
+    G = gpu_tree(x, y, z, c["S"])
+    T = oracle.Tree(x, y, z, c["S"])
+    assert_same_tree(G, T)
+    xs, ys, zs, ms = T.sorted_bodies(x, y, z, m)
+    h = afmm.P2P(eps2=c["eps2"])
+    h.set_bodies(*[_dev(v) for v in (xs, ys, zs, ms)])
+    h.set_tree(G["leaf_start"], G["leaf_count"], G["u_off"], G["u_idx"])
+    out = [torch.empty(xs.shape[0], device="cuda") for _ in range(4)]
+    st = h.eval(*out, stats=True)
+    ax, ay, az, phi = (o.cpu().numpy() for o in out)
+    got = [phi, ax, ay, az]                           # the oracle's order
+    h.close()
+    rng = np.random.default_rng(seed)
+    tg = np.sort(rng.choice(T.L, size=min(n_sample_leaves, T.L), replace=False)).astype(np.int32)
+    tg = np.unique(np.concatenate([tg, [0, T.L - 1, int(np.argmax(T.leaf_count))]])).astype(np.int32)
+    ref = oracle.p2p(xs, ys, zs, ms, T.leaf_start, T.leaf_count, T.u_off, T.u_idx, 1.0, c["eps2"],
+                     targets=tg, with_scale=True)
+    sel = np.zeros(xs.shape[0], bool)
+    for t in tg:
+        sel[T.leaf_start[t]:T.leaf_start[t] + T.leaf_count[t]] = True
+    _tol.check([g[sel] for g in got], [r[sel] for r in ref[:4]], ref[4][sel])
+    assert np.isfinite(np.stack(got)).all()
+    return st
+
+
+def test_c4_end_to_end_sampled():
+    """16M Plummer, S=256 (BASELINE configs[3]) on one GPU: >= 4096 sampled leaves."""
+    st = _end_to_end("C4", 4096, seed=4)
+    assert st["interactions_total"] > 3e10
+
+
+def test_c3_end_to_end_sampled():
+    _end_to_end("C3", 4096, seed=3)
