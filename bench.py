@@ -1,0 +1,430 @@
+#!/usr/bin/env python
+"""Benchmark of the AFMM near-field P2P hot path on B200 (BASELINE.json metric:
+"near-field P2P interactions/s (and % FP32 peak) at 1/2/4/8 B200").
+
+One step = one pass of the whole hot path over the workload, with inputs
+resident in HBM: body ingest (pack; broadcast from rank 0 when N > 1), the
+P2P kernel over this rank's target leaves, and (N > 1) the gather of every
+rank's output slice (grouped broadcasts = allgatherv over NCCL).  The tree is
+built once, on the GPU, by the product builder (afmm_tree_build) -- the
+workload is static (BASELINE configs[1], a fixed 1M-body Plummer sphere).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--S 128]
+  torchrun --nproc-per-node N bench.py --gpus N ...       (N > 1)
+  python bench.py --impl reference ...                    (the fp64 oracle, CPU)
+
+Prints ONE JSON line on rank 0.  Timing: CUDA events around each step on the
+library's stream (= torch's current stream), L2 flushed (256 MiB write)
+between steps outside the events, barrier + synchronize on both sides, max
+over ranks.  Interactions = sum_t n_t sum_{s in U(t)} n_s (PAPER L16 SIII.C);
+20 flops per interaction (the all-pairs convention of [14], north_star).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402  (seeded input generator shared by both arms)
+
+FLOPS_PER_INTERACTION = 20
+METRIC = "near-field P2P interactions/s (and % FP32 peak) at 1/2/4/8 B200"
+SWEEP_S = [32, 48, 64, 96, 128, 192, 256, 384, 512]
+WORKLOAD_DESC = {
+    "C1": "4,096 uniform bodies in unit cube, S=64 (BASELINE configs[0])",
+    "C2": "1M-body Plummer sphere (a=1, r<=10), 1 B200 (BASELINE configs[1])",
+    "C3": "4M-body two colliding Plummer spheres, S=128 (BASELINE configs[2])",
+    "C4": "16M-body Plummer sphere, S=256 (BASELINE configs[3])",
+    "C5": "1M-body colliding galaxies (BASELINE configs[4], static snapshot)",
+}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=100)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C2", choices=sorted(synth.CONFIGS))
+    ap.add_argument("--S", type=int, default=None, help="leaf capacity (default: the config's)")
+    ap.add_argument("--no-sweep", action="store_true", help="skip the S sweep (C2, N=1)")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0, help="oracle sample budget")
+    return ap.parse_args()
+
+
+def peak_fp32_tflops(sm_mhz=1965.0):
+    """FP32 roofline from the unit counts (B200_PROFILING.md: 148 SMs; 128 FP32
+    lanes per SM, 2 flop per FFMA) at the max SM clock (MEASURED_PEAKS.json)."""
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            sm_mhz = float(json.load(f).get("sm_max_mhz", sm_mhz))
+    except Exception:
+        pass
+    return 148 * 128 * 2 * sm_mhz * 1e6 / 1e12, sm_mhz
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for ln in self.proc.stdout:
+            self.lines.append(ln.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            p = [v.strip() for v in ln.split(",")]
+            if len(p) < 9:
+                continue
+            try:
+                sm.append(float(p[1]))
+                mx = float(p[2])
+            except ValueError:
+                continue
+            for nm, v in zip(names, p[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+# ------------------------------------------------------------------ oracle legs (CPU)
+
+def _oracle_sample(xs, ys, zs, ms, T, eps2, budget_s, seed=0):
+    """Time the oracle's naive P2P on a seeded sample of target leaves sized to
+    about budget_s seconds of CPU work.  Returns (interactions/s, desc, cores)."""
+    import oracle
+    I = oracle.interactions(T.leaf_count, T.u_off, T.u_idx)
+    rng = np.random.default_rng(seed)
+    order = rng.permutation(T.L).astype(np.int32)
+    # probe ~0.2% of the work to estimate the rate
+    cum = np.cumsum(I[order])
+    k = int(np.searchsorted(cum, max(cum[-1] * 0.002, 1)) + 1)
+    t0 = time.perf_counter()
+    oracle.p2p(xs, ys, zs, ms, T.leaf_start, T.leaf_count, T.u_off, T.u_idx, 1.0, eps2,
+               targets=np.sort(order[:k]))
+    rate = cum[k - 1] / max(time.perf_counter() - t0, 1e-6)
+    want = min(cum[-1], rate * budget_s)
+    k = int(min(T.L, np.searchsorted(cum, want) + 1))
+    tg = np.sort(order[:k])
+    t0 = time.perf_counter()
+    oracle.p2p(xs, ys, zs, ms, T.leaf_start, T.leaf_count, T.u_off, T.u_idx, 1.0, eps2, targets=tg)
+    dt = time.perf_counter() - t0
+    inter = int(I[tg].sum())
+    cores = len(os.sched_getaffinity(0))
+    desc = (f"{k} of {T.L} target leaves ({inter:.4g} of {int(I.sum()):.4g} interactions, "
+            f"{100.0 * inter / I.sum():.1f}%), seeded random, fp64 oracle_p2p, OpenMP {cores} threads")
+    return inter / dt, desc, cores, inter, dt
+
+
+def run_reference(args):
+    """--impl reference: the fp64 CPU oracle (the tier's reference arm) on the
+    same workload, each step a bounded sample; rank 0 only."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import oracle
+    oracle.build()
+    c = synth.CONFIGS[args.config]
+    S = args.S or c["S"]
+    x, y, z, m = synth.make(args.config)
+    T = oracle.Tree(x, y, z, S)
+    xs, ys, zs, ms = T.sorted_bodies(x, y, z, m)
+    steps, warm = max(1, args.steps), max(0, args.warmup)
+    per_step = max(0.5, 150.0 / (steps + warm))
+    rates = []
+    total_i, total_t = 0, 0.0
+    desc = cores = None
+    for i in range(steps + warm):
+        r, desc, cores, inter, dt = _oracle_sample(xs, ys, zs, ms, T, c["eps2"], per_step, seed=i)
+        if i >= warm:
+            rates.append(r)
+            total_i += inter
+            total_t += dt
+    value = total_i / total_t
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "interactions/s",
+            "n_gpus": args.gpus, "steps": steps, "warmup": warm,
+            "ms_per_step": 1e3 * total_t / steps, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": WORKLOAD_DESC[args.config], "S": S, "n": int(x.shape[0]),
+                       "eps2": c["eps2"], "seed": c["seed"]},
+            "cpu_baseline": {"value": value, "unit": "interactions/s", "cores": cores, "kind": "oracle",
+                             "sample": "per step: " + desc},
+            "e2e": {"value": value, "unit": "interactions/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------ our arm
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ipps_overmanpmm13_b200 as afmm
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    # a dedicated (non-default) stream shared by torch and the library, so the
+    # step events, the NCCL calls and the kernels are ordered on one stream
+    stream = torch.cuda.Stream(dev)
+    torch.cuda.set_stream(stream)
+
+    c = synth.CONFIGS[args.config]
+    S = args.S or c["S"]
+    eps2 = c["eps2"]
+    x, y, z, m = synth.make(args.config)
+    n = int(x.shape[0])
+
+    # ---- setup (untimed): product GPU tree, bodies into tree order on device
+    X, Y, Z, M = (torch.from_numpy(v).to(dev) for v in (x, y, z, m))
+    tree = afmm.GpuTree(local, stream=stream.cuda_stream)
+    t0 = time.perf_counter()
+    tree.build(X, Y, Z, S)
+    tree_s = time.perf_counter() - t0
+    T = tree.copy_out(n)
+    bod = torch.empty((4, n), device=dev)
+    for a, src in enumerate((X, Y, Z, M)):
+        tree.gather(src, bod[a])
+    h = afmm.P2P(device=local, rank=rank, world=world, G=1.0, eps2=eps2, stream=stream.cuda_stream)
+    h.set_bodies(bod[0], bod[1], bod[2], bod[3])
+    t0 = time.perf_counter()
+    h.set_tree(T["leaf_start"], T["leaf_count"], T["u_off"], T["u_idx"])
+    set_tree_s = time.perf_counter() - t0
+    out = torch.empty((4, n), device=dev)           # ax, ay, az, phi
+    flush = torch.empty(64 << 20, dtype=torch.float32, device=dev)   # 256 MiB > 126 MB L2
+
+    def gather_slices():
+        ls, bs = h.get_partition()
+        for r in range(world):
+            lo, hi = int(bs[r]), int(bs[r + 1])
+            if hi > lo:
+                for a in range(4):
+                    dist.broadcast(out[a, lo:hi], src=r)
+
+    def step():
+        if world > 1:
+            for a in range(4):
+                dist.broadcast(bod[a], src=0)                 # a4: source replication
+        h.set_bodies(bod[0], bod[1], bod[2], bod[3])          # a1: pack (1 kernel)
+        h.eval(out[0], out[1], out[2], out[3])                # a5/a6: P2P (1 kernel)
+        if world > 1:
+            gather_slices()                                   # a7: allgatherv of slices
+
+    # ---- warm-up (+ incremental rebalance from measured kernel times, L18 SIV.D)
+    rebalanced = 0
+    for i in range(max(3, args.warmup)):
+        step()
+        if world > 1:
+            kt = torch.tensor([h.kernel_times(1)[-1]], dtype=torch.float64, device=dev)
+            allk = [torch.zeros_like(kt) for _ in range(world)]
+            dist.all_gather(allk, kt)
+            rebalanced += int(h.rebalance(np.array([float(v.item()) for v in allk]), 0.02))
+    torch.cuda.synchronize()
+
+    # ---- timed region
+    K = args.steps
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        for k in range(K):
+            flush.zero_()                                     # L2 flush, outside the step events
+            ev[k][0].record(stream)
+            step()
+            ev[k][1].record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    kern_ms = h.kernel_times(K)
+    st = h.stats()
+    tot = torch.tensor([sum(step_ms), float(np.mean(kern_ms))], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(tot, op=dist.ReduceOp.MAX)
+    total_ms, kern_max = float(tot[0]), float(tot[1])
+    inter = st["interactions_total"]
+    value = inter * K / (total_ms * 1e-3)
+
+    # ---- end to end through the public API with host buffers (H2D + D2H in the timed region)
+    hx = [torch.empty(n, dtype=torch.float32).pin_memory() for _ in range(4)]
+    for a in range(4):
+        hx[a].copy_(bod[a].cpu())
+    ho = [torch.empty(n, dtype=torch.float32).pin_memory() for _ in range(4)]
+    Ke = max(3, K // 2)
+
+    def step_e2e():
+        if world == 1:
+            h.set_bodies(*hx)                                 # afmm_p2p_set_bodies_host (H2D + pack)
+            h.eval(*ho)                                       # afmm_p2p_eval_host (kernel + D2H, blocking)
+        else:
+            if rank == 0:
+                for a in range(4):
+                    bod[a].copy_(hx[a], non_blocking=True)
+            step()
+            if rank == 0:
+                for a in range(4):
+                    ho[a].copy_(out[a], non_blocking=True)
+            torch.cuda.synchronize()
+
+    step_e2e()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    for _ in range(Ke):
+        step_e2e()
+    torch.cuda.synchronize()
+    e2e_s = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(e2e_s, op=dist.ReduceOp.MAX)
+    e2e_value = inter * Ke / float(e2e_s[0])
+
+    # ---- roofline of the dominant kernel (the P2P kernel): FP32 ALU bound
+    peak, sm_max = peak_fp32_tflops()
+    kern_mean = float(np.mean(kern_ms))
+    achieved = FLOPS_PER_INTERACTION * st["interactions_rank"] / (kern_mean * 1e-3) / 1e12
+    prof_traffic = None
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            tr = json.load(f)
+            if tr.get("config") == args.config and tr.get("S") == S:
+                prof_traffic = tr.get("dram_bytes_per_launch")
+    except Exception:
+        pass
+
+    extra = {}
+    if rank == 0 and world == 1:
+        try:
+            extra["fp32_measured"] = afmm.fp32_peak(local)
+        except Exception as e:  # noqa: BLE001
+            extra["fp32_measured"] = {"error": str(e)}
+        if args.config == "C2" and not args.no_sweep:
+            sweep = {}
+            for s2 in SWEEP_S:
+                tr2 = afmm.GpuTree(local, stream=stream.cuda_stream)
+                tr2.build(X, Y, Z, s2)
+                T2 = tr2.copy_out(n)
+                b2 = torch.empty((4, n), device=dev)
+                for a, src in enumerate((X, Y, Z, M)):
+                    tr2.gather(src, b2[a])
+                h2 = afmm.P2P(device=local, eps2=eps2, stream=stream.cuda_stream)
+                h2.set_bodies(b2[0], b2[1], b2[2], b2[3])
+                h2.set_tree(T2["leaf_start"], T2["leaf_count"], T2["u_off"], T2["u_idx"])
+                for _ in range(8):
+                    h2.eval(out[0], out[1], out[2], out[3])
+                km = float(np.median(h2.kernel_times(5)))
+                s2st = h2.stats()
+                ips = s2st["interactions_total"] / (km * 1e-3)
+                sweep[str(s2)] = {"n_leaves": T2["n_leaves"], "interactions": s2st["interactions_total"],
+                                  "kernel_ms": round(km, 4), "interactions_per_s": ips,
+                                  "frac_fp32": FLOPS_PER_INTERACTION * ips / (peak * 1e12)}
+                h2.close()
+                tr2.close()
+            extra["sweep_S"] = sweep
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        try:
+            import oracle
+            oracle.build()
+            To = oracle.Tree(x, y, z, S)
+            xs, ys, zs, ms = To.sorted_bodies(x, y, z, m)
+            r, desc, cores, _, _ = _oracle_sample(xs, ys, zs, ms, To, eps2, args.cpu_seconds)
+            cpu = {"value": r, "unit": "interactions/s", "cores": cores, "kind": "oracle", "sample": desc}
+        except Exception as e:  # noqa: BLE001
+            cpu = {"value": None, "unit": "interactions/s", "cores": None, "kind": "oracle",
+                   "sample": f"failed: {e}"}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "interactions/s", "n_gpus": world,
+            "steps": K, "warmup": max(3, args.warmup), "ms_per_step": total_ms / K,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic",
+            "config": {"workload": WORKLOAD_DESC[args.config], "S": S, "n": n, "eps2": eps2,
+                       "seed": c["seed"], "n_leaves": T["n_leaves"], "u_nnz": T["nnz"],
+                       "interactions_per_step": inter,
+                       "l2": "flushed between steps (256 MiB write outside the step events)",
+                       "step": ("pack + P2P kernel" if world == 1 else
+                                "broadcast bodies + pack + P2P kernel + allgatherv of output slices"),
+                       "parallelism": f"leaf-partition x{world} (cost model, PAPER L16)",
+                       "tree_build_s": round(tree_s, 4), "set_tree_s": round(set_tree_s, 4)},
+            "kernel_ms": {"mean": kern_mean, "max_over_ranks": kern_max},
+            "gpu_time_interactions_per_s": inter / (kern_max * 1e-3),
+            "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
+                         "frac": achieved / peak, "traffic": prof_traffic,
+                         "peak_note": (f"derived: 148 SM x 128 FP32 lanes x 2 flop x {sm_max:.0f} MHz "
+                                       "(no FP32 entry in MEASURED_PEAKS.json); 20 flop/interaction"),
+                         "kernel": "afmm::p2p_kernel"},
+            "clocks": clk.summary(),
+            "e2e": {"value": e2e_value, "unit": "interactions/s", "h2d_bytes_per_step": 16 * n,
+                    "d2h_bytes_per_step": 16 * n, "steps": Ke},
+            "gpu_launches": 2 * K,
+            "rebalanced_in_warmup": rebalanced,
+            "cpu_baseline": cpu,
+            "paper_context": "98x whole-AFMM speedup, 10 CPU cores + 4 Tesla C2050 vs 1 core, 1M Plummer (L24 SVIII.E)",
+        }
+        line.update(extra)
+        print(json.dumps(line), flush=True)
+    h.close()
+    tree.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

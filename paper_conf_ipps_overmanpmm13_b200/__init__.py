@@ -78,6 +78,7 @@ _sig("afmm_p2p_eval", _i, _p, _p, _p, _p, _p, C.POINTER(Stats))
 _sig("afmm_p2p_eval_host", _i, _p, _p, _p, _p, _p, C.POINTER(Stats))
 _sig("afmm_p2p_stats_get", _i, _p, C.POINTER(Stats))
 _sig("afmm_p2p_stream", _p, _p)
+_sig("afmm_p2p_kernel_times", _i, _p, _i, _p)
 _sig("afmm_p2p_destroy", None, _p)
 _sig("afmm_p2p_last_error", C.c_char_p, _p)
 _sig("afmm_interactions", _i, _i, _p, _p, _p, _p)
@@ -100,6 +101,7 @@ EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
             "afmm_p2p_set_bodies_host", "afmm_p2p_bodies_buffer", "afmm_p2p_set_tree",
             "afmm_p2p_set_partition", "afmm_p2p_get_partition", "afmm_p2p_rebalance",
             "afmm_p2p_eval", "afmm_p2p_eval_host", "afmm_p2p_stats_get", "afmm_p2p_stream",
+            "afmm_p2p_kernel_times",
             "afmm_p2p_destroy", "afmm_p2p_last_error", "afmm_interactions",
             "afmm_partition_literal", "afmm_partition_weighted", "afmm_fp32_peak", "afmm_version",
             "afmm_tree_create", "afmm_tree_build", "afmm_tree_info", "afmm_tree_copy_out",
@@ -121,6 +123,12 @@ def _ptr(a):
     if isinstance(a, np.ndarray):
         return a.ctypes.data
     return a.data_ptr()
+
+
+def _check_host_tensor(t, n):
+    import torch
+    if t.is_cuda or t.dtype != torch.float32 or not t.is_contiguous() or t.shape[0] != n:
+        raise TypeError("host tensors must be contiguous float32 CPU tensors of length n")
 
 
 def _is_device(a) -> bool:
@@ -190,9 +198,9 @@ class P2P:
             raise AfmmError(st, f"{what}: {_lib.afmm_p2p_last_error(self._h).decode()}")
 
     def close(self):
-        if getattr(self, "_h", None):
+        if getattr(self, "_h", None) and _lib is not None:   # _lib is None at interpreter exit
             _lib.afmm_p2p_destroy(self._h)
-            self._h = None
+        self._h = None
 
     __del__ = close
 
@@ -211,6 +219,11 @@ class P2P:
         if _is_device(x):
             self._check(_lib.afmm_p2p_set_bodies(self._h, n, _ptr(x), _ptr(y), _ptr(z), _ptr(m)),
                         "afmm_p2p_set_bodies")
+        elif not isinstance(x, np.ndarray):          # torch CPU (e.g. pinned) tensors
+            for v in (x, y, z, m):
+                _check_host_tensor(v, n)
+            self._check(_lib.afmm_p2p_set_bodies_host(self._h, n, _ptr(x), _ptr(y), _ptr(z), _ptr(m)),
+                        "afmm_p2p_set_bodies_host")
         else:
             x, y, z, m = (_np(v, np.float32) for v in (x, y, z, m))
             self._check(_lib.afmm_p2p_set_bodies_host(self._h, n, _ptr(x), _ptr(y), _ptr(z), _ptr(m)),
@@ -254,12 +267,23 @@ class P2P:
                         "afmm_p2p_eval")
         else:
             for a in (ax, ay, az, phi):
-                if not (isinstance(a, np.ndarray) and a.dtype == np.float32 and a.flags.c_contiguous):
-                    raise TypeError("host outputs must be contiguous float32 numpy arrays")
+                if isinstance(a, np.ndarray):
+                    if not (a.dtype == np.float32 and a.flags.c_contiguous):
+                        raise TypeError("host outputs must be contiguous float32 arrays")
+                else:
+                    _check_host_tensor(a, int(a.shape[0]))
             sp = C.byref(s)
             self._check(_lib.afmm_p2p_eval_host(self._h, _ptr(ax), _ptr(ay), _ptr(az), _ptr(phi), sp),
                         "afmm_p2p_eval_host")
         return s.as_dict() if (stats or not _is_device(ax)) else None
+
+    def kernel_times(self, max_count=64):
+        """Kernel ms of the last <= 64 evals (oldest first); synchronises."""
+        buf = np.empty(max(1, max_count), np.float64)
+        cnt = _lib.afmm_p2p_kernel_times(self._h, int(max_count), _ptr(buf))
+        if cnt < 0:
+            self._check(cnt, "afmm_p2p_kernel_times")
+        return buf[:cnt].copy()
 
     def stats(self):
         s = Stats()
@@ -284,9 +308,9 @@ class GpuTree:
             raise AfmmError(st, f"{what}: {_lib.afmm_tree_last_error(self._h).decode()}")
 
     def close(self):
-        if getattr(self, "_h", None):
+        if getattr(self, "_h", None) and _lib is not None:
             _lib.afmm_tree_destroy(self._h)
-            self._h = None
+        self._h = None
 
     __del__ = close
 

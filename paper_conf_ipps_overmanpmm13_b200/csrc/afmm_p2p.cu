@@ -67,7 +67,10 @@ struct afmm_p2p {
     long long rank_interactions = 0;
     long long bucket_inter[8] = {0};
 
-    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;   // aliases of the newest ring entry
+    static constexpr int kRing = 64;             // kernel-time history (afmm_p2p_kernel_times)
+    cudaEvent_t ring0[kRing] = {}, ring1[kRing] = {};
+    long long n_evals = 0;
     bool evaluated = false;
     afmm_p2p_stats last{};
 };
@@ -233,8 +236,10 @@ extern "C" afmm_status afmm_p2p_create(const afmm_p2p_config *cfg, afmm_p2p **ou
             e = cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking);
             h->own_stream = (e == cudaSuccess);
         }
-        if (e == cudaSuccess) e = cudaEventCreate(&h->ev0);
-        if (e == cudaSuccess) e = cudaEventCreate(&h->ev1);
+        for (int i = 0; i < afmm_p2p::kRing && e == cudaSuccess; ++i) {
+            e = cudaEventCreate(&h->ring0[i]);
+            if (e == cudaSuccess) e = cudaEventCreate(&h->ring1[i]);
+        }
         if (e == cudaSuccess) e = cudaMalloc(&h->d_queue, sizeof(int));
         if (e == cudaSuccess) e = cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, cfg->device);
         if (e == cudaSuccess)
@@ -265,8 +270,10 @@ extern "C" void afmm_p2p_destroy(afmm_p2p *h) {
     cudaFree(h->d_chunks);
     cudaFree(h->d_segs);
     cudaFree(h->d_queue);
-    if (h->ev0) cudaEventDestroy(h->ev0);
-    if (h->ev1) cudaEventDestroy(h->ev1);
+    for (int i = 0; i < afmm_p2p::kRing; ++i) {
+        if (h->ring0[i]) cudaEventDestroy(h->ring0[i]);
+        if (h->ring1[i]) cudaEventDestroy(h->ring1[i]);
+    }
     if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
     delete h;
 }
@@ -648,6 +655,9 @@ static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, flo
     p.eps2 = h->cfg.eps2;
     p.G = (double)h->cfg.G;
     CUDA_TRY(h, cudaMemsetAsync(h->d_queue, 0, sizeof(int), h->stream));
+    const int ri = (int)(h->n_evals % afmm_p2p::kRing);
+    h->ev0 = h->ring0[ri];
+    h->ev1 = h->ring1[ri];
     CUDA_TRY(h, cudaEventRecord(h->ev0, h->stream));
     int nlaunch = 0;
     if (p.n_items > 0) {
@@ -657,6 +667,7 @@ static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, flo
         nlaunch = 1;
     }
     CUDA_TRY(h, cudaEventRecord(h->ev1, h->stream));
+    h->n_evals++;
     h->evaluated = true;
     h->last.n_launches = nlaunch;
     return AFMM_OK;
@@ -726,4 +737,26 @@ extern "C" afmm_status afmm_p2p_stats_get(afmm_p2p *h, afmm_p2p_stats *stats) {
     afmm_status st = set_device(h);
     if (st) return st;
     return fill_stats(h, stats);
+}
+
+extern "C" int afmm_p2p_kernel_times(afmm_p2p *h, int max_count, double *ms) {
+    if (!h || h->poisoned || max_count < 0 || (max_count > 0 && !ms)) return AFMM_EINVAL;
+    if (set_device(h)) return AFMM_ECUDA;
+    if (cudaStreamSynchronize(h->stream) != cudaSuccess) {
+        fail(h, AFMM_ECUDA, "kernel_times: stream sync failed");
+        return AFMM_ECUDA;
+    }
+    long long avail = std::min<long long>(h->n_evals, afmm_p2p::kRing);
+    const int cnt = (int)std::min<long long>(avail, max_count);
+    for (int i = 0; i < cnt; ++i) {
+        const long long ev = h->n_evals - cnt + i;      // oldest first
+        const int ri = (int)(ev % afmm_p2p::kRing);
+        float f = 0.f;
+        if (cudaEventElapsedTime(&f, h->ring0[ri], h->ring1[ri]) != cudaSuccess) {
+            fail(h, AFMM_ECUDA, "kernel_times: cudaEventElapsedTime failed");
+            return AFMM_ECUDA;
+        }
+        ms[i] = f;
+    }
+    return cnt;
 }

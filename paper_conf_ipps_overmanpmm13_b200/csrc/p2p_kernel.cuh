@@ -6,36 +6,42 @@
 //     phi_i -= G m_j / r,   a_i += G m_j d / r^3,   d = x_j - x_i,  r^2 = |d|^2 + eps2.
 //
 // B200 design:
-//  * persistent CTAs (256 threads) pull work items from an atomic queue that
-//    the host ordered largest-cost-first;
-//  * the item's sources -- a handful of contiguous body segments, the self leaf
-//    first -- are staged into shared memory with 1-D TMA bulk copies
-//    (cp.async.bulk ... mbarrier::complete_tx), double-buffered so the next
-//    chunk lands while this one is consumed;
-//  * lane mapping: 2 targets per thread (FFMA2 packed math with the source
+//  * persistent, warp-specialised CTAs: 8 consumer warps + 1 producer warp.
+//    The producer pulls work items from an atomic queue (ordered largest-cost-
+//    first by the host), loads the chunk/segment descriptors lane-parallel and
+//    stages each chunk's source segments (the self leaf first, then merged runs
+//    of consecutive U-list leaves) into a kStages-deep shared-memory ring with
+//    1-D TMA bulk copies (cp.async.bulk ... mbarrier::complete_tx).  Full/empty
+//    mbarriers per stage; consumers never wait on the producer's metadata
+//    latency unless the ring runs dry.
+//  * lane mapping: 2 targets per consumer thread (FFMA2 packed math, the source
 //    coordinate broadcast as the .F32 operand), g = ceil(n_t/2) lanes per
-//    "copy", C = 256/g copies per CTA; copy c consumes sources c, c+C, ...
-//    so leaves of any size 1..512 keep >= 95% of the lanes busy (the paper's
-//    one-thread-per-target blocks idle the rest, L16 SIII.C);
-//  * accumulation: fp32 partials over <= FOLD sources per copy, folded into fp64;
-//    copies reduced in fixed order in fp64 through shared memory; one RN
-//    rounding to fp32 at the end.  Deterministic and independent of the
-//    partition (bit-identical across world sizes).
+//    "copy", C = min(256/g, kMaxCopies) copies; copy c consumes sources c, c+C,
+//    ... so leaves of any size keep the lanes busy (the paper's one-thread-per-
+//    target blocks idle the rest, L16 SIII.C).
+//  * accumulation: fp32 partials over <= kFold sources per copy, folded into
+//    fp64 accumulators in shared memory; copies reduced in fixed order in fp64
+//    (one consumer-only named barrier per item); one RN rounding to fp32.
+//    Deterministic and independent of the partition (bit-identical across
+//    world sizes).
 #pragma once
 #include <cstdint>
 #include <cuda_runtime.h>
 
 namespace afmm {
 
-constexpr int kThreads = 256;        // threads per CTA
-constexpr int kCap = 1024;           // bodies per shared-memory stage (16 KiB)
-constexpr int kMaxTargets = 512;     // targets per work item (2 per thread)
-constexpr int kFold = 32;            // fp32 partial length per copy before the fp64 fold
-constexpr int kMinBlocksPerSM = 4;
-constexpr int kStageBytes = 2 * kCap * 16;                   // two TMA stages
-constexpr int kDynSmem = kStageBytes + 8 * kThreads * 8;     // + fp64 accumulators
+constexpr int kConsumers = 256;                 // consumer threads (8 warps)
+constexpr int kThreads = kConsumers + 32;       // + 1 producer warp
+constexpr int kCap = 1024;                      // bodies per shared-memory stage (16 KiB)
+constexpr int kStages = 3;                      // TMA ring depth
+constexpr int kMaxTargets = 512;                // targets per work item (2 per thread)
+constexpr int kMaxCopies = 64;                  // source-split copies per item
+constexpr int kFold = 64;                       // fp32 partial length per copy before the fp64 fold
+constexpr int kMinBlocksPerSM = 3;
+constexpr int kStageBytes = kStages * kCap * 16;
+constexpr int kDynSmem = kStageBytes + 8 * kConsumers * 8;    // + fp64 accumulators
 
-// Work item: targets [tgt_start, tgt_start+tgt_count) of leaf starting at
+// Work item: targets [tgt_start, tgt_start+tgt_count) of the leaf starting at
 // self_start; its sources are chunks [chunk_begin, chunk_begin+chunk_count).
 struct Item {
     int tgt_start, tgt_count, self_start, self_len, chunk_begin, chunk_count, pad0, pad1;
@@ -91,6 +97,10 @@ __device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
         "DONE:\n"
         "}\n" ::"r"(smem_u32(b)), "r"(parity) : "memory");
 }
+// named barrier among the consumer warps only (the producer never joins)
+__device__ __forceinline__ void consumer_sync() {
+    asm volatile("bar.sync 1, %0;" ::"n"(kConsumers) : "memory");
+}
 // 1-D bulk async copy global -> shared, completion counted on an mbarrier (TMA).
 __device__ __forceinline__ void tma_load_1d(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
     asm volatile(
@@ -131,11 +141,11 @@ __device__ __forceinline__ void interact2(const float4 q, const float2 nx, const
     az = __ffma2_rn(s, dz, az);
 }
 
-// fp64 accumulators live in shared memory, [8][kThreads] (bank-conflict free),
-// so the fp32 inner loop keeps its registers; folded every kFold sources.
+// fp64 accumulators live in shared memory, [8][kConsumers] (conflict free), so
+// the fp32 inner loop keeps its registers; folded every kFold sources.
 struct Acc64 {
     double *p;   // &acc[0][tid]
-    __device__ __forceinline__ void add(int u, float v) { p[u * kThreads] += (double)v; }
+    __device__ __forceinline__ void add(int u, float v) { p[u * kConsumers] += (double)v; }
 };
 
 // Consume sources k = k0, k0+C, ... < kend of one staged chunk.
@@ -156,87 +166,106 @@ __device__ __forceinline__ void consume(const float4 *__restrict__ src, int &k, 
     }
 }
 
-__device__ __forceinline__ void produce(int s, const P2PParams &p, float4 (*stage)[kCap],
-                                        uint64_t *full, int *meta_item, int *meta_chunk,
-                                        int &p_item, int &p_chunk, int &p_nchunks, int lane) {
-    int item = -1, chunk = 0;
-    if (lane == 0) {
-        if (p_item < p.n_items && p_chunk >= p_nchunks) {
-            p_item = atomicAdd(p.queue, 1);
-            p_chunk = 0;
-            p_nchunks = (p_item < p.n_items) ? p.items[p_item].chunk_count : 0;
-            if (p_item > p.n_items) p_item = p.n_items;
+struct StageMeta {
+    int item, chunk;
+};
+
+// Producer warp: walk the queue, stage every chunk of every claimed item.
+__device__ __forceinline__ void producer_loop(const P2PParams &p, float4 (*stage)[kCap],
+                                              uint64_t *full, uint64_t *empty, StageMeta *meta,
+                                              int lane) {
+    int st = 0;
+    uint32_t phase = 0;
+    int item = -1, chunk = 0, nchunks = 0, chunk_begin = 0;
+    for (;;) {
+        if (chunk >= nchunks) {                    // claim the next item
+            int it = 0;
+            if (lane == 0) it = atomicAdd(p.queue, 1);
+            it = __shfl_sync(0xffffffffu, it, 0);
+            if (it >= p.n_items) {
+                item = -1;
+            } else {
+                item = it;
+                const Item w = p.items[it];
+                nchunks = w.chunk_count;
+                chunk_begin = w.chunk_begin;
+                chunk = 0;
+            }
         }
-        if (p_item < p.n_items) {
-            item = p_item;
-            chunk = p_chunk++;
+        mbar_wait(&empty[st], phase ^ 1u);         // slot free (passes at once on the first lap)
+        if (item < 0) {
+            if (lane == 0) {
+                meta[st].item = -1;
+                mbar_arrive(&full[st]);
+            }
+            return;
         }
-    }
-    item = __shfl_sync(0xffffffffu, item, 0);
-    chunk = __shfl_sync(0xffffffffu, chunk, 0);
-    if (item < 0) {
+        const Chunk ch = p.chunks[chunk_begin + chunk];
+        // lane-parallel descriptor loads (one L2 round trip for up to 32 segments)
+        Seg sg = {0, 0, 0, 0};
+        if (lane < ch.seg_count) sg = p.segs[ch.seg_begin + lane];
         if (lane == 0) {
-            meta_item[s] = -1;
-            mbar_arrive(&full[s]);
+            meta[st].item = item;
+            meta[st].chunk = chunk;
+            fence_proxy_async();
+            mbar_arrive_expect_tx(&full[st], (uint32_t)ch.nbodies * 16u);
         }
-        return;
-    }
-    const Chunk ch = p.chunks[p.items[item].chunk_begin + chunk];
-    if (lane == 0) {
-        meta_item[s] = item;
-        meta_chunk[s] = chunk;
-        mbar_arrive_expect_tx(&full[s], (uint32_t)ch.nbodies * 16u);
-    }
-    if (lane == 0) {
-        // one elected thread issues the bulk copies (UBLKCP takes uniform operands)
-        for (int sg = 0; sg < ch.seg_count; ++sg) {
-            const Seg g = p.segs[ch.seg_begin + sg];
-            tma_load_1d(&stage[s][g.soff], p.bodies + g.gstart, (uint32_t)g.len * 16u, &full[s]);
+        __syncwarp();
+        if (lane < ch.seg_count)
+            tma_load_1d(&stage[st][sg.soff], p.bodies + sg.gstart, (uint32_t)sg.len * 16u, &full[st]);
+        for (int base = 32; base < ch.seg_count; base += 32) {      // rare: > 32 segments
+            if (base + lane < ch.seg_count) {
+                const Seg s2 = p.segs[ch.seg_begin + base + lane];
+                tma_load_1d(&stage[st][s2.soff], p.bodies + s2.gstart, (uint32_t)s2.len * 16u, &full[st]);
+            }
+        }
+        ++chunk;
+        if (++st == kStages) {
+            st = 0;
+            phase ^= 1u;
         }
     }
 }
 
 __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel(const P2PParams p) {
     extern __shared__ __align__(128) unsigned char dsmem[];
-    float4 (*stage)[kCap] = reinterpret_cast<float4 (*)[kCap]>(dsmem);                 // [2][kCap]
-    double (*acc)[kThreads] = reinterpret_cast<double (*)[kThreads]>(dsmem + kStageBytes); // [8][kThreads]
-    __shared__ __align__(8) uint64_t full[2];
-    __shared__ int meta_item[2], meta_chunk[2];
+    float4 (*stage)[kCap] = reinterpret_cast<float4 (*)[kCap]>(dsmem);                      // [kStages][kCap]
+    double (*acc)[kConsumers] = reinterpret_cast<double (*)[kConsumers]>(dsmem + kStageBytes); // [8][kConsumers]
+    __shared__ __align__(8) uint64_t full[kStages], empty[kStages];
+    __shared__ StageMeta meta[kStages];
 
     const int tid = threadIdx.x;
-    const int lane = tid & 31;
-    const bool producer = tid < 32;
-    int p_item = -1, p_chunk = 0, p_nchunks = 0;   // producer cursor (lane 0 of warp 0)
-
     if (tid == 0) {
-        mbar_init(&full[0], 1);
-        mbar_init(&full[1], 1);
+        for (int s = 0; s < kStages; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], kConsumers / 32);       // one arrive per consumer warp
+        }
         fence_mbar_init();
     }
     __syncthreads();
-    if (producer) {
-        produce(0, p, stage, full, meta_item, meta_chunk, p_item, p_chunk, p_nchunks, lane);
-        produce(1, p, stage, full, meta_item, meta_chunk, p_item, p_chunk, p_nchunks, lane);
+    if (tid >= kConsumers) {                             // ---- producer warp
+        producer_loop(p, stage, full, empty, meta, tid & 31);
+        return;
     }
 
+    // ---- consumer warps
     const float2 e2 = make_float2(p.eps2, p.eps2);
     float2 nx = make_float2(0.f, 0.f), ny = nx, nz = nx;
-    Acc64 A{&acc[0][threadIdx.x]};
-    int g = 1, C = 1, c = 0, l = 0, m0 = -1, m1 = -1;
+    Acc64 A{&acc[0][tid]};
+    int g = 1, C = 1, c = 0, m0 = -1, m1 = -1;
     bool active = false;
-
-    for (int q = 0;; ++q) {
-        const int s = q & 1;
-        mbar_wait(&full[s], (uint32_t)((q >> 1) & 1));
-        const int item = meta_item[s];
-        if (item < 0) break;
-        const int chunk = meta_chunk[s];
-        const Item it = p.items[item];
-        if (chunk == 0) {
+    int st = 0;
+    uint32_t phase = 0;
+    for (;;) {
+        mbar_wait(&full[st], phase);
+        const StageMeta sm = meta[st];
+        if (sm.item < 0) break;
+        const Item it = p.items[sm.item];
+        if (sm.chunk == 0) {
             g = (it.tgt_count + 1) >> 1;
-            C = kThreads / g;
+            C = min(kConsumers / g, kMaxCopies);
             c = tid / g;
-            l = tid - c * g;
+            const int l = tid - c * g;
             active = c < C;
             const int i0 = 2 * l;
             const int i1 = min(2 * l + 1, it.tgt_count - 1);
@@ -254,40 +283,40 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel(const P2
             for (int u = 0; u < 8; ++u) acc[u][tid] = 0.0;
         }
         if (active) {
-            const int nb = p.chunks[it.chunk_begin + chunk].nbodies;
-            const int kself = (chunk == 0) ? it.self_len : 0;
+            const int nb = p.chunks[it.chunk_begin + sm.chunk].nbodies;
+            const int kself = (sm.chunk == 0) ? it.self_len : 0;
             int k = c;
-            consume<true>(stage[s], k, kself, C, nx, ny, nz, e2, m0, m1, A);
-            consume<false>(stage[s], k, nb, C, nx, ny, nz, e2, m0, m1, A);
+            consume<true>(stage[st], k, kself, C, nx, ny, nz, e2, m0, m1, A);
+            consume<false>(stage[st], k, nb, C, nx, ny, nz, e2, m0, m1, A);
         }
-        if (chunk == it.chunk_count - 1) {
-            // fixed-order fp64 reduction across copies (shared-memory accumulators)
-            __syncthreads();
-            if (tid < g) {
-                double v[8];
-#pragma unroll
-                for (int u = 0; u < 8; ++u) v[u] = acc[u][tid];
-                for (int cc = 1; cc < C; ++cc) {
-#pragma unroll
-                    for (int u = 0; u < 8; ++u) v[u] += acc[u][cc * g + tid];
+        __syncwarp();
+        if ((tid & 31) == 0) mbar_arrive(&empty[st]);     // this warp is done with the stage
+        if (sm.chunk == it.chunk_count - 1) {
+            // fixed-order fp64 reduction across copies: thread j < 8g reduces
+            // component u = j / g of lane l = j % g over the C copies
+            consumer_sync();
+            for (int j = tid; j < 8 * g; j += kConsumers) {
+                const int u = j / g, l = j - u * g;
+                double v0 = 0.0, v1 = 0.0;
+                int cc = 0;
+                for (; cc + 1 < C; cc += 2) {
+                    v0 += acc[u][cc * g + l];
+                    v1 += acc[u][(cc + 1) * g + l];
                 }
-                const int i0 = it.tgt_start + 2 * tid;
-                p.ax[i0] = (float)(p.G * v[0]);
-                p.ay[i0] = (float)(p.G * v[1]);
-                p.az[i0] = (float)(p.G * v[2]);
-                p.phi[i0] = (float)(-p.G * v[3]);
-                if (2 * tid + 1 < it.tgt_count) {
-                    p.ax[i0 + 1] = (float)(p.G * v[4]);
-                    p.ay[i0 + 1] = (float)(p.G * v[5]);
-                    p.az[i0 + 1] = (float)(p.G * v[6]);
-                    p.phi[i0 + 1] = (float)(-p.G * v[7]);
+                if (cc < C) v0 += acc[u][cc * g + l];
+                const double v = v0 + v1;
+                const int tgt = 2 * l + (u >> 2);
+                if (tgt < it.tgt_count) {
+                    const int comp = u & 3;
+                    float *dst = comp == 0 ? p.ax : comp == 1 ? p.ay : comp == 2 ? p.az : p.phi;
+                    dst[it.tgt_start + tgt] = (float)(comp == 3 ? -p.G * v : p.G * v);
                 }
             }
+            consumer_sync();                              // acc free for the next item
         }
-        __syncthreads();               // stage s fully consumed
-        if (producer) {
-            fence_proxy_async();
-            produce(s, p, stage, full, meta_item, meta_chunk, p_item, p_chunk, p_nchunks, lane);
+        if (++st == kStages) {
+            st = 0;
+            phase ^= 1u;
         }
     }
 }

@@ -79,7 +79,7 @@ extern "C" afmm_status afmm_fp32_peak(int device, double *tflops_ffma, double *t
         if (cudaGetLastError() != cudaSuccess) st = AFMM_ECUDA;
         if (tflops_ffma) *tflops_ffma = lanes * 2.0 / (best1 * 1e-3) / 1e12;
         if (tflops_ffma2) *tflops_ffma2 = lanes * 4.0 / (best2 * 1e-3) / 1e12;
-        // one block's loop cycles vs the whole launch's duration (upper bound on the clock)
+        // block 0's loop cycles over the launch duration: a lower bound on the SM clock
         if (sm_mhz) *sm_mhz = (double)cyc / (best1 * 1e-3) / 1e6;
     }
     cudaFree(out);
