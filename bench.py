@@ -245,32 +245,26 @@ def main():
     out = torch.empty((4, n), device=dev)           # ax, ay, az, phi
     flush = torch.empty(64 << 20, dtype=torch.float32, device=dev)   # 256 MiB > 126 MB L2
 
-    def gather_slices():
-        ls, bs = h.get_partition()
-        for r in range(world):
-            lo, hi = int(bs[r]), int(bs[r + 1])
-            if hi > lo:
-                for a in range(4):
-                    dist.broadcast(out[a, lo:hi], src=r)
+    from paper_conf_ipps_overmanpmm13_b200 import dist as pdist
+    bsplit = [h.get_partition()[1]]
 
     def step():
         if world > 1:
-            for a in range(4):
-                dist.broadcast(bod[a], src=0)                 # a4: source replication
+            pdist.replicate([bod[a] for a in range(4)], src=0)    # a4: source replication
         h.set_bodies(bod[0], bod[1], bod[2], bod[3])          # a1: pack (1 kernel)
         h.eval(out[0], out[1], out[2], out[3])                # a5/a6: P2P (1 kernel)
         if world > 1:
-            gather_slices()                                   # a7: allgatherv of slices
+            pdist.gather_slices([out[a] for a in range(4)], bsplit[0])   # a7: allgatherv
 
     # ---- warm-up (+ incremental rebalance from measured kernel times, L18 SIV.D)
     rebalanced = 0
     for i in range(max(3, args.warmup)):
         step()
         if world > 1:
-            kt = torch.tensor([h.kernel_times(1)[-1]], dtype=torch.float64, device=dev)
-            allk = [torch.zeros_like(kt) for _ in range(world)]
-            dist.all_gather(allk, kt)
-            rebalanced += int(h.rebalance(np.array([float(v.item()) for v in allk]), 0.02))
+            times = pdist.allgather_scalar(h.kernel_times(1)[-1], dev)
+            if h.rebalance(times, 0.02):
+                rebalanced += 1
+                bsplit[0] = h.get_partition()[1]
     torch.cuda.synchronize()
 
     # ---- timed region

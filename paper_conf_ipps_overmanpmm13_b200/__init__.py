@@ -18,7 +18,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libafmm_p2p.so")
+LIB_PATH = os.environ.get("AFMM_LIB_OVERRIDE") or os.path.join(_HERE, "libafmm_p2p.so")  # override: tools/tune only
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} not built: run `make` (or __graft_entry__.build()) first; "
@@ -84,6 +84,7 @@ _sig("afmm_p2p_last_error", C.c_char_p, _p)
 _sig("afmm_interactions", _i, _i, _p, _p, _p, _p)
 _sig("afmm_partition_literal", _i, _i, _p, _i, _p)
 _sig("afmm_partition_weighted", _i, _i, _p, _i, _p)
+_sig("afmm_partition_rebalance", _i, _i, _p, _p, _i, _p, _p, _d, _p, C.POINTER(_i))
 _sig("afmm_fp32_peak", _i, _i, C.POINTER(_d), C.POINTER(_d), C.POINTER(_d))
 _sig("afmm_version", C.c_char_p)
 _sig("afmm_tree_create", _i, _i, _p, C.POINTER(_p))
@@ -103,7 +104,8 @@ EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
             "afmm_p2p_eval", "afmm_p2p_eval_host", "afmm_p2p_stats_get", "afmm_p2p_stream",
             "afmm_p2p_kernel_times",
             "afmm_p2p_destroy", "afmm_p2p_last_error", "afmm_interactions",
-            "afmm_partition_literal", "afmm_partition_weighted", "afmm_fp32_peak", "afmm_version",
+            "afmm_partition_literal", "afmm_partition_weighted", "afmm_partition_rebalance",
+            "afmm_fp32_peak", "afmm_version",
             "afmm_tree_create", "afmm_tree_build", "afmm_tree_info", "afmm_tree_copy_out",
             "afmm_tree_gather", "afmm_tree_scatter", "afmm_tree_destroy", "afmm_tree_last_error"]
 
@@ -164,6 +166,20 @@ def partition_weighted(w, G: int) -> np.ndarray:
     if st:
         raise AfmmError(st, "afmm_partition_weighted")
     return out
+
+
+def partition_rebalance(leaf_count, I, cur_split, rank_ms, threshold=0.02):
+    """Host-only rebalance rule (see afmm_partition_rebalance) -> (new_split, changed)."""
+    lc, I = _np(leaf_count, np.int32), _np(I, np.int64)
+    cs, rm = _np(cur_split, np.int64), _np(rank_ms, np.float64)
+    G = cs.shape[0] - 1
+    out = np.empty(G + 1, np.int64)
+    ch = _i()
+    st = _lib.afmm_partition_rebalance(lc.shape[0], _ptr(lc), _ptr(I), G, _ptr(cs), _ptr(rm),
+                                       float(threshold), _ptr(out), C.byref(ch))
+    if st:
+        raise AfmmError(st, "afmm_partition_rebalance")
+    return out, bool(ch.value)
 
 
 def fp32_peak(device: int = 0):

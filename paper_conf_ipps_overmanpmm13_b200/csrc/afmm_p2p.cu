@@ -20,9 +20,8 @@
 #include "../../include/afmm_p2p.h"
 #include "p2p_kernel.cuh"
 
-using afmm::Chunk;
-using afmm::Item;
 using afmm::Seg;
+using afmm::Task;
 
 struct afmm_p2p {
     afmm_p2p_config cfg{};
@@ -56,13 +55,11 @@ struct afmm_p2p {
     std::vector<long long> leaf_split, body_split;
 
     // this rank's work list
-    std::vector<Item> h_items;
-    std::vector<Chunk> h_chunks;
+    std::vector<Task> h_tasks;
     std::vector<Seg> h_segs;
-    Item *d_items = nullptr;
-    Chunk *d_chunks = nullptr;
+    Task *d_tasks = nullptr;
     Seg *d_segs = nullptr;
-    size_t items_cap = 0, chunks_cap = 0, segs_cap = 0;
+    size_t tasks_cap = 0, segs_cap = 0;
     int *d_queue = nullptr;
     long long rank_interactions = 0;
     long long bucket_inter[8] = {0};
@@ -266,8 +263,7 @@ extern "C" void afmm_p2p_destroy(afmm_p2p *h) {
     cudaFree(h->d_bodies);
     cudaFree(h->d_soa);
     cudaFree(h->d_out);
-    cudaFree(h->d_items);
-    cudaFree(h->d_chunks);
+    cudaFree(h->d_tasks);
     cudaFree(h->d_segs);
     cudaFree(h->d_queue);
     for (int i = 0; i < afmm_p2p::kRing; ++i) {
@@ -367,94 +363,7 @@ static void compute_body_split(afmm_p2p *h) {
     }
 }
 
-// Build this rank's work list on the host and upload it.
-static afmm_status build_worklist(afmm_p2p *h) {
-    const int r = h->cfg.rank;
-    const long long lo = h->leaf_split[r], hi = h->leaf_split[r + 1];
-    h->h_items.clear();
-    h->h_chunks.clear();
-    h->h_segs.clear();
-    h->rank_interactions = 0;
-    std::fill(h->bucket_inter, h->bucket_inter + 8, 0LL);
-    std::vector<long long> cost;
-    std::vector<Seg> segs;   // staged list of one leaf: self first, then merged neighbours
-    for (long long t = lo; t < hi; ++t) {
-        const int ts = h->leaf_start[t], tn = h->leaf_count[t];
-        segs.clear();
-        bool has_self = false;
-        for (long long u = h->u_off[t]; u < h->u_off[t + 1]; ++u)
-            if (h->u_idx[u] == t) has_self = true;
-        if (has_self) segs.push_back(Seg{ts, tn, 0, 0});
-        // merge runs of leaves whose body ranges are contiguous (consecutive leaf ids)
-        const size_t first_other = segs.size();
-        for (long long u = h->u_off[t]; u < h->u_off[t + 1]; ++u) {
-            const int s = h->u_idx[u];
-            if (s == t) continue;
-            const int bs = h->leaf_start[s], bn = h->leaf_count[s];
-            if (segs.size() > first_other && segs.back().gstart + segs.back().len == bs) {
-                segs.back().len += bn;
-            } else {
-                segs.push_back(Seg{bs, bn, 0, 0});
-            }
-        }
-        // cut the staged list into chunks of <= kCap bodies (self stays in chunk 0)
-        const int chunk_begin = (int)h->h_chunks.size();
-        int cur_bodies = 0;
-        Chunk cur{(int)h->h_segs.size(), 0, 0, 0};
-        long long nsrc = 0;
-        for (const Seg &sg0 : segs) {
-            Seg sg = sg0;
-            nsrc += sg.len;
-            while (sg.len > 0) {
-                if (cur_bodies == afmm::kCap) {
-                    h->h_chunks.push_back(cur);
-                    cur = Chunk{(int)h->h_segs.size(), 0, 0, 0};
-                    cur_bodies = 0;
-                }
-                const int take = std::min(sg.len, afmm::kCap - cur_bodies);
-                h->h_segs.push_back(Seg{sg.gstart, take, cur_bodies, 0});
-                cur.seg_count++;
-                cur.nbodies += take;
-                cur_bodies += take;
-                sg.gstart += take;
-                sg.len -= take;
-            }
-        }
-        if (cur.seg_count > 0 || h->h_chunks.size() == (size_t)chunk_begin) h->h_chunks.push_back(cur);
-        const int chunk_count = (int)h->h_chunks.size() - chunk_begin;
-        for (int a = 0; a < tn; a += afmm::kMaxTargets) {
-            const int cnt = std::min(afmm::kMaxTargets, tn - a);
-            h->h_items.push_back(Item{ts + a, cnt, ts, has_self ? tn : 0, chunk_begin, chunk_count, 0, 0});
-            cost.push_back((long long)(((cnt + 1) / 2) * 2) * std::max<long long>(nsrc, 1));
-        }
-        h->rank_interactions += h->I[t];
-        h->bucket_inter[bucket_of(tn)] += h->I[t];
-    }
-    // largest-cost-first order (stable for determinism of scheduling inputs)
-    std::vector<int> order(h->h_items.size());
-    std::iota(order.begin(), order.end(), 0);
-    std::stable_sort(order.begin(), order.end(), [&](int a, int b) { return cost[a] > cost[b]; });
-    std::vector<Item> sorted(order.size());
-    for (size_t i = 0; i < order.size(); ++i) sorted[i] = h->h_items[order[i]];
-    h->h_items.swap(sorted);
-
-    afmm_status st;
-    if ((st = ensure_device(h, &h->d_items, h->items_cap, h->h_items.size()))) return st;
-    if ((st = ensure_device(h, &h->d_chunks, h->chunks_cap, h->h_chunks.size()))) return st;
-    if ((st = ensure_device(h, &h->d_segs, h->segs_cap, h->h_segs.size()))) return st;
-    if (!h->h_items.empty())
-        CUDA_TRY(h, cudaMemcpyAsync(h->d_items, h->h_items.data(), h->h_items.size() * sizeof(Item),
-                                    cudaMemcpyHostToDevice, h->stream));
-    if (!h->h_chunks.empty())
-        CUDA_TRY(h, cudaMemcpyAsync(h->d_chunks, h->h_chunks.data(), h->h_chunks.size() * sizeof(Chunk),
-                                    cudaMemcpyHostToDevice, h->stream));
-    if (!h->h_segs.empty())
-        CUDA_TRY(h, cudaMemcpyAsync(h->d_segs, h->h_segs.data(), h->h_segs.size() * sizeof(Seg),
-                                    cudaMemcpyHostToDevice, h->stream));
-    CUDA_TRY(h, cudaStreamSynchronize(h->stream));
-    h->evaluated = false;
-    return AFMM_OK;
-}
+#include "worklist.inc"
 
 extern "C" afmm_status afmm_p2p_set_tree(afmm_p2p *h, int n_leaves, const int *leaf_start,
                                          const int *leaf_count, const long long *u_off,
@@ -569,41 +478,42 @@ static bool solve_small(std::vector<double> M, std::vector<double> b, int k, std
     return true;
 }
 
-extern "C" afmm_status afmm_p2p_rebalance(afmm_p2p *h, const double *rank_ms, double threshold,
-                                          int *changed) {
-    CHECK_HANDLE(h);
+extern "C" afmm_status afmm_partition_rebalance(int n_leaves, const int *leaf_count, const long long *I,
+                                                int G, const long long *cur_split, const double *rank_ms,
+                                                double threshold, long long *new_split, int *changed) {
     if (changed) *changed = 0;
-    if (!h->have_tree) return fail(h, AFMM_ESTATE, "rebalance: no tree");
-    if (!rank_ms) return fail(h, AFMM_EINVAL, "rebalance: rank_ms is null");
-    const int W = h->cfg.world;
-    if (W == 1) return AFMM_OK;
-    for (int r = 0; r < W; ++r)
-        if (!(rank_ms[r] >= 0.0) || !std::isfinite(rank_ms[r]))
-            return fail(h, AFMM_EINVAL, "rebalance: rank_ms[%d] invalid", r);
-    // per-rank bucket interaction counts for the CURRENT partition (all ranks)
-    std::vector<double> B((size_t)W * 8, 0.0);
+    if (n_leaves < 1 || G < 1 || !leaf_count || !I || !cur_split || !rank_ms || !new_split)
+        return AFMM_EINVAL;
+    if (cur_split[0] != 0 || cur_split[G] != n_leaves) return AFMM_EINVAL;
+    for (int r = 0; r < G; ++r)
+        if (cur_split[r + 1] < cur_split[r] || !(rank_ms[r] >= 0.0) || !std::isfinite(rank_ms[r]))
+            return AFMM_EINVAL;
+    std::copy(cur_split, cur_split + G + 1, new_split);
+    if (G == 1) return AFMM_OK;
+    // per-rank bucket interaction counts for the current cut
+    std::vector<double> B((size_t)G * 8, 0.0);
     double Isum = 0, Tsum = 0;
-    for (int r = 0; r < W; ++r) {
-        for (long long t = h->leaf_split[r]; t < h->leaf_split[r + 1]; ++t)
-            B[r * 8 + bucket_of(h->leaf_count[t])] += (double)h->I[t];
+    for (int r = 0; r < G; ++r) {
+        for (long long t = cur_split[r]; t < cur_split[r + 1]; ++t)
+            B[r * 8 + bucket_of(leaf_count[t])] += (double)I[t];
         Tsum += rank_ms[r];
     }
     for (double v : B) Isum += v;
     if (Isum <= 0 || Tsum <= 0) return AFMM_OK;
-    const double k0 = Tsum / Isum;     // the paper's GPU coefficient, all ranks (L18 SIV.D)
+    const double k0 = Tsum / Isum;     // the paper's GPU coefficient over all GPUs (L18 SIV.D)
     // ridge-regularised least squares for per-bucket coefficients around k0:
-    // min sum_r (sum_b B_rb c_b - T_r)^2 + lam * sum_b (Bsum_b/W)^2 (c_b - k0)^2
+    // min sum_r (sum_b B_rb c_b - T_r)^2 + lam * sum_b (Bsum_b/G)^2 (c_b - k0)^2
     std::vector<double> M(64, 0.0), rhs(8, 0.0), Bs(8, 0.0);
-    for (int r = 0; r < W; ++r)
+    for (int r = 0; r < G; ++r)
         for (int b = 0; b < 8; ++b) Bs[b] += B[r * 8 + b];
     const double lam = 0.1;
-    for (int r = 0; r < W; ++r)
+    for (int r = 0; r < G; ++r)
         for (int a = 0; a < 8; ++a) {
             for (int b = 0; b < 8; ++b) M[a * 8 + b] += B[r * 8 + a] * B[r * 8 + b];
             rhs[a] += B[r * 8 + a] * rank_ms[r];
         }
     for (int b = 0; b < 8; ++b) {
-        const double wgt = lam * (Bs[b] / W) * (Bs[b] / W) + 1e-30;
+        const double wgt = lam * (Bs[b] / G) * (Bs[b] / G) + 1e-30;
         M[b * 8 + b] += wgt;
         rhs[b] += wgt * k0;
     }
@@ -611,27 +521,46 @@ extern "C" afmm_status afmm_p2p_rebalance(afmm_p2p *h, const double *rank_ms, do
     if (!solve_small(M, rhs, 8, coef)) coef.assign(8, k0);
     for (double &c : coef)
         if (!(c > 0.05 * k0)) c = 0.05 * k0;      // keep weights positive
-    std::vector<double> w(h->L);
-    for (int t = 0; t < h->L; ++t) w[t] = (double)h->I[t] * coef[bucket_of(h->leaf_count[t])];
-    std::vector<long long> split(W + 1);
-    afmm_partition_weighted(h->L, w.data(), W, split.data());
-    // predicted imbalance of the new cut vs the measured one
+    std::vector<double> w(n_leaves);
+    for (int t = 0; t < n_leaves; ++t) w[t] = (double)I[t] * coef[bucket_of(leaf_count[t])];
+    std::vector<long long> split(G + 1);
+    afmm_partition_weighted(n_leaves, w.data(), G, split.data());
+    // adopt only if the predicted imbalance beats the measured one by > threshold
+    // (hysteresis in the spirit of the paper's 5% observation rule, L22 SVII.B)
     double tmax = 0, pmax = 0, psum = 0;
-    for (int r = 0; r < W; ++r) tmax = std::max(tmax, rank_ms[r]);
-    for (int r = 0; r < W; ++r) {
-        double p = 0;
-        for (long long t = split[r]; t < split[r + 1]; ++t) p += w[t];
-        pmax = std::max(pmax, p);
-        psum += p;
+    for (int r = 0; r < G; ++r) tmax = std::max(tmax, rank_ms[r]);
+    for (int r = 0; r < G; ++r) {
+        double pr = 0;
+        for (long long t = split[r]; t < split[r + 1]; ++t) pr += w[t];
+        pmax = std::max(pmax, pr);
+        psum += pr;
     }
-    const double cur_imb = tmax / (Tsum / W);
-    const double new_imb = psum > 0 ? pmax / (psum / W) : 1.0;
-    if (cur_imb - new_imb > threshold && split != h->leaf_split) {
+    const double cur_imb = tmax / (Tsum / G);
+    const double new_imb = psum > 0 ? pmax / (psum / G) : 1.0;
+    if (cur_imb - new_imb > threshold && !std::equal(split.begin(), split.end(), cur_split)) {
+        std::copy(split.begin(), split.end(), new_split);
+        if (changed) *changed = 1;
+    }
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_p2p_rebalance(afmm_p2p *h, const double *rank_ms, double threshold,
+                                          int *changed) {
+    CHECK_HANDLE(h);
+    if (changed) *changed = 0;
+    if (!h->have_tree) return fail(h, AFMM_ESTATE, "rebalance: no tree");
+    if (!rank_ms) return fail(h, AFMM_EINVAL, "rebalance: rank_ms is null");
+    const int W = h->cfg.world;
+    std::vector<long long> split(W + 1);
+    int ch = 0;
+    afmm_status st = afmm_partition_rebalance(h->L, h->leaf_count.data(), h->I.data(), W,
+                                              h->leaf_split.data(), rank_ms, threshold, split.data(), &ch);
+    if (st) return fail(h, st, "rebalance: invalid rank_ms or partition");
+    if (ch) {
         h->leaf_split = split;
         h->user_partition = true;
         compute_body_split(h);
-        afmm_status st = set_device(h);
-        if (st) return st;
+        if ((st = set_device(h))) return st;
         if ((st = build_worklist(h))) return st;
         if (changed) *changed = 1;
     }
@@ -643,10 +572,9 @@ extern "C" afmm_status afmm_p2p_rebalance(afmm_p2p *h, const double *rank_ms, do
 static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, float *phi) {
     afmm::P2PParams p;
     p.bodies = h->d_bodies;
-    p.items = h->d_items;
-    p.chunks = h->d_chunks;
+    p.tasks = h->d_tasks;
     p.segs = h->d_segs;
-    p.n_items = (int)h->h_items.size();
+    p.n_tasks = (int)h->h_tasks.size();
     p.queue = h->d_queue;
     p.ax = ax;
     p.ay = ay;
@@ -660,8 +588,9 @@ static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, flo
     h->ev1 = h->ring1[ri];
     CUDA_TRY(h, cudaEventRecord(h->ev0, h->stream));
     int nlaunch = 0;
-    if (p.n_items > 0) {
-        const int grid = std::max(1, std::min(p.n_items, h->num_sms * h->blocks_per_sm));
+    if (p.n_tasks > 0) {
+        const int grid = std::max(1, std::min((p.n_tasks + afmm::kWarps - 1) / afmm::kWarps,
+                                              h->num_sms * h->blocks_per_sm));
         afmm::p2p_kernel<<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(p);
         CUDA_TRY(h, cudaGetLastError());
         nlaunch = 1;
@@ -685,7 +614,7 @@ static afmm_status fill_stats(afmm_p2p *h, afmm_p2p_stats *s) {
     o.leaf_hi = h->leaf_split[h->cfg.rank + 1];
     o.body_lo = h->body_split[h->cfg.rank];
     o.body_hi = h->body_split[h->cfg.rank + 1];
-    o.n_work_items = (int)h->h_items.size();
+    o.n_work_items = (int)h->h_tasks.size();
     o.n_launches = h->last.n_launches;
     for (int b = 0; b < 8; ++b) o.bucket_interactions[b] = h->bucket_inter[b];
     h->last = o;

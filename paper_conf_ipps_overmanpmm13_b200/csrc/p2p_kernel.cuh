@@ -1,67 +1,88 @@
 // p2p_kernel.cuh -- the near-field P2P kernel for sm_100a.
 //
 // What it computes (PAPER.md L12 SI.C, L16 SIII.C; pair law reading R1-R3 in
-// DESIGN.md): for every target body i of a work item (a chunk of <= 512 bodies
-// of one target leaf t) and every source body j of U(t), j != i,
+// DESIGN.md): for every target body i of a target leaf t and every source body
+// j of U(t), j != i,
 //     phi_i -= G m_j / r,   a_i += G m_j d / r^3,   d = x_j - x_i,  r^2 = |d|^2 + eps2.
 //
-// B200 design:
-//  * persistent, warp-specialised CTAs: 8 consumer warps + 1 producer warp.
-//    The producer pulls work items from an atomic queue (ordered largest-cost-
-//    first by the host), loads the chunk/segment descriptors lane-parallel and
-//    stages each chunk's source segments (the self leaf first, then merged runs
-//    of consecutive U-list leaves) into a kStages-deep shared-memory ring with
-//    1-D TMA bulk copies (cp.async.bulk ... mbarrier::complete_tx).  Full/empty
-//    mbarriers per stage; consumers never wait on the producer's metadata
-//    latency unless the ring runs dry.
-//  * lane mapping: 2 targets per consumer thread (FFMA2 packed math, the source
-//    coordinate broadcast as the .F32 operand), g = ceil(n_t/2) lanes per
-//    "copy", C = min(256/g, kMaxCopies) copies; copy c consumes sources c, c+C,
-//    ... so leaves of any size keep the lanes busy (the paper's one-thread-per-
-//    target blocks idle the rest, L16 SIII.C).
-//  * accumulation: fp32 partials over <= kFold sources per copy, folded into
-//    fp64 accumulators in shared memory; copies reduced in fixed order in fp64
-//    (one consumer-only named barrier per item); one RN rounding to fp32.
-//    Deterministic and independent of the partition (bit-identical across
-//    world sizes).
+// B200 design: every warp is an autonomous pipeline.
+//  * Work = tasks of <= 128 targets (one leaf, or a 128-target slice of a big
+//    leaf), ordered largest-cost-first by the host; warps claim tasks from an
+//    atomic queue one task ahead and prefetch its descriptors.
+//  * A task's sources (its own leaf first, then runs of consecutive U-list
+//    leaves merged into contiguous body segments) stream through a private
+//    kWStages x kWCap-body shared-memory ring per warp, filled by 1-D TMA bulk
+//    copies (cp.async.bulk ... mbarrier::complete_tx) one chunk ahead of the
+//    math -- across task boundaries, so the ring never drains between tasks.
+//  * lane mapping: 4 targets per lane as two FFMA2 pairs (the source coordinate
+//    broadcast as the .F32 operand; two independent chains per source),
+//    g = ceil(n/4) lanes per copy and C = 32/g source-split copies per warp, so
+//    adaptive leaves of any size keep the lanes busy (the paper's
+//    one-thread-per-target blocks idle them, L16 SIII.C).  No CTA barrier
+//    anywhere: reductions over copies are warp-local.
+//  * math: rsqrt.approx.ftz; 13 packed FP32 ops + 2 MUFU per two interactions.
+//  * accumulation (reading R17): fp32 partials over <= kFold sources per copy,
+//    folded into fp64 accumulators in shared memory; copies reduced in a fixed
+//    order in fp64; one RN rounding to fp32.  Deterministic and independent of
+//    the partition (bit-identical across world sizes).
 #pragma once
 #include <cstdint>
 #include <cuda_runtime.h>
 
 namespace afmm {
 
-constexpr int kConsumers = 256;                 // consumer threads (8 warps)
-constexpr int kThreads = kConsumers + 32;       // + 1 producer warp
-constexpr int kCap = 1024;                      // bodies per shared-memory stage (16 KiB)
-constexpr int kStages = 3;                      // TMA ring depth
-constexpr int kMaxTargets = 512;                // targets per work item (2 per thread)
-constexpr int kMaxCopies = 64;                  // source-split copies per item
-constexpr int kFold = 64;                       // fp32 partial length per copy before the fp64 fold
-constexpr int kMinBlocksPerSM = 3;
-constexpr int kStageBytes = kStages * kCap * 16;
-constexpr int kDynSmem = kStageBytes + 8 * kConsumers * 8;    // + fp64 accumulators
+// Tuning knobs (overridable with -D for tools/tune builds; defaults are the product's).
+#ifndef AFMM_WCAP
+#define AFMM_WCAP 384
+#endif
+#ifndef AFMM_WSTAGES
+#define AFMM_WSTAGES 2
+#endif
+#ifndef AFMM_WARPS
+#define AFMM_WARPS 12
+#endif
+#ifndef AFMM_MINB
+#define AFMM_MINB 1
+#endif
+#ifndef AFMM_UNROLL
+#define AFMM_UNROLL 4
+#endif
+#ifndef AFMM_FOLD
+#define AFMM_FOLD 128
+#endif
+constexpr int kWarps = AFMM_WARPS;              // warps per CTA (all consumers)
+constexpr int kThreads = 32 * kWarps;
+constexpr int kWCap = AFMM_WCAP;                // bodies per warp stage
+constexpr int kWStages = AFMM_WSTAGES;          // per-warp TMA ring depth
+constexpr int kTPT = 4;                         // targets per lane
+constexpr int kPairs = kTPT / 2;                // FFMA2 pairs per lane
+constexpr int kVals = 4 * kTPT;                 // fp64 accumulators per lane (ax, ay, az, phi per target)
+constexpr int kTaskTargets = kTPT * 32;         // targets per task (128)
+constexpr int kFold = AFMM_FOLD;                // fp32 partial length per copy before the fp64 fold
+constexpr int kMinBlocksPerSM = AFMM_MINB;
+constexpr int kUnroll = AFMM_UNROLL;            // inner-loop unroll (sources)
+constexpr int kStageBytesW = kWStages * kWCap * 16;     // per warp
+constexpr int kAccBytesW = kVals * 32 * 8;              // per warp
+constexpr int kDynSmem = kWarps * (kStageBytesW + kAccBytesW);
 
-// Work item: targets [tgt_start, tgt_start+tgt_count) of the leaf starting at
-// self_start; its sources are chunks [chunk_begin, chunk_begin+chunk_count).
-struct Item {
-    int tgt_start, tgt_count, self_start, self_len, chunk_begin, chunk_count, pad0, pad1;
+// Task: targets [tgt_start, +tgt_count <= 128) of the leaf whose bodies start
+// at self_start; self_len = the leaf's size if it is in its own U-list (then
+// the first segment is the leaf itself), else 0; sources = segments
+// [seg_begin, +seg_count) totalling nsrc bodies.
+struct Task {
+    int tgt_start, tgt_count, self_start, self_len, seg_begin, seg_count, nsrc, pad;
 };
-// Chunk: segments [seg_begin, seg_begin+seg_count) totalling nbodies (<= kCap).
-struct Chunk {
-    int seg_begin, seg_count, nbodies, pad;
-};
-// Segment: bodies [gstart, gstart+len) staged at shared-memory body offset soff.
+// Segment: bodies [gstart, gstart+len).
 struct Seg {
-    int gstart, len, soff, pad;
+    int gstart, len;
 };
 
 struct P2PParams {
     const float4 *bodies;    // packed {x,y,z,m}, tree order
-    const Item *items;
-    const Chunk *chunks;
+    const Task *tasks;
     const Seg *segs;
-    int n_items;
-    int *queue;              // work counter, zeroed before launch
+    int n_tasks;
+    int *queue;              // task counter, zeroed before launch
     float *ax, *ay, *az, *phi;
     float eps2;
     double G;
@@ -83,9 +104,6 @@ __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *b, uint32_t byte
     asm volatile("mbarrier.arrive.expect_tx.release.cta.shared::cta.b64 _, [%0], %1;"
                  ::"r"(smem_u32(b)), "r"(bytes) : "memory");
 }
-__device__ __forceinline__ void mbar_arrive(uint64_t *b) {
-    asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
-}
 __device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
     asm volatile(
         "{\n"
@@ -96,10 +114,6 @@ __device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
         "bra LAB_WAIT;\n"
         "DONE:\n"
         "}\n" ::"r"(smem_u32(b)), "r"(parity) : "memory");
-}
-// named barrier among the consumer warps only (the producer never joins)
-__device__ __forceinline__ void consumer_sync() {
-    asm volatile("bar.sync 1, %0;" ::"n"(kConsumers) : "memory");
 }
 // 1-D bulk async copy global -> shared, completion counted on an mbarrier (TMA).
 __device__ __forceinline__ void tma_load_1d(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
@@ -141,183 +155,238 @@ __device__ __forceinline__ void interact2(const float4 q, const float2 nx, const
     az = __ffma2_rn(s, dz, az);
 }
 
-// fp64 accumulators live in shared memory, [8][kConsumers] (conflict free), so
-// the fp32 inner loop keeps its registers; folded every kFold sources.
-struct Acc64 {
-    double *p;   // &acc[0][tid]
-    __device__ __forceinline__ void add(int u, float v) { p[u * kConsumers] += (double)v; }
+// Targets of one lane: kPairs FFMA2 pairs (negated coordinates) and the
+// staged-list index of each target (-1: padding slot).
+struct Targets {
+    float2 nx[kPairs], ny[kPairs], nz[kPairs];
+    int m[kTPT];
 };
 
-// Consume sources k = k0, k0+C, ... < kend of one staged chunk.
-template <bool kMasked>
-__device__ __forceinline__ void consume(const float4 *__restrict__ src, int &k, int kend, int C,
-                                        const float2 nx, const float2 ny, const float2 nz,
-                                        const float2 e2, int m0, int m1, Acc64 &A) {
-    while (k < kend) {
-        float2 ax = make_float2(0.f, 0.f), ay = ax, az = ax, ph = ax;
-        const int kstop = min(kend, k + kFold * C);
-#pragma unroll 4
-        for (; k < kstop; k += C) {
-            const float4 q = src[k];
-            interact2<kMasked>(q, nx, ny, nz, e2, ax, ay, az, ph, k == m0, k == m1);
+// fp32 partial sums of one copy plus the lane's fp64 accumulators in shared
+// memory ([kVals][32] per warp, conflict free; u = 4*target_slot + component).
+struct Partial {
+    float2 ax[kPairs], ay[kPairs], az[kPairs], ph[kPairs];
+    int cnt;                              // sources since the last fold
+    double *acc;                          // &acc_w[0][lane]
+    __device__ __forceinline__ void clear() {
+#pragma unroll
+        for (int q = 0; q < kPairs; ++q) ax[q] = ay[q] = az[q] = ph[q] = make_float2(0.f, 0.f);
+        cnt = 0;
+    }
+    __device__ __forceinline__ void fold() {
+#pragma unroll
+        for (int q = 0; q < kPairs; ++q) {
+            double *a = acc + 8 * q * 32;
+            a[0 * 32] += (double)ax[q].x; a[1 * 32] += (double)ay[q].x;
+            a[2 * 32] += (double)az[q].x; a[3 * 32] += (double)ph[q].x;
+            a[4 * 32] += (double)ax[q].y; a[5 * 32] += (double)ay[q].y;
+            a[6 * 32] += (double)az[q].y; a[7 * 32] += (double)ph[q].y;
         }
-        A.add(0, ax.x); A.add(1, ay.x); A.add(2, az.x); A.add(3, ph.x);
-        A.add(4, ax.y); A.add(5, ay.y); A.add(6, az.y); A.add(7, ph.y);
+        clear();
+    }
+};
+
+// Consume sources src[k], k = k0, k0+C, ... < kend; fp32 partials are folded
+// into fp64 before they would exceed kFold sources.  Masks compare k with
+// T.m[j] - moff.
+template <bool kMasked>
+__device__ __forceinline__ void consume(const float4 *__restrict__ src, int k, int kend, int C,
+                                        const Targets &T, int moff, const float2 e2, Partial &P) {
+    while (k < kend) {
+        if (P.cnt >= kFold) P.fold();
+        const int kstop = min(kend, k + (kFold - P.cnt) * C);
+        int iters = 0;
+#pragma unroll kUnroll
+        for (; k < kstop; k += C) {
+            const float4 q4 = src[k];
+#pragma unroll
+            for (int q = 0; q < kPairs; ++q)
+                interact2<kMasked>(q4, T.nx[q], T.ny[q], T.nz[q], e2, P.ax[q], P.ay[q], P.az[q], P.ph[q],
+                                   kMasked && k == T.m[2 * q] - moff, kMasked && k == T.m[2 * q + 1] - moff);
+            ++iters;
+        }
+        P.cnt += iters;
     }
 }
 
-struct StageMeta {
-    int item, chunk;
+// Per-stage metadata of a warp's ring (written by lane 0 at issue time).
+struct ChunkMeta {
+    int tgt_start, tgt_count, toff, self_len, first, nb, is_first, is_last;
 };
 
-// Producer warp: walk the queue, stage every chunk of every claimed item.
-__device__ __forceinline__ void producer_loop(const P2PParams &p, float4 (*stage)[kCap],
-                                              uint64_t *full, uint64_t *empty, StageMeta *meta,
-                                              int lane) {
-    int st = 0;
-    uint32_t phase = 0;
-    int item = -1, chunk = 0, nchunks = 0, chunk_begin = 0;
-    for (;;) {
-        if (chunk >= nchunks) {                    // claim the next item
-            int it = 0;
-            if (lane == 0) it = atomicAdd(p.queue, 1);
-            it = __shfl_sync(0xffffffffu, it, 0);
-            if (it >= p.n_items) {
-                item = -1;
-            } else {
-                item = it;
-                const Item w = p.items[it];
-                nchunks = w.chunk_count;
-                chunk_begin = w.chunk_begin;
-                chunk = 0;
-            }
+// Issue side of a warp's pipeline: the task whose sources are being streamed
+// and the task after it (both claimed from the queue, descriptors in lanes:
+// lane i holds segment i).
+struct Stream {
+    int task, nxt;                // task ids (>= n_tasks: none)
+    Task t, tn;                   // descriptors (warp-uniform)
+    Seg sg, sgn;                  // this lane's segment of t / tn
+    int iseg, ioff, staged;       // cursor within t's source list
+};
+
+__device__ __forceinline__ int claim(const P2PParams &p, int lane) {
+    int it = 0;
+    if (lane == 0) it = atomicAdd(p.queue, 1);
+    return __shfl_sync(0xffffffffu, it, 0);
+}
+__device__ __forceinline__ void load_task(const P2PParams &p, int id, Task &t, Seg &sg, int lane) {
+    if (id >= p.n_tasks) return;
+    t = p.tasks[id];
+    sg = Seg{0, 0};
+    if (lane < t.seg_count) sg = p.segs[t.seg_begin + lane];
+}
+
+// Stage the next chunk (<= kWCap bodies) of the stream into `buf`; returns
+// false when no task is left.
+__device__ __forceinline__ bool issue_chunk(const P2PParams &p, Stream &S, float4 *buf, uint64_t *bar,
+                                            ChunkMeta *meta, int lane) {
+    if (S.task >= p.n_tasks) return false;
+    const int nb = min(kWCap, S.t.nsrc - S.staged);
+    if (lane == 0) {
+        ChunkMeta m;
+        m.tgt_start = S.t.tgt_start;
+        m.tgt_count = S.t.tgt_count;
+        m.toff = S.t.tgt_start - S.t.self_start;
+        m.self_len = S.t.self_len;
+        m.first = S.staged;
+        m.nb = nb;
+        m.is_first = S.staged == 0;
+        m.is_last = S.staged + nb >= S.t.nsrc;
+        *meta = m;
+        fence_proxy_async();
+        mbar_arrive_expect_tx(bar, (uint32_t)nb * 16u);
+    }
+    // pieces of the current segments (warp-uniform walk; lane 0 issues)
+    int filled = 0;
+    while (filled < nb) {
+        int gstart = __shfl_sync(0xffffffffu, S.sg.gstart, S.iseg & 31);
+        int len = __shfl_sync(0xffffffffu, S.sg.len, S.iseg & 31);
+        if (S.iseg >= 32) {                               // rare: > 32 segments
+            const Seg s2 = p.segs[S.t.seg_begin + S.iseg];
+            gstart = s2.gstart;
+            len = s2.len;
         }
-        mbar_wait(&empty[st], phase ^ 1u);         // slot free (passes at once on the first lap)
-        if (item < 0) {
-            if (lane == 0) {
-                meta[st].item = -1;
-                mbar_arrive(&full[st]);
-            }
-            return;
+        const int take = min(len - S.ioff, nb - filled);
+        if (lane == 0) tma_load_1d(buf + filled, p.bodies + gstart + S.ioff, (uint32_t)take * 16u, bar);
+        filled += take;
+        S.ioff += take;
+        if (S.ioff == len) {
+            ++S.iseg;
+            S.ioff = 0;
         }
-        const Chunk ch = p.chunks[chunk_begin + chunk];
-        // lane-parallel descriptor loads (one L2 round trip for up to 32 segments)
-        Seg sg = {0, 0, 0, 0};
-        if (lane < ch.seg_count) sg = p.segs[ch.seg_begin + lane];
-        if (lane == 0) {
-            meta[st].item = item;
-            meta[st].chunk = chunk;
-            fence_proxy_async();
-            mbar_arrive_expect_tx(&full[st], (uint32_t)ch.nbodies * 16u);
+    }
+    S.staged += nb;
+    if (S.staged >= S.t.nsrc) {                           // advance to the prefetched task
+        S.task = S.nxt;
+        S.t = S.tn;
+        S.sg = S.sgn;
+        S.iseg = S.ioff = S.staged = 0;
+        S.nxt = claim(p, lane);                           // and prefetch the one after
+        load_task(p, S.nxt, S.tn, S.sgn, lane);
+    }
+    return true;
+}
+
+// Load this lane's targets (4 consecutive of the n targets of the task): from
+// the staged self leaf when present in this stage, else from global memory.
+__device__ __forceinline__ void load_targets(Targets &T, const float4 *__restrict__ stage,
+                                             const float4 *__restrict__ bodies, const ChunkMeta &m,
+                                             int l, bool active) {
+    const bool staged = m.self_len > 0 && m.toff + m.tgt_count <= m.nb;
+#pragma unroll
+    for (int q = 0; q < kPairs; ++q) {
+        float4 b[2];
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            const int j = 2 * q + h;
+            const int i = min(kTPT * l + j, m.tgt_count - 1);     // padding slots repeat the last target
+            T.m[j] = (kTPT * l + j < m.tgt_count) ? m.toff + i : -1;
+            if (active) b[h] = staged ? stage[m.toff + i] : bodies[m.tgt_start + i];
+            else b[h] = make_float4(0.f, 0.f, 0.f, 0.f);
         }
-        __syncwarp();
-        if (lane < ch.seg_count)
-            tma_load_1d(&stage[st][sg.soff], p.bodies + sg.gstart, (uint32_t)sg.len * 16u, &full[st]);
-        for (int base = 32; base < ch.seg_count; base += 32) {      // rare: > 32 segments
-            if (base + lane < ch.seg_count) {
-                const Seg s2 = p.segs[ch.seg_begin + base + lane];
-                tma_load_1d(&stage[st][s2.soff], p.bodies + s2.gstart, (uint32_t)s2.len * 16u, &full[st]);
-            }
-        }
-        ++chunk;
-        if (++st == kStages) {
-            st = 0;
-            phase ^= 1u;
-        }
+        T.nx[q] = make_float2(-b[0].x, -b[1].x);
+        T.ny[q] = make_float2(-b[0].y, -b[1].y);
+        T.nz[q] = make_float2(-b[0].z, -b[1].z);
     }
 }
 
 __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel(const P2PParams p) {
     extern __shared__ __align__(128) unsigned char dsmem[];
-    float4 (*stage)[kCap] = reinterpret_cast<float4 (*)[kCap]>(dsmem);                      // [kStages][kCap]
-    double (*acc)[kConsumers] = reinterpret_cast<double (*)[kConsumers]>(dsmem + kStageBytes); // [8][kConsumers]
-    __shared__ __align__(8) uint64_t full[kStages], empty[kStages];
-    __shared__ StageMeta meta[kStages];
-
-    const int tid = threadIdx.x;
-    if (tid == 0) {
-        for (int s = 0; s < kStages; ++s) {
-            mbar_init(&full[s], 1);
-            mbar_init(&empty[s], kConsumers / 32);       // one arrive per consumer warp
-        }
+    __shared__ __align__(8) uint64_t full_all[kWarps][kWStages];
+    __shared__ ChunkMeta meta_all[kWarps][kWStages];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    float4 (*stage)[kWCap] = reinterpret_cast<float4 (*)[kWCap]>(dsmem + warp * kStageBytesW);
+    double *accw = reinterpret_cast<double *>(dsmem + kWarps * kStageBytesW + warp * kAccBytesW);
+    uint64_t *full = full_all[warp];
+    ChunkMeta *meta = meta_all[warp];
+    if (lane == 0) {
+        for (int s = 0; s < kWStages; ++s) mbar_init(&full[s], 1);
         fence_mbar_init();
     }
-    __syncthreads();
-    if (tid >= kConsumers) {                             // ---- producer warp
-        producer_loop(p, stage, full, empty, meta, tid & 31);
-        return;
-    }
+    __syncwarp();
 
-    // ---- consumer warps
+    // ---- start the stream: claim two tasks, fill the ring but one stage
+    Stream S;
+    S.task = claim(p, lane);
+    load_task(p, S.task, S.t, S.sg, lane);
+    S.nxt = claim(p, lane);
+    load_task(p, S.nxt, S.tn, S.sgn, lane);
+    S.iseg = S.ioff = S.staged = 0;
+    int issued = 0;
+    for (; issued < kWStages - 1; ++issued)
+        if (!issue_chunk(p, S, stage[issued % kWStages], &full[issued % kWStages], &meta[issued % kWStages], lane))
+            break;
+
     const float2 e2 = make_float2(p.eps2, p.eps2);
-    float2 nx = make_float2(0.f, 0.f), ny = nx, nz = nx;
-    Acc64 A{&acc[0][tid]};
-    int g = 1, C = 1, c = 0, m0 = -1, m1 = -1;
+    Targets T;
+    Partial P;
+    P.acc = accw + lane;
+    int g = 1, C = 1, c = 0, l = 0;
     bool active = false;
-    int st = 0;
-    uint32_t phase = 0;
-    for (;;) {
-        mbar_wait(&full[st], phase);
-        const StageMeta sm = meta[st];
-        if (sm.item < 0) break;
-        const Item it = p.items[sm.item];
-        if (sm.chunk == 0) {
-            g = (it.tgt_count + 1) >> 1;
-            C = min(kConsumers / g, kMaxCopies);
-            c = tid / g;
-            const int l = tid - c * g;
+    for (int q = 0; q < issued; ++q) {
+        // keep the ring one chunk ahead (across task boundaries)
+        if (issued == q + kWStages - 1) {
+            const int s2 = issued % kWStages;
+            if (issue_chunk(p, S, stage[s2], &full[s2], &meta[s2], lane)) ++issued;
+        }
+        const int st = q % kWStages;
+        mbar_wait(&full[st], (uint32_t)((q / kWStages) & 1));
+        const ChunkMeta m = meta[st];
+        if (m.is_first) {
+            g = (m.tgt_count + kTPT - 1) / kTPT;
+            C = 32 / g;
+            c = lane / g;
+            l = lane - c * g;
             active = c < C;
-            const int i0 = 2 * l;
-            const int i1 = min(2 * l + 1, it.tgt_count - 1);
-            const int toff = it.tgt_start - it.self_start;
-            m0 = toff + i0;
-            m1 = (2 * l + 1 < it.tgt_count) ? toff + i1 : m0;
-            if (active) {
-                const float4 b0 = p.bodies[it.tgt_start + i0];
-                const float4 b1 = p.bodies[it.tgt_start + i1];
-                nx = make_float2(-b0.x, -b1.x);
-                ny = make_float2(-b0.y, -b1.y);
-                nz = make_float2(-b0.z, -b1.z);
-            }
+            load_targets(T, stage[st], p.bodies, m, l, active);
 #pragma unroll
-            for (int u = 0; u < 8; ++u) acc[u][tid] = 0.0;
+            for (int u = 0; u < kVals; ++u) accw[u * 32 + lane] = 0.0;
+            P.clear();
         }
         if (active) {
-            const int nb = p.chunks[it.chunk_begin + sm.chunk].nbodies;
-            const int kself = (sm.chunk == 0) ? it.self_len : 0;
-            int k = c;
-            consume<true>(stage[st], k, kself, C, nx, ny, nz, e2, m0, m1, A);
-            consume<false>(stage[st], k, nb, C, nx, ny, nz, e2, m0, m1, A);
+            const int kself = min(max(m.self_len - m.first, 0), m.nb);
+            if (kself > 0) consume<true>(stage[st], c, kself, C, T, m.first, e2, P);
+            const int k0 = kself + ((c - kself) % C + C) % C;        // first k >= kself, k = c (mod C)
+            consume<false>(stage[st], k0, m.nb, C, T, 0, e2, P);
         }
-        __syncwarp();
-        if ((tid & 31) == 0) mbar_arrive(&empty[st]);     // this warp is done with the stage
-        if (sm.chunk == it.chunk_count - 1) {
-            // fixed-order fp64 reduction across copies: thread j < 8g reduces
-            // component u = j / g of lane l = j % g over the C copies
-            consumer_sync();
-            for (int j = tid; j < 8 * g; j += kConsumers) {
-                const int u = j / g, l = j - u * g;
-                double v0 = 0.0, v1 = 0.0;
-                int cc = 0;
-                for (; cc + 1 < C; cc += 2) {
-                    v0 += acc[u][cc * g + l];
-                    v1 += acc[u][(cc + 1) * g + l];
-                }
-                if (cc < C) v0 += acc[u][cc * g + l];
-                const double v = v0 + v1;
-                const int tgt = 2 * l + (u >> 2);
-                if (tgt < it.tgt_count) {
+        if (m.is_last) {
+            if (active) P.fold();
+            __syncwarp();
+            // fixed-order fp64 reduction over the warp's copies
+            for (int j = lane; j < kVals * g; j += 32) {
+                const int u = j / g, l2 = j - u * g;
+                const double *a = accw + u * 32 + l2;
+                double v = 0.0;
+                for (int cc = 0; cc < C; ++cc) v += a[cc * g];
+                const int tgt = kTPT * l2 + (u >> 2);
+                if (tgt < m.tgt_count) {
                     const int comp = u & 3;
                     float *dst = comp == 0 ? p.ax : comp == 1 ? p.ay : comp == 2 ? p.az : p.phi;
-                    dst[it.tgt_start + tgt] = (float)(comp == 3 ? -p.G * v : p.G * v);
+                    dst[m.tgt_start + tgt] = (float)(comp == 3 ? -p.G * v : p.G * v);
                 }
             }
-            consumer_sync();                              // acc free for the next item
         }
-        if (++st == kStages) {
-            st = 0;
-            phase ^= 1u;
-        }
+        __syncwarp();                     // stage st (and the accumulators) free again
     }
 }
 

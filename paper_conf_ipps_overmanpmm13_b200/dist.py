@@ -1,0 +1,49 @@
+"""torch.distributed plumbing for the multi-GPU path.
+
+No arithmetic of the method lives here: these helpers only move the library's
+inputs and outputs between ranks (NCCL over NVLink/NVSwitch on B200; gloo on
+CPU in the tests).
+
+* replicate(tensors, src)      -- a4: "building the data to send to the GPUs"
+                                  (PAPER L16 SIII.C): every rank holds all bodies.
+* gather_slices(rows, split)   -- a7: every rank's disjoint output slice to all
+                                  ranks (allgatherv as one broadcast per owner);
+                                  the paper's blocking copy "into known
+                                  locations" (L16 SIII.D).
+* allgather_scalar(v, device)  -- a8: per-rank kernel times for the GPU time
+                                  (max over GPUs, L20 SVII.A) and the rebalance.
+"""
+from __future__ import annotations
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+
+def body_split_from(leaf_split, leaf_start, n):
+    """Rank r owns output bodies [body_split[r], body_split[r+1])."""
+    ls = np.asarray(leaf_split, np.int64)
+    L = len(leaf_start)
+    return np.array([n if v >= L else int(leaf_start[v]) for v in ls], np.int64)
+
+
+def replicate(tensors, src=0):
+    for t in tensors:
+        dist.broadcast(t, src=src)
+
+
+def gather_slices(rows, body_split):
+    """rows: list of 1-D tensors (length n) owned piecewise by the ranks."""
+    world = len(body_split) - 1
+    for r in range(world):
+        lo, hi = int(body_split[r]), int(body_split[r + 1])
+        if hi > lo:
+            for row in rows:
+                dist.broadcast(row[lo:hi], src=r)
+
+
+def allgather_scalar(v: float, device) -> np.ndarray:
+    t = torch.tensor([float(v)], dtype=torch.float64, device=device)
+    out = [torch.zeros_like(t) for _ in range(dist.get_world_size())]
+    dist.all_gather(out, t)
+    return np.array([float(o.item()) for o in out])
