@@ -90,7 +90,7 @@ class ClockSampler:
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
-                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+                 "-lms", "20"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
         except Exception:
@@ -256,6 +256,9 @@ def main():
         if world > 1:
             pdist.gather_slices([out[a] for a in range(4)], bsplit[0])   # a7: allgatherv
 
+    # clocks are sampled from the warm-up through the timed region
+    clk = ClockSampler(local).__enter__()
+
     # ---- warm-up (+ incremental rebalance from measured kernel times, L18 SIV.D)
     rebalanced = 0
     for i in range(max(3, args.warmup)):
@@ -273,13 +276,13 @@ def main():
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    with ClockSampler(local) as clk:
-        for k in range(K):
-            flush.zero_()                                     # L2 flush, outside the step events
-            ev[k][0].record(stream)
-            step()
-            ev[k][1].record(stream)
-        torch.cuda.synchronize()
+    for k in range(K):
+        flush.zero_()                                         # L2 flush, outside the step events
+        ev[k][0].record(stream)
+        step()
+        ev[k][1].record(stream)
+    torch.cuda.synchronize()
+    clk.__exit__(None, None, None)
     if world > 1:
         dist.barrier()
     step_ms = [a.elapsed_time(b) for a, b in ev]
