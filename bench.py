@@ -60,6 +60,8 @@ def parse():
     ap.add_argument("--no-sweep", action="store_true", help="skip the S sweep (C2, N=1)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="oracle sample budget")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="gloo + AFMM_BENCH_SAME_DEVICE=1 exercises the N>1 flow on one GPU (testing only)")
     return ap.parse_args()
 
 
@@ -212,9 +214,14 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if os.environ.get("AFMM_BENCH_SAME_DEVICE") == "1":     # functional test of the N>1 flow on one GPU
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group("gloo")
     dev = torch.device("cuda", local)
     # a dedicated (non-default) stream shared by torch and the library, so the
     # step events, the NCCL calls and the kernels are ordered on one stream
