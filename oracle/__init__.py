@@ -61,6 +61,12 @@ def _L():
                                    i64, p, p, p, p, p, p]
         lib.oracle_interactions.restype = None
         lib.oracle_interactions.argtypes = [i64, p, p, p, p]
+        lib.oracle_tree_enforce.restype = p
+        lib.oracle_tree_enforce.argtypes = [p, i64, p, p, p, C.c_int]
+        lib.oracle_kick.restype = None
+        lib.oracle_kick.argtypes = [i64, p, p, p, p, p, p, C.c_double]
+        lib.oracle_drift.restype = None
+        lib.oracle_drift.argtypes = [i64, p, p, p, p, p, p, C.c_double]
         lib.oracle_partition_literal.restype = None
         lib.oracle_partition_literal.argtypes = [i64, p, C.c_int, p, p]
         _lib = lib
@@ -76,56 +82,92 @@ def _c(a, dt):
 
 
 class Tree:
-    """Adaptive octree + U-list of the oracle (fields are numpy copies)."""
+    """Adaptive octree + U-list of the oracle (fields are numpy copies).
 
-    def __init__(self, x, y, z, S, domain=None, ulist=True):
-        x, y, z = (_c(v, np.float32) for v in (x, y, z))
-        n = x.shape[0]
+    Keeps its C handle so that ``enforce`` (Enforce_S, L20 SVI.A) can walk it."""
+
+    def __init__(self, x=None, y=None, z=None, S=None, domain=None, ulist=True, _handle=None, _n=None):
         lib = _L()
-        lo = np.zeros(3)
-        k = 0
-        fixed = 0
-        if domain is not None:
-            lo = _c(domain[0], np.float64)
-            k = int(domain[1])
-            fixed = 1
-        h = lib.oracle_tree_build(n, _ptr(x), _ptr(y), _ptr(z), int(S), fixed, _ptr(lo), k)
+        if _handle is None:
+            x, y, z = (_c(v, np.float32) for v in (x, y, z))
+            n = x.shape[0]
+            lo = np.zeros(3)
+            k = 0
+            fixed = 0
+            if domain is not None:
+                lo = _c(domain[0], np.float64)
+                k = int(domain[1])
+                fixed = 1
+            h = lib.oracle_tree_build(n, _ptr(x), _ptr(y), _ptr(z), int(S), fixed, _ptr(lo), k)
+            if not h:
+                raise ValueError("oracle_tree_build failed")
+        else:
+            h, n = _handle, _n
+        self._h = h
+        self._fill(lib, h, n, int(S), ulist)
+
+    def _fill(self, lib, h, n, S, ulist):
+        L = lib.oracle_tree_nleaves(h)
+        self.n, self.S, self.L = n, S, int(L)
+        self.perm = np.empty(n, np.int32)
+        self.leaf_start = np.empty(L, np.int32)
+        self.leaf_count = np.empty(L, np.int32)
+        self.leaf_level = np.empty(L, np.int32)
+        self.leaf_prefix = np.empty(L, np.uint64)
+        lo_out = np.empty(3)
+        k_out = np.zeros(1, np.int32)
+        lib.oracle_tree_get(h, _ptr(self.perm), _ptr(self.leaf_start), _ptr(self.leaf_count),
+                            _ptr(self.leaf_level), _ptr(self.leaf_prefix), _ptr(lo_out), _ptr(k_out))
+        self.lo, self.k = lo_out, int(k_out[0])
+        nn = lib.oracle_tree_nnodes(h)
+        self.node_level = np.empty(nn, np.int32)
+        self.node_prefix = np.empty(nn, np.uint64)
+        self.node_b = np.empty(nn, np.int64)
+        self.node_e = np.empty(nn, np.int64)
+        self.node_is_leaf = np.empty(nn, np.int32)
+        lib.oracle_tree_nodes(h, _ptr(self.node_level), _ptr(self.node_prefix), _ptr(self.node_b),
+                              _ptr(self.node_e), _ptr(self.node_is_leaf))
+        if ulist:
+            nnz = lib.oracle_ulist_build(h)
+            self.u_off = np.empty(L + 1, np.int64)
+            self.u_idx = np.empty(max(nnz, 1), np.int32)
+            lib.oracle_ulist_get(h, _ptr(self.u_off), _ptr(self.u_idx))
+            self.u_idx = self.u_idx[:nnz]
+
+    def enforce(self, x, y, z, S=None, ulist=True):
+        """Enforce_S (L20 SVI.A) for new positions of the same bodies -> new Tree.
+        x, y, z are given in THIS tree's body order (positions after a drift)."""
+        x, y, z = (_c(v, np.float32) for v in (x, y, z))
+        S = self.S if S is None else int(S)
+        h = _L().oracle_tree_enforce(self._h, x.shape[0], _ptr(x), _ptr(y), _ptr(z), S)
         if not h:
-            raise ValueError("oracle_tree_build failed")
-        try:
-            L = lib.oracle_tree_nleaves(h)
-            self.n, self.S, self.L = n, int(S), int(L)
-            self.perm = np.empty(n, np.int32)
-            self.leaf_start = np.empty(L, np.int32)
-            self.leaf_count = np.empty(L, np.int32)
-            self.leaf_level = np.empty(L, np.int32)
-            self.leaf_prefix = np.empty(L, np.uint64)
-            lo_out = np.empty(3)
-            k_out = np.zeros(1, np.int32)
-            lib.oracle_tree_get(h, _ptr(self.perm), _ptr(self.leaf_start), _ptr(self.leaf_count),
-                                _ptr(self.leaf_level), _ptr(self.leaf_prefix), _ptr(lo_out),
-                                _ptr(k_out))
-            self.lo, self.k = lo_out, int(k_out[0])
-            nn = lib.oracle_tree_nnodes(h)
-            self.node_level = np.empty(nn, np.int32)
-            self.node_prefix = np.empty(nn, np.uint64)
-            self.node_b = np.empty(nn, np.int64)
-            self.node_e = np.empty(nn, np.int64)
-            self.node_is_leaf = np.empty(nn, np.int32)
-            lib.oracle_tree_nodes(h, _ptr(self.node_level), _ptr(self.node_prefix),
-                                  _ptr(self.node_b), _ptr(self.node_e), _ptr(self.node_is_leaf))
-            if ulist:
-                nnz = lib.oracle_ulist_build(h)
-                self.u_off = np.empty(L + 1, np.int64)
-                self.u_idx = np.empty(max(nnz, 1), np.int32)
-                lib.oracle_ulist_get(h, _ptr(self.u_off), _ptr(self.u_idx))
-                self.u_idx = self.u_idx[:nnz]
-        finally:
-            lib.oracle_tree_free(h)
+            raise ValueError("oracle_tree_enforce failed")
+        return Tree(S=S, ulist=ulist, _handle=h, _n=x.shape[0])
+
+    def __del__(self):
+        if getattr(self, "_h", None) and _lib is not None:
+            _lib.oracle_tree_free(self._h)
+            self._h = None
 
     def sorted_bodies(self, *arrs):
-        """Permute original-order arrays into tree (Morton) order."""
+        """Permute input-order arrays into tree (Morton) order."""
         return tuple(_c(a, np.float32)[self.perm] for a in arrs)
+
+
+def kick(vx, vy, vz, ax, ay, az, h):
+    """Leapfrog kick v <- v + h a (fp64 arithmetic on fp32 state, one rounding)."""
+    v = [np.array(a, np.float32) for a in (vx, vy, vz)]
+    a = [_c(t, np.float32) for t in (ax, ay, az)]
+    _L().oracle_kick(v[0].shape[0], *[_ptr(t) for t in v], *[_ptr(t) for t in a], float(h))
+    return tuple(v)
+
+
+def drift(x, y, z, vx, vy, vz, dt):
+    """Leapfrog drift x <- x + dt v (fp64 arithmetic on fp32 state, one rounding)."""
+    p = [np.array(a, np.float32) for a in (x, y, z)]
+    v = [_c(t, np.float32) for t in (vx, vy, vz)]
+    _L().oracle_drift(p[0].shape[0], *[_ptr(t) for t in p], *[_ptr(t) for t in v], float(dt))
+    return tuple(p)
 
 
 def domain(x, y, z):

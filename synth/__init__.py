@@ -126,6 +126,65 @@ def colliding(n: int, seed: int):
     return _as_f32_bodies(np.concatenate([pa, pb]), n)
 
 
+def _plummer_velocities(pos: np.ndarray, mass: float, seed: int, stream: int) -> np.ndarray:
+    """Isotropic Plummer velocities (a = 1, G = 1, sphere mass `mass`): speed
+    v = q * v_esc(r), v_esc = sqrt(2 mass) (1 + r^2)^(-1/4), q drawn by rejection
+    from g(q) = q^2 (1 - q^2)^(7/2) (Aarseth-Henon-Wielen).  Draw index for body
+    i, attempt a, component c: (i*64 + a)*4 + c."""
+    n = pos.shape[0]
+    idx = np.arange(n, dtype=np.uint64)
+    q = np.full(n, 0.5)
+    done = np.zeros(n, dtype=bool)
+    for a in range(64):
+        todo = np.nonzero(~done)[0]
+        if todo.size == 0:
+            break
+        base = (idx[todo] * np.uint64(64) + np.uint64(a)) * np.uint64(4)
+        qq = uniform01(seed, stream, base)
+        gg = 0.1 * uniform01(seed, stream, base + np.uint64(1))
+        ok = gg < qq * qq * (1.0 - qq * qq) ** 3.5
+        q[todo[ok]] = qq[ok]
+        done[todo[ok]] = True
+    base = idx * np.uint64(64 * 4) + np.uint64(64 * 4 - 2)      # direction draws (disjoint indices)
+    ct = 2.0 * uniform01(seed, stream + 100, base) - 1.0
+    ph = 2.0 * np.pi * uniform01(seed, stream + 100, base + np.uint64(1))
+    r2 = (pos ** 2).sum(1)
+    v = q * np.sqrt(2.0 * mass) * (1.0 + r2) ** -0.25
+    st = np.sqrt(np.maximum(0.0, 1.0 - ct * ct))
+    return np.stack([v * st * np.cos(ph), v * st * np.sin(ph), v * ct], 1)
+
+
+COLLIDE_BULK = ((0.5, 0.0, 0.0), (-0.5, 0.0, 0.0))
+
+
+def colliding_with_velocities(n: int, seed: int):
+    """C5 initial state: the colliding pair of `colliding` plus velocities --
+    bulk (+0.5, 0, 0) for the sphere at x = -5 and (-0.5, 0, 0) for the one at
+    x = +5 (approach along x), plus isotropic Plummer internal velocities.
+    Returns fp32 (x, y, z, m, vx, vy, vz)."""
+    na = n // 2
+    pa = _plummer_positions(na, seed, 3)
+    pb = _plummer_positions(n - na, seed, 4)
+    va = _plummer_velocities(pa, na / n, seed, 5) + np.array(COLLIDE_BULK[0])
+    vb = _plummer_velocities(pb, (n - na) / n, seed, 6) + np.array(COLLIDE_BULK[1])
+    pos = np.concatenate([pa + np.array(COLLIDE_CENTRES[0]), pb + np.array(COLLIDE_CENTRES[1])])
+    vel = np.concatenate([va, vb])
+    x, y, z, m = _as_f32_bodies(pos, n)
+    return x, y, z, m, vel[:, 0].astype(np.float32), vel[:, 1].astype(np.float32), vel[:, 2].astype(np.float32)
+
+
+def c5_domain(x, y, z):
+    """Fixed C5 domain (reading R9, "initially contained within 1/64 th
+    of the simulation space"): the initial power-of-two cube (lo, k) grown 4x per
+    axis (side 2^(k+2)) and centred on the initial cube.  Returns (lo[3], k)."""
+    P = np.stack([x, y, z], 1).astype(np.float64)
+    lo = P.min(0)
+    ext = (P.max(0) - lo).max()
+    k = int(np.frexp(ext)[1]) if ext > 0 else 0
+    side = 2.0 ** k
+    return lo - 1.5 * side, k + 2
+
+
 def lattice(M: int):
     """One body at each cell centre of an M^3 grid on [0,1)^3 (U-list closed-form pin)."""
     c = (np.arange(M, dtype=np.float64) + 0.5) / M
