@@ -85,10 +85,15 @@ _sig("afmm_interactions", _i, _i, _p, _p, _p, _p)
 _sig("afmm_partition_literal", _i, _i, _p, _i, _p)
 _sig("afmm_partition_weighted", _i, _i, _p, _i, _p)
 _sig("afmm_partition_rebalance", _i, _i, _p, _p, _i, _p, _p, _d, _p, C.POINTER(_i))
+_sig("afmm_cost_fit", _i, _i, _p, _p, _p)
+_sig("afmm_p2p_set_cost_coef", _i, _p, _p)
+_sig("afmm_kick", _i, _ll, _p, _p, _p, _p, _p, _p, C.c_float, _p)
+_sig("afmm_drift", _i, _ll, _p, _p, _p, _p, _p, _p, C.c_float, _p)
 _sig("afmm_fp32_peak", _i, _i, C.POINTER(_d), C.POINTER(_d), C.POINTER(_d))
 _sig("afmm_version", C.c_char_p)
 _sig("afmm_tree_create", _i, _i, _p, C.POINTER(_p))
 _sig("afmm_tree_build", _i, _p, _ll, _p, _p, _p, _i, _i, _p, _i)
+_sig("afmm_tree_enforce", _i, _p, _ll, _p, _p, _p, _i)
 _sig("afmm_tree_info", _i, _p, C.POINTER(_i), C.POINTER(_ll), _p, C.POINTER(_i), C.POINTER(_i),
      C.POINTER(_ll))
 _sig("afmm_tree_copy_out", _i, _p, _p, _p, _p, _p, _p, _p, _p)
@@ -105,8 +110,9 @@ EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
             "afmm_p2p_kernel_times",
             "afmm_p2p_destroy", "afmm_p2p_last_error", "afmm_interactions",
             "afmm_partition_literal", "afmm_partition_weighted", "afmm_partition_rebalance",
+            "afmm_cost_fit", "afmm_p2p_set_cost_coef", "afmm_kick", "afmm_drift",
             "afmm_fp32_peak", "afmm_version",
-            "afmm_tree_create", "afmm_tree_build", "afmm_tree_info", "afmm_tree_copy_out",
+            "afmm_tree_create", "afmm_tree_build", "afmm_tree_enforce", "afmm_tree_info", "afmm_tree_copy_out",
             "afmm_tree_gather", "afmm_tree_scatter", "afmm_tree_destroy", "afmm_tree_last_error"]
 
 
@@ -180,6 +186,33 @@ def partition_rebalance(leaf_count, I, cur_split, rank_ms, threshold=0.02):
     if st:
         raise AfmmError(st, "afmm_partition_rebalance")
     return out, bool(ch.value)
+
+
+def cost_fit(bucket_inter, rank_ms):
+    """Per-bucket cost coefficients (afmm_cost_fit); bucket_inter: [G, 8]."""
+    B = _np(bucket_inter, np.float64).reshape(-1, N_BUCKETS)
+    r = _np(rank_ms, np.float64)
+    out = np.empty(N_BUCKETS, np.float64)
+    st = _lib.afmm_cost_fit(B.shape[0], _ptr(B), _ptr(r), _ptr(out))
+    if st:
+        raise AfmmError(st, "afmm_cost_fit")
+    return out
+
+
+def kick(vx, vy, vz, ax, ay, az, h, stream=None):
+    """Leapfrog kick v <- v + h a on device tensors (afmm_kick)."""
+    st = _lib.afmm_kick(int(vx.shape[0]), _ptr(vx), _ptr(vy), _ptr(vz), _ptr(ax), _ptr(ay), _ptr(az),
+                        float(h), stream)
+    if st:
+        raise AfmmError(st, "afmm_kick")
+
+
+def drift(x, y, z, vx, vy, vz, dt, stream=None):
+    """Leapfrog drift x <- x + dt v on device tensors (afmm_drift)."""
+    st = _lib.afmm_drift(int(x.shape[0]), _ptr(x), _ptr(y), _ptr(z), _ptr(vx), _ptr(vy), _ptr(vz),
+                         float(dt), stream)
+    if st:
+        raise AfmmError(st, "afmm_drift")
 
 
 def fp32_peak(device: int = 0):
@@ -259,6 +292,10 @@ class P2P:
     def set_partition(self, leaf_split=None):
         ls = None if leaf_split is None else _np(leaf_split, np.int64)
         self._check(_lib.afmm_p2p_set_partition(self._h, _ptr(ls)), "afmm_p2p_set_partition")
+
+    def set_cost_coef(self, coef=None):
+        c = None if coef is None else _np(coef, np.float64)
+        self._check(_lib.afmm_p2p_set_cost_coef(self._h, _ptr(c)), "afmm_p2p_set_cost_coef")
 
     def get_partition(self):
         ls = np.empty(self.world + 1, np.int64)
@@ -341,6 +378,12 @@ class GpuTree:
             fixed = 1
         self._check(_lib.afmm_tree_build(self._h, int(x.shape[0]), _ptr(x), _ptr(y), _ptr(z), int(S),
                                          fixed, _ptr(lo), k), "afmm_tree_build")
+        return self.info()
+
+    def enforce(self, x, y, z, S):
+        """Enforce_S on the last build for moved bodies (afmm_tree_enforce)."""
+        self._check(_lib.afmm_tree_enforce(self._h, int(x.shape[0]), _ptr(x), _ptr(y), _ptr(z), int(S)),
+                    "afmm_tree_enforce")
         return self.info()
 
     def info(self):

@@ -52,6 +52,8 @@ struct afmm_p2p {
 
     // partition
     bool user_partition = false;
+    bool have_coef = false;                 // per-bucket cost coefficients for set_tree's cut
+    double coef[8] = {1, 1, 1, 1, 1, 1, 1, 1};
     std::vector<long long> leaf_split, body_split;
 
     // this rank's work list
@@ -411,7 +413,13 @@ extern "C" afmm_status afmm_p2p_set_tree(afmm_p2p *h, int n_leaves, const int *l
     if (!h->user_partition || (long long)h->leaf_split.size() != W + 1 || h->leaf_split[W] != n_leaves) {
         h->user_partition = false;
         h->leaf_split.assign(W + 1, 0);
-        afmm_partition_literal(n_leaves, h->I.data(), W, h->leaf_split.data());
+        if (h->have_coef && W > 1) {        // incremental adjustment carried across trees (L18 SIV.D)
+            std::vector<double> w(n_leaves);
+            for (int t = 0; t < n_leaves; ++t) w[t] = (double)h->I[t] * h->coef[bucket_of(leaf_count[t])];
+            afmm_partition_weighted(n_leaves, w.data(), W, h->leaf_split.data());
+        } else {
+            afmm_partition_literal(n_leaves, h->I.data(), W, h->leaf_split.data());
+        }
     }
     compute_body_split(h);
     h->have_tree = true;
@@ -439,6 +447,19 @@ extern "C" afmm_status afmm_p2p_set_partition(afmm_p2p *h, const long long *leaf
     if (st) return st;
     compute_body_split(h);
     return build_worklist(h);
+}
+
+extern "C" afmm_status afmm_p2p_set_cost_coef(afmm_p2p *h, const double *coef) {
+    CHECK_HANDLE(h);
+    if (!coef) {
+        h->have_coef = false;
+        return AFMM_OK;
+    }
+    for (int b = 0; b < 8; ++b)
+        if (!(coef[b] > 0.0) || !std::isfinite(coef[b])) return fail(h, AFMM_EINVAL, "set_cost_coef: coef[%d] invalid", b);
+    std::copy(coef, coef + 8, h->coef);
+    h->have_coef = true;
+    return AFMM_OK;
 }
 
 extern "C" afmm_status afmm_p2p_get_partition(const afmm_p2p *h, long long *leaf_split,
@@ -478,6 +499,48 @@ static bool solve_small(std::vector<double> M, std::vector<double> b, int k, std
     return true;
 }
 
+// Per-bucket GPU cost coefficients (ms per interaction) from per-rank kernel
+// times: the paper's observational coefficient "dividing the maximum kernel
+// time by the total number of P2P operations" (L18 SIV.D) refined per
+// target-leaf-size bucket by ridge-regularised least squares over ranks:
+//   min sum_r (sum_b B_rb c_b - T_r)^2 + lam sum_b (Bsum_b/G)^2 (c_b - k0)^2,
+// k0 = sum T / sum I; coefficients kept >= 0.05 k0.
+extern "C" afmm_status afmm_cost_fit(int G, const double *bucket_inter, const double *rank_ms, double *coef) {
+    if (G < 1 || !bucket_inter || !rank_ms || !coef) return AFMM_EINVAL;
+    double Isum = 0, Tsum = 0;
+    for (int r = 0; r < G; ++r) {
+        if (!(rank_ms[r] >= 0.0) || !std::isfinite(rank_ms[r])) return AFMM_EINVAL;
+        Tsum += rank_ms[r];
+        for (int b = 0; b < 8; ++b) {
+            if (!(bucket_inter[r * 8 + b] >= 0.0)) return AFMM_EINVAL;
+            Isum += bucket_inter[r * 8 + b];
+        }
+    }
+    if (Isum <= 0 || Tsum <= 0) {
+        for (int b = 0; b < 8; ++b) coef[b] = 1.0;
+        return AFMM_OK;
+    }
+    const double k0 = Tsum / Isum;
+    std::vector<double> M(64, 0.0), rhs(8, 0.0), Bs(8, 0.0);
+    for (int r = 0; r < G; ++r)
+        for (int b = 0; b < 8; ++b) Bs[b] += bucket_inter[r * 8 + b];
+    const double lam = 0.1;
+    for (int r = 0; r < G; ++r)
+        for (int a = 0; a < 8; ++a) {
+            for (int b = 0; b < 8; ++b) M[a * 8 + b] += bucket_inter[r * 8 + a] * bucket_inter[r * 8 + b];
+            rhs[a] += bucket_inter[r * 8 + a] * rank_ms[r];
+        }
+    for (int b = 0; b < 8; ++b) {
+        const double wgt = lam * (Bs[b] / G) * (Bs[b] / G) + 1e-30;
+        M[b * 8 + b] += wgt;
+        rhs[b] += wgt * k0;
+    }
+    std::vector<double> c;
+    if (!solve_small(M, rhs, 8, c)) c.assign(8, k0);
+    for (int b = 0; b < 8; ++b) coef[b] = (c[b] > 0.05 * k0) ? c[b] : 0.05 * k0;
+    return AFMM_OK;
+}
+
 extern "C" afmm_status afmm_partition_rebalance(int n_leaves, const int *leaf_count, const long long *I,
                                                 int G, const long long *cur_split, const double *rank_ms,
                                                 double threshold, long long *new_split, int *changed) {
@@ -492,35 +555,16 @@ extern "C" afmm_status afmm_partition_rebalance(int n_leaves, const int *leaf_co
     if (G == 1) return AFMM_OK;
     // per-rank bucket interaction counts for the current cut
     std::vector<double> B((size_t)G * 8, 0.0);
-    double Isum = 0, Tsum = 0;
+    double Tsum = 0;
     for (int r = 0; r < G; ++r) {
         for (long long t = cur_split[r]; t < cur_split[r + 1]; ++t)
             B[r * 8 + bucket_of(leaf_count[t])] += (double)I[t];
         Tsum += rank_ms[r];
     }
-    for (double v : B) Isum += v;
-    if (Isum <= 0 || Tsum <= 0) return AFMM_OK;
-    const double k0 = Tsum / Isum;     // the paper's GPU coefficient over all GPUs (L18 SIV.D)
-    // ridge-regularised least squares for per-bucket coefficients around k0:
-    // min sum_r (sum_b B_rb c_b - T_r)^2 + lam * sum_b (Bsum_b/G)^2 (c_b - k0)^2
-    std::vector<double> M(64, 0.0), rhs(8, 0.0), Bs(8, 0.0);
-    for (int r = 0; r < G; ++r)
-        for (int b = 0; b < 8; ++b) Bs[b] += B[r * 8 + b];
-    const double lam = 0.1;
-    for (int r = 0; r < G; ++r)
-        for (int a = 0; a < 8; ++a) {
-            for (int b = 0; b < 8; ++b) M[a * 8 + b] += B[r * 8 + a] * B[r * 8 + b];
-            rhs[a] += B[r * 8 + a] * rank_ms[r];
-        }
-    for (int b = 0; b < 8; ++b) {
-        const double wgt = lam * (Bs[b] / G) * (Bs[b] / G) + 1e-30;
-        M[b * 8 + b] += wgt;
-        rhs[b] += wgt * k0;
-    }
-    std::vector<double> coef;
-    if (!solve_small(M, rhs, 8, coef)) coef.assign(8, k0);
-    for (double &c : coef)
-        if (!(c > 0.05 * k0)) c = 0.05 * k0;      // keep weights positive
+    if (Tsum <= 0) return AFMM_OK;
+    double coef[8];
+    afmm_status fst = afmm_cost_fit(G, B.data(), rank_ms, coef);
+    if (fst) return fst;
     std::vector<double> w(n_leaves);
     for (int t = 0; t < n_leaves; ++t) w[t] = (double)I[t] * coef[bucket_of(leaf_count[t])];
     std::vector<long long> split(G + 1);

@@ -104,16 +104,41 @@ struct Nodes {
     unsigned long long *prefix;
 };
 
-// For each node of the current level: split if > S bodies and level < 21.
+// Internal nodes of the previous build, for Enforce_S: per level, node prefixes
+// in ascending order ([base[l], base[l+1])) and their child counts.
+struct PrevTree {
+    const unsigned long long *prefix;
+    const int *nchild;
+    const long long *base;      // device, levels + 1 entries
+    int levels;                 // 0: no previous tree (fresh build)
+};
+
+__device__ __forceinline__ bool prev_internal(const PrevTree &pv, int lev, unsigned long long prefix) {
+    if (lev >= pv.levels) return false;
+    long long lo = pv.base[lev], hi = pv.base[lev + 1];
+    while (lo < hi) {
+        const long long mid = lo + ((hi - lo) >> 1);
+        if (pv.prefix[mid] < prefix) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo < pv.base[lev + 1] && pv.prefix[lo] == prefix && pv.nchild[lo] > 0;
+}
+
+// For each node of the current level: split if > S bodies and level < 21
+// (L10 SI.B).  Enforce_S (L20 SVI.A; pv.levels > 0) additionally keeps a node
+// with exactly S bodies split when it was a parent before: Collapse applies only
+// to parents with FEWER than S bodies, PushDown only to leaves with MORE than S.
 // Child ranges by binary search on the octant digit inside [b, e).
 __global__ void split_count_kernel(int m, int base, Nodes nd, const unsigned long long *__restrict__ keys,
-                                   int S, int *__restrict__ cb, int *__restrict__ nc) {
+                                   int S, PrevTree pv, int *__restrict__ cb, int *__restrict__ nc) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= m) return;
     const int id = base + i;
     const int b = nd.b[id], e = nd.e[id], lev = nd.level[id];
     int cnt = 0;
-    if (e - b > S && lev < kMaxLevel) {
+    const bool split = lev < kMaxLevel &&
+                       (e - b > S || (e - b == S && pv.levels > 0 && prev_internal(pv, lev, nd.prefix[id])));
+    if (split) {
         const int shift = 3 * (kMaxLevel - 1 - lev);
         int bound[9];
         bound[0] = b;
@@ -275,6 +300,13 @@ struct afmm_tree {
     long long *u_off = nullptr;
     int *u_idx = nullptr;
     std::vector<void *> owned;
+    // node arrays of the last build (level-major, prefixes ascending per level):
+    // the "previous tree" of the next afmm_tree_enforce
+    unsigned long long *pv_prefix = nullptr;
+    int *pv_nchild = nullptr;
+    long long *pv_base = nullptr;
+    size_t pv_cap = 0;
+    int pv_levels = 0;
 };
 
 namespace {
@@ -368,15 +400,17 @@ extern "C" void afmm_tree_destroy(afmm_tree *t) {
     cudaSetDevice(t->device);
     if (t->stream) cudaStreamSynchronize(t->stream);
     free_all(t);
+    cudaFree(t->pv_prefix);
+    cudaFree(t->pv_nchild);
+    cudaFree(t->pv_base);
     if (t->own_stream && t->stream) cudaStreamDestroy(t->stream);
     delete t;
 }
 
 extern "C" const char *afmm_tree_last_error(const afmm_tree *t) { return t ? t->err.c_str() : "null handle"; }
 
-extern "C" afmm_status afmm_tree_build(afmm_tree *t, long long n, const float *x, const float *y,
-                                       const float *z, int S, int fixed_domain, const double *lo_in,
-                                       int k_in) {
+static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const float *y, const float *z,
+                              int S, int fixed_domain, const double *lo_in, int k_in, bool enforce) {
     if (!t) return AFMM_EINVAL;
     if (t->poisoned) return AFMM_ESTATE;
     if (n < 1 || n >= (1LL << 31)) return tfail(t, AFMM_EINVAL, "tree_build: n=%lld out of range", n);
@@ -465,6 +499,8 @@ extern "C" afmm_status afmm_tree_build(afmm_tree *t, long long n, const float *x
         TCU(t, cudaMemcpyAsync(nd.prefix, &p0, sizeof(p0), cudaMemcpyHostToDevice, st));
         TCU(t, cudaStreamSynchronize(st));
     }
+    PrevTree pv{t->pv_prefix, t->pv_nchild, t->pv_base, enforce ? t->pv_levels : 0};
+    std::vector<long long> lvl_base;
     long long base = 0, m = 1;     // current level occupies [base, base+m)
     int level = 0;
     int *cb = nullptr, *nc = nullptr, *off = nullptr;
@@ -485,7 +521,7 @@ extern "C" afmm_status afmm_tree_build(afmm_tree *t, long long n, const float *x
                 scan_tmp_bytes = need;
             }
         }
-        split_count_kernel<<<grid_for(m, TH), TH, 0, st>>>((int)m, (int)base, nd, t->keys_sorted, S, cb, nc);
+        split_count_kernel<<<grid_for(m, TH), TH, 0, st>>>((int)m, (int)base, nd, t->keys_sorted, S, pv, cb, nc);
         TCU(t, cudaGetLastError());
         TCU(t, cudaMemsetAsync(nc + m, 0, sizeof(int), st));
         size_t sb = scan_tmp_bytes;
@@ -510,12 +546,31 @@ extern "C" afmm_status afmm_tree_build(afmm_tree *t, long long n, const float *x
         split_write_kernel<<<grid_for(m, TH), TH, 0, st>>>((int)m, (int)base, (int)next_base, nd, cb, nc, off);
         TCU(t, cudaGetLastError());
         t->max_level = level;
+        lvl_base.push_back(base);
         base = next_base;
         m = total;
         ++level;
     }
     const long long nn = base;     // total nodes
     t->n_nodes = nn;
+    lvl_base.push_back(nn);
+    // keep this tree's nodes as the "previous tree" of the next Enforce_S
+    if ((size_t)nn > t->pv_cap) {
+        cudaFree(t->pv_prefix);
+        cudaFree(t->pv_nchild);
+        t->pv_prefix = nullptr;
+        t->pv_nchild = nullptr;
+        t->pv_cap = 0;
+        TCU(t, cudaMalloc(&t->pv_prefix, (size_t)nn * sizeof(unsigned long long)));
+        TCU(t, cudaMalloc(&t->pv_nchild, (size_t)nn * sizeof(int)));
+        t->pv_cap = (size_t)nn;
+    }
+    if (!t->pv_base) TCU(t, cudaMalloc(&t->pv_base, (kMaxLevel + 2) * sizeof(long long)));
+    TCU(t, cudaMemcpyAsync(t->pv_prefix, nd.prefix, nn * sizeof(unsigned long long), cudaMemcpyDeviceToDevice, st));
+    TCU(t, cudaMemcpyAsync(t->pv_nchild, nd.nchild, nn * sizeof(int), cudaMemcpyDeviceToDevice, st));
+    TCU(t, cudaMemcpyAsync(t->pv_base, lvl_base.data(), lvl_base.size() * sizeof(long long),
+                           cudaMemcpyHostToDevice, st));
+    t->pv_levels = (int)lvl_base.size() - 1;
 
     // 5. leaves in Morton order: flag first bodies, scan
     int *flag, *leaf_at, *node_leaf;
@@ -570,6 +625,25 @@ extern "C" afmm_status afmm_tree_build(afmm_tree *t, long long n, const float *x
     t->n = n;
     t->built = true;
     return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_tree_build(afmm_tree *t, long long n, const float *x, const float *y,
+                                       const float *z, int S, int fixed_domain, const double *lo_in,
+                                       int k_in) {
+    return build_impl(t, n, x, y, z, S, fixed_domain, lo_in, k_in, false);
+}
+
+// Enforce_S (PAPER L20 SVI.A): the tree the last build becomes after its bodies
+// moved -- same domain; a node splits iff it holds > S bodies, or exactly S and
+// it was a parent in the previous tree (see split_count_kernel).
+extern "C" afmm_status afmm_tree_enforce(afmm_tree *t, long long n, const float *x, const float *y,
+                                         const float *z, int S) {
+    if (!t) return AFMM_EINVAL;
+    if (t->poisoned) return AFMM_ESTATE;
+    if (!t->built || t->pv_levels < 1) return tfail(t, AFMM_ESTATE, "tree_enforce: no previous tree");
+    if (n != t->n) return tfail(t, AFMM_EINVAL, "tree_enforce: n=%lld differs from the previous tree (%lld)", n, t->n);
+    const double lo[3] = {t->lo[0], t->lo[1], t->lo[2]};
+    return build_impl(t, n, x, y, z, S, 1, lo, t->k, true);
 }
 
 extern "C" afmm_status afmm_tree_info(const afmm_tree *t, int *n_leaves, long long *nnz, double *lo,

@@ -1,0 +1,143 @@
+"""C5 dynamic workload (BASELINE configs[4]): kick-drift-
+kick leapfrog steps with Enforce_S tree maintenance and the incremental
+partition rebalance, all through the C ABI (orchestration only -- every
+arithmetic step runs in libafmm_p2p.so kernels).
+
+Per time step (PAPER L16 SIII.D "the particle positions are updated ... and
+then any tree optimizations are done to improve the run on the next time step";
+L20 SVI.A Enforce_S; L18 SIV.D observational coefficients):
+  1. kick(dt/2) with the current accelerations      (afmm_kick, own slice)
+  2. drift(dt)                                        (afmm_drift, own slice)
+  3. N > 1: replicate positions and velocities        (allgatherv of slices)
+  4. Enforce_S on the moved bodies (fixed domain)     (afmm_tree_enforce)
+  5. carry the state into the new tree order          (afmm_tree_gather)
+  6. set_bodies / set_tree; N > 1: the cut uses the per-bucket cost
+     coefficients fitted to the previous step's kernel times (afmm_cost_fit)
+  7. near-field P2P                                    (afmm_p2p_eval)
+  8. kick(dt/2) with the new accelerations
+
+Note: the far field is out of scope (S10), so bodies move under the
+near-field force only; C5 is a dynamic load for the GPU path, not a physical
+simulation.
+"""
+from __future__ import annotations
+
+import time
+
+import numpy as np
+import torch
+
+from . import GpuTree, P2P, cost_fit, drift, kick
+
+
+class TimeLoop:
+    def __init__(self, x, y, z, m, vx, vy, vz, S, eps2, dt, domain, device=0, rank=0, world=1, G=1.0):
+        self.dev = torch.device("cuda", device)
+        self.stream = torch.cuda.Stream(self.dev)
+        torch.cuda.set_stream(self.stream)
+        self.S, self.eps2, self.dt, self.rank, self.world = int(S), float(eps2), float(dt), rank, world
+        self.n = int(x.shape[0])
+        n = self.n
+        # state in tree order: rows x, y, z, m, vx, vy, vz
+        src = torch.stack([torch.as_tensor(np.asarray(v, np.float32)) for v in (x, y, z, m, vx, vy, vz)]).to(self.dev)
+        self.state = torch.empty((7, n), device=self.dev)
+        self.tmp = torch.empty((7, n), device=self.dev)
+        self.acc = torch.zeros((4, n), device=self.dev)        # ax, ay, az, phi
+        self.tree = GpuTree(device, stream=self.stream.cuda_stream)
+        self.tree.build(src[0], src[1], src[2], self.S, domain=domain)
+        for a in range(7):
+            self.tree.gather(src[a], self.state[a])
+        self.h = P2P(device=device, rank=rank, world=world, G=G, eps2=eps2, stream=self.stream.cuda_stream)
+        self.step_no = 0
+        self.log = []
+        self._load_tree()
+        self._eval()
+
+    # ------------------------------------------------------------------ pieces
+    def _load_tree(self):
+        T = self.tree.copy_out(self.n)
+        self.T = T
+        s = self.state
+        self.h.set_bodies(s[0], s[1], s[2], s[3])
+        self.h.set_tree(T["leaf_start"], T["leaf_count"], T["u_off"], T["u_idx"])
+        self.body_split = self.h.get_partition()[1]
+
+    def _slice(self):
+        lo, hi = int(self.body_split[self.rank]), int(self.body_split[self.rank + 1])
+        return lo, hi
+
+    def _eval(self):
+        a = self.acc
+        self.h.eval(a[0], a[1], a[2], a[3])
+
+    def _kick(self):
+        lo, hi = self._slice()
+        s, a = self.state, self.acc
+        kick(s[4, lo:hi], s[5, lo:hi], s[6, lo:hi], a[0, lo:hi], a[1, lo:hi], a[2, lo:hi], 0.5 * self.dt,
+             self.stream.cuda_stream)
+
+    def _drift(self):
+        lo, hi = self._slice()
+        s = self.state
+        drift(s[0, lo:hi], s[1, lo:hi], s[2, lo:hi], s[4, lo:hi], s[5, lo:hi], s[6, lo:hi], self.dt,
+              self.stream.cuda_stream)
+
+    def _refit(self):
+        """N > 1: per-bucket coefficients from this step's kernel times (L18 SIV.D)."""
+        if self.world == 1:
+            return
+        import torch.distributed as dist
+        st = self.h.stats()
+        mine = torch.tensor([st["kernel_ms"]] + [float(v) for v in st["bucket_interactions"]],
+                            dtype=torch.float64, device=self.dev)
+        allv = [torch.zeros_like(mine) for _ in range(self.world)]
+        dist.all_gather(allv, mine)
+        arr = np.stack([v.cpu().numpy() for v in allv])
+        self.h.set_cost_coef(cost_fit(arr[:, 1:], arr[:, 0]))
+
+    # ------------------------------------------------------------------ one step
+    def step(self, hooks=None):
+        """One KDK step.  hooks (optional dict of callables) receive the state
+        for verification: 'pre_enforce'(x, y, z) with positions in the old tree
+        order, 'post_eval'(loop) after the new accelerations."""
+        ev = [torch.cuda.Event(enable_timing=True) for _ in range(6)]
+        t0 = time.perf_counter()
+        ev[0].record(self.stream)
+        self._refit()
+        self._kick()
+        self._drift()
+        if self.world > 1:
+            from . import dist as pdist
+            pdist.gather_slices([self.state[a] for a in (0, 1, 2, 4, 5, 6)], self.body_split)
+        ev[1].record(self.stream)
+        s = self.state
+        if hooks and "pre_enforce" in hooks:
+            torch.cuda.synchronize()
+            hooks["pre_enforce"](s[0].cpu().numpy(), s[1].cpu().numpy(), s[2].cpu().numpy())
+        self.tree.enforce(s[0], s[1], s[2], self.S)
+        for a in range(7):
+            self.tree.gather(s[a], self.tmp[a])
+        self.state, self.tmp = self.tmp, self.state
+        ev[2].record(self.stream)
+        self._load_tree()
+        ev[3].record(self.stream)
+        self._eval()
+        ev[4].record(self.stream)
+        self._kick()
+        ev[5].record(self.stream)
+        torch.cuda.synchronize()
+        st = self.h.stats()
+        rec = {"step": self.step_no, "n_leaves": self.T["n_leaves"], "interactions": st["interactions_total"],
+               "kernel_ms": st["kernel_ms"], "kick_drift_ms": ev[0].elapsed_time(ev[1]),
+               "enforce_ms": ev[1].elapsed_time(ev[2]), "set_tree_ms": ev[2].elapsed_time(ev[3]),
+               "eval_ms": ev[3].elapsed_time(ev[4]), "step_ms": 1e3 * (time.perf_counter() - t0),
+               "leaf_split": self.h.get_partition()[0].tolist()}
+        self.log.append(rec)
+        self.step_no += 1
+        if hooks and "post_eval" in hooks:
+            hooks["post_eval"](self)
+        return rec
+
+    def close(self):
+        self.h.close()
+        self.tree.close()
