@@ -307,6 +307,11 @@ struct afmm_tree {
     long long *pv_base = nullptr;
     size_t pv_cap = 0;
     int pv_levels = 0;
+    // workspace arena: one grow-only device buffer per call site (no cudaMalloc
+    // in steady state -- the tree is rebuilt every time step in C5)
+    std::vector<void *> ws_ptr;
+    std::vector<size_t> ws_cap;
+    size_t node_cap = 1024;
 };
 
 namespace {
@@ -334,8 +339,9 @@ afmm_status tfail(afmm_tree *t, afmm_status st, const char *fmt, ...) {
     } while (0)
 
 void free_all(afmm_tree *t) {
-    for (void *p : t->owned) cudaFree(p);
-    t->owned.clear();
+    for (void *p : t->ws_ptr) cudaFree(p);
+    t->ws_ptr.clear();
+    t->ws_cap.clear();
     t->perm = nullptr;
     t->keys_sorted = nullptr;
     t->ls = t->lc = t->ll = nullptr;
@@ -344,29 +350,38 @@ void free_all(afmm_tree *t) {
     t->u_idx = nullptr;
 }
 
+// grow-only workspace buffer for call site `slot` (contents not preserved on growth)
 template <typename T>
-afmm_status dalloc(afmm_tree *t, T **p, size_t count) {
-    void *q = nullptr;
-    TCU(t, cudaMalloc(&q, std::max<size_t>(count, 1) * sizeof(T)));
-    t->owned.push_back(q);
-    *p = static_cast<T *>(q);
+afmm_status wsalloc(afmm_tree *t, int slot, T **p, size_t count) {
+    const size_t bytes = std::max<size_t>(count, 1) * sizeof(T);
+    if ((size_t)slot >= t->ws_ptr.size()) {
+        t->ws_ptr.resize(slot + 1, nullptr);
+        t->ws_cap.resize(slot + 1, 0);
+    }
+    if (t->ws_cap[slot] < bytes) {
+        cudaFree(t->ws_ptr[slot]);
+        t->ws_ptr[slot] = nullptr;
+        t->ws_cap[slot] = 0;
+        const size_t want = bytes + bytes / 4;
+        TCU(t, cudaMalloc(&t->ws_ptr[slot], want));
+        t->ws_cap[slot] = want;
+    }
+    *p = static_cast<T *>(t->ws_ptr[slot]);
     return AFMM_OK;
 }
 
-// scoped temporaries
-struct Tmp {
-    std::vector<void *> v;
-    ~Tmp() {
-        for (void *p : v) cudaFree(p);
-    }
+enum Slot {
+    kPart, kKeys, kIdx, kKeysSorted, kPerm, kSortTmp, kNodeA, kNodeB = kNodeA + 6, kCb = kNodeB + 6, kNc, kOff,
+    kScanTmp, kFlag, kLeafAt, kNodeLeaf, kScan2, kLs, kLc, kLl, kLp, kLeafNode, kCounts, kUoff, kScan3, kUidx
 };
-template <typename T>
-afmm_status talloc(afmm_tree *t, Tmp &tmp, T **p, size_t count) {
-    void *q = nullptr;
-    TCU(t, cudaMalloc(&q, std::max<size_t>(count, 1) * sizeof(T)));
-    tmp.v.push_back(q);
-    *p = static_cast<T *>(q);
-    return AFMM_OK;
+
+__global__ void root_kernel(Nodes nd, int n) {
+    nd.b[0] = 0;
+    nd.e[0] = n;
+    nd.first_child[0] = -1;
+    nd.nchild[0] = 0;
+    nd.level[0] = 0;
+    nd.prefix[0] = 0ull;
 }
 
 }  // namespace
@@ -420,10 +435,8 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
                          !std::isfinite(lo_in[2]) || k_in < -1000 || k_in > 1000))
         return tfail(t, AFMM_EINVAL, "tree_build: bad fixed domain");
     TCU(t, cudaSetDevice(t->device));
-    free_all(t);
     t->built = false;
     cudaStream_t st = t->stream;
-    Tmp tmp;
     const int TH = 256;
 
     // 1. domain (reading R6): lo = min, side = smallest power of two > max extent
@@ -433,7 +446,7 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     } else {
         const int g = 296;
         float *part;
-        if (afmm_status s = talloc(t, tmp, &part, (size_t)g * 6)) return s;
+        if (afmm_status s = wsalloc(t, kPart, &part, (size_t)g * 6)) return s;
         minmax_kernel<<<g, TH, 0, st>>>(n, x, y, z, part);
         TCU(t, cudaGetLastError());
         std::vector<float> h(g * 6);
@@ -458,10 +471,10 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     // 2. keys; 3. stable radix sort by (key, index)
     unsigned long long *keys;
     int *idx;
-    if (afmm_status s = talloc(t, tmp, &keys, n)) return s;
-    if (afmm_status s = talloc(t, tmp, &idx, n)) return s;
-    if (afmm_status s = dalloc(t, &t->keys_sorted, n)) return s;
-    if (afmm_status s = dalloc(t, &t->perm, n)) return s;
+    if (afmm_status s = wsalloc(t, kKeys, &keys, n)) return s;
+    if (afmm_status s = wsalloc(t, kIdx, &idx, n)) return s;
+    if (afmm_status s = wsalloc(t, kKeysSorted, &t->keys_sorted, n)) return s;
+    if (afmm_status s = wsalloc(t, kPerm, &t->perm, n)) return s;
     keys_kernel<<<grid_for(n, TH), TH, 0, st>>>(n, x, y, z, t->lo[0], t->lo[1], t->lo[2], scale, keys, idx);
     TCU(t, cudaGetLastError());
     {
@@ -469,36 +482,27 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
         TCU(t, cub::DeviceRadixSort::SortPairs(nullptr, tb, keys, t->keys_sorted, idx, t->perm, (int)n, 0,
                                                3 * kMaxLevel, st));
         void *tbuf;
-        if (afmm_status s = talloc(t, tmp, reinterpret_cast<char **>(&tbuf), tb)) return s;
+        if (afmm_status s = wsalloc(t, kSortTmp, reinterpret_cast<char **>(&tbuf), tb)) return s;
         TCU(t, cub::DeviceRadixSort::SortPairs(tbuf, tb, keys, t->keys_sorted, idx, t->perm, (int)n, 0,
                                                3 * kMaxLevel, st));
     }
 
     // 4. level-synchronous split into one node array (level-major)
-    size_t cap = 1024;
-    std::vector<void *> node_bufs;
+    size_t cap = t->node_cap;                 // grow-only across builds
     Nodes nd{};
-    auto alloc_nodes = [&](size_t c, Nodes &o) -> afmm_status {
-        if (afmm_status s = talloc(t, tmp, &o.b, c)) return s;
-        if (afmm_status s = talloc(t, tmp, &o.e, c)) return s;
-        if (afmm_status s = talloc(t, tmp, &o.first_child, c)) return s;
-        if (afmm_status s = talloc(t, tmp, &o.nchild, c)) return s;
-        if (afmm_status s = talloc(t, tmp, &o.level, c)) return s;
-        if (afmm_status s = talloc(t, tmp, &o.prefix, c)) return s;
+    int node_set = kNodeA;
+    auto alloc_nodes = [&](size_t c, Nodes &o, int set) -> afmm_status {
+        if (afmm_status s = wsalloc(t, set + 0, &o.b, c)) return s;
+        if (afmm_status s = wsalloc(t, set + 1, &o.e, c)) return s;
+        if (afmm_status s = wsalloc(t, set + 2, &o.first_child, c)) return s;
+        if (afmm_status s = wsalloc(t, set + 3, &o.nchild, c)) return s;
+        if (afmm_status s = wsalloc(t, set + 4, &o.level, c)) return s;
+        if (afmm_status s = wsalloc(t, set + 5, &o.prefix, c)) return s;
         return AFMM_OK;
     };
-    if (afmm_status s = alloc_nodes(cap, nd)) return s;
-    {
-        const int zero = 0, nn = (int)n, lv = 0, m1 = -1;
-        const unsigned long long p0 = 0;
-        TCU(t, cudaMemcpyAsync(nd.b, &zero, sizeof(int), cudaMemcpyHostToDevice, st));
-        TCU(t, cudaMemcpyAsync(nd.e, &nn, sizeof(int), cudaMemcpyHostToDevice, st));
-        TCU(t, cudaMemcpyAsync(nd.first_child, &m1, sizeof(int), cudaMemcpyHostToDevice, st));
-        TCU(t, cudaMemcpyAsync(nd.nchild, &zero, sizeof(int), cudaMemcpyHostToDevice, st));
-        TCU(t, cudaMemcpyAsync(nd.level, &lv, sizeof(int), cudaMemcpyHostToDevice, st));
-        TCU(t, cudaMemcpyAsync(nd.prefix, &p0, sizeof(p0), cudaMemcpyHostToDevice, st));
-        TCU(t, cudaStreamSynchronize(st));
-    }
+    if (afmm_status s = alloc_nodes(cap, nd, node_set)) return s;
+    root_kernel<<<1, 1, 0, st>>>(nd, (int)n);
+    TCU(t, cudaGetLastError());
     PrevTree pv{t->pv_prefix, t->pv_nchild, t->pv_base, enforce ? t->pv_levels : 0};
     std::vector<long long> lvl_base;
     long long base = 0, m = 1;     // current level occupies [base, base+m)
@@ -507,17 +511,16 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     size_t lvl_cap = 0;
     void *scan_tmp = nullptr;
     size_t scan_tmp_bytes = 0;
-    Tmp lvl_tmp_holder;
     while (m > 0) {
         if ((size_t)m + 1 > lvl_cap) {
             lvl_cap = std::max<size_t>((size_t)m + 1, 2 * lvl_cap);
-            if (afmm_status s = talloc(t, tmp, &cb, lvl_cap * 9)) return s;
-            if (afmm_status s = talloc(t, tmp, &nc, lvl_cap)) return s;
-            if (afmm_status s = talloc(t, tmp, &off, lvl_cap)) return s;
+            if (afmm_status s = wsalloc(t, kCb, &cb, lvl_cap * 9)) return s;
+            if (afmm_status s = wsalloc(t, kNc, &nc, lvl_cap)) return s;
+            if (afmm_status s = wsalloc(t, kOff, &off, lvl_cap)) return s;
             size_t need = 0;
             TCU(t, cub::DeviceScan::ExclusiveSum(nullptr, need, nc, off, (int)lvl_cap, st));
             if (need > scan_tmp_bytes) {
-                if (afmm_status s = talloc(t, tmp, reinterpret_cast<char **>(&scan_tmp), need)) return s;
+                if (afmm_status s = wsalloc(t, kScanTmp, reinterpret_cast<char **>(&scan_tmp), need)) return s;
                 scan_tmp_bytes = need;
             }
         }
@@ -533,7 +536,8 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
         if ((size_t)(next_base + total) > cap) {
             size_t ncap = std::max<size_t>(2 * cap, (size_t)(next_base + total));
             Nodes n2{};
-            if (afmm_status s = alloc_nodes(ncap, n2)) return s;
+            node_set = node_set == kNodeA ? kNodeB : kNodeA;
+            if (afmm_status s = alloc_nodes(ncap, n2, node_set)) return s;
             TCU(t, cudaMemcpyAsync(n2.b, nd.b, next_base * sizeof(int), cudaMemcpyDeviceToDevice, st));
             TCU(t, cudaMemcpyAsync(n2.e, nd.e, next_base * sizeof(int), cudaMemcpyDeviceToDevice, st));
             TCU(t, cudaMemcpyAsync(n2.first_child, nd.first_child, next_base * sizeof(int), cudaMemcpyDeviceToDevice, st));
@@ -553,6 +557,7 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     }
     const long long nn = base;     // total nodes
     t->n_nodes = nn;
+    t->node_cap = cap;
     lvl_base.push_back(nn);
     // keep this tree's nodes as the "previous tree" of the next Enforce_S
     if ((size_t)nn > t->pv_cap) {
@@ -574,9 +579,9 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
 
     // 5. leaves in Morton order: flag first bodies, scan
     int *flag, *leaf_at, *node_leaf;
-    if (afmm_status s = talloc(t, tmp, &flag, n + 1)) return s;
-    if (afmm_status s = talloc(t, tmp, &leaf_at, n + 1)) return s;
-    if (afmm_status s = talloc(t, tmp, &node_leaf, nn)) return s;
+    if (afmm_status s = wsalloc(t, kFlag, &flag, n + 1)) return s;
+    if (afmm_status s = wsalloc(t, kLeafAt, &leaf_at, n + 1)) return s;
+    if (afmm_status s = wsalloc(t, kNodeLeaf, &node_leaf, nn)) return s;
     TCU(t, cudaMemsetAsync(flag, 0, (n + 1) * sizeof(int), st));
     leaf_flag_kernel<<<grid_for(nn, TH), TH, 0, st>>>((int)nn, nd, flag);
     TCU(t, cudaGetLastError());
@@ -584,28 +589,28 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
         size_t sb = 0;
         TCU(t, cub::DeviceScan::ExclusiveSum(nullptr, sb, flag, leaf_at, (int)(n + 1), st));
         char *sbuf;
-        if (afmm_status s = talloc(t, tmp, &sbuf, sb)) return s;
+        if (afmm_status s = wsalloc(t, kScan2, &sbuf, sb)) return s;
         TCU(t, cub::DeviceScan::ExclusiveSum(sbuf, sb, flag, leaf_at, (int)(n + 1), st));
     }
     int L = 0;
     TCU(t, cudaMemcpyAsync(&L, leaf_at + n, sizeof(int), cudaMemcpyDeviceToHost, st));
     TCU(t, cudaStreamSynchronize(st));
     t->L = L;
-    if (afmm_status s = dalloc(t, &t->ls, L)) return s;
-    if (afmm_status s = dalloc(t, &t->lc, L)) return s;
-    if (afmm_status s = dalloc(t, &t->ll, L)) return s;
-    if (afmm_status s = dalloc(t, &t->lp, L)) return s;
+    if (afmm_status s = wsalloc(t, kLs, &t->ls, L)) return s;
+    if (afmm_status s = wsalloc(t, kLc, &t->lc, L)) return s;
+    if (afmm_status s = wsalloc(t, kLl, &t->ll, L)) return s;
+    if (afmm_status s = wsalloc(t, kLp, &t->lp, L)) return s;
     leaf_write_kernel<<<grid_for(nn, TH), TH, 0, st>>>((int)nn, nd, leaf_at, node_leaf, t->ls, t->lc, t->ll, t->lp);
     TCU(t, cudaGetLastError());
     int *leaf_node;
-    if (afmm_status s = talloc(t, tmp, &leaf_node, L)) return s;
+    if (afmm_status s = wsalloc(t, kLeafNode, &leaf_node, L)) return s;
     leaf_node_kernel<<<grid_for(nn, TH), TH, 0, st>>>((int)nn, node_leaf, leaf_node);
     TCU(t, cudaGetLastError());
 
     // 6. U-lists: count, scan, fill
     long long *counts;
-    if (afmm_status s = talloc(t, tmp, &counts, (size_t)L + 1)) return s;
-    if (afmm_status s = dalloc(t, &t->u_off, (size_t)L + 1)) return s;
+    if (afmm_status s = wsalloc(t, kCounts, &counts, (size_t)L + 1)) return s;
+    if (afmm_status s = wsalloc(t, kUoff, &t->u_off, (size_t)L + 1)) return s;
     TCU(t, cudaMemsetAsync(counts + L, 0, sizeof(long long), st));
     ulist_kernel<<<grid_for(L, 128), 128, 0, st>>>(L, nd, node_leaf, leaf_node, nullptr, nullptr, counts);
     TCU(t, cudaGetLastError());
@@ -613,12 +618,12 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
         size_t sb = 0;
         TCU(t, cub::DeviceScan::ExclusiveSum(nullptr, sb, counts, t->u_off, L + 1, st));
         char *sbuf;
-        if (afmm_status s = talloc(t, tmp, &sbuf, sb)) return s;
+        if (afmm_status s = wsalloc(t, kScan3, &sbuf, sb)) return s;
         TCU(t, cub::DeviceScan::ExclusiveSum(sbuf, sb, counts, t->u_off, L + 1, st));
     }
     TCU(t, cudaMemcpyAsync(&t->nnz, t->u_off + L, sizeof(long long), cudaMemcpyDeviceToHost, st));
     TCU(t, cudaStreamSynchronize(st));
-    if (afmm_status s = dalloc(t, &t->u_idx, (size_t)t->nnz)) return s;
+    if (afmm_status s = wsalloc(t, kUidx, &t->u_idx, (size_t)t->nnz)) return s;
     ulist_kernel<<<grid_for(L, 128), 128, 0, st>>>(L, nd, node_leaf, leaf_node, t->u_off, t->u_idx, nullptr);
     TCU(t, cudaGetLastError());
     TCU(t, cudaStreamSynchronize(st));
