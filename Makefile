@@ -6,7 +6,7 @@ PKG       := paper_conf_ipps_overmanpmm13_b200
 SRC       := $(PKG)/csrc
 LIB       := $(PKG)/libafmm_p2p.so
 CU_SRCS   := $(SRC)/afmm_p2p.cu $(SRC)/peak.cu $(SRC)/tree_build.cu $(SRC)/step.cu
-CU_HDRS   := $(SRC)/p2p_kernel.cuh $(SRC)/worklist.inc include/afmm_p2p.h include/afmm_tree.h include/afmm_step.h
+CU_HDRS   := $(SRC)/p2p_kernel.cuh $(SRC)/worklist.inc $(SRC)/worklist_dev.cuh include/afmm_p2p.h include/afmm_tree.h include/afmm_step.h
 ORACLE    := oracle/liboracle.so
 
 all: $(LIB) $(ORACLE)

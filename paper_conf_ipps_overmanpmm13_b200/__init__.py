@@ -72,6 +72,8 @@ _sig("afmm_p2p_set_bodies_host", _i, _p, _ll, _p, _p, _p, _p)
 _sig("afmm_p2p_bodies_buffer", _i, _p, C.POINTER(_p), C.POINTER(_ll))
 _sig("afmm_p2p_set_tree", _i, _p, _i, _p, _p, _p, _p)
 _sig("afmm_p2p_set_partition", _i, _p, _p)
+_sig("afmm_p2p_set_tree_device", _i, _p, _i, _p, _p, _p, _p)
+_sig("afmm_tree_device_arrays", _i, _p, C.POINTER(_p), C.POINTER(_p), C.POINTER(_p), C.POINTER(_p), C.POINTER(_p))
 _sig("afmm_p2p_get_partition", _i, _p, _p, _p)
 _sig("afmm_p2p_rebalance", _i, _p, _p, _d, C.POINTER(_i))
 _sig("afmm_p2p_eval", _i, _p, _p, _p, _p, _p, C.POINTER(Stats))
@@ -106,6 +108,7 @@ _sig("afmm_tree_last_error", C.c_char_p, _p)
 EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
             "afmm_p2p_set_bodies_host", "afmm_p2p_bodies_buffer", "afmm_p2p_set_tree",
             "afmm_p2p_set_partition", "afmm_p2p_get_partition", "afmm_p2p_rebalance",
+            "afmm_p2p_set_tree_device", "afmm_tree_device_arrays",
             "afmm_p2p_eval", "afmm_p2p_eval_host", "afmm_p2p_stats_get", "afmm_p2p_stream",
             "afmm_p2p_kernel_times",
             "afmm_p2p_destroy", "afmm_p2p_last_error", "afmm_interactions",
@@ -289,6 +292,12 @@ class P2P:
         self._check(_lib.afmm_p2p_set_tree(self._h, ls.shape[0], _ptr(ls), _ptr(lc), _ptr(uo), _ptr(ui)),
                     "afmm_p2p_set_tree")
 
+    def set_tree_device(self, n_leaves, leaf_start, leaf_count, u_off, u_idx):
+        """Tree ingest from device pointers (ints) or torch CUDA tensors."""
+        ptr = lambda a: a if isinstance(a, int) else _ptr(a)  # noqa: E731
+        self._check(_lib.afmm_p2p_set_tree_device(self._h, int(n_leaves), ptr(leaf_start), ptr(leaf_count),
+                                                  ptr(u_off), ptr(u_idx)), "afmm_p2p_set_tree_device")
+
     def set_partition(self, leaf_split=None):
         ls = None if leaf_split is None else _np(leaf_split, np.int64)
         self._check(_lib.afmm_p2p_set_partition(self._h, _ptr(ls)), "afmm_p2p_set_partition")
@@ -408,6 +417,12 @@ class GpuTree:
         out["u_idx"] = out["u_idx"][:nnz]
         out.update(inf)
         return out
+
+    def device_arrays(self):
+        """Device pointers (ints) of the last build: perm, leaf_start, leaf_count, u_off, u_idx."""
+        ps = [_p() for _ in range(5)]
+        self._check(_lib.afmm_tree_device_arrays(self._h, *[C.byref(q) for q in ps]), "afmm_tree_device_arrays")
+        return {k: q.value for k, q in zip(("perm", "leaf_start", "leaf_count", "u_off", "u_idx"), ps)}
 
     def gather(self, src, dst):
         """dst[p] = src[perm[p]] (device tensors)."""

@@ -63,6 +63,11 @@ struct afmm_p2p {
     Seg *d_segs = nullptr;
     size_t tasks_cap = 0, segs_cap = 0;
     int *d_queue = nullptr;
+    int n_tasks = 0;                        // tasks of the current work list (host or device built)
+    bool tree_on_device = false;            // set_tree_device: no host mirror of the tree
+    // device-ingest workspace (grow-only)
+    std::vector<void *> dws_ptr;
+    std::vector<size_t> dws_cap;
     long long rank_interactions = 0;
     long long bucket_inter[8] = {0};
 
@@ -267,6 +272,7 @@ extern "C" void afmm_p2p_destroy(afmm_p2p *h) {
     cudaFree(h->d_out);
     cudaFree(h->d_tasks);
     cudaFree(h->d_segs);
+    for (void *q : h->dws_ptr) cudaFree(q);
     cudaFree(h->d_queue);
     for (int i = 0; i < afmm_p2p::kRing; ++i) {
         if (h->ring0[i]) cudaEventDestroy(h->ring0[i]);
@@ -366,6 +372,7 @@ static void compute_body_split(afmm_p2p *h) {
 }
 
 #include "worklist.inc"
+#include "worklist_dev.cuh"
 
 extern "C" afmm_status afmm_p2p_set_tree(afmm_p2p *h, int n_leaves, const int *leaf_start,
                                          const int *leaf_count, const long long *u_off,
@@ -426,8 +433,172 @@ extern "C" afmm_status afmm_p2p_set_tree(afmm_p2p *h, int n_leaves, const int *l
     return build_worklist(h);
 }
 
+
+// grow-only device workspace for set_tree_device
+template <typename T>
+static afmm_status dws(afmm_p2p *h, int slot, T **p, size_t count) {
+    const size_t bytes = std::max<size_t>(count, 1) * sizeof(T);
+    if ((size_t)slot >= h->dws_ptr.size()) {
+        h->dws_ptr.resize(slot + 1, nullptr);
+        h->dws_cap.resize(slot + 1, 0);
+    }
+    if (h->dws_cap[slot] < bytes) {
+        cudaFree(h->dws_ptr[slot]);
+        h->dws_ptr[slot] = nullptr;
+        h->dws_cap[slot] = 0;
+        const size_t want = bytes + bytes / 4;
+        CUDA_TRY(h, cudaMalloc(&h->dws_ptr[slot], want));
+        h->dws_cap[slot] = want;
+    }
+    *p = static_cast<T *>(h->dws_ptr[slot]);
+    return AFMM_OK;
+}
+
+__global__ void body_split_kernel(int G, int L, long long n, const long long *__restrict__ split,
+                                  const int *__restrict__ ls, long long *__restrict__ bsplit) {
+    const int r = threadIdx.x;
+    if (r <= G) bsplit[r] = split[r] >= L ? n : ls[split[r]];
+}
+
+extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const int *leaf_start,
+                                                const int *leaf_count, const long long *u_off,
+                                                const int *u_idx) {
+    using namespace afmm;
+    CHECK_HANDLE(h);
+    if (h->n < 1 || !h->d_bodies) return fail(h, AFMM_ESTATE, "set_tree_device: call set_bodies first");
+    if (n_leaves < 1 || !leaf_start || !leaf_count || !u_off || !u_idx)
+        return fail(h, AFMM_EINVAL, "set_tree_device: n_leaves=%d / null pointer", n_leaves);
+    afmm_status st = set_device(h);
+    if (st) return st;
+    cudaStream_t s = h->stream;
+    const int L = n_leaves, W = h->cfg.world, TH = 256;
+    auto grid = [&](long long m) { return (int)std::max<long long>(1, (m + TH - 1) / TH); };
+    enum { sI, sP, sW, sPW, sSplit, sErr, sNseg, sNtask, sNsrc, sSegOff, sTaskOff, sStats, sKeys, sVals, sKeys2,
+           sVals2, sTasksU, sCoef, sTmp, sBsplit };
+    long long *I, *P, *split, *nsrc, *bsplit;
+    int *err, *nseg, *ntask, *seg_off, *task_off, *vals, *vals2;
+    unsigned long long *stats, *keys, *keys2;
+    if ((st = dws(h, sI, &I, L)) || (st = dws(h, sP, &P, L)) || (st = dws(h, sSplit, &split, W + 1)) ||
+        (st = dws(h, sErr, &err, 1)) || (st = dws(h, sBsplit, &bsplit, W + 1)))
+        return st;
+    // 1. validation + Interactions(t)
+    CUDA_TRY(h, cudaMemsetAsync(err, 0, sizeof(int), s));
+    dev::validate_interactions_kernel<<<grid(L), TH, 0, s>>>(L, h->n, h->cfg.max_leaf, leaf_start, leaf_count,
+                                                            u_off, u_idx, I, err);
+    CUDA_TRY(h, cudaGetLastError());
+    int herr = 0;
+    CUDA_TRY(h, cudaMemcpyAsync(&herr, err, sizeof(int), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(h, cudaStreamSynchronize(s));
+    if (herr)
+        return fail(h, AFMM_EINVAL, "set_tree_device: invalid tree (flags 0x%x: 1 start, 2 count, 4 cover, "
+                                    "8 u_off, 16 u_idx range, 32 row order)", herr);
+    // 2. partition (literal rule, or the per-bucket coefficients of the last step)
+    {
+        size_t tb = 0;
+        CUDA_TRY(h, cub::DeviceScan::InclusiveSum(nullptr, tb, I, P, L, s));
+        char *tmp;
+        if ((st = dws(h, sTmp, &tmp, tb))) return st;
+        CUDA_TRY(h, cub::DeviceScan::InclusiveSum(tmp, tb, I, P, L, s));
+    }
+    if (h->user_partition && (long long)h->leaf_split.size() == W + 1 && h->leaf_split[W] == L) {
+        CUDA_TRY(h, cudaMemcpyAsync(split, h->leaf_split.data(), (W + 1) * sizeof(long long),
+                                    cudaMemcpyHostToDevice, s));
+    } else if (h->have_coef && W > 1) {
+        double *w, *pw, *coef;
+        if ((st = dws(h, sW, &w, L)) || (st = dws(h, sPW, &pw, L)) || (st = dws(h, sCoef, &coef, 8))) return st;
+        CUDA_TRY(h, cudaMemcpyAsync(coef, h->coef, 8 * sizeof(double), cudaMemcpyHostToDevice, s));
+        dev::weights_kernel<<<grid(L), TH, 0, s>>>(L, leaf_count, I, coef, w);
+        size_t tb = 0;
+        CUDA_TRY(h, cub::DeviceScan::InclusiveSum(nullptr, tb, w, pw, L, s));
+        char *tmp;
+        if ((st = dws(h, sTmp, &tmp, tb))) return st;
+        CUDA_TRY(h, cub::DeviceScan::InclusiveSum(tmp, tb, w, pw, L, s));
+        dev::weighted_cut_kernel<<<1, 1, 0, s>>>(L, W, pw, split);
+        h->user_partition = false;
+    } else {
+        dev::literal_cut_kernel<<<1, 1, 0, s>>>(L, W, P, split);
+        h->user_partition = false;
+    }
+    CUDA_TRY(h, cudaGetLastError());
+    body_split_kernel<<<1, 64, 0, s>>>(W, L, h->n, split, leaf_start, bsplit);
+    h->leaf_split.assign(W + 1, 0);
+    h->body_split.assign(W + 1, 0);
+    CUDA_TRY(h, cudaMemcpyAsync(h->leaf_split.data(), split, (W + 1) * sizeof(long long), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(h, cudaMemcpyAsync(h->body_split.data(), bsplit, (W + 1) * sizeof(long long), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(h, cudaMemcpyAsync(&h->I_total, P + (L - 1), sizeof(long long), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(h, cudaStreamSynchronize(s));
+    // 3. this rank's work list
+    const int r = h->cfg.rank;
+    const int lo = (int)h->leaf_split[r], m = (int)(h->leaf_split[r + 1] - h->leaf_split[r]);
+    if ((st = dws(h, sNseg, &nseg, (size_t)m + 1)) || (st = dws(h, sNtask, &ntask, (size_t)m + 1)) ||
+        (st = dws(h, sNsrc, &nsrc, (size_t)m + 1)) || (st = dws(h, sSegOff, &seg_off, (size_t)m + 1)) ||
+        (st = dws(h, sTaskOff, &task_off, (size_t)m + 1)) || (st = dws(h, sStats, &stats, 9)))
+        return st;
+    CUDA_TRY(h, cudaMemsetAsync(stats, 0, 9 * sizeof(unsigned long long), s));
+    CUDA_TRY(h, cudaMemsetAsync(nseg + m, 0, sizeof(int), s));
+    CUDA_TRY(h, cudaMemsetAsync(ntask + m, 0, sizeof(int), s));
+    if (m > 0) {
+        dev::count_kernel<<<grid(m), TH, 0, s>>>(m, lo, leaf_start, leaf_count, u_off, u_idx, I, nseg, ntask, nsrc,
+                                                stats);
+        CUDA_TRY(h, cudaGetLastError());
+    }
+    {
+        size_t tb = 0;
+        CUDA_TRY(h, cub::DeviceScan::ExclusiveSum(nullptr, tb, nseg, seg_off, m + 1, s));
+        char *tmp;
+        if ((st = dws(h, sTmp, &tmp, tb))) return st;
+        CUDA_TRY(h, cub::DeviceScan::ExclusiveSum(tmp, tb, nseg, seg_off, m + 1, s));
+        CUDA_TRY(h, cub::DeviceScan::ExclusiveSum(tmp, tb, ntask, task_off, m + 1, s));
+    }
+    int totals[2] = {0, 0};
+    unsigned long long hstats[9];
+    CUDA_TRY(h, cudaMemcpyAsync(&totals[0], seg_off + m, sizeof(int), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(h, cudaMemcpyAsync(&totals[1], task_off + m, sizeof(int), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(h, cudaMemcpyAsync(hstats, stats, sizeof(hstats), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(h, cudaStreamSynchronize(s));
+    const int nsegs = totals[0], nt = totals[1];
+    if ((st = ensure_device(h, &h->d_segs, h->segs_cap, (size_t)nsegs))) return st;
+    if ((st = ensure_device(h, &h->d_tasks, h->tasks_cap, (size_t)nt))) return st;
+    Task *tasks_u;
+    if ((st = dws(h, sTasksU, &tasks_u, nt)) || (st = dws(h, sKeys, &keys, nt)) || (st = dws(h, sVals, &vals, nt)) ||
+        (st = dws(h, sKeys2, &keys2, nt)) || (st = dws(h, sVals2, &vals2, nt)))
+        return st;
+    if (m > 0) {
+        dev::write_kernel<<<grid(m), TH, 0, s>>>(m, lo, leaf_start, leaf_count, u_off, u_idx, seg_off, task_off,
+                                                ntask, nsrc, h->d_segs, tasks_u, keys, vals);
+        CUDA_TRY(h, cudaGetLastError());
+    }
+    if (nt > 0) {
+        size_t tb = 0;
+        CUDA_TRY(h, cub::DeviceRadixSort::SortPairs(nullptr, tb, keys, keys2, vals, vals2, nt, 0, 64, s));
+        char *tmp;
+        if ((st = dws(h, sTmp, &tmp, tb))) return st;
+        CUDA_TRY(h, cub::DeviceRadixSort::SortPairs(tmp, tb, keys, keys2, vals, vals2, nt, 0, 64, s));
+        dev::gather_tasks_kernel<<<grid(nt), TH, 0, s>>>(nt, vals2, tasks_u, h->d_tasks);
+        CUDA_TRY(h, cudaGetLastError());
+    }
+    h->n_tasks = nt;
+    h->L = L;
+    h->rank_interactions = (long long)hstats[0];
+    for (int b = 0; b < 8; ++b) h->bucket_inter[b] = (long long)hstats[1 + b];
+    h->tree_on_device = true;
+    h->have_tree = true;
+    h->h_tasks.clear();
+    h->h_segs.clear();
+    h->leaf_start.clear();
+    h->leaf_count.clear();
+    h->u_off.clear();
+    h->u_idx.clear();
+    h->I.clear();
+    h->evaluated = false;
+    return AFMM_OK;
+}
+
 extern "C" afmm_status afmm_p2p_set_partition(afmm_p2p *h, const long long *leaf_split) {
     CHECK_HANDLE(h);
+    if (h->tree_on_device && h->have_tree)
+        return fail(h, AFMM_ESTATE, "set_partition: the tree was ingested from device memory; "
+                                    "set the partition before set_tree_device or use set_tree");
     const int W = h->cfg.world;
     if (!leaf_split) {
         h->user_partition = false;
@@ -593,6 +764,9 @@ extern "C" afmm_status afmm_p2p_rebalance(afmm_p2p *h, const double *rank_ms, do
     CHECK_HANDLE(h);
     if (changed) *changed = 0;
     if (!h->have_tree) return fail(h, AFMM_ESTATE, "rebalance: no tree");
+    if (h->tree_on_device)
+        return fail(h, AFMM_ESTATE, "rebalance: the tree was ingested from device memory; "
+                                    "use afmm_cost_fit + afmm_p2p_set_cost_coef before the next set_tree_device");
     if (!rank_ms) return fail(h, AFMM_EINVAL, "rebalance: rank_ms is null");
     const int W = h->cfg.world;
     std::vector<long long> split(W + 1);
@@ -618,7 +792,7 @@ static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, flo
     p.bodies = h->d_bodies;
     p.tasks = h->d_tasks;
     p.segs = h->d_segs;
-    p.n_tasks = (int)h->h_tasks.size();
+    p.n_tasks = h->n_tasks;
     p.queue = h->d_queue;
     p.ax = ax;
     p.ay = ay;
@@ -658,7 +832,7 @@ static afmm_status fill_stats(afmm_p2p *h, afmm_p2p_stats *s) {
     o.leaf_hi = h->leaf_split[h->cfg.rank + 1];
     o.body_lo = h->body_split[h->cfg.rank];
     o.body_hi = h->body_split[h->cfg.rank + 1];
-    o.n_work_items = (int)h->h_tasks.size();
+    o.n_work_items = h->n_tasks;
     o.n_launches = h->last.n_launches;
     for (int b = 0; b < 8; ++b) o.bucket_interactions[b] = h->bucket_inter[b];
     h->last = o;

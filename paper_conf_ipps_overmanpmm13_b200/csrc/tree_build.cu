@@ -686,6 +686,19 @@ extern "C" afmm_status afmm_tree_copy_out(const afmm_tree *tc, int *perm, int *l
     return AFMM_OK;
 }
 
+extern "C" afmm_status afmm_tree_device_arrays(const afmm_tree *t, const int **perm, const int **leaf_start,
+                                               const int **leaf_count, const long long **u_off,
+                                               const int **u_idx) {
+    if (!t) return AFMM_EINVAL;
+    if (!t->built) return AFMM_ESTATE;
+    if (perm) *perm = t->perm;
+    if (leaf_start) *leaf_start = t->ls;
+    if (leaf_count) *leaf_count = t->lc;
+    if (u_off) *u_off = t->u_off;
+    if (u_idx) *u_idx = t->u_idx;
+    return AFMM_OK;
+}
+
 extern "C" afmm_status afmm_tree_gather(afmm_tree *t, const float *in, float *out) {
     if (!t || !in || !out) return AFMM_EINVAL;
     if (!t->built) return AFMM_ESTATE;

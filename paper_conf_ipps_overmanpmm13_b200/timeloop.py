@@ -50,16 +50,19 @@ class TimeLoop:
         self.h = P2P(device=device, rank=rank, world=world, G=G, eps2=eps2, stream=self.stream.cuda_stream)
         self.step_no = 0
         self.log = []
-        self._load_tree()
+        self._load_tree(host_copy=True)
         self._eval()
 
     # ------------------------------------------------------------------ pieces
-    def _load_tree(self):
-        T = self.tree.copy_out(self.n)
-        self.T = T
+    def _load_tree(self, host_copy=False):
+        """Device-side ingest of the GPU tree (afmm_p2p_set_tree_device): no host
+        round trip; a host copy of the tree is kept only for verification hooks."""
+        info = self.tree.info()
+        d = self.tree.device_arrays()
         s = self.state
         self.h.set_bodies(s[0], s[1], s[2], s[3])
-        self.h.set_tree(T["leaf_start"], T["leaf_count"], T["u_off"], T["u_idx"])
+        self.h.set_tree_device(info["n_leaves"], d["leaf_start"], d["leaf_count"], d["u_off"], d["u_idx"])
+        self.T = self.tree.copy_out(self.n) if host_copy else info
         self.body_split = self.h.get_partition()[1]
 
     def _slice(self):
@@ -119,7 +122,7 @@ class TimeLoop:
             self.tree.gather(s[a], self.tmp[a])
         self.state, self.tmp = self.tmp, self.state
         ev[2].record(self.stream)
-        self._load_tree()
+        self._load_tree(host_copy=bool(hooks))
         ev[3].record(self.stream)
         self._eval()
         ev[4].record(self.stream)

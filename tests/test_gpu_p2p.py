@@ -273,3 +273,75 @@ def test_fp32_peak_sane():
     afmm = _afmm()
     p = afmm.fp32_peak(0)
     assert 30 < p["ffma_tflops"] < 90 and 20 < p["ffma2_tflops"] < 180
+
+
+@pytest.mark.parametrize("world,coef", [(1, None), (3, None), (4, [1.0, 1.0, 2.0, 1.5, 1.0, 1.0, 1.0, 1.0])])
+def test_set_tree_device_matches_host_ingest(world, coef):
+    """afmm_p2p_set_tree_device (kernels) == afmm_p2p_set_tree (host): same
+    partition, stats and bit-identical outputs, straight from the GPU tree."""
+    afmm = _afmm()
+    x, y, z, m = synth.make("plummer", 150000, 12)
+    n = x.shape[0]
+    tree = afmm.GpuTree(0)
+    X, Y, Z, M = (torch.from_numpy(v).cuda() for v in (x, y, z, m))
+    info = tree.build(X, Y, Z, 48)
+    T = tree.copy_out(n)
+    d = tree.device_arrays()
+    bod = torch.empty((4, n), device="cuda")
+    for a, src in enumerate((X, Y, Z, M)):
+        tree.gather(src, bod[a])
+    outs = []
+    for mode in ("host", "device"):
+        out = torch.full((4, n), float("nan"), device="cuda")
+        splits, stats = [], []
+        for r in range(world):
+            h = afmm.P2P(rank=r, world=world, eps2=1e-6)
+            h.set_bodies(bod[0], bod[1], bod[2], bod[3])
+            if coef is not None:
+                h.set_cost_coef(coef)
+            if mode == "host":
+                h.set_tree(T["leaf_start"], T["leaf_count"], T["u_off"], T["u_idx"])
+            else:
+                h.set_tree_device(info["n_leaves"], d["leaf_start"], d["leaf_count"], d["u_off"], d["u_idx"])
+            stats.append(h.eval(out[0], out[1], out[2], out[3], stats=True))
+            splits.append(h.get_partition())
+            h.close()
+        torch.cuda.synchronize()
+        outs.append((out.cpu().numpy(), splits, stats))
+    (oh, sh, th), (od, sd, td) = outs
+    assert np.array_equal(oh, od) and np.isfinite(od).all()
+    for a, b in zip(sh, sd):
+        if coef is None:
+            assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
+        else:                                   # fp64 prefix sums of the weights may tie-break differently
+            assert np.abs(a[0] - b[0]).max() <= 1
+    for a, b in zip(th, td):
+        assert a["interactions_total"] == b["interactions_total"]
+        if coef is None:
+            assert a["interactions_rank"] == b["interactions_rank"]
+            assert a["bucket_interactions"] == b["bucket_interactions"]
+            assert a["n_work_items"] == b["n_work_items"]
+    tree.close()
+
+
+def test_set_tree_device_rejects_invalid_tree():
+    afmm = _afmm()
+    h = afmm.P2P(max_leaf=64)
+    xs = torch.rand(8, device="cuda")
+    h.set_bodies(xs, xs, xs, xs)
+    dev = lambda a, dt: torch.tensor(a, dtype=dt, device="cuda")  # noqa: E731
+    bad = [([0, 4], [4, 3], [0, 1, 2], [0, 1]), ([0, 4], [4, 4], [0, 2, 3], [1, 0, 1]),
+           ([0, 4], [4, 4], [0, 1, 2], [0, 2]), ([0, 4], [4, 4], [1, 1, 2], [0, 1])]
+    for ls, lc, uo, ui in bad:
+        with pytest.raises(afmm.AfmmError) as e:
+            h.set_tree_device(2, dev(ls, torch.int32), dev(lc, torch.int32), dev(uo, torch.int64),
+                              dev(ui, torch.int32))
+        assert e.value.status == afmm.AFMM_EINVAL
+    h.set_tree_device(2, dev([0, 4], torch.int32), dev([4, 4], torch.int32), dev([0, 2, 4], torch.int64),
+                      dev([0, 1, 0, 1], torch.int32))
+    out = [torch.zeros(8, device="cuda") for _ in range(4)]
+    h.eval(*out, stats=True)
+    with pytest.raises(afmm.AfmmError) as e:
+        h.rebalance([1.0], 0.02)
+    assert e.value.status == afmm.AFMM_ESTATE
+    h.close()
