@@ -125,7 +125,10 @@ afmm_status ensure_device(afmm_p2p *h, T **ptr, size_t &cap, size_t count) {
     if (*ptr) cudaFree(*ptr);
     *ptr = nullptr;
     cap = 0;
+    // grow-only with 50% headroom: a time-stepping caller re-ingests slowly
+    // growing trees every step, and cudaMalloc/cudaFree are device-wide syncs
     size_t c = std::max<size_t>(count, 1);
+    c += c / 2;
     CUDA_TRY(h, cudaMalloc(reinterpret_cast<void **>(ptr), c * sizeof(T)));
     cap = c;
     return AFMM_OK;
@@ -446,7 +449,7 @@ static afmm_status dws(afmm_p2p *h, int slot, T **p, size_t count) {
         cudaFree(h->dws_ptr[slot]);
         h->dws_ptr[slot] = nullptr;
         h->dws_cap[slot] = 0;
-        const size_t want = bytes + bytes / 4;
+        const size_t want = bytes + bytes / 2;
         CUDA_TRY(h, cudaMalloc(&h->dws_ptr[slot], want));
         h->dws_cap[slot] = want;
     }

@@ -362,7 +362,7 @@ afmm_status wsalloc(afmm_tree *t, int slot, T **p, size_t count) {
         cudaFree(t->ws_ptr[slot]);
         t->ws_ptr[slot] = nullptr;
         t->ws_cap[slot] = 0;
-        const size_t want = bytes + bytes / 4;
+        const size_t want = bytes + bytes / 2;
         TCU(t, cudaMalloc(&t->ws_ptr[slot], want));
         t->ws_cap[slot] = want;
     }

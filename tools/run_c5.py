@@ -76,6 +76,10 @@ print(json.dumps({
     "step_interactions_per_s": tot_int / sum(r["step_ms"] * 1e-3 for r in L),
     "mean_ms": {k: float(np.mean([r[k] for r in L])) for k in
                 ("kernel_ms", "kick_drift_ms", "enforce_ms", "set_tree_ms", "eval_ms", "step_ms")},
+    "step_ms_by_quarter": [round(float(np.mean([r["step_ms"] for r in L[q * len(L) // 4:(q + 1) * len(L) // 4]])), 3)
+                           for q in range(4)],
+    "set_tree_ms_by_quarter": [round(float(np.mean([r["set_tree_ms"] for r in L[q * len(L) // 4:(q + 1) * len(L) // 4]])), 3)
+                               for q in range(4)],
     "n_leaves": [L[0]["n_leaves"], L[len(L) // 2]["n_leaves"], L[-1]["n_leaves"]],
     "interactions_per_step": [L[0]["interactions"], L[len(L) // 2]["interactions"], L[-1]["interactions"]],
     "checks": checks}))
