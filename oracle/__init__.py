@@ -67,6 +67,9 @@ def _L():
         lib.oracle_kick.argtypes = [i64, p, p, p, p, p, p, C.c_double]
         lib.oracle_drift.restype = None
         lib.oracle_drift.argtypes = [i64, p, p, p, p, p, p, C.c_double]
+        lib.oracle_stokeslet.restype = None
+        lib.oracle_stokeslet.argtypes = [i64, p, p, p, p, p, p, i64, p, p, p, p, C.c_double, C.c_double,
+                                         i64, p, p, p, p, p]
         lib.oracle_partition_literal.restype = None
         lib.oracle_partition_literal.argtypes = [i64, p, C.c_int, p, p]
         _lib = lib
@@ -195,6 +198,22 @@ def p2p(x, y, z, m, leaf_start, leaf_count, u_off, u_idx, G=1.0, eps2=0.0, targe
                     _ptr(leaf_count), _ptr(u_off), _ptr(u_idx), float(G), float(eps2),
                     0 if tg is None else tg.shape[0], _ptr(tg),
                     *[_ptr(o) for o in out[:4]], _ptr(out[4]) if with_scale else None)
+    return tuple(out)
+
+
+def stokeslet(x, y, z, fx, fy, fz, leaf_start, leaf_count, u_off, u_idx, mu=1.0, eps2=1e-6,
+              targets=None, with_scale=False):
+    """fp64 regularized-Stokeslet near field (reading R26) over bodies in tree
+    order; self term included.  Returns (ux, uy, uz[, A])."""
+    arrs = [_c(v, np.float32) for v in (x, y, z, fx, fy, fz)]
+    leaf_start, leaf_count = _c(leaf_start, np.int32), _c(leaf_count, np.int32)
+    u_off, u_idx = _c(u_off, np.int64), _c(u_idx, np.int32)
+    n = arrs[0].shape[0]
+    out = [np.full(n, np.nan) for _ in range(4 if with_scale else 3)]
+    tg = None if targets is None else _c(targets, np.int32)
+    _L().oracle_stokeslet(n, *[_ptr(a) for a in arrs], leaf_start.shape[0], _ptr(leaf_start), _ptr(leaf_count),
+                          _ptr(u_off), _ptr(u_idx), float(mu), float(eps2), 0 if tg is None else tg.shape[0],
+                          _ptr(tg), *[_ptr(o) for o in out[:3]], _ptr(out[3]) if with_scale else None)
     return tuple(out)
 
 

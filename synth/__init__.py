@@ -212,3 +212,16 @@ def make(name_or_dist: str, n: int | None = None, seed: int | None = None):
         return GENERATORS[c["dist"]](n if n is not None else c["n"],
                                      seed if seed is not None else c["seed"])
     return GENERATORS[name_or_dist](n, seed)
+
+
+def uniform_with_forces(n: int, seed: int):
+    """Stokeslet workload (PAPER L26 SIX.B: "ten million sources in a uniform
+    distribution"): positions uniform in [0,1)^3, forces with independent
+    components uniform in [-1, 1).  Returns fp32 (x, y, z, fx, fy, fz)."""
+    x, y, z, _ = uniform_cube(n, seed)
+    k = np.arange(n, dtype=np.uint64)
+    f = [(2.0 * uniform01(seed, 7, k * np.uint64(3) + np.uint64(c)) - 1.0).astype(np.float32) for c in range(3)]
+    return x, y, z, f[0], f[1], f[2]
+
+
+CONFIGS["C6"] = dict(dist="stokeslet", n=10_000_000, S=128, seed=6, eps2=1e-6)
