@@ -59,6 +59,7 @@ def parse():
     ap.add_argument("--S", type=int, default=None, help="leaf capacity (default: the config's)")
     ap.add_argument("--no-sweep", action="store_true", help="skip the S sweep (C2, N=1)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-stokeslet", action="store_true", help="skip the C6 Stokeslet line (N=1)")
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="oracle sample budget")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="gloo + AFMM_BENCH_SAME_DEVICE=1 exercises the N>1 flow on one GPU (testing only)")
@@ -378,6 +379,36 @@ def main():
                 h2.close()
                 tr2.close()
             extra["sweep_S"] = sweep
+
+    if rank == 0 and world == 1 and not args.no_stokeslet:
+        # row f4: the regularized-Stokeslet law on its paper workload (C6: 10M uniform sources, L26 SIX.B)
+        c6 = synth.CONFIGS["C6"]
+        sx, sy, sz, sfx, sfy, sfz = synth.uniform_with_forces(c6["n"], c6["seed"])
+        n6 = sx.shape[0]
+        D = [torch.from_numpy(v).to(dev) for v in (sx, sy, sz, sfx, sfy, sfz)]
+        tr6 = afmm.GpuTree(local, stream=stream.cuda_stream)
+        inf6 = tr6.build(D[0], D[1], D[2], c6["S"])
+        d6 = tr6.device_arrays()
+        B6 = torch.empty((6, n6), device=dev)
+        for a in range(6):
+            tr6.gather(D[a], B6[a])
+        h6 = afmm.P2P(device=local, eps2=c6["eps2"], stream=stream.cuda_stream, law=afmm.LAW_STOKESLET)
+        h6.set_bodies_stokeslet(*[B6[a] for a in range(6)])
+        h6.set_tree_device(inf6["n_leaves"], d6["leaf_start"], d6["leaf_count"], d6["u_off"], d6["u_idx"])
+        o6 = torch.empty((4, n6), device=dev)
+        for _ in range(6):
+            h6.eval(o6[0], o6[1], o6[2], o6[3])
+        k6 = float(np.median(h6.kernel_times(4)))
+        st6 = h6.stats()
+        ips6 = st6["interactions_total"] / (k6 * 1e-3)
+        extra["stokeslet_C6"] = {
+            "workload": "C6: 10M uniform Stokeslet sources, S=128, eps2=1e-6 (PAPER L26 SIX.B; reading R26)",
+            "interactions": st6["interactions_total"], "kernel_ms": k6, "interactions_per_s": ips6,
+            "flop_per_interaction": 32, "frac_fp32": 32 * ips6 / (peak * 1e12),
+            "note": "19 packed FP32 ops + 2 MUFU per two interactions; FMA=2 flop, rsqrt=1"}
+        h6.close()
+        tr6.close()
+        del D, B6, o6
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:

@@ -39,7 +39,11 @@ class AfmmError(RuntimeError):
 
 class Config(C.Structure):
     _fields_ = [("device", C.c_int), ("rank", C.c_int), ("world", C.c_int), ("G", C.c_float),
-                ("eps2", C.c_float), ("max_leaf", C.c_int), ("stream", C.c_void_p)]
+                ("eps2", C.c_float), ("max_leaf", C.c_int), ("stream", C.c_void_p), ("law", C.c_int),
+                ("mu", C.c_float)]
+
+
+LAW_GRAVITY, LAW_STOKESLET = 0, 1
 
 
 class Stats(C.Structure):
@@ -70,6 +74,7 @@ _sig("afmm_p2p_create", _i, C.POINTER(Config), C.POINTER(_p))
 _sig("afmm_p2p_set_bodies", _i, _p, _ll, _p, _p, _p, _p)
 _sig("afmm_p2p_set_bodies_host", _i, _p, _ll, _p, _p, _p, _p)
 _sig("afmm_p2p_bodies_buffer", _i, _p, C.POINTER(_p), C.POINTER(_ll))
+_sig("afmm_p2p_set_bodies_stokeslet", _i, _p, _ll, _p, _p, _p, _p, _p, _p)
 _sig("afmm_p2p_set_tree", _i, _p, _i, _p, _p, _p, _p)
 _sig("afmm_p2p_set_partition", _i, _p, _p)
 _sig("afmm_p2p_set_tree_device", _i, _p, _i, _p, _p, _p, _p)
@@ -107,6 +112,7 @@ _sig("afmm_tree_last_error", C.c_char_p, _p)
 # every symbol include/*.h declares (checked by tests/test_abi.py)
 EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
             "afmm_p2p_set_bodies_host", "afmm_p2p_bodies_buffer", "afmm_p2p_set_tree",
+            "afmm_p2p_set_bodies_stokeslet",
             "afmm_p2p_set_partition", "afmm_p2p_get_partition", "afmm_p2p_rebalance",
             "afmm_p2p_set_tree_device", "afmm_tree_device_arrays",
             "afmm_p2p_eval", "afmm_p2p_eval_host", "afmm_p2p_stats_get", "afmm_p2p_stream",
@@ -232,12 +238,14 @@ def fp32_peak(device: int = 0):
 class P2P:
     """One afmm_p2p handle (one per rank / GPU)."""
 
-    def __init__(self, device=0, rank=0, world=1, G=1.0, eps2=0.0, max_leaf=1024, stream=None):
+    def __init__(self, device=0, rank=0, world=1, G=1.0, eps2=0.0, max_leaf=1024, stream=None,
+                 law=LAW_GRAVITY, mu=1.0):
         cfg = Config()
         _lib.afmm_p2p_config_init(C.byref(cfg))
         cfg.device, cfg.rank, cfg.world = int(device), int(rank), int(world)
         cfg.G, cfg.eps2, cfg.max_leaf = float(G), float(eps2), int(max_leaf)
         cfg.stream = stream
+        cfg.law, cfg.mu = int(law), float(mu)
         h = _p()
         st = _lib.afmm_p2p_create(C.byref(cfg), C.byref(h))
         if st:
@@ -280,6 +288,12 @@ class P2P:
             x, y, z, m = (_np(v, np.float32) for v in (x, y, z, m))
             self._check(_lib.afmm_p2p_set_bodies_host(self._h, n, _ptr(x), _ptr(y), _ptr(z), _ptr(m)),
                         "afmm_p2p_set_bodies_host")
+
+    def set_bodies_stokeslet(self, x, y, z, fx, fy, fz):
+        """Stokeslet bodies: torch CUDA tensors (device pointers), tree order."""
+        self._check(_lib.afmm_p2p_set_bodies_stokeslet(self._h, int(x.shape[0]), *[_ptr(a) for a in
+                                                                                  (x, y, z, fx, fy, fz)]),
+                    "afmm_p2p_set_bodies_stokeslet")
 
     def bodies_buffer(self):
         p, b = _p(), _ll()

@@ -217,6 +217,8 @@ extern "C" afmm_status afmm_p2p_config_init(afmm_p2p_config *cfg) {
     cfg->eps2 = 0.0f;
     cfg->max_leaf = 1024;
     cfg->stream = nullptr;
+    cfg->law = AFMM_LAW_GRAVITY;
+    cfg->mu = 1.0f;
     return AFMM_OK;
 }
 
@@ -229,7 +231,8 @@ extern "C" afmm_status afmm_p2p_create(const afmm_p2p_config *cfg, afmm_p2p **ou
     if (cfg->max_leaf > 1024) return AFMM_ENOTSUP;
     if (cfg->max_leaf < 1 || cfg->world < 1 || cfg->rank < 0 || cfg->rank >= cfg->world ||
         !std::isfinite(cfg->G) || !std::isfinite(cfg->eps2) || !(cfg->eps2 >= 0.0f) ||
-        cfg->device < 0)
+        cfg->device < 0 || (cfg->law != AFMM_LAW_GRAVITY && cfg->law != AFMM_LAW_STOKESLET) ||
+        !std::isfinite(cfg->mu) || !(cfg->mu > 0.0f))
         return AFMM_EINVAL;
     afmm_p2p *h = new (std::nothrow) afmm_p2p();
     if (!h) return AFMM_ENOMEM;
@@ -250,10 +253,13 @@ extern "C" afmm_status afmm_p2p_create(const afmm_p2p_config *cfg, afmm_p2p **ou
         if (e == cudaSuccess) e = cudaMalloc(&h->d_queue, sizeof(int));
         if (e == cudaSuccess) e = cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, cfg->device);
         if (e == cudaSuccess)
-            e = cudaFuncSetAttribute(afmm::p2p_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+            e = cudaFuncSetAttribute(afmm::p2p_kernel_t<afmm::Gravity>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                      afmm::kDynSmem);
         if (e == cudaSuccess)
-            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&h->blocks_per_sm, afmm::p2p_kernel,
+            e = cudaFuncSetAttribute(afmm::p2p_kernel_t<afmm::Stokeslet>,
+                                     cudaFuncAttributeMaxDynamicSharedMemorySize, afmm::kDynSmem);
+        if (e == cudaSuccess)
+            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&h->blocks_per_sm, afmm::p2p_kernel_t<afmm::Gravity>,
                                                               afmm::kThreads, afmm::kDynSmem);
         if (e != cudaSuccess) st = fail(h, AFMM_ECUDA, "create: %s", cudaGetErrorString(e));
         if (h->blocks_per_sm < 1) h->blocks_per_sm = 1;
@@ -294,13 +300,16 @@ extern "C" void *afmm_p2p_stream(const afmm_p2p *h) { return h ? (void *)h->stre
 
 // ------------------------------------------------------------------ bodies
 
+static int words_of(const afmm_p2p *h) { return h->cfg.law == AFMM_LAW_STOKESLET ? 2 : 1; }
+
 static afmm_status alloc_bodies(afmm_p2p *h, long long n) {
-    if (n > h->bodies_cap) {
+    const long long words = n * words_of(h);       // float4 per body: 1 (gravity) or 2 (Stokeslet)
+    if (words > h->bodies_cap) {
         cudaFree(h->d_bodies);
         h->d_bodies = nullptr;
         h->bodies_cap = 0;
-        CUDA_TRY(h, cudaMalloc(&h->d_bodies, (size_t)n * sizeof(float4)));
-        h->bodies_cap = n;
+        CUDA_TRY(h, cudaMalloc(&h->d_bodies, (size_t)words * sizeof(float4)));
+        h->bodies_cap = words;
     }
     if (h->n != n) h->have_tree = false;   // a tree for another n is stale
     h->n = n;
@@ -320,6 +329,7 @@ static afmm_status pack(afmm_p2p *h, const float *x, const float *y, const float
 extern "C" afmm_status afmm_p2p_set_bodies(afmm_p2p *h, long long n, const float *x,
                                            const float *y, const float *z, const float *m) {
     CHECK_HANDLE(h);
+    if (h->cfg.law != AFMM_LAW_GRAVITY) return fail(h, AFMM_EINVAL, "set_bodies: handle law is not gravity");
     if (n < 1 || n >= (1LL << 31)) return fail(h, AFMM_EINVAL, "set_bodies: n=%lld out of [1, 2^31)", n);
     const int nn = (x != nullptr) + (y != nullptr) + (z != nullptr) + (m != nullptr);
     if (nn != 0 && nn != 4) return fail(h, AFMM_EINVAL, "set_bodies: pass all four pointers or none");
@@ -333,6 +343,7 @@ extern "C" afmm_status afmm_p2p_set_bodies(afmm_p2p *h, long long n, const float
 extern "C" afmm_status afmm_p2p_set_bodies_host(afmm_p2p *h, long long n, const float *x,
                                                 const float *y, const float *z, const float *m) {
     CHECK_HANDLE(h);
+    if (h->cfg.law != AFMM_LAW_GRAVITY) return fail(h, AFMM_EINVAL, "set_bodies_host: handle law is not gravity");
     if (n < 1 || n >= (1LL << 31)) return fail(h, AFMM_EINVAL, "set_bodies_host: n=%lld out of [1, 2^31)", n);
     if (!x || !y || !z || !m) return fail(h, AFMM_EINVAL, "set_bodies_host: null pointer");
     afmm_status st = set_device(h);
@@ -355,11 +366,31 @@ extern "C" afmm_status afmm_p2p_set_bodies_host(afmm_p2p *h, long long n, const 
     return AFMM_OK;
 }
 
+extern "C" afmm_status afmm_p2p_set_bodies_stokeslet(afmm_p2p *h, long long n, const float *x, const float *y,
+                                                     const float *z, const float *fx, const float *fy,
+                                                     const float *fz) {
+    CHECK_HANDLE(h);
+    if (h->cfg.law != AFMM_LAW_STOKESLET)
+        return fail(h, AFMM_EINVAL, "set_bodies_stokeslet: handle law is not the Stokeslet");
+    if (n < 1 || n >= (1LL << 31)) return fail(h, AFMM_EINVAL, "set_bodies_stokeslet: n=%lld out of [1, 2^31)", n);
+    const int nn = !!x + !!y + !!z + !!fx + !!fy + !!fz;
+    if (nn != 0 && nn != 6) return fail(h, AFMM_EINVAL, "set_bodies_stokeslet: pass all six pointers or none");
+    afmm_status st = set_device(h);
+    if (st) return st;
+    if ((st = alloc_bodies(h, n))) return st;
+    if (nn == 0) return AFMM_OK;
+    const int threads = 256;
+    long long blocks = std::min<long long>((n + threads - 1) / threads, (long long)h->num_sms * 16);
+    afmm::pack_stokeslet_kernel<<<(int)blocks, threads, 0, h->stream>>>(n, x, y, z, fx, fy, fz, h->d_bodies);
+    CUDA_TRY(h, cudaGetLastError());
+    return AFMM_OK;
+}
+
 extern "C" afmm_status afmm_p2p_bodies_buffer(afmm_p2p *h, void **dev_ptr, long long *bytes) {
     CHECK_HANDLE(h);
     if (!h->d_bodies || h->n < 1) return fail(h, AFMM_ESTATE, "bodies_buffer: no bodies set");
     if (dev_ptr) *dev_ptr = h->d_bodies;
-    if (bytes) *bytes = h->n * (long long)sizeof(float4);
+    if (bytes) *bytes = h->n * (long long)sizeof(float4) * words_of(h);
     return AFMM_OK;
 }
 
@@ -802,7 +833,8 @@ static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, flo
     p.az = az;
     p.phi = phi;
     p.eps2 = h->cfg.eps2;
-    p.G = (double)h->cfg.G;
+    p.G = h->cfg.law == AFMM_LAW_STOKESLET ? 1.0 / (8.0 * 3.14159265358979323846 * (double)h->cfg.mu)
+                                           : (double)h->cfg.G;
     CUDA_TRY(h, cudaMemsetAsync(h->d_queue, 0, sizeof(int), h->stream));
     const int ri = (int)(h->n_evals % afmm_p2p::kRing);
     h->ev0 = h->ring0[ri];
@@ -812,7 +844,10 @@ static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, flo
     if (p.n_tasks > 0) {
         const int grid = std::max(1, std::min((p.n_tasks + afmm::kWarps - 1) / afmm::kWarps,
                                               h->num_sms * h->blocks_per_sm));
-        afmm::p2p_kernel<<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(p);
+        if (h->cfg.law == AFMM_LAW_STOKESLET)
+            afmm::p2p_kernel_t<afmm::Stokeslet><<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(p);
+        else
+            afmm::p2p_kernel_t<afmm::Gravity><<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(p);
         CUDA_TRY(h, cudaGetLastError());
         nlaunch = 1;
     }

@@ -85,7 +85,7 @@ struct P2PParams {
     int *queue;              // task counter, zeroed before launch
     float *ax, *ay, *az, *phi;
     float eps2;
-    double G;
+    double G;                // output scale: G (gravity) or 1/(8 pi mu) (Stokeslet)
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
@@ -155,6 +155,63 @@ __device__ __forceinline__ void interact2(const float4 q, const float2 nx, const
     az = __ffma2_rn(s, dz, az);
 }
 
+// ---- pair laws.  A source occupies kWords float4 in the staged ring; the
+// four fp32 partial pairs are (ax, ay, az, phi) for gravity and (ux, uy, uz, -)
+// for Stokeslets.
+struct Gravity {
+    static constexpr int kWords = 1;
+    static constexpr bool kMaskSelf = true;        // reading R2: the j == i pair is excluded
+    template <bool kMasked>
+    __device__ __forceinline__ static void apply(const float4 *__restrict__ src, int k, const float2 nx,
+                                                 const float2 ny, const float2 nz, const float2 e2, float2 &a0,
+                                                 float2 &a1, float2 &a2, float2 &a3, bool s0, bool s1) {
+        interact2<kMasked>(src[k], nx, ny, nz, e2, a0, a1, a2, a3, s0, s1);
+    }
+    // a = G v, phi = -G v
+    __device__ __forceinline__ static float out(int comp, double v, double scale) {
+        return (float)(comp == 3 ? -scale * v : scale * v);
+    }
+};
+
+// Regularized Stokeslet (reading R26; PAPER L22 SVIII.B "method of regularized
+// Stokeslets as described in [15]"): u_i += [f_k (r^2 + 2 e^2) + (f_k . d) d] /
+// (r^2 + e^2)^{3/2} (times 1/(8 pi mu) at the end); the self term is finite and
+// included.  Source words: {x, y, z, fx}, {fy, fz, 0, 0}.  Per two interactions:
+// 19 packed FP32 ops + 2 MUFU.RSQ.
+struct Stokeslet {
+    static constexpr int kWords = 2;
+    static constexpr bool kMaskSelf = false;
+    template <bool kMasked>
+    __device__ __forceinline__ static void apply(const float4 *__restrict__ src, int k, const float2 nx,
+                                                 const float2 ny, const float2 nz, const float2 e2, float2 &ux,
+                                                 float2 &uy, float2 &uz, float2 &, bool, bool) {
+        const float4 q0 = src[2 * k], q1 = src[2 * k + 1];
+        const float2 dx = __fadd2_rn(make_float2(q0.x, q0.x), nx);
+        const float2 dy = __fadd2_rn(make_float2(q0.y, q0.y), ny);
+        const float2 dz = __fadd2_rn(make_float2(q0.z, q0.z), nz);
+        float2 r2 = __ffma2_rn(dx, dx, e2);                      // r^2 + e^2
+        r2 = __ffma2_rn(dy, dy, r2);
+        r2 = __ffma2_rn(dz, dz, r2);
+        float2 inv;
+        inv.x = rsqrt_ftz(r2.x);
+        inv.y = rsqrt_ftz(r2.y);
+        const float2 i3 = __fmul2_rn(__fmul2_rn(inv, inv), inv);  // (r^2 + e^2)^{-3/2}
+        const float2 fx = make_float2(q0.w, q0.w), fy = make_float2(q1.x, q1.x), fz = make_float2(q1.y, q1.y);
+        float2 fd = __fmul2_rn(fx, dx);
+        fd = __ffma2_rn(fy, dy, fd);
+        fd = __ffma2_rn(fz, dz, fd);
+        const float2 a = __ffma2_rn(e2, i3, inv);                 // (r^2 + 2 e^2) (r^2 + e^2)^{-3/2}
+        const float2 b = __fmul2_rn(fd, i3);                      // (f . d) (r^2 + e^2)^{-3/2}
+        ux = __ffma2_rn(b, dx, __ffma2_rn(a, fx, ux));
+        uy = __ffma2_rn(b, dy, __ffma2_rn(a, fy, uy));
+        uz = __ffma2_rn(b, dz, __ffma2_rn(a, fz, uz));
+    }
+    // u = v / (8 pi mu); the fourth output is zero
+    __device__ __forceinline__ static float out(int comp, double v, double scale) {
+        return comp == 3 ? 0.0f : (float)(scale * v);
+    }
+};
+
 // Targets of one lane: kPairs FFMA2 pairs (negated coordinates) and the
 // staged-list index of each target (-1: padding slot).
 struct Targets {
@@ -189,7 +246,7 @@ struct Partial {
 // Consume sources src[k], k = k0, k0+C, ... < kend; fp32 partials are folded
 // into fp64 before they would exceed kFold sources.  Masks compare k with
 // T.m[j] - moff.
-template <bool kMasked>
+template <class Law, bool kMasked>
 __device__ __forceinline__ void consume(const float4 *__restrict__ src, int k, int kend, int C,
                                         const Targets &T, int moff, const float2 e2, Partial &P) {
     while (k < kend) {
@@ -198,11 +255,11 @@ __device__ __forceinline__ void consume(const float4 *__restrict__ src, int k, i
         int iters = 0;
 #pragma unroll kUnroll
         for (; k < kstop; k += C) {
-            const float4 q4 = src[k];
 #pragma unroll
             for (int q = 0; q < kPairs; ++q)
-                interact2<kMasked>(q4, T.nx[q], T.ny[q], T.nz[q], e2, P.ax[q], P.ay[q], P.az[q], P.ph[q],
-                                   kMasked && k == T.m[2 * q] - moff, kMasked && k == T.m[2 * q + 1] - moff);
+                Law::template apply<kMasked>(src, k, T.nx[q], T.ny[q], T.nz[q], e2, P.ax[q], P.ay[q], P.az[q],
+                                             P.ph[q], kMasked && k == T.m[2 * q] - moff,
+                                             kMasked && k == T.m[2 * q + 1] - moff);
             ++iters;
         }
         P.cnt += iters;
@@ -238,10 +295,11 @@ __device__ __forceinline__ void load_task(const P2PParams &p, int id, Task &t, S
 
 // Stage the next chunk (<= kWCap bodies) of the stream into `buf`; returns
 // false when no task is left.
+template <int kWords>
 __device__ __forceinline__ bool issue_chunk(const P2PParams &p, Stream &S, float4 *buf, uint64_t *bar,
                                             ChunkMeta *meta, int lane) {
     if (S.task >= p.n_tasks) return false;
-    const int nb = min(kWCap, S.t.nsrc - S.staged);
+    const int nb = min(kWCap / kWords, S.t.nsrc - S.staged);
     if (lane == 0) {
         ChunkMeta m;
         m.tgt_start = S.t.tgt_start;
@@ -254,7 +312,7 @@ __device__ __forceinline__ bool issue_chunk(const P2PParams &p, Stream &S, float
         m.is_last = S.staged + nb >= S.t.nsrc;
         *meta = m;
         fence_proxy_async();
-        mbar_arrive_expect_tx(bar, (uint32_t)nb * 16u);
+        mbar_arrive_expect_tx(bar, (uint32_t)nb * 16u * kWords);
     }
     // pieces of the current segments (warp-uniform walk; lane 0 issues)
     int filled = 0;
@@ -267,7 +325,9 @@ __device__ __forceinline__ bool issue_chunk(const P2PParams &p, Stream &S, float
             len = s2.len;
         }
         const int take = min(len - S.ioff, nb - filled);
-        if (lane == 0) tma_load_1d(buf + filled, p.bodies + gstart + S.ioff, (uint32_t)take * 16u, bar);
+        if (lane == 0)
+            tma_load_1d(buf + (size_t)filled * kWords, p.bodies + (size_t)(gstart + S.ioff) * kWords,
+                        (uint32_t)take * 16u * kWords, bar);
         filled += take;
         S.ioff += take;
         if (S.ioff == len) {
@@ -289,6 +349,7 @@ __device__ __forceinline__ bool issue_chunk(const P2PParams &p, Stream &S, float
 
 // Load this lane's targets (4 consecutive of the n targets of the task): from
 // the staged self leaf when present in this stage, else from global memory.
+template <int kWords>
 __device__ __forceinline__ void load_targets(Targets &T, const float4 *__restrict__ stage,
                                              const float4 *__restrict__ bodies, const ChunkMeta &m,
                                              int l, bool active) {
@@ -301,7 +362,7 @@ __device__ __forceinline__ void load_targets(Targets &T, const float4 *__restric
             const int j = 2 * q + h;
             const int i = min(kTPT * l + j, m.tgt_count - 1);     // padding slots repeat the last target
             T.m[j] = (kTPT * l + j < m.tgt_count) ? m.toff + i : -1;
-            if (active) b[h] = staged ? stage[m.toff + i] : bodies[m.tgt_start + i];
+            if (active) b[h] = staged ? stage[(size_t)(m.toff + i) * kWords] : bodies[(size_t)(m.tgt_start + i) * kWords];
             else b[h] = make_float4(0.f, 0.f, 0.f, 0.f);
         }
         T.nx[q] = make_float2(-b[0].x, -b[1].x);
@@ -310,7 +371,8 @@ __device__ __forceinline__ void load_targets(Targets &T, const float4 *__restric
     }
 }
 
-__global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel(const P2PParams p) {
+template <class Law>
+__global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const P2PParams p) {
     extern __shared__ __align__(128) unsigned char dsmem[];
     __shared__ __align__(8) uint64_t full_all[kWarps][kWStages];
     __shared__ ChunkMeta meta_all[kWarps][kWStages];
@@ -334,7 +396,8 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel(const P2
     S.iseg = S.ioff = S.staged = 0;
     int issued = 0;
     for (; issued < kWStages - 1; ++issued)
-        if (!issue_chunk(p, S, stage[issued % kWStages], &full[issued % kWStages], &meta[issued % kWStages], lane))
+        if (!issue_chunk<Law::kWords>(p, S, stage[issued % kWStages], &full[issued % kWStages],
+                                      &meta[issued % kWStages], lane))
             break;
 
     const float2 e2 = make_float2(p.eps2, p.eps2);
@@ -347,7 +410,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel(const P2
         // keep the ring one chunk ahead (across task boundaries)
         if (issued == q + kWStages - 1) {
             const int s2 = issued % kWStages;
-            if (issue_chunk(p, S, stage[s2], &full[s2], &meta[s2], lane)) ++issued;
+            if (issue_chunk<Law::kWords>(p, S, stage[s2], &full[s2], &meta[s2], lane)) ++issued;
         }
         const int st = q % kWStages;
         mbar_wait(&full[st], (uint32_t)((q / kWStages) & 1));
@@ -358,16 +421,16 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel(const P2
             c = lane / g;
             l = lane - c * g;
             active = c < C;
-            load_targets(T, stage[st], p.bodies, m, l, active);
+            load_targets<Law::kWords>(T, stage[st], p.bodies, m, l, active);
 #pragma unroll
             for (int u = 0; u < kVals; ++u) accw[u * 32 + lane] = 0.0;
             P.clear();
         }
         if (active) {
-            const int kself = min(max(m.self_len - m.first, 0), m.nb);
-            if (kself > 0) consume<true>(stage[st], c, kself, C, T, m.first, e2, P);
+            const int kself = Law::kMaskSelf ? min(max(m.self_len - m.first, 0), m.nb) : 0;
+            if (kself > 0) consume<Law, true>(stage[st], c, kself, C, T, m.first, e2, P);
             const int k0 = kself + ((c - kself) % C + C) % C;        // first k >= kself, k = c (mod C)
-            consume<false>(stage[st], k0, m.nb, C, T, 0, e2, P);
+            consume<Law, false>(stage[st], k0, m.nb, C, T, 0, e2, P);
         }
         if (m.is_last) {
             if (active) P.fold();
@@ -382,11 +445,23 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel(const P2
                 if (tgt < m.tgt_count) {
                     const int comp = u & 3;
                     float *dst = comp == 0 ? p.ax : comp == 1 ? p.ay : comp == 2 ? p.az : p.phi;
-                    dst[m.tgt_start + tgt] = (float)(comp == 3 ? -p.G * v : p.G * v);
+                    dst[m.tgt_start + tgt] = Law::out(comp, v, p.G);
                 }
             }
         }
         __syncwarp();                     // stage st (and the accumulators) free again
+    }
+}
+
+// Stokeslet bodies: {x, y, z, fx}, {fy, fz, 0, 0}
+__global__ void pack_stokeslet_kernel(long long n, const float *__restrict__ x, const float *__restrict__ y,
+                                      const float *__restrict__ z, const float *__restrict__ fx,
+                                      const float *__restrict__ fy, const float *__restrict__ fz,
+                                      float4 *__restrict__ out) {
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n;
+         i += (long long)gridDim.x * blockDim.x) {
+        out[2 * i] = make_float4(x[i], y[i], z[i], fx[i]);
+        out[2 * i + 1] = make_float4(fy[i], fz[i], 0.f, 0.f);
     }
 }
 

@@ -34,3 +34,22 @@ def check(gpu, ref, A, rel=REL):
     assert (ea[well] <= rel).all(), stats
     assert (da[~well] <= ABS_A * A[~well] + 1e-300).all(), stats
     return stats
+
+
+def check_vec(gpu, ref, A, rel=REL):
+    """Vector-only version of `check` (Stokeslet velocities): gpu/ref = (ux, uy, uz)."""
+    u = np.stack([np.asarray(v, np.float64) for v in gpu], 1)
+    r = np.stack([np.asarray(v, np.float64) for v in ref], 1)
+    du = np.linalg.norm(u - r, axis=1)
+    nr = np.linalg.norm(r, axis=1)
+    glob = np.linalg.norm(u - r) / max(np.linalg.norm(r), 1e-300)
+    kappa = np.where(nr > 0, A / np.where(nr > 0, nr, 1.0), np.inf)
+    well = kappa <= KAPPA
+    eu = np.where(nr > 0, du / np.where(nr > 0, nr, 1.0), 0.0)
+    stats = {"u_global_rel": float(glob), "u_max_rel_well": float(eu[well].max()) if well.any() else 0.0,
+             "n_ill": int((~well).sum())}
+    assert np.isfinite(u).all(), stats
+    assert glob <= rel, stats
+    assert (eu[well] <= rel).all(), stats
+    assert (du[~well] <= ABS_A * A[~well] + 1e-300).all(), stats
+    return stats

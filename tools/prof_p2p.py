@@ -19,10 +19,15 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="C2")
 ap.add_argument("--S", type=int, default=None)
 ap.add_argument("--evals", type=int, default=4)
+ap.add_argument("--law", default="gravity", choices=["gravity", "stokeslet"])
 a = ap.parse_args()
 c = synth.CONFIGS[a.config]
 S = a.S or c["S"]
-x, y, z, m = synth.make(a.config)
+if a.law == "stokeslet":
+    x, y, z, fx, fy, fz = synth.uniform_with_forces(c["n"], c["seed"])
+    m = fx
+else:
+    x, y, z, m = synth.make(a.config)
 n = x.shape[0]
 dev = torch.device("cuda", 0)
 st = torch.cuda.Stream(dev)
@@ -34,8 +39,16 @@ T = t.copy_out(n)
 b = torch.empty((4, n), device=dev)
 for i, s in enumerate((X, Y, Z, M)):
     t.gather(s, b[i])
-h = afmm.P2P(eps2=c["eps2"], stream=st.cuda_stream)
-h.set_bodies(b[0], b[1], b[2], b[3])
+if a.law == "stokeslet":
+    F = [torch.from_numpy(v).to(dev) for v in (fx, fy, fz)]
+    Fs = torch.empty((3, n), device=dev)
+    for i in range(3):
+        t.gather(F[i], Fs[i])
+    h = afmm.P2P(eps2=c["eps2"], stream=st.cuda_stream, law=afmm.LAW_STOKESLET)
+    h.set_bodies_stokeslet(b[0], b[1], b[2], Fs[0], Fs[1], Fs[2])
+else:
+    h = afmm.P2P(eps2=c["eps2"], stream=st.cuda_stream)
+    h.set_bodies(b[0], b[1], b[2], b[3])
 h.set_tree(T["leaf_start"], T["leaf_count"], T["u_off"], T["u_idx"])
 out = torch.empty((4, n), device=dev)
 for _ in range(a.evals):
