@@ -70,6 +70,8 @@ def _L():
         lib.oracle_stokeslet.restype = None
         lib.oracle_stokeslet.argtypes = [i64, p, p, p, p, p, p, i64, p, p, p, p, C.c_double, C.c_double,
                                          i64, p, p, p, p, p]
+        lib.oracle_farfield_counts.restype = None
+        lib.oracle_farfield_counts.argtypes = [p, p]
         lib.oracle_partition_literal.restype = None
         lib.oracle_partition_literal.argtypes = [i64, p, C.c_int, p, p]
         _lib = lib
@@ -146,6 +148,12 @@ class Tree:
         if not h:
             raise ValueError("oracle_tree_enforce failed")
         return Tree(S=S, ulist=ulist, _handle=h, _n=x.shape[0])
+
+    def farfield_counts(self):
+        """M(Op) for P2M, M2M, M2L, L2L, L2P, P2P (L18 SIV.D; reading R27)."""
+        out = np.zeros(6, np.int64)
+        _L().oracle_farfield_counts(self._h, _ptr(out))
+        return out
 
     def __del__(self):
         if getattr(self, "_h", None) and _lib is not None:

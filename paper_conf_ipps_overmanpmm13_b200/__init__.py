@@ -101,6 +101,7 @@ _sig("afmm_version", C.c_char_p)
 _sig("afmm_tree_create", _i, _i, _p, C.POINTER(_p))
 _sig("afmm_tree_build", _i, _p, _ll, _p, _p, _p, _i, _i, _p, _i)
 _sig("afmm_tree_enforce", _i, _p, _ll, _p, _p, _p, _i)
+_sig("afmm_tree_farfield_counts", _i, _p, _p)
 _sig("afmm_tree_info", _i, _p, C.POINTER(_i), C.POINTER(_ll), _p, C.POINTER(_i), C.POINTER(_i),
      C.POINTER(_ll))
 _sig("afmm_tree_copy_out", _i, _p, _p, _p, _p, _p, _p, _p, _p)
@@ -108,6 +109,20 @@ _sig("afmm_tree_gather", _i, _p, _p, _p)
 _sig("afmm_tree_scatter", _i, _p, _p, _p)
 _sig("afmm_tree_destroy", None, _p)
 _sig("afmm_tree_last_error", C.c_char_p, _p)
+
+class LbConfig(C.Structure):
+    _fields_ = [("S_init", C.c_int), ("S_min", C.c_int), ("S_max", C.c_int), ("dS", C.c_int),
+                ("balance_rel", C.c_double), ("observe_rel", C.c_double)]
+
+
+LB_SEARCH, LB_INCREMENTAL, LB_OBSERVATION = 0, 1, 2
+LB_KEEP, LB_REBUILD, LB_ENFORCE, LB_FINE = 0, 1, 2, 3
+_sig("afmm_lb_config_init", _i, C.POINTER(LbConfig))
+_sig("afmm_lb_create", _i, C.POINTER(LbConfig), C.POINTER(_p))
+_sig("afmm_lb_step", _i, _p, _d, _d, C.POINTER(_i), C.POINTER(_i))
+_sig("afmm_lb_predicted", _i, _p, _d, C.POINTER(_i))
+_sig("afmm_lb_state", _i, _p, C.POINTER(_i), C.POINTER(_i), C.POINTER(_d))
+_sig("afmm_lb_destroy", None, _p)
 
 # every symbol include/*.h declares (checked by tests/test_abi.py)
 EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
@@ -121,7 +136,9 @@ EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
             "afmm_partition_literal", "afmm_partition_weighted", "afmm_partition_rebalance",
             "afmm_cost_fit", "afmm_p2p_set_cost_coef", "afmm_kick", "afmm_drift",
             "afmm_fp32_peak", "afmm_version",
-            "afmm_tree_create", "afmm_tree_build", "afmm_tree_enforce", "afmm_tree_info", "afmm_tree_copy_out",
+            "afmm_tree_create", "afmm_tree_build", "afmm_tree_enforce", "afmm_tree_info",
+            "afmm_tree_farfield_counts", "afmm_lb_config_init", "afmm_lb_create", "afmm_lb_step",
+            "afmm_lb_predicted", "afmm_lb_state", "afmm_lb_destroy", "afmm_tree_copy_out",
             "afmm_tree_gather", "afmm_tree_scatter", "afmm_tree_destroy", "afmm_tree_last_error"]
 
 
@@ -432,6 +449,12 @@ class GpuTree:
         out.update(inf)
         return out
 
+    def farfield_counts(self):
+        """M(Op) = [P2M, M2M, M2L, L2L, L2P, P2P] of the last build (L18 SIV.D)."""
+        out = np.zeros(6, np.int64)
+        self._check(_lib.afmm_tree_farfield_counts(self._h, _ptr(out)), "afmm_tree_farfield_counts")
+        return out
+
     def device_arrays(self):
         """Device pointers (ints) of the last build: perm, leaf_start, leaf_count, u_off, u_idx."""
         ps = [_p() for _ in range(5)]
@@ -444,3 +467,46 @@ class GpuTree:
 
     def scatter(self, src, dst):
         self._check(_lib.afmm_tree_scatter(self._h, _ptr(src), _ptr(dst)), "afmm_tree_scatter")
+
+
+# ------------------------------------------------------------------ load balancer (row f3)
+
+class LoadBalancer:
+    """afmm_lb: the paper's Search / Incremental / Observation controller (L18 SV, L20-L22)."""
+
+    def __init__(self, S_init=128, S_min=8, S_max=2048, dS=8, balance_rel=0.15, observe_rel=0.05):
+        cfg = LbConfig()
+        _lib.afmm_lb_config_init(C.byref(cfg))
+        cfg.S_init, cfg.S_min, cfg.S_max, cfg.dS = int(S_init), int(S_min), int(S_max), int(dS)
+        cfg.balance_rel, cfg.observe_rel = float(balance_rel), float(observe_rel)
+        h = _p()
+        st = _lib.afmm_lb_create(C.byref(cfg), C.byref(h))
+        if st:
+            raise AfmmError(st, "afmm_lb_create")
+        self._h = h
+
+    def step(self, t_cpu, t_gpu):
+        a, S = _i(), _i()
+        st = _lib.afmm_lb_step(self._h, float(t_cpu), float(t_gpu), C.byref(a), C.byref(S))
+        if st:
+            raise AfmmError(st, "afmm_lb_step")
+        return a.value, S.value
+
+    def predicted(self, t_pred):
+        a = _i()
+        st = _lib.afmm_lb_predicted(self._h, float(t_pred), C.byref(a))
+        if st:
+            raise AfmmError(st, "afmm_lb_predicted")
+        return a.value
+
+    def state(self):
+        s, S, b = _i(), _i(), _d()
+        _lib.afmm_lb_state(self._h, C.byref(s), C.byref(S), C.byref(b))
+        return {"state": s.value, "S": S.value, "best": b.value}
+
+    def close(self):
+        if getattr(self, "_h", None) and _lib is not None:
+            _lib.afmm_lb_destroy(self._h)
+        self._h = None
+
+    __del__ = close

@@ -260,6 +260,67 @@ __global__ void leaf_node_kernel(int nn, const int *__restrict__ node_leaf, int 
     if (l >= 0) leaf_node[l] = i;
 }
 
+// index of (lev, prefix) among the previous build's nodes, or -1
+__device__ __forceinline__ long long find_node(const PrevTree &pv, int lev, unsigned long long prefix) {
+    if (lev >= pv.levels || lev < 0) return -1;
+    long long lo = pv.base[lev], hi = pv.base[lev + 1];
+    while (lo < hi) {
+        const long long mid = lo + ((hi - lo) >> 1);
+        if (pv.prefix[mid] < prefix) lo = mid + 1;
+        else hi = mid;
+    }
+    return (lo < pv.base[lev + 1] && pv.prefix[lo] == prefix) ? lo : -1;
+}
+
+// M2L count (L18 SIV.D M(Op); reading R27): for node b (level >= 2), the
+// children of the colleagues of parent(b) -- same-level nodes in the 3x3x3
+// cells around it, parent included -- whose boxes do not touch b.
+__global__ void vlist_count_kernel(long long nn, PrevTree pv, unsigned long long *__restrict__ out) {
+    const long long b = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (b >= nn) return;
+    int lev = 0;
+    while (lev + 1 < pv.levels && pv.base[lev + 1] <= b) ++lev;
+    if (lev < 2) return;
+    const unsigned long long pre = pv.prefix[b];
+    long long Ab[3], wb;
+    box_of(lev, pre, Ab, wb);
+    const int plev = lev - 1;
+    const unsigned long long ppre = pre >> 3;
+    const long long pc[3] = {(long long)compact3(ppre), (long long)compact3(ppre >> 1), (long long)compact3(ppre >> 2)};
+    const long long M = 1LL << plev;
+    unsigned long long cnt = 0;
+    for (int dz = -1; dz <= 1; ++dz)
+        for (int dy = -1; dy <= 1; ++dy)
+            for (int dx = -1; dx <= 1; ++dx) {
+                const long long qx = pc[0] + dx, qy = pc[1] + dy, qz = pc[2] + dz;
+                if (qx < 0 || qy < 0 || qz < 0 || qx >= M || qy >= M || qz >= M) continue;
+                const unsigned long long qpre = spread3(qx) | (spread3(qy) << 1) | (spread3(qz) << 2);
+                const long long q = find_node(pv, plev, qpre);
+                if (q < 0 || pv.nchild[q] == 0) continue;
+                for (int o = 0; o < 8; ++o) {
+                    const unsigned long long cpre = (qpre << 3) | (unsigned long long)o;
+                    if (find_node(pv, lev, cpre) < 0) continue;
+                    long long Ac[3], wc;
+                    box_of(lev, cpre, Ac, wc);
+                    bool touch = true;
+#pragma unroll
+                    for (int a = 0; a < 3; ++a) touch &= (Ab[a] <= Ac[a] + wc) && (Ac[a] <= Ab[a] + wb);
+                    cnt += !touch;
+                }
+            }
+    if (cnt) atomicAdd(out, cnt);
+}
+
+// sum_t n_t * sum_{s in U(t)} n_s
+__global__ void p2p_count_kernel(int L, const int *__restrict__ lc, const long long *__restrict__ uo,
+                                 const int *__restrict__ ui, unsigned long long *__restrict__ out) {
+    const int t = blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= L) return;
+    unsigned long long src = 0;
+    for (long long u = uo[t]; u < uo[t + 1]; ++u) src += (unsigned long long)lc[ui[u]];
+    atomicAdd(out, src * (unsigned long long)lc[t]);
+}
+
 __global__ void gather_kernel(long long n, const int *__restrict__ perm, const float *__restrict__ in,
                               float *__restrict__ out) {
     for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n;
@@ -372,7 +433,8 @@ afmm_status wsalloc(afmm_tree *t, int slot, T **p, size_t count) {
 
 enum Slot {
     kPart, kKeys, kIdx, kKeysSorted, kPerm, kSortTmp, kNodeA, kNodeB = kNodeA + 6, kCb = kNodeB + 6, kNc, kOff,
-    kScanTmp, kFlag, kLeafAt, kNodeLeaf, kScan2, kLs, kLc, kLl, kLp, kLeafNode, kCounts, kUoff, kScan3, kUidx
+    kScanTmp, kFlag, kLeafAt, kNodeLeaf, kScan2, kLs, kLc, kLl, kLp, kLeafNode, kCounts, kUoff, kScan3, kUidx,
+    kFarfield
 };
 
 __global__ void root_kernel(Nodes nd, int n) {
@@ -683,6 +745,30 @@ extern "C" afmm_status afmm_tree_copy_out(const afmm_tree *tc, int *perm, int *l
     if (u_idx && t->nnz > 0)
         TCU(t, cudaMemcpyAsync(u_idx, t->u_idx, t->nnz * sizeof(int), cudaMemcpyDeviceToHost, st));
     TCU(t, cudaStreamSynchronize(st));
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_tree_farfield_counts(afmm_tree *t, long long *counts) {
+    if (!t || !counts) return AFMM_EINVAL;
+    if (!t->built) return AFMM_ESTATE;
+    TCU(t, cudaSetDevice(t->device));
+    unsigned long long *d = nullptr;
+    if (afmm_status s = wsalloc(t, kFarfield, &d, 2)) return s;
+    TCU(t, cudaMemsetAsync(d, 0, 2 * sizeof(unsigned long long), t->stream));
+    PrevTree pv{t->pv_prefix, t->pv_nchild, t->pv_base, t->pv_levels};
+    vlist_count_kernel<<<grid_for(t->n_nodes, 256), 256, 0, t->stream>>>(t->n_nodes, pv, d);
+    TCU(t, cudaGetLastError());
+    p2p_count_kernel<<<grid_for(t->L, 256), 256, 0, t->stream>>>(t->L, t->lc, t->u_off, t->u_idx, d + 1);
+    TCU(t, cudaGetLastError());
+    unsigned long long h[2];
+    TCU(t, cudaMemcpyAsync(h, d, sizeof(h), cudaMemcpyDeviceToHost, t->stream));
+    TCU(t, cudaStreamSynchronize(t->stream));
+    counts[0] = t->L;
+    counts[1] = t->n_nodes - 1;
+    counts[2] = (long long)h[0];
+    counts[3] = t->n_nodes - 1;
+    counts[4] = t->L;
+    counts[5] = (long long)h[1];
     return AFMM_OK;
 }
 

@@ -15,7 +15,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 def _declared():
     names = []
-    for h in ("afmm_p2p.h", "afmm_tree.h", "afmm_step.h"):
+    for h in ("afmm_p2p.h", "afmm_tree.h", "afmm_step.h", "afmm_balance.h"):
         src = open(os.path.join(ROOT, "include", h)).read()
         src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
         names += re.findall(r"\b(afmm_\w+)\s*\(", src)
