@@ -5,7 +5,7 @@ NVFLAGS   := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -Xcompiler -O2 --
 PKG       := paper_conf_ipps_overmanpmm13_b200
 SRC       := $(PKG)/csrc
 LIB       := $(PKG)/libafmm_p2p.so
-CU_SRCS   := $(SRC)/afmm_p2p.cu $(SRC)/peak.cu $(SRC)/tree_build.cu $(SRC)/step.cu $(SRC)/balance.cpp
+CU_SRCS   := $(SRC)/afmm_p2p.cu $(SRC)/peak.cu $(SRC)/tree_build.cu $(SRC)/step.cu $(SRC)/balance.cpp $(SRC)/finegrained.cpp
 CU_HDRS   := $(SRC)/p2p_kernel.cuh $(SRC)/worklist.inc $(SRC)/worklist_dev.cuh include/afmm_p2p.h include/afmm_tree.h include/afmm_step.h include/afmm_balance.h
 ORACLE    := oracle/liboracle.so
 

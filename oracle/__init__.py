@@ -63,6 +63,8 @@ def _L():
         lib.oracle_interactions.argtypes = [i64, p, p, p, p]
         lib.oracle_tree_enforce.restype = p
         lib.oracle_tree_enforce.argtypes = [p, i64, p, p, p, C.c_int]
+        lib.oracle_tree_rebuild.restype = p
+        lib.oracle_tree_rebuild.argtypes = [p, i64, p, p, p, C.c_int, C.c_int, i64, p, p, p]
         lib.oracle_kick.restype = None
         lib.oracle_kick.argtypes = [i64, p, p, p, p, p, p, C.c_double]
         lib.oracle_drift.restype = None
@@ -147,6 +149,21 @@ class Tree:
         h = _L().oracle_tree_enforce(self._h, x.shape[0], _ptr(x), _ptr(y), _ptr(z), S)
         if not h:
             raise ValueError("oracle_tree_enforce failed")
+        return Tree(S=S, ulist=ulist, _handle=h, _n=x.shape[0])
+
+    def rebuild(self, x, y, z, S=None, mode=2, edits=(), ulist=True):
+        """Rebuild for new positions with the previous structure (mode 2, KEEP)
+        or the Enforce_S rule (mode 1), then Collapse (1) / PushDown (2) edits
+        given as (level, prefix, action) triples (L18 SIV.B-C, L20 SVI.B; R27)."""
+        x, y, z = (_c(v, np.float32) for v in (x, y, z))
+        S = self.S if S is None else int(S)
+        lev = _c([e[0] for e in edits] or [0], np.int32)
+        pre = _c([e[1] for e in edits] or [0], np.uint64)
+        act = _c([e[2] for e in edits] or [0], np.int32)
+        h = _L().oracle_tree_rebuild(self._h, x.shape[0], _ptr(x), _ptr(y), _ptr(z), S, int(mode),
+                                     len(edits), _ptr(lev), _ptr(pre), _ptr(act))
+        if not h:
+            raise ValueError("oracle_tree_rebuild failed")
         return Tree(S=S, ulist=ulist, _handle=h, _n=x.shape[0])
 
     def farfield_counts(self):

@@ -124,6 +124,19 @@ _sig("afmm_lb_predicted", _i, _p, _d, C.POINTER(_i))
 _sig("afmm_lb_state", _i, _p, C.POINTER(_i), C.POINTER(_i), C.POINTER(_d))
 _sig("afmm_lb_destroy", None, _p)
 
+
+class FgResult(C.Structure):
+    _fields_ = [("direction", C.c_int), ("groups_tried", C.c_int), ("groups_applied", C.c_int),
+                ("nodes_changed", C.c_longlong), ("t_before", C.c_double), ("t_after", C.c_double),
+                ("t_cpu_after", C.c_double), ("t_gpu_after", C.c_double)]
+
+
+TREE_ENFORCE, TREE_KEEP = 1, 2
+COLLAPSE, PUSHDOWN = 1, 2
+_sig("afmm_tree_rebuild", _i, _p, _ll, _p, _p, _p, _i, _i, _i, _p, _p, _p)
+_sig("afmm_tree_nodes", _i, _p, _p, _p, _p)
+_sig("afmm_fine_grained", _i, _p, _ll, _p, _p, _p, _i, _p, _i, _d, _i, C.POINTER(FgResult))
+
 # every symbol include/*.h declares (checked by tests/test_abi.py)
 EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
             "afmm_p2p_set_bodies_host", "afmm_p2p_bodies_buffer", "afmm_p2p_set_tree",
@@ -139,7 +152,8 @@ EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
             "afmm_tree_create", "afmm_tree_build", "afmm_tree_enforce", "afmm_tree_info",
             "afmm_tree_farfield_counts", "afmm_lb_config_init", "afmm_lb_create", "afmm_lb_step",
             "afmm_lb_predicted", "afmm_lb_state", "afmm_lb_destroy", "afmm_tree_copy_out",
-            "afmm_tree_gather", "afmm_tree_scatter", "afmm_tree_destroy", "afmm_tree_last_error"]
+            "afmm_tree_gather", "afmm_tree_scatter", "afmm_tree_destroy", "afmm_tree_last_error",
+            "afmm_tree_rebuild", "afmm_tree_nodes", "afmm_fine_grained"]
 
 
 def version() -> str:
@@ -425,6 +439,35 @@ class GpuTree:
         self._check(_lib.afmm_tree_enforce(self._h, int(x.shape[0]), _ptr(x), _ptr(y), _ptr(z), int(S)),
                     "afmm_tree_enforce")
         return self.info()
+
+    def rebuild(self, x, y, z, S, mode=TREE_KEEP, edits=()):
+        """afmm_tree_rebuild: previous structure (TREE_KEEP) or Enforce_S rule
+        (TREE_ENFORCE), then (level, prefix, COLLAPSE|PUSHDOWN) edits."""
+        lev = _np([e[0] for e in edits] or [0], np.int32)
+        pre = _np([e[1] for e in edits] or [0], np.uint64)
+        act = _np([e[2] for e in edits] or [0], np.int32)
+        self._check(_lib.afmm_tree_rebuild(self._h, int(x.shape[0]), _ptr(x), _ptr(y), _ptr(z), int(S), int(mode),
+                                           len(edits), _ptr(lev), _ptr(pre), _ptr(act)), "afmm_tree_rebuild")
+        return self.info()
+
+    def nodes(self):
+        """All nodes of the last build: level, prefix, nchild (numpy)."""
+        nn = self.info()["n_nodes"]
+        out = {"level": np.empty(nn, np.int32), "prefix": np.empty(nn, np.uint64), "nchild": np.empty(nn, np.int32)}
+        self._check(_lib.afmm_tree_nodes(self._h, _ptr(out["level"]), _ptr(out["prefix"]), _ptr(out["nchild"])),
+                    "afmm_tree_nodes")
+        return out
+
+    def fine_grained(self, x, y, z, S, coef, direction=0, group_frac=0.05, max_groups=16):
+        """FineGrainedOptimize (afmm_fine_grained, L20 SVI.B) -> result dict."""
+        c = _np(coef, np.float64)
+        if c.shape != (6,):
+            raise ValueError("coef must hold 6 values (P2M, M2M, M2L, L2L, L2P, P2P)")
+        r = FgResult()
+        self._check(_lib.afmm_fine_grained(self._h, int(x.shape[0]), _ptr(x), _ptr(y), _ptr(z), int(S), _ptr(c),
+                                           int(direction), float(group_frac), int(max_groups), C.byref(r)),
+                    "afmm_fine_grained")
+        return {k: getattr(r, k) for k, _ in FgResult._fields_}
 
     def info(self):
         L, nnz, k, ml, nn = _i(), _ll(), _i(), _i(), _ll()

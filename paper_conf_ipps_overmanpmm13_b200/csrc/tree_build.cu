@@ -124,20 +124,53 @@ __device__ __forceinline__ bool prev_internal(const PrevTree &pv, int lev, unsig
     return lo < pv.base[lev + 1] && pv.prefix[lo] == prefix && pv.nchild[lo] > 0;
 }
 
+// Per-node edits of FineGrainedOptimize (L20 SVI.B): per level, ascending
+// prefixes with an action (1 = Collapse: stay a leaf, 2 = PushDown: split).
+struct Edits {
+    const unsigned long long *prefix;
+    const int *action;
+    const long long *base;      // device, kMaxLevel + 2 entries
+    int n;                      // 0: none
+};
+
+__device__ __forceinline__ int edit_of(const Edits &ed, int lev, unsigned long long prefix) {
+    long long lo = ed.base[lev], hi = ed.base[lev + 1];
+    const long long end = hi;
+    while (lo < hi) {
+        const long long mid = lo + ((hi - lo) >> 1);
+        if (ed.prefix[mid] < prefix) lo = mid + 1;
+        else hi = mid;
+    }
+    return (lo < end && ed.prefix[lo] == prefix) ? ed.action[lo] : 0;
+}
+
+enum { kModeFresh = 0, kModeEnforce = 1, kModeKeep = 2 };
+
 // For each node of the current level: split if > S bodies and level < 21
 // (L10 SI.B).  Enforce_S (L20 SVI.A; pv.levels > 0) additionally keeps a node
 // with exactly S bodies split when it was a parent before: Collapse applies only
 // to parents with FEWER than S bodies, PushDown only to leaves with MORE than S.
 // Child ranges by binary search on the octant digit inside [b, e).
 __global__ void split_count_kernel(int m, int base, Nodes nd, const unsigned long long *__restrict__ keys,
-                                   int S, PrevTree pv, int *__restrict__ cb, int *__restrict__ nc) {
+                                   int S, int mode, PrevTree pv, Edits ed, int *__restrict__ cb,
+                                   int *__restrict__ nc) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= m) return;
     const int id = base + i;
     const int b = nd.b[id], e = nd.e[id], lev = nd.level[id];
     int cnt = 0;
-    const bool split = lev < kMaxLevel &&
-                       (e - b > S || (e - b == S && pv.levels > 0 && prev_internal(pv, lev, nd.prefix[id])));
+    bool split;
+    if (mode == kModeKeep)            // structure kept: split iff it was a parent (Collapse/PushDown edits below)
+        split = pv.levels > 0 && prev_internal(pv, lev, nd.prefix[id]);
+    else
+        split = e - b > S || (mode == kModeEnforce && e - b == S && pv.levels > 0 &&
+                              prev_internal(pv, lev, nd.prefix[id]));
+    if (ed.n > 0) {
+        const int a = edit_of(ed, lev, nd.prefix[id]);
+        if (a == 1) split = false;
+        else if (a == 2) split = true;
+    }
+    split = split && lev < kMaxLevel;
     if (split) {
         const int shift = 3 * (kMaxLevel - 1 - lev);
         int bound[9];
@@ -434,7 +467,7 @@ afmm_status wsalloc(afmm_tree *t, int slot, T **p, size_t count) {
 enum Slot {
     kPart, kKeys, kIdx, kKeysSorted, kPerm, kSortTmp, kNodeA, kNodeB = kNodeA + 6, kCb = kNodeB + 6, kNc, kOff,
     kScanTmp, kFlag, kLeafAt, kNodeLeaf, kScan2, kLs, kLc, kLl, kLp, kLeafNode, kCounts, kUoff, kScan3, kUidx,
-    kFarfield
+    kFarfield, kEditPrefix, kEditAction, kEditBase
 };
 
 __global__ void root_kernel(Nodes nd, int n) {
@@ -487,7 +520,8 @@ extern "C" void afmm_tree_destroy(afmm_tree *t) {
 extern "C" const char *afmm_tree_last_error(const afmm_tree *t) { return t ? t->err.c_str() : "null handle"; }
 
 static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const float *y, const float *z,
-                              int S, int fixed_domain, const double *lo_in, int k_in, bool enforce) {
+                              int S, int fixed_domain, const double *lo_in, int k_in, int mode,
+                              Edits ed = Edits{nullptr, nullptr, nullptr, 0}) {
     if (!t) return AFMM_EINVAL;
     if (t->poisoned) return AFMM_ESTATE;
     if (n < 1 || n >= (1LL << 31)) return tfail(t, AFMM_EINVAL, "tree_build: n=%lld out of range", n);
@@ -565,7 +599,7 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     if (afmm_status s = alloc_nodes(cap, nd, node_set)) return s;
     root_kernel<<<1, 1, 0, st>>>(nd, (int)n);
     TCU(t, cudaGetLastError());
-    PrevTree pv{t->pv_prefix, t->pv_nchild, t->pv_base, enforce ? t->pv_levels : 0};
+    PrevTree pv{t->pv_prefix, t->pv_nchild, t->pv_base, mode != kModeFresh ? t->pv_levels : 0};
     std::vector<long long> lvl_base;
     long long base = 0, m = 1;     // current level occupies [base, base+m)
     int level = 0;
@@ -586,7 +620,8 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
                 scan_tmp_bytes = need;
             }
         }
-        split_count_kernel<<<grid_for(m, TH), TH, 0, st>>>((int)m, (int)base, nd, t->keys_sorted, S, pv, cb, nc);
+        split_count_kernel<<<grid_for(m, TH), TH, 0, st>>>((int)m, (int)base, nd, t->keys_sorted, S, mode, pv, ed,
+                                                            cb, nc);
         TCU(t, cudaGetLastError());
         TCU(t, cudaMemsetAsync(nc + m, 0, sizeof(int), st));
         size_t sb = scan_tmp_bytes;
@@ -697,7 +732,7 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
 extern "C" afmm_status afmm_tree_build(afmm_tree *t, long long n, const float *x, const float *y,
                                        const float *z, int S, int fixed_domain, const double *lo_in,
                                        int k_in) {
-    return build_impl(t, n, x, y, z, S, fixed_domain, lo_in, k_in, false);
+    return build_impl(t, n, x, y, z, S, fixed_domain, lo_in, k_in, kModeFresh);
 }
 
 // Enforce_S (PAPER L20 SVI.A): the tree the last build becomes after its bodies
@@ -710,7 +745,71 @@ extern "C" afmm_status afmm_tree_enforce(afmm_tree *t, long long n, const float 
     if (!t->built || t->pv_levels < 1) return tfail(t, AFMM_ESTATE, "tree_enforce: no previous tree");
     if (n != t->n) return tfail(t, AFMM_EINVAL, "tree_enforce: n=%lld differs from the previous tree (%lld)", n, t->n);
     const double lo[3] = {t->lo[0], t->lo[1], t->lo[2]};
-    return build_impl(t, n, x, y, z, S, 1, lo, t->k, true);
+    return build_impl(t, n, x, y, z, S, 1, lo, t->k, kModeEnforce);
+}
+
+// Rebuild with per-node edits (Collapse / PushDown, L18 SIV.B-C) on top of the
+// KEEP (structure of the last build) or ENFORCE rule -- FineGrainedOptimize's
+// primitive (L20 SVI.B).
+extern "C" afmm_status afmm_tree_rebuild(afmm_tree *t, long long n, const float *x, const float *y,
+                                         const float *z, int S, int mode, int n_edits, const int *edit_level,
+                                         const unsigned long long *edit_prefix, const int *edit_action) {
+    if (!t) return AFMM_EINVAL;
+    if (t->poisoned) return AFMM_ESTATE;
+    if (!t->built || t->pv_levels < 1) return tfail(t, AFMM_ESTATE, "tree_rebuild: no previous tree");
+    if (n != t->n) return tfail(t, AFMM_EINVAL, "tree_rebuild: n=%lld differs from the previous tree", n);
+    if (mode != AFMM_TREE_KEEP && mode != AFMM_TREE_ENFORCE) return tfail(t, AFMM_EINVAL, "tree_rebuild: bad mode");
+    if (n_edits < 0 || (n_edits > 0 && (!edit_level || !edit_prefix || !edit_action)))
+        return tfail(t, AFMM_EINVAL, "tree_rebuild: bad edit list");
+    std::vector<std::pair<std::pair<int, unsigned long long>, int>> e(n_edits);
+    for (int i = 0; i < n_edits; ++i) {
+        if (edit_level[i] < 0 || edit_level[i] > kMaxLevel || (edit_action[i] != 1 && edit_action[i] != 2))
+            return tfail(t, AFMM_EINVAL, "tree_rebuild: edit %d invalid", i);
+        e[i] = {{edit_level[i], edit_prefix[i]}, edit_action[i]};
+    }
+    std::sort(e.begin(), e.end());
+    for (int i = 1; i < n_edits; ++i)
+        if (e[i].first == e[i - 1].first && e[i].second != e[i - 1].second)
+            return tfail(t, AFMM_EINVAL, "tree_rebuild: conflicting edits for one node");
+    std::vector<long long> base(kMaxLevel + 2, 0);
+    std::vector<unsigned long long> pre(std::max(n_edits, 1));
+    std::vector<int> act(std::max(n_edits, 1));
+    for (int i = 0; i < n_edits; ++i) {
+        pre[i] = e[i].first.second;
+        act[i] = e[i].second;
+        base[e[i].first.first + 1]++;
+    }
+    for (int l = 0; l <= kMaxLevel; ++l) base[l + 1] += base[l];
+    TCU(t, cudaSetDevice(t->device));
+    unsigned long long *dp;
+    int *da;
+    long long *db;
+    if (afmm_status s = wsalloc(t, kEditPrefix, &dp, pre.size())) return s;
+    if (afmm_status s = wsalloc(t, kEditAction, &da, act.size())) return s;
+    if (afmm_status s = wsalloc(t, kEditBase, &db, base.size())) return s;
+    TCU(t, cudaMemcpyAsync(dp, pre.data(), pre.size() * sizeof(unsigned long long), cudaMemcpyHostToDevice, t->stream));
+    TCU(t, cudaMemcpyAsync(da, act.data(), act.size() * sizeof(int), cudaMemcpyHostToDevice, t->stream));
+    TCU(t, cudaMemcpyAsync(db, base.data(), base.size() * sizeof(long long), cudaMemcpyHostToDevice, t->stream));
+    const double lo[3] = {t->lo[0], t->lo[1], t->lo[2]};
+    return build_impl(t, n, x, y, z, S, 1, lo, t->k, mode == AFMM_TREE_KEEP ? kModeKeep : kModeEnforce,
+                      Edits{dp, da, db, n_edits});
+}
+
+// All nodes of the last build (host outputs, nullable): level, prefix, child count.
+extern "C" afmm_status afmm_tree_nodes(afmm_tree *t, int *level, unsigned long long *prefix, int *nchild) {
+    if (!t) return AFMM_EINVAL;
+    if (!t->built) return AFMM_ESTATE;
+    TCU(t, cudaSetDevice(t->device));
+    const long long nn = t->n_nodes;
+    std::vector<long long> base(t->pv_levels + 1);
+    TCU(t, cudaMemcpyAsync(base.data(), t->pv_base, base.size() * sizeof(long long), cudaMemcpyDeviceToHost, t->stream));
+    if (prefix) TCU(t, cudaMemcpyAsync(prefix, t->pv_prefix, nn * sizeof(unsigned long long), cudaMemcpyDeviceToHost, t->stream));
+    if (nchild) TCU(t, cudaMemcpyAsync(nchild, t->pv_nchild, nn * sizeof(int), cudaMemcpyDeviceToHost, t->stream));
+    TCU(t, cudaStreamSynchronize(t->stream));
+    if (level)
+        for (int l = 0; l < t->pv_levels; ++l)
+            for (long long i = base[l]; i < base[l + 1]; ++i) level[i] = l;
+    return AFMM_OK;
 }
 
 extern "C" afmm_status afmm_tree_info(const afmm_tree *t, int *n_leaves, long long *nnz, double *lo,

@@ -118,12 +118,10 @@ __device__ __forceinline__ int slices_for(int tn, long long nsrc) {
     int kbest = kmin;
     double best = 1e300;
     for (int k = kmin; k <= kmin + 3 && k <= tn; ++k) {
-        double slots = 0.0;
-        for (int i = 0; i < k; ++i) {
-            const int m = (int)(((long long)tn * (i + 1)) / k - ((long long)tn * i) / k);
-            const int g = (m + kTPT - 1) / kTPT;
-            slots += 32.0 / (32 / g);
-        }
+        // slice sizes are q+1 (r of them) and q (k - r): floor(tn (i+1)/k) - floor(tn i/k)
+        const int q = tn / k, r = tn - q * k;
+        const int g1 = (q + 1 + kTPT - 1) / kTPT, g0 = (q + kTPT - 1) / kTPT;
+        double slots = (double)r * (32.0 / (32 / g1)) + (double)(k - r) * (q > 0 ? 32.0 / (32 / g0) : 0.0);
         slots = slots * (double)(nsrc > 1 ? nsrc : 1) + kTaskOverhead * k;
         if (slots < best - 1e-9) {
             best = slots;
