@@ -25,6 +25,7 @@ if not os.path.exists(LIB_PATH):
                       "there is no CPU fallback for the AFMM P2P path")
 _lib = C.CDLL(LIB_PATH)
 
+MAX_LEAF = 1 << 30     # AFMM_MAX_LEAF of include/afmm_p2p.h
 AFMM_OK, AFMM_EINVAL, AFMM_ESTATE, AFMM_ENOMEM, AFMM_ECUDA, AFMM_ENCCL, AFMM_ENOTSUP = 0, -1, -2, -3, -4, -5, -6
 _STATUS = {0: "AFMM_OK", -1: "AFMM_EINVAL", -2: "AFMM_ESTATE", -3: "AFMM_ENOMEM", -4: "AFMM_ECUDA",
            -5: "AFMM_ENCCL", -6: "AFMM_ENOTSUP"}
@@ -269,12 +270,14 @@ def fp32_peak(device: int = 0):
 class P2P:
     """One afmm_p2p handle (one per rank / GPU)."""
 
-    def __init__(self, device=0, rank=0, world=1, G=1.0, eps2=0.0, max_leaf=1024, stream=None,
+    def __init__(self, device=0, rank=0, world=1, G=1.0, eps2=0.0, max_leaf=None, stream=None,
                  law=LAW_GRAVITY, mu=1.0):
         cfg = Config()
         _lib.afmm_p2p_config_init(C.byref(cfg))
         cfg.device, cfg.rank, cfg.world = int(device), int(rank), int(world)
-        cfg.G, cfg.eps2, cfg.max_leaf = float(G), float(eps2), int(max_leaf)
+        cfg.G, cfg.eps2 = float(G), float(eps2)
+        if max_leaf is not None:
+            cfg.max_leaf = int(max_leaf)
         cfg.stream = stream
         cfg.law, cfg.mu = int(law), float(mu)
         h = _p()

@@ -215,7 +215,7 @@ extern "C" afmm_status afmm_p2p_config_init(afmm_p2p_config *cfg) {
     cfg->world = 1;
     cfg->G = 1.0f;
     cfg->eps2 = 0.0f;
-    cfg->max_leaf = 1024;
+    cfg->max_leaf = AFMM_MAX_LEAF;
     cfg->stream = nullptr;
     cfg->law = AFMM_LAW_GRAVITY;
     cfg->mu = 1.0f;
@@ -228,7 +228,7 @@ extern "C" afmm_status afmm_p2p_create(const afmm_p2p_config *cfg, afmm_p2p **ou
     if (!out) return AFMM_EINVAL;
     *out = nullptr;
     if (!cfg) return AFMM_EINVAL;
-    if (cfg->max_leaf > 1024) return AFMM_ENOTSUP;
+    if (cfg->max_leaf > AFMM_MAX_LEAF) return AFMM_ENOTSUP;
     if (cfg->max_leaf < 1 || cfg->world < 1 || cfg->rank < 0 || cfg->rank >= cfg->world ||
         !std::isfinite(cfg->G) || !std::isfinite(cfg->eps2) || !(cfg->eps2 >= 0.0f) ||
         cfg->device < 0 || (cfg->law != AFMM_LAW_GRAVITY && cfg->law != AFMM_LAW_STOKESLET) ||

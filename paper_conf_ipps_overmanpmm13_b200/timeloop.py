@@ -16,6 +16,18 @@ L20 SVI.A Enforce_S; L18 SIV.D observational coefficients):
   7. near-field P2P                                    (afmm_p2p_eval)
   8. kick(dt/2) with the new accelerations
 
+With a load balancer (lb=LoadBalancer(...)) step 4 follows
+the controller's action from the previous step instead (PAPER L18 SV, L20-L22):
+  KEEP     afmm_tree_rebuild(KEEP): the structure is kept, bodies re-binned
+  REBUILD  afmm_tree_build with the new S (fixed domain)
+  ENFORCE  afmm_tree_enforce(S), predict, and FineGrainedOptimize if the
+           controller asks (afmm_fine_grained), predict again
+  FINE     KEEP + afmm_fine_grained
+and after step 7 the controller sees T_gpu = the measured P2P kernel time (max
+over ranks) and T_cpu = sum_op C_op M(op), the far-field time MODELLED from the
+operation counts of the tree (afmm_tree_farfield_counts; reading R29: the CPU
+far field is out of scope, so its time is a model with per-op costs cpu_coef).
+
 Note: the far field is out of scope (S10), so bodies move under the
 near-field force only; C5 is a dynamic load for the GPU path, not a physical
 simulation.
@@ -27,16 +39,31 @@ import time
 import numpy as np
 import torch
 
-from . import GpuTree, P2P, cost_fit, drift, kick
+from . import (LB_ENFORCE, LB_FINE, LB_KEEP, LB_REBUILD, TREE_KEEP, GpuTree, P2P, cost_fit, drift,
+               kick)
+
+# Default modelled far-field costs (seconds per operation: P2M, M2M, M2L, L2L,
+# L2P), reading R29: translation operators of an order-p expansion cost
+# O(p^4) flops and P2M / L2P O(p^2) per body; the default puts one M2L at 1 ns
+# so that the modelled far field and the measured B200 near field cross near
+# the S the bench sweep finds (not a measurement of any CPU).
+CPU_COEF_DEFAULT = (0.5e-9, 1.0e-9, 1.0e-9, 1.0e-9, 0.5e-9)
 
 
 class TimeLoop:
-    def __init__(self, x, y, z, m, vx, vy, vz, S, eps2, dt, domain, device=0, rank=0, world=1, G=1.0):
+    def __init__(self, x, y, z, m, vx, vy, vz, S, eps2, dt, domain, device=0, rank=0, world=1, G=1.0,
+                 lb=None, cpu_coef=CPU_COEF_DEFAULT, fine_group=0.05, fine_max_groups=16):
         self.dev = torch.device("cuda", device)
         self.stream = torch.cuda.Stream(self.dev)
         torch.cuda.set_stream(self.stream)
         self.S, self.eps2, self.dt, self.rank, self.world = int(S), float(eps2), float(dt), rank, world
         self.n = int(x.shape[0])
+        self.domain = domain
+        self.lb = lb
+        self.cpu_coef = np.asarray(cpu_coef, np.float64)
+        self.fine_group, self.fine_max_groups = float(fine_group), int(fine_max_groups)
+        self.next_action = LB_KEEP
+        self.c_p2p = None                                       # s per interaction, observed (L18 SIV.D)
         n = self.n
         # state in tree order: rows x, y, z, m, vx, vy, vz
         src = torch.stack([torch.as_tensor(np.asarray(v, np.float32)) for v in (x, y, z, m, vx, vy, vz)]).to(self.dev)
@@ -98,11 +125,67 @@ class TimeLoop:
         arr = np.stack([v.cpu().numpy() for v in allv])
         self.h.set_cost_coef(cost_fit(arr[:, 1:], arr[:, 0]))
 
+    # ------------------------------------------------------------------ load balancing
+    def _times(self):
+        """(T_cpu modelled, T_gpu measured max over ranks, counts) of this step."""
+        ms = float(self.h.stats()["kernel_ms"])
+        if self.world > 1:
+            import torch.distributed as dist
+            t = torch.tensor([ms], dtype=torch.float64, device=self.dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms = float(t.item())
+        c = self.tree.farfield_counts()
+        return float(np.dot(self.cpu_coef, c[:5])), 1e-3 * ms, c
+
+    def _coef6(self):
+        return np.concatenate([self.cpu_coef, [self.c_p2p or 0.0]])
+
+    def _predict(self):
+        c = self.tree.farfield_counts()
+        return max(float(np.dot(self.cpu_coef, c[:5])), (self.c_p2p or 0.0) * float(c[5]))
+
+    def _maintain(self, x, y, z):
+        """Tree maintenance of this step (step 4): Enforce_S without a balancer,
+        else the controller's pending action."""
+        rec = {"action": None}
+        if self.lb is None:
+            self.tree.enforce(x, y, z, self.S)
+            return rec
+        a = self.next_action
+        rec["action"] = ("keep", "rebuild", "enforce", "fine")[a]
+        if a == LB_REBUILD:
+            self.tree.build(x, y, z, self.S, domain=self.domain)
+        elif a == LB_ENFORCE:
+            self.tree.enforce(x, y, z, self.S)
+            rec["t_pred"] = self._predict()
+            if self.lb.predicted(rec["t_pred"]) == LB_FINE:
+                r = self.tree.fine_grained(x, y, z, self.S, self._coef6(), 0, self.fine_group, self.fine_max_groups)
+                rec["fine"] = r
+                self.lb.predicted(r["t_after"])
+        else:
+            self.tree.rebuild(x, y, z, self.S, mode=TREE_KEEP)
+            if a == LB_FINE:
+                r = self.tree.fine_grained(x, y, z, self.S, self._coef6(), 0, self.fine_group, self.fine_max_groups)
+                rec["fine"] = r
+                self.lb.predicted(r["t_after"])
+        return rec
+
+    def _balance(self, rec):
+        t_cpu, t_gpu, c = self._times()
+        if c[5] > 0:
+            self.c_p2p = t_gpu / float(c[5])
+        a, S = self.lb.step(t_cpu, t_gpu)
+        self.next_action, self.S = a, S
+        st = self.lb.state()
+        rec.update({"t_cpu_model": t_cpu, "t_gpu": t_gpu, "compute": max(t_cpu, t_gpu), "lb_state": st["state"],
+                    "S_next": S, "next": ("keep", "rebuild", "enforce", "fine")[a]})
+
     # ------------------------------------------------------------------ one step
     def step(self, hooks=None):
         """One KDK step.  hooks (optional dict of callables) receive the state
         for verification: 'pre_enforce'(x, y, z) with positions in the old tree
-        order, 'post_eval'(loop) after the new accelerations."""
+        order, 'post_maintain'(loop, rec) after the tree maintenance (loop.tree
+        holds the new tree), 'post_eval'(loop) after the new accelerations."""
         ev = [torch.cuda.Event(enable_timing=True) for _ in range(6)]
         t0 = time.perf_counter()
         ev[0].record(self.stream)
@@ -117,7 +200,9 @@ class TimeLoop:
         if hooks and "pre_enforce" in hooks:
             torch.cuda.synchronize()
             hooks["pre_enforce"](s[0].cpu().numpy(), s[1].cpu().numpy(), s[2].cpu().numpy())
-        self.tree.enforce(s[0], s[1], s[2], self.S)
+        lbrec = self._maintain(s[0], s[1], s[2])
+        if hooks and "post_maintain" in hooks:
+            hooks["post_maintain"](self, lbrec)
         for a in range(7):
             self.tree.gather(s[a], self.tmp[a])
         self.state, self.tmp = self.tmp, self.state
@@ -134,7 +219,12 @@ class TimeLoop:
                "kernel_ms": st["kernel_ms"], "kick_drift_ms": ev[0].elapsed_time(ev[1]),
                "enforce_ms": ev[1].elapsed_time(ev[2]), "set_tree_ms": ev[2].elapsed_time(ev[3]),
                "eval_ms": ev[3].elapsed_time(ev[4]), "step_ms": 1e3 * (time.perf_counter() - t0),
-               "leaf_split": self.h.get_partition()[0].tolist()}
+               "leaf_split": self.h.get_partition()[0].tolist(), "S": self.S}
+        if self.lb is not None:
+            t1 = time.perf_counter()
+            rec.update(lbrec)
+            self._balance(rec)
+            rec["lb_ms"] = 1e3 * (time.perf_counter() - t1)
         self.log.append(rec)
         self.step_no += 1
         if hooks and "post_eval" in hooks:

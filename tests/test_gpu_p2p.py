@@ -23,7 +23,7 @@ def _dev(a):
     return torch.from_numpy(np.ascontiguousarray(a, np.float32)).cuda()
 
 
-def gpu_eval(xs, ys, zs, ms, T, eps2, G=1.0, world=1, max_leaf=1024, leaf_split=None):
+def gpu_eval(xs, ys, zs, ms, T, eps2, G=1.0, world=1, max_leaf=None, leaf_split=None):
     """Run the library for every rank of `world` on this one GPU and merge the
     disjoint output slices (ranks write only their own bodies)."""
     afmm = _afmm()
@@ -88,10 +88,12 @@ def test_c3_colliding_parity_full():
 
 @pytest.mark.parametrize("dist,n,S,eps2", [("uniform", 20000, 1, 1e-6), ("uniform", 20000, 7, 0.0),
                                            ("plummer", 50000, 300, 1e-4), ("colliding", 30000, 33, 1e-6),
-                                           ("plummer", 1000, 5000, 1e-6)])
+                                           ("plummer", 1000, 5000, 1e-6), ("plummer", 40000, 3000, 1e-6),
+                                           ("uniform", 30000, 12000, 1e-6)])
 def test_ragged_leaf_sizes(dist, n, S, eps2):
     """Leaves of every size 1..S (ragged tails of the lane mapping), eps2 = 0,
-    one-leaf trees (N <= S), sources spanning several 1024-body stages."""
+    one-leaf trees (N <= S), sources spanning several 1024-body stages, leaves
+    far above 1024 bodies (the KEEP rule of the load balancer lets leaves grow)."""
     x, y, z, m = synth.make(dist, n, 17)
     _parity(x, y, z, m, S, eps2)
 
@@ -196,7 +198,7 @@ def test_host_pointer_api_matches_device_api():
 def test_error_statuses():
     afmm = _afmm()
     with pytest.raises(afmm.AfmmError) as e:
-        afmm.P2P(max_leaf=2048)
+        afmm.P2P(max_leaf=afmm.MAX_LEAF + 1)
     assert e.value.status == afmm.AFMM_ENOTSUP
     for kw in ({"eps2": -1.0}, {"G": float("inf")}, {"world": 0}, {"rank": 2, "world": 2}):
         with pytest.raises(afmm.AfmmError) as e:

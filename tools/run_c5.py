@@ -23,11 +23,22 @@ ap.add_argument("--S", type=int, default=128)
 ap.add_argument("--dt", type=float, default=0.05)
 ap.add_argument("--eps2", type=float, default=1e-4)
 ap.add_argument("--check-every", type=int, default=0)
+ap.add_argument("--lb", action="store_true", help="drive S and the tree with the load balancer (row f3)")
+ap.add_argument("--cpu-coef", default="", help="modelled far-field costs P2M,M2M,M2L,L2L,L2P (s/op)")
+ap.add_argument("--no-fine", action="store_true", help="load balancer without FineGrainedOptimize")
 a = ap.parse_args()
 x, y, z, m, vx, vy, vz = synth.colliding_with_velocities(a.n, 5)
 dom = synth.c5_domain(x, y, z)
 t0 = time.perf_counter()
-loop = TimeLoop(x, y, z, m, vx, vy, vz, a.S, a.eps2, a.dt, dom)
+kw = {}
+if a.lb:
+    import paper_conf_ipps_overmanpmm13_b200 as afmm
+    kw["lb"] = afmm.LoadBalancer(S_init=a.S)
+    if a.cpu_coef:
+        kw["cpu_coef"] = [float(v) for v in a.cpu_coef.split(",")]
+    if a.no_fine:
+        kw["fine_max_groups"] = 0
+loop = TimeLoop(x, y, z, m, vx, vy, vz, a.S, a.eps2, a.dt, dom, **kw)
 setup_s = time.perf_counter() - t0
 checks = []
 otree = [None]
@@ -82,5 +93,13 @@ print(json.dumps({
                                for q in range(4)],
     "n_leaves": [L[0]["n_leaves"], L[len(L) // 2]["n_leaves"], L[-1]["n_leaves"]],
     "interactions_per_step": [L[0]["interactions"], L[len(L) // 2]["interactions"], L[-1]["interactions"]],
-    "checks": checks}))
+    "checks": checks,
+    **({"lb": {"cpu_coef": list(map(float, loop.cpu_coef)),
+               "trajectory": [{k: (round(v, 7) if isinstance(v, float) else v) for k, v in r.items()
+                               if k in ("step", "S", "action", "lb_state", "t_cpu_model", "t_gpu", "compute",
+                                        "n_leaves", "lb_ms", "step_ms")} for r in L],
+               "fine": [dict(step=r["step"], **r["fine"]) for r in L if "fine" in r],
+               "compute_ms_by_quarter": [round(1e3 * float(np.mean([r["compute"] for r in
+                                                                    L[q * len(L) // 4:(q + 1) * len(L) // 4]])), 4)
+                                         for q in range(4)]}} if a.lb else {})}))
 loop.close()
