@@ -245,22 +245,22 @@ struct Partial {
 
 // Consume sources src[k], k = k0, k0+C, ... < kend; fp32 partials are folded
 // into fp64 before they would exceed kFold sources.  Masks compare k with
-// T.m[j] - moff.
+// T.m[j] - moff.  rcpC = ceil(2^16 / C): floor(N rcpC / 2^16) == floor(N / C)
+// exactly for 0 <= N < 2048, C <= 32 (no integer division in the loop setup).
 template <class Law, bool kMasked>
-__device__ __forceinline__ void consume(const float4 *__restrict__ src, int k, int kend, int C,
+__device__ __forceinline__ void consume(const float4 *__restrict__ src, int k, int kend, int C, int rcpC,
                                         const Targets &T, int moff, const float2 e2, Partial &P) {
     while (k < kend) {
         if (P.cnt >= kFold) P.fold();
-        const int kstop = min(kend, k + (kFold - P.cnt) * C);
-        int iters = 0;
+        const int span = min(kend - k, (kFold - P.cnt) * C);
+        const int iters = ((span + C - 1) * rcpC) >> 16;            // ceil(span / C)
 #pragma unroll kUnroll
-        for (; k < kstop; k += C) {
+        for (int it = 0; it < iters; ++it, k += C) {
 #pragma unroll
             for (int q = 0; q < kPairs; ++q)
                 Law::template apply<kMasked>(src, k, T.nx[q], T.ny[q], T.nz[q], e2, P.ax[q], P.ay[q], P.az[q],
                                              P.ph[q], kMasked && k == T.m[2 * q] - moff,
                                              kMasked && k == T.m[2 * q + 1] - moff);
-            ++iters;
         }
         P.cnt += iters;
     }
@@ -404,7 +404,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
     Targets T;
     Partial P;
     P.acc = accw + lane;
-    int g = 1, C = 1, c = 0, l = 0;
+    int g = 1, C = 1, rcpC = 65536, c = 0, l = 0;
     bool active = false;
     for (int q = 0; q < issued; ++q) {
         // keep the ring one chunk ahead (across task boundaries)
@@ -418,6 +418,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
         if (m.is_first) {
             g = (m.tgt_count + kTPT - 1) / kTPT;
             C = 32 / g;
+            rcpC = (65536 + C - 1) / C;
             c = lane / g;
             l = lane - c * g;
             active = c < C;
@@ -428,9 +429,10 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
         }
         if (active) {
             const int kself = Law::kMaskSelf ? min(max(m.self_len - m.first, 0), m.nb) : 0;
-            if (kself > 0) consume<Law, true>(stage[st], c, kself, C, T, m.first, e2, P);
-            const int k0 = kself + ((c - kself) % C + C) % C;        // first k >= kself, k = c (mod C)
-            consume<Law, false>(stage[st], k0, m.nb, C, T, 0, e2, P);
+            if (kself > 0) consume<Law, true>(stage[st], c, kself, C, rcpC, T, m.first, e2, P);
+            // first k >= kself with k = c (mod C)
+            const int k0 = kself <= c ? c : c + C * (((kself - c + C - 1) * rcpC) >> 16);
+            consume<Law, false>(stage[st], k0, m.nb, C, rcpC, T, 0, e2, P);
         }
         if (m.is_last) {
             if (active) P.fold();
