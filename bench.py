@@ -37,6 +37,7 @@ sys.path.insert(0, ROOT)
 
 import synth  # noqa: E402  (seeded input generator shared by both arms)
 
+E2E_PIECES = 4             # pieces of the pipelined host-to-host evaluation (e2e)
 FLOPS_PER_INTERACTION = 20
 METRIC = "near-field P2P interactions/s (and % FP32 peak) at 1/2/4/8 B200"
 SWEEP_S = [32, 48, 64, 96, 128, 192, 256, 384, 512]
@@ -312,8 +313,8 @@ def main():
 
     def step_e2e():
         if world == 1:
-            h.set_bodies(*hx)                                 # afmm_p2p_set_bodies_host (H2D + pack)
-            h.eval(*ho)                                       # afmm_p2p_eval_host (kernel + D2H, blocking)
+            # afmm_p2p_eval_host_pipelined: H2D + pack, kernel pieces, D2H overlapped; blocking
+            h.eval_host_pipelined(*hx, *ho, pieces=E2E_PIECES)
         else:
             if rank == 0:
                 for a in range(4):
@@ -446,7 +447,9 @@ def main():
                          "kernel": "afmm::p2p_kernel"},
             "clocks": clk.summary(),
             "e2e": {"value": e2e_value, "unit": "interactions/s", "h2d_bytes_per_step": 16 * n,
-                    "d2h_bytes_per_step": 16 * n, "steps": Ke},
+                    "d2h_bytes_per_step": 16 * n, "steps": Ke,
+                    "path": f"afmm_p2p_eval_host_pipelined ({E2E_PIECES} pieces) from pinned host arrays" if world == 1
+                    else "rank 0 H2D + step + D2H"},
             "gpu_launches": 2 * K,
             "rebalanced_in_warmup": rebalanced,
             "cpu_baseline": cpu,

@@ -84,6 +84,7 @@ _sig("afmm_p2p_get_partition", _i, _p, _p, _p)
 _sig("afmm_p2p_rebalance", _i, _p, _p, _d, C.POINTER(_i))
 _sig("afmm_p2p_eval", _i, _p, _p, _p, _p, _p, C.POINTER(Stats))
 _sig("afmm_p2p_eval_host", _i, _p, _p, _p, _p, _p, C.POINTER(Stats))
+_sig("afmm_p2p_eval_host_pipelined", _i, _p, _ll, _p, _p, _p, _p, _p, _p, _p, _p, _i, C.POINTER(Stats))
 _sig("afmm_p2p_stats_get", _i, _p, C.POINTER(Stats))
 _sig("afmm_p2p_stream", _p, _p)
 _sig("afmm_p2p_kernel_times", _i, _p, _i, _p)
@@ -154,7 +155,7 @@ EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
             "afmm_tree_farfield_counts", "afmm_lb_config_init", "afmm_lb_create", "afmm_lb_step",
             "afmm_lb_predicted", "afmm_lb_state", "afmm_lb_destroy", "afmm_tree_copy_out",
             "afmm_tree_gather", "afmm_tree_scatter", "afmm_tree_destroy", "afmm_tree_last_error",
-            "afmm_tree_rebuild", "afmm_tree_nodes", "afmm_fine_grained"]
+            "afmm_tree_rebuild", "afmm_tree_nodes", "afmm_fine_grained", "afmm_p2p_eval_host_pipelined"]
 
 
 def version() -> str:
@@ -386,6 +387,25 @@ class P2P:
             self._check(_lib.afmm_p2p_eval_host(self._h, _ptr(ax), _ptr(ay), _ptr(az), _ptr(phi), sp),
                         "afmm_p2p_eval_host")
         return s.as_dict() if (stats or not _is_device(ax)) else None
+
+    def eval_host_pipelined(self, x, y, z, m, ax, ay, az, phi, pieces=8):
+        """afmm_p2p_eval_host_pipelined: host inputs (tree order) -> host outputs,
+        transfers overlapped with the kernel pieces.  Host tensors or numpy
+        float32 arrays (pinned torch tensors for the overlap)."""
+        arrs = (x, y, z, m, ax, ay, az, phi)
+        n = int(x.shape[0])
+        for a in arrs:
+            if _is_device(a):
+                raise TypeError("eval_host_pipelined takes host arrays")
+            if isinstance(a, np.ndarray):
+                if not (a.dtype == np.float32 and a.flags.c_contiguous and a.shape[0] == n):
+                    raise TypeError("host arrays must be contiguous float32 of length n")
+            else:
+                _check_host_tensor(a, n)
+        s = Stats()
+        self._check(_lib.afmm_p2p_eval_host_pipelined(self._h, n, *[_ptr(a) for a in arrs], int(pieces), C.byref(s)),
+                    "afmm_p2p_eval_host_pipelined")
+        return s.as_dict()
 
     def kernel_times(self, max_count=64):
         """Kernel ms of the last <= 64 evals (oldest first); synchronises."""

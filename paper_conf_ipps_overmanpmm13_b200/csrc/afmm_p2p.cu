@@ -7,6 +7,7 @@
 // cudaEvent timing (PAPER L20 SVII.A).  Rows a4/a7 (replication, gather) are
 // collectives issued by the caller on the buffers this library exposes.
 #include <algorithm>
+#include <climits>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -15,6 +16,7 @@
 #include <string>
 #include <vector>
 
+#include <cuda.h>               // driver types for cuStreamWaitValue32 (resolved at run time)
 #include <cuda_runtime.h>
 
 #include "../../include/afmm_p2p.h"
@@ -77,6 +79,19 @@ struct afmm_p2p {
     long long n_evals = 0;
     bool evaluated = false;
     afmm_p2p_stats last{};
+
+    // pipelined host evaluation (afmm_p2p_eval_host_pipelined): the rank's tasks
+    // regrouped into P Morton-contiguous pieces, LPT order kept inside each
+    bool pipe_valid = false;
+    int pipe_P = 0;
+    std::vector<int> pipe_off;                       // P + 1 offsets into d_ptasks
+    std::vector<long long> pipe_need, pipe_lo, pipe_hi;   // bodies needed (prefix), output range per piece
+    afmm::Task *d_ptasks = nullptr;
+    size_t ptasks_cap = 0;
+    int *d_pqueue = nullptr;                         // kMaxPieces counters
+    cudaStream_t s_in = nullptr, s_out = nullptr;
+    void *wait_value32 = nullptr;                    // cuStreamWaitValue32 (driver entry point)
+    cudaEvent_t ev_start = nullptr, ev_in[64] = {}, ev_k[64] = {}, ev_done = nullptr;
 };
 
 namespace {
@@ -283,6 +298,17 @@ extern "C" void afmm_p2p_destroy(afmm_p2p *h) {
     cudaFree(h->d_segs);
     for (void *q : h->dws_ptr) cudaFree(q);
     cudaFree(h->d_queue);
+    cudaFree(h->d_ptasks);
+    cudaFree(h->d_pqueue);
+    if (h->s_in) cudaStreamSynchronize(h->s_in), cudaStreamDestroy(h->s_in);
+    if (h->s_out) cudaStreamSynchronize(h->s_out), cudaStreamDestroy(h->s_out);
+
+    for (int i = 0; i < 64; ++i) {
+        if (h->ev_in[i]) cudaEventDestroy(h->ev_in[i]);
+        if (h->ev_k[i]) cudaEventDestroy(h->ev_k[i]);
+    }
+    if (h->ev_start) cudaEventDestroy(h->ev_start);
+    if (h->ev_done) cudaEventDestroy(h->ev_done);
     for (int i = 0; i < afmm_p2p::kRing; ++i) {
         if (h->ring0[i]) cudaEventDestroy(h->ring0[i]);
         if (h->ring1[i]) cudaEventDestroy(h->ring1[i]);
@@ -612,6 +638,7 @@ extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const
         CUDA_TRY(h, cudaGetLastError());
     }
     h->n_tasks = nt;
+    h->pipe_valid = false;
     h->L = L;
     h->rank_interactions = (long long)hstats[0];
     for (int b = 0; b < 8; ++b) h->bucket_inter[b] = (long long)hstats[1 + b];
@@ -835,6 +862,7 @@ static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, flo
     p.eps2 = h->cfg.eps2;
     p.G = h->cfg.law == AFMM_LAW_STOKESLET ? 1.0 / (8.0 * 3.14159265358979323846 * (double)h->cfg.mu)
                                            : (double)h->cfg.G;
+    p.done = nullptr;
     CUDA_TRY(h, cudaMemsetAsync(h->d_queue, 0, sizeof(int), h->stream));
     const int ri = (int)(h->n_evals % afmm_p2p::kRing);
     h->ev0 = h->ring0[ri];
@@ -913,6 +941,198 @@ extern "C" afmm_status afmm_p2p_eval_host(afmm_p2p *h, float *ax, float *ay, flo
         for (int a = 0; a < 4; ++a)
             CUDA_TRY(h, cudaMemcpyAsync(hp[a] + lo, d[a] + lo, (size_t)(hi - lo) * sizeof(float),
                                         cudaMemcpyDeviceToHost, h->stream));
+    return fill_stats(h, stats);
+}
+
+// ------------------------------------------------------------------ pipelined host evaluation
+
+static constexpr int kMaxPieces = 64;
+
+// Regroup this rank's tasks into P pieces of consecutive targets (equal modelled
+// cost tgt_count * nsrc, cut in tgt_start order); inside a piece the tasks keep
+// the work list's largest-cost-first order.  Per piece: the output body range and
+// the prefix of bodies [0, need) its sources and targets lie in.
+static afmm_status build_pipe(afmm_p2p *h, int P) {
+    const int nt = h->n_tasks;
+    std::vector<afmm::Task> t(nt);
+    if (nt) CUDA_TRY(h, cudaMemcpy(t.data(), h->d_tasks, nt * sizeof(afmm::Task), cudaMemcpyDeviceToHost));
+    int nseg = 0;
+    for (const auto &x : t) nseg = std::max(nseg, x.seg_begin + x.seg_count);
+    std::vector<afmm::Seg> sg(nseg);
+    if (nseg) CUDA_TRY(h, cudaMemcpy(sg.data(), h->d_segs, nseg * sizeof(afmm::Seg), cudaMemcpyDeviceToHost));
+    std::vector<int> ord(nt);
+    for (int i = 0; i < nt; ++i) ord[i] = i;
+    std::stable_sort(ord.begin(), ord.end(), [&](int a, int b) { return t[a].tgt_start < t[b].tgt_start; });
+    double total = 0.0;
+    for (const auto &x : t) total += (double)x.tgt_count * (double)std::max(x.nsrc, 1);
+    std::vector<int> piece(nt, 0);
+    double acc = 0.0;
+    int p = 0;
+    for (int r = 0; r < nt; ++r) {
+        const afmm::Task &x = t[ord[r]];
+        // a leaf's slices share tgt_start ranges that are disjoint; cut only between leaves' first slices
+        while (p < P - 1 && acc >= total * (p + 1) / P && (r == 0 || x.self_start != t[ord[r - 1]].self_start)) ++p;
+        piece[ord[r]] = p;
+        acc += (double)x.tgt_count * (double)std::max(x.nsrc, 1);
+    }
+    h->pipe_off.assign(P + 1, 0);
+    h->pipe_need.assign(P, 0);
+    h->pipe_lo.assign(P, LLONG_MAX);
+    h->pipe_hi.assign(P, 0);
+    for (int i = 0; i < nt; ++i) {
+        const int q = piece[i];
+        h->pipe_off[q + 1]++;
+        long long need = (long long)t[i].tgt_start + t[i].tgt_count;
+        for (int j = 0; j < t[i].seg_count; ++j) {
+            const afmm::Seg &z = sg[t[i].seg_begin + j];
+            need = std::max(need, (long long)z.gstart + z.len);
+        }
+        h->pipe_need[q] = std::max(h->pipe_need[q], need);
+        h->pipe_lo[q] = std::min(h->pipe_lo[q], (long long)t[i].tgt_start);
+        h->pipe_hi[q] = std::max(h->pipe_hi[q], (long long)t[i].tgt_start + t[i].tgt_count);
+    }
+    for (int q = 0; q < P; ++q) {
+        h->pipe_off[q + 1] += h->pipe_off[q];
+        if (q > 0) h->pipe_need[q] = std::max(h->pipe_need[q], h->pipe_need[q - 1]);
+        if (h->pipe_lo[q] > h->pipe_hi[q]) h->pipe_lo[q] = h->pipe_hi[q] = 0;   // empty piece
+    }
+    std::vector<afmm::Task> grouped(std::max(nt, 1));
+    std::vector<int> fill(h->pipe_off.begin(), h->pipe_off.end() - 1);
+    for (int i = 0; i < nt; ++i) {                                              // stable: LPT kept
+        afmm::Task x = t[i];
+        x.piece = piece[i];
+        grouped[fill[piece[i]]++] = x;
+    }
+    afmm_status st = ensure_device(h, &h->d_ptasks, h->ptasks_cap, grouped.size());
+    if (st) return st;
+    CUDA_TRY(h, cudaMemcpy(h->d_ptasks, grouped.data(), grouped.size() * sizeof(afmm::Task), cudaMemcpyHostToDevice));
+    h->pipe_P = P;
+    h->pipe_valid = true;
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, const float *x, const float *y,
+                                                    const float *z, const float *m, float *ax, float *ay,
+                                                    float *az, float *phi, int n_pieces, afmm_p2p_stats *stats) {
+    CHECK_HANDLE(h);
+    if (h->cfg.law != AFMM_LAW_GRAVITY) return fail(h, AFMM_EINVAL, "eval_host_pipelined: gravity handles only");
+    if (!h->have_tree || !h->d_bodies) return fail(h, AFMM_ESTATE, "eval_host_pipelined: set_bodies and set_tree first");
+    if (n != h->n) return fail(h, AFMM_EINVAL, "eval_host_pipelined: n=%lld differs from the tree's %lld", n, h->n);
+    if (!x || !y || !z || !m || !ax || !ay || !az || !phi)
+        return fail(h, AFMM_EINVAL, "eval_host_pipelined: null pointer");
+    if (n_pieces < 1 || n_pieces > kMaxPieces)
+        return fail(h, AFMM_EINVAL, "eval_host_pipelined: n_pieces=%d outside [1, %d]", n_pieces, kMaxPieces);
+    afmm_status st = set_device(h);
+    if (st) return st;
+    if (!h->s_in) {
+        CUDA_TRY(h, cudaStreamCreateWithFlags(&h->s_in, cudaStreamNonBlocking));
+        CUDA_TRY(h, cudaStreamCreateWithFlags(&h->s_out, cudaStreamNonBlocking));
+        CUDA_TRY(h, cudaEventCreateWithFlags(&h->ev_start, cudaEventDisableTiming));
+        CUDA_TRY(h, cudaEventCreateWithFlags(&h->ev_done, cudaEventDisableTiming));
+        for (int i = 0; i < kMaxPieces; ++i) {
+            CUDA_TRY(h, cudaEventCreateWithFlags(&h->ev_in[i], cudaEventDisableTiming));
+            CUDA_TRY(h, cudaEventCreateWithFlags(&h->ev_k[i], cudaEventDisableTiming));
+        }
+        CUDA_TRY(h, cudaMalloc(&h->d_pqueue, (kMaxPieces + 1) * sizeof(int)));
+        cudaDriverEntryPointQueryResult q;
+        CUDA_TRY(h, cudaGetDriverEntryPoint("cuStreamWaitValue32", &h->wait_value32, cudaEnableDefault, &q));
+        if (q != cudaDriverEntryPointSuccess || !h->wait_value32)
+            return fail(h, AFMM_ENOTSUP, "eval_host_pipelined: cuStreamWaitValue32 unavailable");
+    }
+    if (4 * n > h->soa_cap) {
+        cudaFree(h->d_soa);
+        h->d_soa = nullptr;
+        h->soa_cap = 0;
+        CUDA_TRY(h, cudaMalloc(&h->d_soa, (size_t)(4 * n) * sizeof(float)));
+        h->soa_cap = 4 * n;
+    }
+    if (4 * n > h->out_cap) {
+        cudaFree(h->d_out);
+        h->d_out = nullptr;
+        h->out_cap = 0;
+        CUDA_TRY(h, cudaMalloc(&h->d_out, (size_t)(4 * n) * sizeof(float)));
+        h->out_cap = 4 * n;
+    }
+    if (!h->pipe_valid || h->pipe_P != n_pieces)
+        if ((st = build_pipe(h, n_pieces))) return st;
+    const int P = n_pieces;
+    float *dsoa[4] = {h->d_soa, h->d_soa + n, h->d_soa + 2 * n, h->d_soa + 3 * n};
+    float *dout[4] = {h->d_out, h->d_out + n, h->d_out + 2 * n, h->d_out + 3 * n};
+    const float *hin[4] = {x, y, z, m};
+    float *hout[4] = {ax, ay, az, phi};
+    // One launch over the piece-major task list: a piece's tail overlaps the
+    // next piece; warps count finished tasks per piece (P2PParams.done) and the
+    // copy-out stream waits on each counter (cuStreamWaitValue32) before copying
+    // that piece's outputs back, while later pieces still run.  The inputs go in
+    // first (sources of a piece may lie anywhere in the tree order).
+    using WaitFn = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+    const WaitFn wait32 = reinterpret_cast<WaitFn>(h->wait_value32);
+    int *queue = h->d_pqueue, *done = h->d_pqueue + 1;
+    CUDA_TRY(h, cudaMemsetAsync(h->d_pqueue, 0, (P + 1) * sizeof(int), h->stream));
+    CUDA_TRY(h, cudaEventRecord(h->ev_start, h->stream));      // earlier readers of the bodies / outputs
+    CUDA_TRY(h, cudaStreamWaitEvent(h->s_in, h->ev_start, 0));
+    CUDA_TRY(h, cudaStreamWaitEvent(h->s_out, h->ev_start, 0));
+    const size_t b = (size_t)n * sizeof(float);
+    const long long half = n / 2;
+    for (int part = 0; part < 2; ++part) {                     // two halves: pack of the first overlaps the second copy
+        const long long lo = part ? half : 0, hi = part ? n : half;
+        if (hi <= lo) continue;
+        for (int a = 0; a < 4; ++a)
+            CUDA_TRY(h, cudaMemcpyAsync(dsoa[a] + lo, hin[a] + lo, (size_t)(hi - lo) * sizeof(float),
+                                        cudaMemcpyHostToDevice, h->s_in));
+        const int threads = 256;
+        const int blocks = (int)std::min<long long>((hi - lo + threads - 1) / threads, (long long)h->num_sms * 16);
+        afmm::pack_bodies_kernel<<<blocks, threads, 0, h->s_in>>>(hi - lo, dsoa[0] + lo, dsoa[1] + lo, dsoa[2] + lo,
+                                                                 dsoa[3] + lo, h->d_bodies + lo);
+        CUDA_TRY(h, cudaGetLastError());
+    }
+    (void)b;
+    CUDA_TRY(h, cudaEventRecord(h->ev_in[0], h->s_in));
+    CUDA_TRY(h, cudaStreamWaitEvent(h->stream, h->ev_in[0], 0));
+    const int ri = (int)(h->n_evals % afmm_p2p::kRing);
+    h->ev0 = h->ring0[ri];
+    h->ev1 = h->ring1[ri];
+    CUDA_TRY(h, cudaEventRecord(h->ev0, h->stream));
+    const int nt = h->pipe_off[P];
+    int nlaunch = 0;
+    if (nt > 0) {
+        afmm::P2PParams prm;
+        prm.bodies = h->d_bodies;
+        prm.tasks = h->d_ptasks;
+        prm.segs = h->d_segs;
+        prm.n_tasks = nt;
+        prm.queue = queue;
+        prm.ax = dout[0];
+        prm.ay = dout[1];
+        prm.az = dout[2];
+        prm.phi = dout[3];
+        prm.eps2 = h->cfg.eps2;
+        prm.G = (double)h->cfg.G;
+        prm.done = done;
+        const int grid = std::max(1, std::min((nt + afmm::kWarps - 1) / afmm::kWarps, h->num_sms * h->blocks_per_sm));
+        afmm::p2p_kernel_t<afmm::Gravity><<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(prm);
+        CUDA_TRY(h, cudaGetLastError());
+        nlaunch = 1;
+    }
+    CUDA_TRY(h, cudaEventRecord(h->ev1, h->stream));
+    // the launch must be enqueued before the copy-out stream starts waiting on its counters
+    for (int q = 0; q < P; ++q) {
+        const long long lo = h->pipe_lo[q], hi = h->pipe_hi[q];
+        const int cnt = h->pipe_off[q + 1] - h->pipe_off[q];
+        if (hi <= lo || cnt == 0) continue;
+        const CUresult r = wait32((CUstream)h->s_out, (CUdeviceptr)(done + q), (cuuint32_t)cnt, CU_STREAM_WAIT_VALUE_GEQ);
+        if (r != CUDA_SUCCESS) return fail(h, AFMM_ECUDA, "eval_host_pipelined: cuStreamWaitValue32 failed (%d)", (int)r);
+        for (int a = 0; a < 4; ++a)
+            CUDA_TRY(h, cudaMemcpyAsync(hout[a] + lo, dout[a] + lo, (size_t)(hi - lo) * sizeof(float),
+                                        cudaMemcpyDeviceToHost, h->s_out));
+    }
+    // safety net: nothing on s_out may outlive the kernel's stream order
+    CUDA_TRY(h, cudaStreamWaitEvent(h->s_out, h->ev1, 0));
+    CUDA_TRY(h, cudaEventRecord(h->ev_done, h->s_out));
+    CUDA_TRY(h, cudaStreamWaitEvent(h->stream, h->ev_done, 0));
+    h->n_evals++;
+    h->evaluated = true;
+    h->last.n_launches = nlaunch;
     return fill_stats(h, stats);
 }
 

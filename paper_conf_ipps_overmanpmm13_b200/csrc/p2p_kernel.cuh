@@ -70,7 +70,8 @@ constexpr int kDynSmem = kWarps * (kStageBytesW + kAccBytesW);
 // the first segment is the leaf itself), else 0; sources = segments
 // [seg_begin, +seg_count) totalling nsrc bodies.
 struct Task {
-    int tgt_start, tgt_count, self_start, self_len, seg_begin, seg_count, nsrc, pad;
+    int tgt_start, tgt_count, self_start, self_len, seg_begin, seg_count, nsrc;
+    int piece;               // completion counter index (pipelined host evaluation), else 0
 };
 // Segment: bodies [gstart, gstart+len).
 struct Seg {
@@ -86,6 +87,7 @@ struct P2PParams {
     float *ax, *ay, *az, *phi;
     float eps2;
     double G;                // output scale: G (gravity) or 1/(8 pi mu) (Stokeslet)
+    int *done;               // nullptr, or per-piece counters of finished tasks (afmm_p2p_eval_host_pipelined)
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
@@ -268,7 +270,7 @@ __device__ __forceinline__ void consume(const float4 *__restrict__ src, int k, i
 
 // Per-stage metadata of a warp's ring (written by lane 0 at issue time).
 struct ChunkMeta {
-    int tgt_start, tgt_count, toff, self_len, first, nb, is_first, is_last;
+    int tgt_start, tgt_count, toff, self_len, first, nb, is_first, is_last, piece;
 };
 
 // Issue side of a warp's pipeline: the task whose sources are being streamed
@@ -310,6 +312,7 @@ __device__ __forceinline__ bool issue_chunk(const P2PParams &p, Stream &S, float
         m.nb = nb;
         m.is_first = S.staged == 0;
         m.is_last = S.staged + nb >= S.t.nsrc;
+        m.piece = S.t.piece;
         *meta = m;
         fence_proxy_async();
         mbar_arrive_expect_tx(bar, (uint32_t)nb * 16u * kWords);
@@ -449,6 +452,11 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
                     float *dst = comp == 0 ? p.ax : comp == 1 ? p.ay : comp == 2 ? p.az : p.phi;
                     dst[m.tgt_start + tgt] = Law::out(comp, v, p.G);
                 }
+            }
+            if (p.done) {                 // publish the task's outputs (pipelined copy-back waits on it)
+                __threadfence();
+                __syncwarp();
+                if (lane == 0) atomicAdd(p.done + m.piece, 1);
             }
         }
         __syncwarp();                     // stage st (and the accumulators) free again

@@ -347,3 +347,72 @@ def test_set_tree_device_rejects_invalid_tree():
         h.rebalance([1.0], 0.02)
     assert e.value.status == afmm.AFMM_ESTATE
     h.close()
+
+
+@pytest.mark.parametrize("world,pieces,ingest", [(1, 1, "host"), (1, 8, "host"), (1, 64, "device"), (2, 5, "host"),
+                                                 (3, 8, "device")])
+def test_eval_host_pipelined_bit_identical(world, pieces, ingest):
+    """afmm_p2p_eval_host_pipelined (H2D / kernel pieces / D2H overlapped) ==
+    afmm_p2p_eval on device buffers, bit for bit, on every rank's slice; the
+    handle's bodies afterwards are the host ones (a plain eval agrees too)."""
+    afmm = _afmm()
+    x, y, z, m = synth.make("plummer", 200000, 21)
+    n = x.shape[0]
+    tree = afmm.GpuTree(0)
+    X, Y, Z, M = (torch.from_numpy(v).cuda() for v in (x, y, z, m))
+    info = tree.build(X, Y, Z, 64)
+    T = tree.copy_out(n)
+    d = tree.device_arrays()
+    bod = torch.empty((4, n), device="cuda")
+    for a, src in enumerate((X, Y, Z, M)):
+        tree.gather(src, bod[a])
+    hb = [bod[a].cpu().pin_memory() for a in range(4)]
+    ref = torch.full((4, n), float("nan"), device="cuda")
+    got = [torch.full((n,), float("nan")).pin_memory() for _ in range(4)]
+    again = torch.full((4, n), float("nan"), device="cuda")
+    for r in range(world):
+        h = afmm.P2P(rank=r, world=world, eps2=1e-6)
+        h.set_bodies(bod[0], bod[1], bod[2], bod[3])
+        if ingest == "host":
+            h.set_tree(T["leaf_start"], T["leaf_count"], T["u_off"], T["u_idx"])
+        else:
+            h.set_tree_device(info["n_leaves"], d["leaf_start"], d["leaf_count"], d["u_off"], d["u_idx"])
+        h.eval(ref[0], ref[1], ref[2], ref[3])
+        h.set_bodies(*[torch.zeros(n, device="cuda") for _ in range(4)])   # stale device bodies
+        for _ in range(2):                                                  # plan reused on the 2nd call
+            st = h.eval_host_pipelined(*hb, *got, pieces=pieces)
+        assert st["n_launches"] <= pieces and st["n_launches"] >= 1
+        h.eval(again[0], again[1], again[2], again[3])
+        h.close()
+    torch.cuda.synchronize()
+    r_ = ref.cpu().numpy()
+    assert np.isfinite(r_).all()
+    for a in range(4):
+        assert np.array_equal(got[a].numpy(), r_[a])
+    assert np.array_equal(again.cpu().numpy(), r_)
+    tree.close()
+
+
+def test_eval_host_pipelined_errors():
+    afmm = _afmm()
+    h = afmm.P2P(eps2=1e-6)
+    a = [np.zeros(10, np.float32) for _ in range(8)]
+    with pytest.raises(afmm.AfmmError) as e:
+        h.eval_host_pipelined(*a)
+    assert e.value.status == afmm.AFMM_ESTATE
+    x, y, z, m = synth.make("uniform", 1000, 3)
+    T, dd = _tree(x, y, z, 32)
+    h.set_bodies(*T.sorted_bodies(x, y, z, m))
+    h.set_tree(dd["leaf_start"], dd["leaf_count"], dd["u_off"], dd["u_idx"])
+    b = [np.zeros(1000, np.float32) for _ in range(8)]
+    for p in (0, 65):
+        with pytest.raises(afmm.AfmmError) as e:
+            h.eval_host_pipelined(*b, pieces=p)
+        assert e.value.status == afmm.AFMM_EINVAL
+    with pytest.raises(afmm.AfmmError):
+        h.eval_host_pipelined(*[np.zeros(999, np.float32) for _ in range(8)])
+    h.close()
+    s = afmm.P2P(law=afmm.LAW_STOKESLET)
+    with pytest.raises(afmm.AfmmError) as e:
+        s.eval_host_pipelined(*b)
+    s.close()
