@@ -274,13 +274,16 @@ struct ChunkMeta {
 };
 
 // Issue side of a warp's pipeline: the task whose sources are being streamed
-// and the task after it (both claimed from the queue, descriptors in lanes:
-// lane i holds segment i).
+// and the task after it (claimed one task ahead; a deeper prefetch costs more
+// registers than its latency saves).  Descriptors are warp-uniform; segments live in lanes (lane i holds segment i of its task) and
+// `pre` is the exclusive prefix of the current task's segment lengths, so every
+// lane can issue the bulk copy of its own segment's part of a chunk.
 struct Stream {
     int task, nxt;                // task ids (>= n_tasks: none)
     Task t, tn;                   // descriptors (warp-uniform)
     Seg sg, sgn;                  // this lane's segment of t / tn
-    int iseg, ioff, staged;       // cursor within t's source list
+    int pre;                      // sum of the lengths of t's segments before this lane's (seg_count <= 32)
+    int staged;                   // sources of t already staged
 };
 
 __device__ __forceinline__ int claim(const P2PParams &p, int lane) {
@@ -294,9 +297,30 @@ __device__ __forceinline__ void load_task(const P2PParams &p, int id, Task &t, S
     sg = Seg{0, 0};
     if (lane < t.seg_count) sg = p.segs[t.seg_begin + lane];
 }
+__device__ __forceinline__ int excl_prefix(int v, int lane) {
+    int inc = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int u = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc += u;
+    }
+    return inc - v;
+}
+
+// Bulk copies of the part of segment (gstart, len), whose first source has index
+// `pre` in the task's source list, that falls in the chunk [lo, hi).
+template <int kWords>
+__device__ __forceinline__ void copy_piece(const P2PParams &p, float4 *buf, uint64_t *bar, int gstart, int len,
+                                           int pre, int lo, int hi) {
+    const int a = max(pre, lo), b = min(pre + len, hi);
+    if (a < b)
+        tma_load_1d(buf + (size_t)(a - lo) * kWords, p.bodies + (size_t)(gstart + a - pre) * kWords,
+                    (uint32_t)(b - a) * 16u * kWords, bar);
+}
 
 // Stage the next chunk (<= kWCap bodies) of the stream into `buf`; returns
-// false when no task is left.
+// false when no task is left.  Lane 0 posts the byte count, then every lane
+// whose segment overlaps the chunk issues that piece (no warp-serial walk).
 template <int kWords>
 __device__ __forceinline__ bool issue_chunk(const P2PParams &p, Stream &S, float4 *buf, uint64_t *bar,
                                             ChunkMeta *meta, int lane) {
@@ -317,33 +341,27 @@ __device__ __forceinline__ bool issue_chunk(const P2PParams &p, Stream &S, float
         fence_proxy_async();
         mbar_arrive_expect_tx(bar, (uint32_t)nb * 16u * kWords);
     }
-    // pieces of the current segments (warp-uniform walk; lane 0 issues)
-    int filled = 0;
-    while (filled < nb) {
-        int gstart = __shfl_sync(0xffffffffu, S.sg.gstart, S.iseg & 31);
-        int len = __shfl_sync(0xffffffffu, S.sg.len, S.iseg & 31);
-        if (S.iseg >= 32) {                               // rare: > 32 segments
-            const Seg s2 = p.segs[S.t.seg_begin + S.iseg];
-            gstart = s2.gstart;
-            len = s2.len;
-        }
-        const int take = min(len - S.ioff, nb - filled);
-        if (lane == 0)
-            tma_load_1d(buf + (size_t)filled * kWords, p.bodies + (size_t)(gstart + S.ioff) * kWords,
-                        (uint32_t)take * 16u * kWords, bar);
-        filled += take;
-        S.ioff += take;
-        if (S.ioff == len) {
-            ++S.iseg;
-            S.ioff = 0;
+    __syncwarp();
+    const int lo = S.staged, hi = S.staged + nb;
+    if (S.t.seg_count <= 32) {
+        copy_piece<kWords>(p, buf, bar, S.sg.gstart, S.sg.len, S.pre, lo, hi);
+    } else {                                              // rare: > 32 segments, windows of 32
+        int base = 0;
+        for (int w = 0; w < S.t.seg_count && base < hi; w += 32) {
+            Seg sw{0, 0};
+            if (w + lane < S.t.seg_count) sw = p.segs[S.t.seg_begin + w + lane];
+            const int pre = base + excl_prefix(sw.len, lane);
+            copy_piece<kWords>(p, buf, bar, sw.gstart, sw.len, pre, lo, hi);
+            base = __shfl_sync(0xffffffffu, pre + sw.len, 31);
         }
     }
-    S.staged += nb;
+    S.staged = hi;
     if (S.staged >= S.t.nsrc) {                           // advance to the prefetched task
         S.task = S.nxt;
         S.t = S.tn;
         S.sg = S.sgn;
-        S.iseg = S.ioff = S.staged = 0;
+        S.staged = 0;
+        S.pre = excl_prefix(S.sg.len, lane);
         S.nxt = claim(p, lane);                           // and prefetch the one after
         load_task(p, S.nxt, S.tn, S.sgn, lane);
     }
@@ -396,7 +414,8 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
     load_task(p, S.task, S.t, S.sg, lane);
     S.nxt = claim(p, lane);
     load_task(p, S.nxt, S.tn, S.sgn, lane);
-    S.iseg = S.ioff = S.staged = 0;
+    S.staged = 0;
+    S.pre = excl_prefix(S.sg.len, lane);
     int issued = 0;
     for (; issued < kWStages - 1; ++issued)
         if (!issue_chunk<Law::kWords>(p, S, stage[issued % kWStages], &full[issued % kWStages],
@@ -408,6 +427,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
     Partial P;
     P.acc = accw + lane;
     int g = 1, C = 1, rcpC = 65536, c = 0, l = 0;
+    int q32_u = 0, q32_l = 0, s32_u = 0, s32_l = 0;   // lane/g, lane%g, 32/g, 32%g
     bool active = false;
     for (int q = 0; q < issued; ++q) {
         // keep the ring one chunk ahead (across task boundaries)
@@ -425,6 +445,10 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
             c = lane / g;
             l = lane - c * g;
             active = c < C;
+            q32_u = c;
+            q32_l = l;
+            s32_u = C;               // 32/g == C
+            s32_l = 32 - C * g;
             load_targets<Law::kWords>(T, stage[st], p.bodies, m, l, active);
 #pragma unroll
             for (int u = 0; u < kVals; ++u) accw[u * 32 + lane] = 0.0;
@@ -440,9 +464,10 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
         if (m.is_last) {
             if (active) P.fold();
             __syncwarp();
-            // fixed-order fp64 reduction over the warp's copies
+            // fixed-order fp64 reduction over the warp's copies: value j = u*g + l2
+            // (u = 4*slot + component of lane l2); lanes walk j by 32 without dividing
+            int u = q32_u, l2 = q32_l;
             for (int j = lane; j < kVals * g; j += 32) {
-                const int u = j / g, l2 = j - u * g;
                 const double *a = accw + u * 32 + l2;
                 double v = 0.0;
                 for (int cc = 0; cc < C; ++cc) v += a[cc * g];
@@ -451,6 +476,12 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
                     const int comp = u & 3;
                     float *dst = comp == 0 ? p.ax : comp == 1 ? p.ay : comp == 2 ? p.az : p.phi;
                     dst[m.tgt_start + tgt] = Law::out(comp, v, p.G);
+                }
+                u += s32_u;
+                l2 += s32_l;
+                if (l2 >= g) {
+                    l2 -= g;
+                    ++u;
                 }
             }
             if (p.done) {                 // publish the task's outputs (pipelined copy-back waits on it)
