@@ -65,6 +65,76 @@ constexpr int kStageBytesW = kWStages * kWCap * 16;     // per warp
 constexpr int kAccBytesW = kVals * 32 * 8;              // per warp
 constexpr int kDynSmem = kWarps * (kStageBytesW + kAccBytesW);
 
+// ---- target slicing (host and device worklist builders share this; SURVEY
+// S8(a) a5 "leaves bucketed by size, so adaptive leaves of 1..S bodies do not
+// idle lanes").  A slice of m <= 128 targets runs on g = ceil(m/4) lanes per
+// copy and C = 32/g source-split copies, i.e. ceil(nsrc/C) warp iterations.
+// Only the largest m of each C matters (a smaller slice with the same C costs
+// the same), so the candidates are m in {4,8,12,16,20,24,32,40,64,128}.  A leaf
+// of tn targets is cut into slices by an exact integer DP minimising
+//     sum_slices ceil(nsrc / C(m)) + kSliceTaskCost,
+// the second term standing for a task's fixed cost (descriptors, first-chunk
+// latency, copy reduction) in warp iterations.  Integer arithmetic only, so the
+// host and device builders produce identical task lists.
+#ifndef AFMM_TASK_COST
+#define AFMM_TASK_COST 32
+#endif
+constexpr int kSliceCands = 10;
+constexpr long long kSliceTaskCost = AFMM_TASK_COST;
+constexpr int kMaxDpSlices = 64;                // slices of the DP part (<= 255 targets, >= 4 each)
+__host__ __device__ __forceinline__ int slice_cand_m(int i) {
+    return i < 6 ? 4 * (i + 1) : i == 6 ? 32 : i == 7 ? 40 : i == 8 ? 64 : 128;
+}
+__host__ __device__ __forceinline__ int slice_copies(int m) {   // C = 32 / ceil(m / 4)
+    return 32 / ((m + 3) / 4);
+}
+__host__ __device__ __forceinline__ long long slice_iters(long long nsrc, int m) {
+    const long long C = slice_copies(m), ns = nsrc > 1 ? nsrc : 1;
+    return (ns + C - 1) / C;
+}
+// Leaves above 255 targets first take full 128-target slices (100% lane use)
+// until <= 255 targets remain (tn % 128 + 128, so the remainder may still merge
+// with one full block); the DP cuts the rest.  Returns the number of DP slices
+// and writes their sizes (each 1..128) to sz[0..k); *n_full = leading full slices.
+__host__ __device__ inline int plan_slices(int tn, long long nsrc, int *n_full, unsigned char *sz) {
+    int rest = tn, full = 0;
+    if (tn > 255) {
+        rest = tn % 128 + 128;
+        full = (tn - rest) / 128;
+    }
+    *n_full = full;
+    long long cost[kSliceCands];
+    for (int i = 0; i < kSliceCands; ++i) cost[i] = slice_iters(nsrc, slice_cand_m(i)) + kSliceTaskCost;
+    long long f[129];                           // f(a) for the last 129 values of a (ring)
+    unsigned char arg[256];
+    f[0] = 0;
+    for (int a = 1; a <= rest; ++a) {
+        long long best = -1;
+        int bi = 0;
+        for (int i = 0; i < kSliceCands; ++i) {
+            const int m = slice_cand_m(i), prev = a > m ? a - m : 0;
+            const long long v = f[prev % 129] + cost[i];
+            if (best < 0 || v < best) {
+                best = v;
+                bi = i;
+            }
+        }
+        f[a % 129] = best;
+        arg[a] = (unsigned char)bi;
+    }
+    int k = 0;
+    for (int a = rest; a > 0;) {
+        const int m = slice_cand_m(arg[a]) < a ? slice_cand_m(arg[a]) : a;
+        sz[k++] = (unsigned char)m;
+        a -= m;
+    }
+    return k;
+}
+// Size of slice j of a plan (full slices first).
+__host__ __device__ __forceinline__ int plan_size(int j, int n_full, const unsigned char *sz) {
+    return j < n_full ? kTaskTargets : sz[j - n_full];
+}
+
 // Task: targets [tgt_start, +tgt_count <= 128) of the leaf whose bodies start
 // at self_start; self_len = the leaf's size if it is in its own U-list (then
 // the first segment is the leaf itself), else 0; sources = segments

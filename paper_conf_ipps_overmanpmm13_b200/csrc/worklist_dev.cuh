@@ -110,25 +110,11 @@ __global__ void weighted_cut_kernel(int L, int G, const double *__restrict__ P, 
     for (int r = g + 1; r <= G; ++r) split[r] = L;
 }
 
-// k near-equal target slices for a leaf of tn targets and nsrc sources (same
-// model as worklist.inc).
 __device__ __forceinline__ int slices_for(int tn, long long nsrc) {
-    constexpr double kTaskOverhead = 1280.0;
-    const int kmin = (tn + kTaskTargets - 1) / kTaskTargets;
-    int kbest = kmin;
-    double best = 1e300;
-    for (int k = kmin; k <= kmin + 3 && k <= tn; ++k) {
-        // slice sizes are q+1 (r of them) and q (k - r): floor(tn (i+1)/k) - floor(tn i/k)
-        const int q = tn / k, r = tn - q * k;
-        const int g1 = (q + 1 + kTPT - 1) / kTPT, g0 = (q + kTPT - 1) / kTPT;
-        double slots = (double)r * (32.0 / (32 / g1)) + (double)(k - r) * (q > 0 ? 32.0 / (32 / g0) : 0.0);
-        slots = slots * (double)(nsrc > 1 ? nsrc : 1) + kTaskOverhead * k;
-        if (slots < best - 1e-9) {
-            best = slots;
-            kbest = k;
-        }
-    }
-    return kbest;
+    unsigned char sz[kMaxDpSlices];
+    int n_full = 0;
+    const int k = plan_slices(tn, nsrc, &n_full, sz);
+    return n_full + k;
 }
 
 // pass 1 over this rank's leaves [lo, lo+m): segment and slice counts, nsrc,
@@ -185,15 +171,15 @@ __global__ void write_kernel(int m, int lo, const int *__restrict__ ls, const in
         if (w > first_other && segs[w - 1].gstart + segs[w - 1].len == ls[s]) segs[w - 1].len += lc[s];
         else segs[w++] = Seg{ls[s], lc[s]};
     }
-    const int k = ntask[i];
     const long long src = nsrc[i];
-    for (int j = 0; j < k; ++j) {
-        const int a = (int)(((long long)tn * j) / k);
-        const int cnt = (int)(((long long)tn * (j + 1)) / k) - a;
+    unsigned char sz[kMaxDpSlices];
+    int n_full = 0;
+    const int k_dp = plan_slices(tn, src, &n_full, sz);   // n_full + k_dp == ntask[i] (same plan as count_kernel)
+    for (int j = 0, a = 0; j < n_full + k_dp; a += plan_size(j, n_full, sz), ++j) {
         const int q = task_off[i] + j;
+        const int cnt = plan_size(j, n_full, sz);
         tasks[q] = Task{ts + a, cnt, ts, self ? tn : 0, seg_begin, w - seg_begin, (int)src, 0};
-        const int g = (cnt + kTPT - 1) / kTPT;
-        const unsigned long long cost = (unsigned long long)(32 / (32 / g)) * (unsigned long long)(src > 1 ? src : 1);
+        const unsigned long long cost = (unsigned long long)slice_iters(src, cnt);
         keys[q] = ~cost;                              // ascending sort of ~cost = largest cost first
         vals[q] = q;
     }
