@@ -41,6 +41,37 @@ __device__ __forceinline__ void interact2_rcp(const float4 q, const float2 nx, c
     ay = __ffma2_rn(s, dy, ay);
     az = __ffma2_rn(s, dz, az);
 }
+// Variant 4: the three acceleration FFMA2s of one pair in one PTX block (so
+// ptxas may issue them back to back with s in the same operand slot -> .reuse)
+__device__ __forceinline__ unsigned long long f2u(float2 v) {
+    unsigned long long r;
+    asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(v.x), "f"(v.y));
+    return r;
+}
+__device__ __forceinline__ float2 u2f(unsigned long long r) {
+    float2 v;
+    asm("mov.b64 {%0, %1}, %2;" : "=f"(v.x), "=f"(v.y) : "l"(r));
+    return v;
+}
+__device__ __forceinline__ void interact2_blk(const float4 q, const float2 nx, const float2 ny, const float2 nz,
+                                              const float2 e2, unsigned long long &ax, unsigned long long &ay,
+                                              unsigned long long &az, float2 &ph) {
+    const float2 dx = __fadd2_rn(make_float2(q.x, q.x), nx);
+    const float2 dy = __fadd2_rn(make_float2(q.y, q.y), ny);
+    const float2 dz = __fadd2_rn(make_float2(q.z, q.z), nz);
+    float2 r2 = __ffma2_rn(dx, dx, e2);
+    r2 = __ffma2_rn(dy, dy, r2);
+    r2 = __ffma2_rn(dz, dz, r2);
+    float2 inv;
+    inv.x = rsqrt_ftz(r2.x);
+    inv.y = rsqrt_ftz(r2.y);
+    const float2 t = __fmul2_rn(make_float2(q.w, q.w), inv);
+    ph = __fadd2_rn(ph, t);
+    const float2 i2 = __fmul2_rn(inv, inv);
+    const float2 s = __fmul2_rn(t, i2);
+    asm volatile("{\n\tfma.rn.f32x2 %0, %3, %4, %0;\n\tfma.rn.f32x2 %1, %3, %5, %1;\n\tfma.rn.f32x2 %2, %3, %6, %2;\n}"
+                 : "+l"(ax), "+l"(ay), "+l"(az) : "l"(f2u(s)), "l"(f2u(dx)), "l"(f2u(dy)), "l"(f2u(dz)));
+}
 // Variant 2: scalar FP32 ops (no FFMA2)
 __device__ __forceinline__ void interact1(const float4 q, float nx, float ny, float nz, float e2, float &ax,
                                           float &ay, float &az, float &ph) {
@@ -81,6 +112,11 @@ __global__ void __launch_bounds__(32 * kWarpsT, 1) loop_kernel(const float4 *__r
                 for (int q = 0; q < 2; ++q) {
                     if (kVar == 0 || (kVar == 1 && q == 1))
                         interact2<false>(s[k], nx[q], ny[q], nz[q], e2, ax[q], ay[q], az[q], ph[q], false, false);
+                    else if (kVar == 4) {
+                        unsigned long long ux = f2u(ax[q]), uy = f2u(ay[q]), uz = f2u(az[q]);
+                        interact2_blk(s[k], nx[q], ny[q], nz[q], e2, ux, uy, uz, ph[q]);
+                        ax[q] = u2f(ux); ay[q] = u2f(uy); az[q] = u2f(uz);
+                    }
                     else if (kVar == 1 || kVar == 3)
                         interact2_rcp(s[k], nx[q], ny[q], nz[q], e2, ax[q], ay[q], az[q], ph[q]);
                     else {
@@ -151,6 +187,7 @@ int main() {
     run<16, 4, true>(g, out, sms, "16 warps");
     run<12, 2, true>(g, out, sms, "unroll 2");
     run<12, 8, true>(g, out, sms, "unroll 8");
+    run<12, 4, true, 4>(g, out, sms, "a-update asm block");
     run<12, 4, true, 1>(g, out, sms, "rcp on one pair");
     run<12, 4, true, 3>(g, out, sms, "rcp on both pairs");
     run<12, 4, true, 2>(g, out, sms, "scalar FFMA");
