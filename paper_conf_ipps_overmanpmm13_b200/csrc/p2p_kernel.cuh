@@ -33,7 +33,7 @@ namespace afmm {
 
 // Tuning knobs (overridable with -D for tools/tune builds; defaults are the product's).
 #ifndef AFMM_WCAP
-#define AFMM_WCAP 384
+#define AFMM_WCAP 448
 #endif
 #ifndef AFMM_WSTAGES
 #define AFMM_WSTAGES 2
