@@ -4,8 +4,9 @@
 
 One step = one pass of the whole hot path over the workload, with inputs
 resident in HBM: body ingest (pack; broadcast from rank 0 when N > 1), the
-P2P kernel over this rank's target leaves, and (N > 1) the gather of every
-rank's output slice (grouped broadcasts = allgatherv over NCCL).  The tree is
+P2P kernel over this rank's target leaves, which (N > 1) also stores every
+result into every other rank's output array over CUDA-IPC peer windows
+(the fused gather of row a7; a 4-byte all_reduce marks completion).  The tree is
 built once, on the GPU, by the product builder (afmm_tree_build) -- the
 workload is static (BASELINE configs[1], a fixed 1M-body Plummer sphere).
 
@@ -255,15 +256,25 @@ def main():
     flush = torch.empty(64 << 20, dtype=torch.float32, device=dev)   # 256 MiB > 126 MB L2
 
     from paper_conf_ipps_overmanpmm13_b200 import dist as pdist
-    bsplit = [h.get_partition()[1]]
+    close_windows = None
+    if world > 1:
+        # a7 fused: every rank's output array is a peer window of every other
+        # rank's handle (CUDA IPC over NVLink); the P2P kernel stores each result
+        # into all of them as its tasks finish -- no gather after the kernel
+        close_windows = pdist.open_peer_windows(h, out)
+    done = torch.zeros(1, device=dev)
 
     def step():
         if world > 1:
             pdist.replicate([bod[a] for a in range(4)], src=0)    # a4: source replication
         h.set_bodies(bod[0], bod[1], bod[2], bod[3])          # a1: pack (1 kernel)
-        h.eval(out[0], out[1], out[2], out[3])                # a5/a6: P2P (1 kernel)
-        if world > 1:
-            pdist.gather_slices([out[a] for a in range(4)], bsplit[0])   # a7: allgatherv
+        h.eval(out[0], out[1], out[2], out[3])                # a5/a6 + a7: P2P with peer-window stores
+        if world > 1:                                         # completion: all ranks' kernels (and their
+            if args.dist_backend == "nccl":                   # NVLink stores) done before anyone reads
+                dist.all_reduce(done)
+            else:
+                torch.cuda.synchronize()
+                dist.barrier()
 
     # clocks are sampled from the warm-up through the timed region
     clk = ClockSampler(local).__enter__()
@@ -276,7 +287,6 @@ def main():
             times = pdist.allgather_scalar(h.kernel_times(1)[-1], dev)
             if h.rebalance(times, 0.02):
                 rebalanced += 1
-                bsplit[0] = h.get_partition()[1]
     torch.cuda.synchronize()
 
     # ---- timed region
@@ -435,7 +445,8 @@ def main():
                        "interactions_per_step": inter,
                        "l2": "flushed between steps (256 MiB write outside the step events)",
                        "step": ("pack + P2P kernel" if world == 1 else
-                                "broadcast bodies + pack + P2P kernel + allgatherv of output slices"),
+                                "broadcast bodies (NCCL) + pack + P2P kernel storing every result into all "
+                                "ranks' outputs over CUDA-IPC peer windows (fused gather) + 4-byte all_reduce"),
                        "parallelism": f"leaf-partition x{world} (cost model, PAPER L16)",
                        "tree_build_s": round(tree_s, 4), "set_tree_s": round(set_tree_s, 4)},
             "kernel_ms": {"mean": kern_mean, "max_over_ranks": kern_max},
@@ -457,6 +468,8 @@ def main():
         }
         line.update(extra)
         print(json.dumps(line), flush=True)
+    if close_windows is not None:
+        close_windows()
     h.close()
     tree.close()
     if world > 1:

@@ -86,6 +86,16 @@ _sig("afmm_p2p_eval", _i, _p, _p, _p, _p, _p, C.POINTER(Stats))
 _sig("afmm_p2p_eval_host", _i, _p, _p, _p, _p, _p, C.POINTER(Stats))
 _sig("afmm_p2p_eval_host_pipelined", _i, _p, _ll, _p, _p, _p, _p, _p, _p, _p, _p, _i, C.POINTER(Stats))
 _sig("afmm_p2p_stats_get", _i, _p, C.POINTER(Stats))
+_sig("afmm_p2p_set_peer_windows", _i, _p, _i, _p)
+
+
+class IpcHandle(C.Structure):
+    _fields_ = [("handle", C.c_ubyte * 64), ("offset", C.c_longlong)]
+
+
+_sig("afmm_ipc_export", _i, _p, C.POINTER(IpcHandle))
+_sig("afmm_ipc_import", _i, C.POINTER(IpcHandle), C.POINTER(_p), C.POINTER(_p))
+_sig("afmm_ipc_close", _i, _p)
 _sig("afmm_p2p_stream", _p, _p)
 _sig("afmm_p2p_kernel_times", _i, _p, _i, _p)
 _sig("afmm_p2p_destroy", None, _p)
@@ -155,7 +165,35 @@ EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
             "afmm_tree_farfield_counts", "afmm_lb_config_init", "afmm_lb_create", "afmm_lb_step",
             "afmm_lb_predicted", "afmm_lb_state", "afmm_lb_destroy", "afmm_tree_copy_out",
             "afmm_tree_gather", "afmm_tree_scatter", "afmm_tree_destroy", "afmm_tree_last_error",
-            "afmm_tree_rebuild", "afmm_tree_nodes", "afmm_fine_grained", "afmm_p2p_eval_host_pipelined"]
+            "afmm_tree_rebuild", "afmm_tree_nodes", "afmm_fine_grained", "afmm_p2p_eval_host_pipelined",
+            "afmm_p2p_set_peer_windows", "afmm_ipc_export", "afmm_ipc_import", "afmm_ipc_close"]
+
+
+def ipc_export(dev_ptr):
+    """afmm_ipc_export: bytes (64-B cudaIpcMemHandle of the base allocation +
+    8-B offset) describing a device pointer (int) or CUDA tensor."""
+    h = IpcHandle()
+    ptr = dev_ptr.data_ptr() if hasattr(dev_ptr, "data_ptr") else int(dev_ptr)
+    st = _lib.afmm_ipc_export(C.c_void_p(ptr), C.byref(h))
+    if st:
+        raise AfmmError(st, "afmm_ipc_export")
+    return bytes(C.string_at(C.addressof(h), C.sizeof(h)))
+
+
+def ipc_import(blob):
+    """afmm_ipc_import: (device pointer, base) in this process; close with ipc_close(base)."""
+    h = IpcHandle.from_buffer_copy(blob)
+    p, b = _p(), _p()
+    st = _lib.afmm_ipc_import(C.byref(h), C.byref(p), C.byref(b))
+    if st:
+        raise AfmmError(st, "afmm_ipc_import")
+    return p.value, b.value
+
+
+def ipc_close(base):
+    st = _lib.afmm_ipc_close(C.c_void_p(base))
+    if st:
+        raise AfmmError(st, "afmm_ipc_close")
 
 
 def version() -> str:
@@ -387,6 +425,18 @@ class P2P:
             self._check(_lib.afmm_p2p_eval_host(self._h, _ptr(ax), _ptr(ay), _ptr(az), _ptr(phi), sp),
                         "afmm_p2p_eval_host")
         return s.as_dict() if (stats or not _is_device(ax)) else None
+
+    def set_peer_windows(self, windows):
+        """afmm_p2p_set_peer_windows: windows = list of (ax, ay, az, phi) device
+        pointers (ints) or CUDA tensors of n fp32 each; [] clears."""
+        flat = []
+        for w in windows:
+            if len(w) != 4:
+                raise ValueError("a window is (ax, ay, az, phi)")
+            flat += [a.data_ptr() if hasattr(a, "data_ptr") else int(a) for a in w]
+        arr = (C.c_void_p * max(1, len(flat)))(*flat)
+        self._check(_lib.afmm_p2p_set_peer_windows(self._h, len(windows), arr if flat else None),
+                    "afmm_p2p_set_peer_windows")
 
     def eval_host_pipelined(self, x, y, z, m, ax, ay, az, phi, pieces=8):
         """afmm_p2p_eval_host_pipelined: host inputs (tree order) -> host outputs,

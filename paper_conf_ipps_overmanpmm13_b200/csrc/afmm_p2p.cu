@@ -92,6 +92,10 @@ struct afmm_p2p {
     cudaStream_t s_in = nullptr, s_out = nullptr;
     void *wait_value32 = nullptr;                    // cuStreamWaitValue32 (driver entry point)
     cudaEvent_t ev_start = nullptr, ev_in[64] = {}, ev_k[64] = {}, ev_done = nullptr;
+
+    // peer output windows (fused gather, afmm_p2p_set_peer_windows)
+    int n_peers = 0;
+    float *peers[afmm::kMaxWin - 1][4] = {};
 };
 
 namespace {
@@ -848,6 +852,17 @@ extern "C" afmm_status afmm_p2p_rebalance(afmm_p2p *h, const double *rank_ms, do
 
 // ------------------------------------------------------------------ eval
 
+// window 0 = the caller's outputs; windows 1.. = the registered peer windows (fused gather, row a7)
+static void set_windows(afmm_p2p *h, afmm::P2PParams &p, float *ax, float *ay, float *az, float *phi) {
+    p.out[0][0] = ax;
+    p.out[0][1] = ay;
+    p.out[0][2] = az;
+    p.out[0][3] = phi;
+    p.n_win = 1 + h->n_peers;
+    for (int w = 1; w < afmm::kMaxWin; ++w)
+        for (int a = 0; a < 4; ++a) p.out[w][a] = w <= h->n_peers ? h->peers[w - 1][a] : nullptr;
+}
+
 static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, float *phi) {
     afmm::P2PParams p;
     p.bodies = h->d_bodies;
@@ -855,10 +870,7 @@ static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, flo
     p.segs = h->d_segs;
     p.n_tasks = h->n_tasks;
     p.queue = h->d_queue;
-    p.ax = ax;
-    p.ay = ay;
-    p.az = az;
-    p.phi = phi;
+    set_windows(h, p, ax, ay, az, phi);
     p.eps2 = h->cfg.eps2;
     p.G = h->cfg.law == AFMM_LAW_STOKESLET ? 1.0 / (8.0 * 3.14159265358979323846 * (double)h->cfg.mu)
                                            : (double)h->cfg.G;
@@ -1102,10 +1114,11 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
         prm.segs = h->d_segs;
         prm.n_tasks = nt;
         prm.queue = queue;
-        prm.ax = dout[0];
-        prm.ay = dout[1];
-        prm.az = dout[2];
-        prm.phi = dout[3];
+        prm.out[0][0] = dout[0];
+        prm.out[0][1] = dout[1];
+        prm.out[0][2] = dout[2];
+        prm.out[0][3] = dout[3];
+        prm.n_win = 1;
         prm.eps2 = h->cfg.eps2;
         prm.G = (double)h->cfg.G;
         prm.done = done;
@@ -1136,6 +1149,75 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
     return fill_stats(h, stats);
 }
 
+extern "C" afmm_status afmm_p2p_set_peer_windows(afmm_p2p *h, int count, float *const *ptrs) {
+    if (!h) return AFMM_EINVAL;
+    if (count < 0 || count > afmm::kMaxWin - 1)
+        return fail(h, AFMM_EINVAL, "set_peer_windows: count %d outside [0, %d]", count, afmm::kMaxWin - 1);
+    if (count > 0 && !ptrs) return fail(h, AFMM_EINVAL, "set_peer_windows: ptrs is null");
+    for (int k = 0; k < 4 * count; ++k)
+        if (!ptrs[k]) return fail(h, AFMM_EINVAL, "set_peer_windows: pointer %d is null", k);
+    h->n_peers = count;
+    for (int w = 0; w < afmm::kMaxWin - 1; ++w)
+        for (int a = 0; a < 4; ++a) h->peers[w][a] = w < count ? ptrs[4 * w + a] : nullptr;
+    return AFMM_OK;
+}
+
+namespace {
+using RangeFn = CUresult (*)(CUdeviceptr *, size_t *, CUdeviceptr);
+RangeFn address_range_fn() {
+    static RangeFn fn = nullptr;
+    if (!fn) {
+        void *f = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &f, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<RangeFn>(f);
+    }
+    return fn;
+}
+}  // namespace
+
+extern "C" afmm_status afmm_ipc_export(const void *dev_ptr, afmm_ipc_handle *out) {
+    if (!dev_ptr || !out) return AFMM_EINVAL;
+    const RangeFn range = address_range_fn();
+    if (!range) return AFMM_ENOTSUP;
+    CUdeviceptr base = 0;
+    size_t size = 0;
+    if (range(&base, &size, (CUdeviceptr)dev_ptr) != CUDA_SUCCESS) return AFMM_EINVAL;
+    cudaIpcMemHandle_t hd;
+    if (cudaIpcGetMemHandle(&hd, (void *)base) != cudaSuccess) {
+        cudaGetLastError();
+        return AFMM_ECUDA;
+    }
+    static_assert(sizeof(hd) == sizeof(out->handle), "cudaIpcMemHandle_t is 64 bytes");
+    std::memcpy(out->handle, &hd, sizeof(hd));
+    out->offset = (long long)((CUdeviceptr)dev_ptr - base);
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_ipc_import(const afmm_ipc_handle *in, void **dev_ptr, void **base) {
+    if (!in || !dev_ptr || !base || in->offset < 0) return AFMM_EINVAL;
+    cudaIpcMemHandle_t hd;
+    std::memcpy(&hd, in->handle, sizeof(hd));
+    void *b = nullptr;
+    if (cudaIpcOpenMemHandle(&b, hd, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+        cudaGetLastError();
+        return AFMM_ECUDA;
+    }
+    *base = b;
+    *dev_ptr = (char *)b + in->offset;
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_ipc_close(void *base) {
+    if (!base) return AFMM_EINVAL;
+    if (cudaIpcCloseMemHandle(base) != cudaSuccess) {
+        cudaGetLastError();
+        return AFMM_ECUDA;
+    }
+    return AFMM_OK;
+}
+
 extern "C" afmm_status afmm_p2p_stats_get(afmm_p2p *h, afmm_p2p_stats *stats) {
     CHECK_HANDLE(h);
     if (!h->evaluated) return fail(h, AFMM_ESTATE, "stats_get: no eval yet");
@@ -1144,6 +1226,15 @@ extern "C" afmm_status afmm_p2p_stats_get(afmm_p2p *h, afmm_p2p_stats *stats) {
     return fill_stats(h, stats);
 }
 
+#if AFMM_PROF
+// tuning builds only (-DAFMM_PROF=1): the per-warp cycle breakdown of the last P2P launch
+extern "C" int afmm_p2p_prof_read(unsigned long long *host, int n) {
+    const int cap = 148 * 32 * afmm::kProfSlots;
+    n = n < cap ? n : cap;
+    if (cudaMemcpyFromSymbol(host, afmm::afmm_prof_buf, (size_t)n * 8) != cudaSuccess) return -1;
+    return n;
+}
+#endif
 extern "C" int afmm_p2p_kernel_times(afmm_p2p *h, int max_count, double *ms) {
     if (!h || h->poisoned || max_count < 0 || (max_count > 0 && !ms)) return AFMM_EINVAL;
     if (set_device(h)) return AFMM_ECUDA;

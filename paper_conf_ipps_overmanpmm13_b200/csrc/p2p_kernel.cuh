@@ -21,9 +21,9 @@
 //    one-thread-per-target blocks idle them, L16 SIII.C).  No CTA barrier
 //    anywhere: reductions over copies are warp-local.
 //  * math: rsqrt.approx.ftz; 13 packed FP32 ops + 2 MUFU per two interactions.
-//  * accumulation (reading R17): fp32 partials over <= kFold sources per copy,
-//    folded into fp64 accumulators in shared memory; copies reduced in a fixed
-//    order in fp64; one RN rounding to fp32.  Deterministic and independent of
+//  * accumulation (reading R17): fp32 partials over <= kFold (256) sources per
+//    copy, folded into fp64 accumulators in shared memory; at the task's end the
+//    copies are reduced by a fixed-order fp64 shuffle tree; one RN rounding to fp32.  Deterministic and independent of
 //    the partition (bit-identical across world sizes).
 #pragma once
 #include <cstdint>
@@ -48,16 +48,31 @@ namespace afmm {
 #define AFMM_UNROLL 4
 #endif
 #ifndef AFMM_FOLD
-#define AFMM_FOLD 128
+#define AFMM_FOLD 256
+#endif
+#ifndef AFMM_PROF
+#define AFMM_PROF 0                               // per-warp cycle breakdown (tools/prof_breakdown.py)
+#endif
+#if AFMM_PROF
+constexpr int kProfSlots = 16;
+__device__ unsigned long long afmm_prof_buf[148 * 32 * kProfSlots];
+#define PROF_T(v) const long long v = clock64()
+#define PROF_ADD(k, t0) (prof ? (void)(prof[k] += clock64() - (t0)) : (void)0)
+#else
+#define PROF_T(v)
+#define PROF_ADD(k, t0)
 #endif
 constexpr int kWarps = AFMM_WARPS;              // warps per CTA (all consumers)
 constexpr int kThreads = 32 * kWarps;
 constexpr int kWCap = AFMM_WCAP;                // bodies per warp stage
 constexpr int kWStages = AFMM_WSTAGES;          // per-warp TMA ring depth
-constexpr int kTPT = 4;                         // targets per lane
+#ifndef AFMM_TPT
+#define AFMM_TPT 4
+#endif
+constexpr int kTPT = AFMM_TPT;                  // targets per lane (even)
 constexpr int kPairs = kTPT / 2;                // FFMA2 pairs per lane
 constexpr int kVals = 4 * kTPT;                 // fp64 accumulators per lane (ax, ay, az, phi per target)
-constexpr int kTaskTargets = kTPT * 32;         // targets per task (128)
+constexpr int kTaskTargets = kTPT * 32;         // targets per task (32 lanes x kTPT)
 constexpr int kFold = AFMM_FOLD;                // fp32 partial length per copy before the fp64 fold
 constexpr int kMinBlocksPerSM = AFMM_MINB;
 constexpr int kUnroll = AFMM_UNROLL;            // inner-loop unroll (sources)
@@ -81,57 +96,62 @@ constexpr int kDynSmem = kWarps * (kStageBytesW + kAccBytesW);
 #endif
 constexpr int kSliceCands = 10;
 constexpr long long kSliceTaskCost = AFMM_TASK_COST;
-constexpr int kMaxDpSlices = 64;                // slices of the DP part (<= 255 targets, >= 4 each)
-__host__ __device__ __forceinline__ int slice_cand_m(int i) {
-    return i < 6 ? 4 * (i + 1) : i == 6 ? 32 : i == 7 ? 40 : i == 8 ? 64 : 128;
+constexpr int kMaxDpSlices = 2 * kTaskTargets / kTPT + 1;   // slices of the DP part (< 2 kTaskTargets targets)
+// candidate copy counts C (each the largest g = 32 / C lanes per copy), and the
+// largest slice for each: m = kTPT * floor(32 / C)
+__host__ __device__ __forceinline__ int slice_cand_C(int i) {
+    return i == 0 ? 32 : i == 1 ? 16 : i == 2 ? 10 : i == 3 ? 8 : i == 4 ? 6 : i == 5 ? 5 : i == 6 ? 4 : i == 7 ? 3
+         : i == 8 ? 2 : 1;
 }
-__host__ __device__ __forceinline__ int slice_copies(int m) {   // C = 32 / ceil(m / 4)
-    return 32 / ((m + 3) / 4);
+__host__ __device__ __forceinline__ int slice_cand_m(int i) { return kTPT * (32 / slice_cand_C(i)); }
+__host__ __device__ __forceinline__ int slice_copies(int m) {   // C = 32 / ceil(m / kTPT)
+    return 32 / ((m + kTPT - 1) / kTPT);
 }
 __host__ __device__ __forceinline__ long long slice_iters(long long nsrc, int m) {
     const long long C = slice_copies(m), ns = nsrc > 1 ? nsrc : 1;
     return (ns + C - 1) / C;
 }
-// Leaves above 255 targets first take full 128-target slices (100% lane use)
-// until <= 255 targets remain (tn % 128 + 128, so the remainder may still merge
-// with one full block); the DP cuts the rest.  Returns the number of DP slices
-// and writes their sizes (each 1..128) to sz[0..k); *n_full = leading full slices.
-__host__ __device__ inline int plan_slices(int tn, long long nsrc, int *n_full, unsigned char *sz) {
+// Leaves of 2 kTaskTargets or more targets first take full kTaskTargets slices
+// (100% lane use) until < 2 kTaskTargets remain (tn % kTaskTargets + kTaskTargets,
+// so the remainder may still merge with one full block); the DP cuts the rest.  Returns the number of DP slices
+// and writes their sizes (each 1..kTaskTargets) to sz[0..k); *n_full = leading full slices.
+__host__ __device__ inline int plan_slices(int tn, long long nsrc, int *n_full, unsigned short *sz) {
     int rest = tn, full = 0;
-    if (tn > 255) {
-        rest = tn % 128 + 128;
-        full = (tn - rest) / 128;
+    if (tn >= 2 * kTaskTargets) {
+        rest = tn % kTaskTargets + kTaskTargets;
+        full = (tn - rest) / kTaskTargets;
     }
     *n_full = full;
     long long cost[kSliceCands];
     for (int i = 0; i < kSliceCands; ++i) cost[i] = slice_iters(nsrc, slice_cand_m(i)) + kSliceTaskCost;
-    long long f[129];                           // f(a) for the last 129 values of a (ring)
-    unsigned char arg[256];
+    constexpr int kRing = kTaskTargets + 1;
+    long long f[kRing];                         // f(a) for the last kRing values of a (ring)
+    unsigned char arg[2 * kTaskTargets];
     f[0] = 0;
     for (int a = 1; a <= rest; ++a) {
         long long best = -1;
         int bi = 0;
         for (int i = 0; i < kSliceCands; ++i) {
             const int m = slice_cand_m(i), prev = a > m ? a - m : 0;
-            const long long v = f[prev % 129] + cost[i];
+            const long long v = f[prev % kRing] + cost[i];
             if (best < 0 || v < best) {
                 best = v;
                 bi = i;
             }
         }
-        f[a % 129] = best;
+        f[a % kRing] = best;
         arg[a] = (unsigned char)bi;
     }
     int k = 0;
     for (int a = rest; a > 0;) {
         const int m = slice_cand_m(arg[a]) < a ? slice_cand_m(arg[a]) : a;
-        sz[k++] = (unsigned char)m;
+        sz[k++] = (unsigned short)m;
         a -= m;
     }
     return k;
 }
 // Size of slice j of a plan (full slices first).
-__host__ __device__ __forceinline__ int plan_size(int j, int n_full, const unsigned char *sz) {
+__host__ __device__ __forceinline__ int plan_size(int j, int n_full, const unsigned short *sz) {
     return j < n_full ? kTaskTargets : sz[j - n_full];
 }
 
@@ -148,13 +168,16 @@ struct Seg {
     int gstart, len;
 };
 
+constexpr int kMaxWin = 8;                     // own outputs + up to 7 peers (one NVSwitch box)
 struct P2PParams {
     const float4 *bodies;    // packed {x,y,z,m}, tree order
     const Task *tasks;
     const Seg *segs;
     int n_tasks;
     int *queue;              // task counter, zeroed before launch
-    float *ax, *ay, *az, *phi;
+    float *out[kMaxWin][4];  // output windows {ax, ay, az, phi}: [0] = this eval's outputs, [1, n_win) = peer
+                             // ranks' output arrays (NVLink P2P / IPC pointers): the fused gather (row a7)
+    int n_win;
     float eps2;
     double G;                // output scale: G (gravity) or 1/(8 pi mu) (Stokeslet)
     int *done;               // nullptr, or per-piece counters of finished tasks (afmm_p2p_eval_host_pipelined)
@@ -193,6 +216,13 @@ __device__ __forceinline__ void tma_load_1d(void *dst, const void *src, uint32_t
         "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
         ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
 }
+#if AFMM_PROF
+__device__ __forceinline__ long long __smid_dummy() {
+    unsigned r;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
+    return r;
+}
+#endif
 __device__ __forceinline__ float rsqrt_ftz(float x) {
     float y;
     asm("rsqrt.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
@@ -393,9 +423,10 @@ __device__ __forceinline__ void copy_piece(const P2PParams &p, float4 *buf, uint
 // whose segment overlaps the chunk issues that piece (no warp-serial walk).
 template <int kWords>
 __device__ __forceinline__ bool issue_chunk(const P2PParams &p, Stream &S, float4 *buf, uint64_t *bar,
-                                            ChunkMeta *meta, int lane) {
+                                            ChunkMeta *meta, int lane, long long *prof = nullptr) {
     if (S.task >= p.n_tasks) return false;
     const int nb = min(kWCap / kWords, S.t.nsrc - S.staged);
+    PROF_T(t_a);
     if (lane == 0) {
         ChunkMeta m;
         m.tgt_start = S.t.tgt_start;
@@ -412,6 +443,8 @@ __device__ __forceinline__ bool issue_chunk(const P2PParams &p, Stream &S, float
         mbar_arrive_expect_tx(bar, (uint32_t)nb * 16u * kWords);
     }
     __syncwarp();
+    PROF_ADD(12, t_a);
+    PROF_T(t_b);
     const int lo = S.staged, hi = S.staged + nb;
     if (S.t.seg_count <= 32) {
         copy_piece<kWords>(p, buf, bar, S.sg.gstart, S.sg.len, S.pre, lo, hi);
@@ -426,6 +459,8 @@ __device__ __forceinline__ bool issue_chunk(const P2PParams &p, Stream &S, float
         }
     }
     S.staged = hi;
+    PROF_ADD(13, t_b);
+    PROF_T(t_c);
     if (S.staged >= S.t.nsrc) {                           // advance to the prefetched task
         S.task = S.nxt;
         S.t = S.tn;
@@ -435,6 +470,7 @@ __device__ __forceinline__ bool issue_chunk(const P2PParams &p, Stream &S, float
         S.nxt = claim(p, lane);                           // and prefetch the one after
         load_task(p, S.nxt, S.tn, S.sgn, lane);
     }
+    PROF_ADD(14, t_c);
     return true;
 }
 
@@ -477,6 +513,12 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
         fence_mbar_init();
     }
     __syncwarp();
+#if AFMM_PROF
+    long long prof[kProfSlots] = {0};
+    unsigned long long gt0;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt0));
+    PROF_T(t_all);
+#endif
 
     // ---- start the stream: claim two tasks, fill the ring but one stage
     Stream S;
@@ -501,13 +543,26 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
     bool active = false;
     for (int q = 0; q < issued; ++q) {
         // keep the ring one chunk ahead (across task boundaries)
+        PROF_T(t_is);
         if (issued == q + kWStages - 1) {
             const int s2 = issued % kWStages;
+#if AFMM_PROF
+            if (issue_chunk<Law::kWords>(p, S, stage[s2], &full[s2], &meta[s2], lane, prof)) ++issued;
+#else
             if (issue_chunk<Law::kWords>(p, S, stage[s2], &full[s2], &meta[s2], lane)) ++issued;
+#endif
         }
+        PROF_ADD(0, t_is);
         const int st = q % kWStages;
+        PROF_T(t_w);
         mbar_wait(&full[st], (uint32_t)((q / kWStages) & 1));
         const ChunkMeta m = meta[st];
+        PROF_ADD(1, t_w);
+        PROF_T(t_f);
+#if AFMM_PROF
+        prof[6] += 1;
+        prof[7] += m.is_first;
+#endif
         if (m.is_first) {
             g = (m.tgt_count + kTPT - 1) / kTPT;
             C = 32 / g;
@@ -524,6 +579,8 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
             for (int u = 0; u < kVals; ++u) accw[u * 32 + lane] = 0.0;
             P.clear();
         }
+        PROF_ADD(2, t_f);
+        PROF_T(t_m);
         if (active) {
             const int kself = Law::kMaskSelf ? min(max(m.self_len - m.first, 0), m.nb) : 0;
             if (kself > 0) consume<Law, true>(stage[st], c, kself, C, rcpC, T, m.first, e2, P);
@@ -531,27 +588,51 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
             const int k0 = kself <= c ? c : c + C * (((kself - c + C - 1) * rcpC) >> 16);
             consume<Law, false>(stage[st], k0, m.nb, C, rcpC, T, 0, e2, P);
         }
+        PROF_ADD(3, t_m);
+        PROF_T(t_l);
         if (m.is_last) {
-            if (active) P.fold();
-            __syncwarp();
-            // fixed-order fp64 reduction over the warp's copies: value j = u*g + l2
-            // (u = 4*slot + component of lane l2); lanes walk j by 32 without dividing
-            int u = q32_u, l2 = q32_l;
-            for (int j = lane; j < kVals * g; j += 32) {
-                const double *a = accw + u * 32 + l2;
-                double v = 0.0;
-                for (int cc = 0; cc < C; ++cc) v += a[cc * g];
-                const int tgt = kTPT * l2 + (u >> 2);
-                if (tgt < m.tgt_count) {
-                    const int comp = u & 3;
-                    float *dst = comp == 0 ? p.ax : comp == 1 ? p.ay : comp == 2 ? p.az : p.phi;
-                    dst[m.tgt_start + tgt] = Law::out(comp, v, p.G);
+            // final per-lane values (fp64 accumulators + the open fp32 partials), then
+            // a fixed-order fp64 tree over the warp's copies (lanes c*g + l2, c < C):
+            // round o adds copy c+o into copy c for c = 0 mod 2o (R17: fixed order).
+            double v[kVals];
+#pragma unroll
+            for (int q = 0; q < kPairs; ++q) {
+                const double *a = P.acc + 8 * q * 32;
+                v[8 * q + 0] = active ? a[0 * 32] + (double)P.ax[q].x : 0.0;
+                v[8 * q + 1] = active ? a[1 * 32] + (double)P.ay[q].x : 0.0;
+                v[8 * q + 2] = active ? a[2 * 32] + (double)P.az[q].x : 0.0;
+                v[8 * q + 3] = active ? a[3 * 32] + (double)P.ph[q].x : 0.0;
+                v[8 * q + 4] = active ? a[4 * 32] + (double)P.ax[q].y : 0.0;
+                v[8 * q + 5] = active ? a[5 * 32] + (double)P.ay[q].y : 0.0;
+                v[8 * q + 6] = active ? a[6 * 32] + (double)P.az[q].y : 0.0;
+                v[8 * q + 7] = active ? a[7 * 32] + (double)P.ph[q].y : 0.0;
+            }
+            for (int o = 1; o < C; o <<= 1) {
+                const bool take = (c & (2 * o - 1)) == 0 && c + o < C;
+#pragma unroll
+                for (int u = 0; u < kVals; ++u) {
+                    const double w = __shfl_down_sync(0xffffffffu, v[u], o * g);
+                    if (take) v[u] += w;
                 }
-                u += s32_u;
-                l2 += s32_l;
-                if (l2 >= g) {
-                    l2 -= g;
-                    ++u;
+            }
+            if (active && c == 0) {
+#pragma unroll
+                for (int j = 0; j < kTPT; ++j) {
+                    const int tgt = kTPT * l + j;
+                    if (tgt < m.tgt_count) {
+                        const int u = 8 * (j >> 1) + 4 * (j & 1), i = m.tgt_start + tgt;
+                        const float o0 = Law::out(0, v[u + 0], p.G), o1 = Law::out(1, v[u + 1], p.G);
+                        const float o2 = Law::out(2, v[u + 2], p.G), o3 = Law::out(3, v[u + 3], p.G);
+#pragma unroll
+                        for (int w = 0; w < kMaxWin; ++w) {     // own outputs, then every peer window
+                            if (w < p.n_win) {
+                                p.out[w][0][i] = o0;
+                                p.out[w][1][i] = o1;
+                                p.out[w][2][i] = o2;
+                                p.out[w][3][i] = o3;
+                            }
+                        }
+                    }
                 }
             }
             if (p.done) {                 // publish the task's outputs (pipelined copy-back waits on it)
@@ -560,8 +641,22 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
                 if (lane == 0) atomicAdd(p.done + m.piece, 1);
             }
         }
+        PROF_ADD(4, t_l);
+        PROF_T(t_s);
         __syncwarp();                     // stage st (and the accumulators) free again
+        PROF_ADD(5, t_s);
     }
+    if (p.n_win > 1) __threadfence_system();   // peer-window stores performed before the kernel completes
+#if AFMM_PROF
+    PROF_ADD(8, t_all);
+    unsigned long long gt1;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt1));
+    prof[9] = (long long)gt0;
+    prof[10] = (long long)gt1;
+    prof[11] = __smid_dummy();
+    if (lane == 0)
+        for (int k = 0; k < kProfSlots; ++k) afmm_prof_buf[(blockIdx.x * kWarps + warp) * kProfSlots + k] = prof[k];
+#endif
 }
 
 // Stokeslet bodies: {x, y, z, fx}, {fy, fz, 0, 0}

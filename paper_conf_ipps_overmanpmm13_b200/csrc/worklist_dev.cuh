@@ -111,7 +111,7 @@ __global__ void weighted_cut_kernel(int L, int G, const double *__restrict__ P, 
 }
 
 __device__ __forceinline__ int slices_for(int tn, long long nsrc) {
-    unsigned char sz[kMaxDpSlices];
+    unsigned short sz[kMaxDpSlices];
     int n_full = 0;
     const int k = plan_slices(tn, nsrc, &n_full, sz);
     return n_full + k;
@@ -172,7 +172,7 @@ __global__ void write_kernel(int m, int lo, const int *__restrict__ ls, const in
         else segs[w++] = Seg{ls[s], lc[s]};
     }
     const long long src = nsrc[i];
-    unsigned char sz[kMaxDpSlices];
+    unsigned short sz[kMaxDpSlices];
     int n_full = 0;
     const int k_dp = plan_slices(tn, src, &n_full, sz);   // n_full + k_dp == ntask[i] (same plan as count_kernel)
     for (int j = 0, a = 0; j < n_full + k_dp; a += plan_size(j, n_full, sz), ++j) {

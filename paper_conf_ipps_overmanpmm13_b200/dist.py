@@ -10,6 +10,12 @@ CPU in the tests).
                                   ranks (allgatherv as one broadcast per owner);
                                   the paper's blocking copy "into known
                                   locations" (L16 SIII.D).
+* open_peer_windows(h, out)    -- a7 fused: every rank's (4, n) output array is
+                                  opened in every other rank over CUDA IPC and
+                                  registered as a peer window of the library
+                                  handle, so the P2P kernel itself stores each
+                                  result into all ranks' arrays over NVLink
+                                  (no NCCL gather); complete after a barrier.
 * allgather_scalar(v, device)  -- a8: per-rank kernel times for the GPU time
                                   (max over GPUs, L20 SVII.A) and the rebalance.
 """
@@ -40,6 +46,35 @@ def gather_slices(rows, body_split):
         if hi > lo:
             for row in rows:
                 dist.broadcast(row[lo:hi], src=r)
+
+
+def open_peer_windows(h, out):
+    """out: this rank's contiguous (4, n) float32 CUDA tensor (ax, ay, az, phi).
+    Exchanges IPC handles (all_gather_object) and registers the peers' rows as
+    the handle's peer windows.  Returns a function that unregisters and closes
+    them."""
+    from . import ipc_close, ipc_export, ipc_import
+    if out.dim() != 2 or out.shape[0] != 4 or not out.is_contiguous():
+        raise ValueError("out must be a contiguous (4, n) tensor")
+    world, rank = dist.get_world_size(), dist.get_rank()
+    blobs = [None] * world
+    dist.all_gather_object(blobs, ipc_export(out))
+    stride = out.shape[1] * out.element_size()
+    windows, bases = [], []
+    for r in range(world):
+        if r == rank:
+            continue
+        ptr, base = ipc_import(blobs[r])
+        bases.append(base)
+        windows.append(tuple(ptr + a * stride for a in range(4)))
+    h.set_peer_windows(windows)
+    dist.barrier()
+
+    def close():
+        h.set_peer_windows([])
+        for b in bases:
+            ipc_close(b)
+    return close
 
 
 def allgather_scalar(v: float, device) -> np.ndarray:
