@@ -257,11 +257,18 @@ def main():
 
     from paper_conf_ipps_overmanpmm13_b200 import dist as pdist
     close_windows = None
+    gather_mode = "none (N = 1)"
     if world > 1:
         # a7 fused: every rank's output array is a peer window of every other
         # rank's handle (CUDA IPC over NVLink); the P2P kernel stores each result
-        # into all of them as its tasks finish -- no gather after the kernel
-        close_windows = pdist.open_peer_windows(h, out)
+        # into all of them as its tasks finish -- no gather after the kernel.
+        # If a box refuses CUDA IPC between its GPUs, the step falls back to the
+        # NCCL allgatherv of the slices (reported in config.gather).
+        try:
+            close_windows = pdist.open_peer_windows(h, out)
+            gather_mode = "fused: P2P kernel stores into CUDA-IPC peer windows"
+        except Exception as e:  # noqa: BLE001
+            gather_mode = f"NCCL allgatherv (peer windows unavailable: {e})"[:200]
     done = torch.zeros(1, device=dev)
 
     def step():
@@ -269,7 +276,9 @@ def main():
             pdist.replicate([bod[a] for a in range(4)], src=0)    # a4: source replication
         h.set_bodies(bod[0], bod[1], bod[2], bod[3])          # a1: pack (1 kernel)
         h.eval(out[0], out[1], out[2], out[3])                # a5/a6 + a7: P2P with peer-window stores
-        if world > 1:                                         # completion: all ranks' kernels (and their
+        if world > 1 and close_windows is None:
+            pdist.gather_slices([out[a] for a in range(4)], h.get_partition()[1])
+        elif world > 1:                                       # completion: all ranks' kernels (and their
             if args.dist_backend == "nccl":                   # NVLink stores) done before anyone reads
                 dist.all_reduce(done)
             else:
@@ -448,6 +457,7 @@ def main():
                                 "broadcast bodies (NCCL) + pack + P2P kernel storing every result into all "
                                 "ranks' outputs over CUDA-IPC peer windows (fused gather) + 4-byte all_reduce"),
                        "parallelism": f"leaf-partition x{world} (cost model, PAPER L16)",
+                       "gather": gather_mode,
                        "tree_build_s": round(tree_s, 4), "set_tree_s": round(set_tree_s, 4)},
             "kernel_ms": {"mean": kern_mean, "max_over_ranks": kern_max},
             "gpu_time_interactions_per_s": inter / (kern_max * 1e-3),

@@ -326,24 +326,55 @@ struct Targets {
 struct Partial {
     float2 ax[kPairs], ay[kPairs], az[kPairs], ph[kPairs];
     int cnt;                              // sources since the last fold
+    bool folded;                          // the fp64 accumulators hold this task's earlier partials
     double *acc;                          // &acc_w[0][lane]
     __device__ __forceinline__ void clear() {
 #pragma unroll
         for (int q = 0; q < kPairs; ++q) ax[q] = ay[q] = az[q] = ph[q] = make_float2(0.f, 0.f);
         cnt = 0;
     }
+    // fp32 partial -> fp64 accumulators (the first fold of a task initialises them,
+    // so nothing is zeroed at task start and tasks that never fold never touch them)
     __device__ __forceinline__ void fold() {
+        if (folded) {
 #pragma unroll
-        for (int q = 0; q < kPairs; ++q) {
-            double *a = acc + 8 * q * 32;
-            a[0 * 32] += (double)ax[q].x; a[1 * 32] += (double)ay[q].x;
-            a[2 * 32] += (double)az[q].x; a[3 * 32] += (double)ph[q].x;
-            a[4 * 32] += (double)ax[q].y; a[5 * 32] += (double)ay[q].y;
-            a[6 * 32] += (double)az[q].y; a[7 * 32] += (double)ph[q].y;
+            for (int q = 0; q < kPairs; ++q) {
+                double *a = acc + 8 * q * 32;
+                a[0 * 32] += (double)ax[q].x; a[1 * 32] += (double)ay[q].x;
+                a[2 * 32] += (double)az[q].x; a[3 * 32] += (double)ph[q].x;
+                a[4 * 32] += (double)ax[q].y; a[5 * 32] += (double)ay[q].y;
+                a[6 * 32] += (double)az[q].y; a[7 * 32] += (double)ph[q].y;
+            }
+        } else {
+#pragma unroll
+            for (int q = 0; q < kPairs; ++q) {
+                double *a = acc + 8 * q * 32;
+                a[0 * 32] = (double)ax[q].x; a[1 * 32] = (double)ay[q].x;
+                a[2 * 32] = (double)az[q].x; a[3 * 32] = (double)ph[q].x;
+                a[4 * 32] = (double)ax[q].y; a[5 * 32] = (double)ay[q].y;
+                a[6 * 32] = (double)az[q].y; a[7 * 32] = (double)ph[q].y;
+            }
         }
+        folded = true;
         clear();
     }
 };
+
+// Lane mapping of a task with g lanes per copy (1 <= g <= 32): C = 32 / g copies,
+// rcpC = ceil(2^16 / C), rcpG = ceil(2^16 / g) (floor(lane * rcpG / 2^16) == lane / g
+// for lane < 32).  Packed {C | rcpC << 8, rcpG}, read from the constant bank.
+struct LaneMapTable {
+    int2 v[33];
+    constexpr LaneMapTable() : v() {
+        for (int g = 1; g <= 32; ++g) {
+            const int C = 32 / g;
+            v[g].x = C | (((65536 + C - 1) / C) << 8);
+            v[g].y = (65536 + g - 1) / g;
+        }
+    }
+};
+__constant__ constexpr LaneMapTable kLaneMap{};
+__device__ __forceinline__ int2 lane_map(int g) { return kLaneMap.v[g]; }
 
 // Consume sources src[k], k = k0, k0+C, ... < kend; fp32 partials are folded
 // into fp64 before they would exceed kFold sources.  Masks compare k with
@@ -381,8 +412,9 @@ struct ChunkMeta {
 struct Stream {
     int task, nxt;                // task ids (>= n_tasks: none)
     Task t, tn;                   // descriptors (warp-uniform)
-    Seg sg, sgn;                  // this lane's segment of t / tn
+    Seg sg;                       // this lane's segment of t
     int pre;                      // sum of the lengths of t's segments before this lane's (seg_count <= 32)
+    bool pre_ok;                  // pre computed (deferred to t's first chunk issue)
     int staged;                   // sources of t already staged
 };
 
@@ -391,11 +423,15 @@ __device__ __forceinline__ int claim(const P2PParams &p, int lane) {
     if (lane == 0) it = atomicAdd(p.queue, 1);
     return __shfl_sync(0xffffffffu, it, 0);
 }
-__device__ __forceinline__ void load_task(const P2PParams &p, int id, Task &t, Seg &sg, int lane) {
-    if (id >= p.n_tasks) return;
-    t = p.tasks[id];
-    sg = Seg{0, 0};
-    if (lane < t.seg_count) sg = p.segs[t.seg_begin + lane];
+__device__ __forceinline__ void load_desc(const P2PParams &p, int id, Task &t) {
+    if (id < p.n_tasks) t = p.tasks[id];
+}
+// this lane's segment of task t (issued when t becomes current; its prefix is
+// taken one chunk later, so the load's latency hides behind a chunk of math)
+__device__ __forceinline__ Seg load_seg(const P2PParams &p, int id, const Task &t, int lane) {
+    Seg sg{0, 0};
+    if (id < p.n_tasks && lane < t.seg_count) sg = p.segs[t.seg_begin + lane];
+    return sg;
 }
 __device__ __forceinline__ int excl_prefix(int v, int lane) {
     int inc = v;
@@ -425,6 +461,10 @@ template <int kWords>
 __device__ __forceinline__ bool issue_chunk(const P2PParams &p, Stream &S, float4 *buf, uint64_t *bar,
                                             ChunkMeta *meta, int lane, long long *prof = nullptr) {
     if (S.task >= p.n_tasks) return false;
+    if (!S.pre_ok) {
+        S.pre = excl_prefix(S.sg.len, lane);
+        S.pre_ok = true;
+    }
     const int nb = min(kWCap / kWords, S.t.nsrc - S.staged);
     PROF_T(t_a);
     if (lane == 0) {
@@ -464,11 +504,11 @@ __device__ __forceinline__ bool issue_chunk(const P2PParams &p, Stream &S, float
     if (S.staged >= S.t.nsrc) {                           // advance to the prefetched task
         S.task = S.nxt;
         S.t = S.tn;
-        S.sg = S.sgn;
+        S.sg = load_seg(p, S.task, S.t, lane);
+        S.pre_ok = false;
         S.staged = 0;
-        S.pre = excl_prefix(S.sg.len, lane);
         S.nxt = claim(p, lane);                           // and prefetch the one after
-        load_task(p, S.nxt, S.tn, S.sgn, lane);
+        load_desc(p, S.nxt, S.tn);
     }
     PROF_ADD(14, t_c);
     return true;
@@ -499,7 +539,7 @@ __device__ __forceinline__ void load_targets(Targets &T, const float4 *__restric
 }
 
 template <class Law>
-__global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const P2PParams p) {
+__global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const __grid_constant__ P2PParams p) {
     extern __shared__ __align__(128) unsigned char dsmem[];
     __shared__ __align__(8) uint64_t full_all[kWarps][kWStages];
     __shared__ ChunkMeta meta_all[kWarps][kWStages];
@@ -523,11 +563,12 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
     // ---- start the stream: claim two tasks, fill the ring but one stage
     Stream S;
     S.task = claim(p, lane);
-    load_task(p, S.task, S.t, S.sg, lane);
+    load_desc(p, S.task, S.t);
+    S.sg = load_seg(p, S.task, S.t, lane);
+    S.pre_ok = false;
     S.nxt = claim(p, lane);
-    load_task(p, S.nxt, S.tn, S.sgn, lane);
+    load_desc(p, S.nxt, S.tn);
     S.staged = 0;
-    S.pre = excl_prefix(S.sg.len, lane);
     int issued = 0;
     for (; issued < kWStages - 1; ++issued)
         if (!issue_chunk<Law::kWords>(p, S, stage[issued % kWStages], &full[issued % kWStages],
@@ -539,8 +580,8 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
     Partial P;
     P.acc = accw + lane;
     int g = 1, C = 1, rcpC = 65536, c = 0, l = 0;
-    int q32_u = 0, q32_l = 0, s32_u = 0, s32_l = 0;   // lane/g, lane%g, 32/g, 32%g
     bool active = false;
+    P.folded = false;
     for (int q = 0; q < issued; ++q) {
         // keep the ring one chunk ahead (across task boundaries)
         PROF_T(t_is);
@@ -564,20 +605,16 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
         prof[7] += m.is_first;
 #endif
         if (m.is_first) {
-            g = (m.tgt_count + kTPT - 1) / kTPT;
-            C = 32 / g;
-            rcpC = (65536 + C - 1) / C;
-            c = lane / g;
+            g = (m.tgt_count + kTPT - 1) / kTPT;          // kTPT is a power of two: a shift
+            const int2 mg = lane_map(g);                  // {C | rcpC << 8, rcpG}: no integer division
+            C = mg.x & 255;
+            rcpC = mg.x >> 8;
+            c = (lane * mg.y) >> 16;                      // lane / g
             l = lane - c * g;
             active = c < C;
-            q32_u = c;
-            q32_l = l;
-            s32_u = C;               // 32/g == C
-            s32_l = 32 - C * g;
             load_targets<Law::kWords>(T, stage[st], p.bodies, m, l, active);
-#pragma unroll
-            for (int u = 0; u < kVals; ++u) accw[u * 32 + lane] = 0.0;
             P.clear();
+            P.folded = false;
         }
         PROF_ADD(2, t_f);
         PROF_T(t_m);
@@ -591,29 +628,52 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
         PROF_ADD(3, t_m);
         PROF_T(t_l);
         if (m.is_last) {
-            // final per-lane values (fp64 accumulators + the open fp32 partials), then
-            // a fixed-order fp64 tree over the warp's copies (lanes c*g + l2, c < C):
-            // round o adds copy c+o into copy c for c = 0 mod 2o (R17: fixed order).
+            // final per-lane values, then a fixed-order tree over the warp's copies
+            // (lanes c*g + l2, c < C): round o adds copy c+o into copy c for c = 0 mod 2o
+            // (R17).  If no lane folded (every copy's sources fit one fp32 partial) the
+            // tree runs on the fp32 partials, else in fp64 on accumulators + partials.
             double v[kVals];
+            if (__any_sync(0xffffffffu, P.folded)) {
 #pragma unroll
-            for (int q = 0; q < kPairs; ++q) {
-                const double *a = P.acc + 8 * q * 32;
-                v[8 * q + 0] = active ? a[0 * 32] + (double)P.ax[q].x : 0.0;
-                v[8 * q + 1] = active ? a[1 * 32] + (double)P.ay[q].x : 0.0;
-                v[8 * q + 2] = active ? a[2 * 32] + (double)P.az[q].x : 0.0;
-                v[8 * q + 3] = active ? a[3 * 32] + (double)P.ph[q].x : 0.0;
-                v[8 * q + 4] = active ? a[4 * 32] + (double)P.ax[q].y : 0.0;
-                v[8 * q + 5] = active ? a[5 * 32] + (double)P.ay[q].y : 0.0;
-                v[8 * q + 6] = active ? a[6 * 32] + (double)P.az[q].y : 0.0;
-                v[8 * q + 7] = active ? a[7 * 32] + (double)P.ph[q].y : 0.0;
-            }
-            for (int o = 1; o < C; o <<= 1) {
-                const bool take = (c & (2 * o - 1)) == 0 && c + o < C;
-#pragma unroll
-                for (int u = 0; u < kVals; ++u) {
-                    const double w = __shfl_down_sync(0xffffffffu, v[u], o * g);
-                    if (take) v[u] += w;
+                for (int q = 0; q < kPairs; ++q) {
+                    const double *a = P.acc + 8 * q * 32;
+                    const bool f = active && P.folded;
+                    v[8 * q + 0] = (f ? a[0 * 32] : 0.0) + (double)P.ax[q].x;
+                    v[8 * q + 1] = (f ? a[1 * 32] : 0.0) + (double)P.ay[q].x;
+                    v[8 * q + 2] = (f ? a[2 * 32] : 0.0) + (double)P.az[q].x;
+                    v[8 * q + 3] = (f ? a[3 * 32] : 0.0) + (double)P.ph[q].x;
+                    v[8 * q + 4] = (f ? a[4 * 32] : 0.0) + (double)P.ax[q].y;
+                    v[8 * q + 5] = (f ? a[5 * 32] : 0.0) + (double)P.ay[q].y;
+                    v[8 * q + 6] = (f ? a[6 * 32] : 0.0) + (double)P.az[q].y;
+                    v[8 * q + 7] = (f ? a[7 * 32] : 0.0) + (double)P.ph[q].y;
                 }
+                for (int o = 1; o < C; o <<= 1) {
+                    const bool take = (c & (2 * o - 1)) == 0 && c + o < C;
+#pragma unroll
+                    for (int u = 0; u < kVals; ++u) {
+                        const double w = __shfl_down_sync(0xffffffffu, v[u], o * g);
+                        if (take) v[u] += w;
+                    }
+                }
+            } else {
+                float f[kVals];
+#pragma unroll
+                for (int q = 0; q < kPairs; ++q) {
+                    f[8 * q + 0] = P.ax[q].x; f[8 * q + 1] = P.ay[q].x;
+                    f[8 * q + 2] = P.az[q].x; f[8 * q + 3] = P.ph[q].x;
+                    f[8 * q + 4] = P.ax[q].y; f[8 * q + 5] = P.ay[q].y;
+                    f[8 * q + 6] = P.az[q].y; f[8 * q + 7] = P.ph[q].y;
+                }
+                for (int o = 1; o < C; o <<= 1) {
+                    const bool take = (c & (2 * o - 1)) == 0 && c + o < C;
+#pragma unroll
+                    for (int u = 0; u < kVals; ++u) {
+                        const float w = __shfl_down_sync(0xffffffffu, f[u], o * g);
+                        if (take) f[u] = __fadd_rn(f[u], w);
+                    }
+                }
+#pragma unroll
+                for (int u = 0; u < kVals; ++u) v[u] = (double)f[u];
             }
             if (active && c == 0) {
 #pragma unroll
@@ -623,9 +683,13 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
                         const int u = 8 * (j >> 1) + 4 * (j & 1), i = m.tgt_start + tgt;
                         const float o0 = Law::out(0, v[u + 0], p.G), o1 = Law::out(1, v[u + 1], p.G);
                         const float o2 = Law::out(2, v[u + 2], p.G), o3 = Law::out(3, v[u + 3], p.G);
-#pragma unroll
-                        for (int w = 0; w < kMaxWin; ++w) {     // own outputs, then every peer window
-                            if (w < p.n_win) {
+                        p.out[0][0][i] = o0;                    // own outputs
+                        p.out[0][1][i] = o1;
+                        p.out[0][2][i] = o2;
+                        p.out[0][3][i] = o3;
+                        if (p.n_win > 1) {                      // then every peer window (fused gather)
+#pragma unroll 1
+                            for (int w = 1; w < p.n_win; ++w) {
                                 p.out[w][0][i] = o0;
                                 p.out[w][1][i] = o1;
                                 p.out[w][2][i] = o2;
