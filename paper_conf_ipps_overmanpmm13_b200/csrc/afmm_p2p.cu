@@ -884,6 +884,7 @@ static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, flo
     if (p.n_tasks > 0) {
         const int grid = std::max(1, std::min((p.n_tasks + afmm::kWarps - 1) / afmm::kWarps,
                                               h->num_sms * h->blocks_per_sm));
+        p.static_rounds = afmm::static_rounds(p.n_tasks, grid * afmm::kWarps);
         if (h->cfg.law == AFMM_LAW_STOKESLET)
             afmm::p2p_kernel_t<afmm::Stokeslet><<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(p);
         else
@@ -1114,6 +1115,7 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
         prm.segs = h->d_segs;
         prm.n_tasks = nt;
         prm.queue = queue;
+        prm.static_rounds = 0;                       // pieces complete in claim order
         prm.out[0][0] = dout[0];
         prm.out[0][1] = dout[1];
         prm.out[0][2] = dout[2];

@@ -91,6 +91,15 @@ constexpr int kDynSmem = kWarps * (kStageBytesW + kAccBytesW);
 // the second term standing for a task's fixed cost (descriptors, first-chunk
 // latency, copy reduction) in warp iterations.  Integer arithmetic only, so the
 // host and device builders produce identical task lists.
+#ifndef AFMM_ALLMASK
+#define AFMM_ALLMASK 0                            // chunks holding self sources run wholly in the masked loop
+#endif
+#ifndef AFMM_STATIC_FRAC
+#define AFMM_STATIC_FRAC 0.9                      // share of the tasks dealt statically (snake rounds) ...
+#endif
+#ifndef AFMM_STATIC_MIN_TASKS
+#define AFMM_STATIC_MIN_TASKS 48                  // ... when there are at least this many tasks per warp
+#endif
 #ifndef AFMM_TASK_COST
 #define AFMM_TASK_COST 32
 #endif
@@ -174,7 +183,9 @@ struct P2PParams {
     const Task *tasks;
     const Seg *segs;
     int n_tasks;
-    int *queue;              // task counter, zeroed before launch
+    int *queue;              // task counter of the dynamic tail, zeroed before launch
+    int static_rounds;       // R: tasks [0, R*W) are dealt to the W warps in snake order (no atomic),
+                             // tasks [R*W, n_tasks) are claimed from `queue`
     float *out[kMaxWin][4];  // output windows {ax, ay, az, phi}: [0] = this eval's outputs, [1, n_win) = peer
                              // ranks' output arrays (NVLink P2P / IPC pointers): the fused gather (row a7)
     int n_win;
@@ -416,12 +427,30 @@ struct Stream {
     int pre;                      // sum of the lengths of t's segments before this lane's (seg_count <= 32)
     bool pre_ok;                  // pre computed (deferred to t's first chunk issue)
     int staged;                   // sources of t already staged
+    int seq;                      // tasks this warp has taken (claim)
 };
 
-__device__ __forceinline__ int claim(const P2PParams &p, int lane) {
+// Rounds of the static deal for n tasks over W warps: floor(frac * n / W) when
+// tasks are small and many (>= AFMM_STATIC_MIN_TASKS per warp, small S: there the
+// claim's atomic latency is a visible share of a task), else 0 (all dynamic: with
+// few, long tasks the cost model's error would unbalance a static deal).  A/B on
+// C2: S = 32 +4.6 %, S = 512 -9 % if dealt statically (DESIGN.md v10).
+__host__ __device__ inline int static_rounds(int n, int W) {
+    if (W <= 0 || n < (long long)AFMM_STATIC_MIN_TASKS * W) return 0;
+    return (int)((double)AFMM_STATIC_FRAC * n / W);
+}
+// The warp's seq-th task.  Tasks are sorted largest-cost-first; the first R
+// rounds of W (= all warps of the grid) are dealt in snake order -- round r
+// gives warp w task r*W + w (r even) or r*W + W-1-w (r odd), an LPT-style deal
+// that needs no atomic and whose ids are known ahead -- and the smaller tasks
+// after them are claimed dynamically, which absorbs the static part's error.
+__device__ __forceinline__ int claim(const P2PParams &p, int &seq, int lane) {
+    const int W = gridDim.x * kWarps, gw = blockIdx.x * kWarps + (threadIdx.x >> 5);
+    const int r = seq++;
+    if (r < p.static_rounds) return r * W + ((r & 1) ? W - 1 - gw : gw);
     int it = 0;
     if (lane == 0) it = atomicAdd(p.queue, 1);
-    return __shfl_sync(0xffffffffu, it, 0);
+    return p.static_rounds * W + __shfl_sync(0xffffffffu, it, 0);
 }
 __device__ __forceinline__ void load_desc(const P2PParams &p, int id, Task &t) {
     if (id < p.n_tasks) t = p.tasks[id];
@@ -507,7 +536,7 @@ __device__ __forceinline__ bool issue_chunk(const P2PParams &p, Stream &S, float
         S.sg = load_seg(p, S.task, S.t, lane);
         S.pre_ok = false;
         S.staged = 0;
-        S.nxt = claim(p, lane);                           // and prefetch the one after
+        S.nxt = claim(p, S.seq, lane);                    // and prefetch the one after
         load_desc(p, S.nxt, S.tn);
     }
     PROF_ADD(14, t_c);
@@ -562,11 +591,12 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
 
     // ---- start the stream: claim two tasks, fill the ring but one stage
     Stream S;
-    S.task = claim(p, lane);
+    S.seq = 0;
+    S.task = claim(p, S.seq, lane);
     load_desc(p, S.task, S.t);
     S.sg = load_seg(p, S.task, S.t, lane);
     S.pre_ok = false;
-    S.nxt = claim(p, lane);
+    S.nxt = claim(p, S.seq, lane);
     load_desc(p, S.nxt, S.tn);
     S.staged = 0;
     int issued = 0;
@@ -620,10 +650,18 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
         PROF_T(t_m);
         if (active) {
             const int kself = Law::kMaskSelf ? min(max(m.self_len - m.first, 0), m.nb) : 0;
+#if AFMM_ALLMASK
+            if (kself > 0) {             // the whole chunk in the masked loop (one call, one remainder)
+                consume<Law, true>(stage[st], c, m.nb, C, rcpC, T, m.first, e2, P);
+            } else {
+                consume<Law, false>(stage[st], c, m.nb, C, rcpC, T, 0, e2, P);
+            }
+#else
             if (kself > 0) consume<Law, true>(stage[st], c, kself, C, rcpC, T, m.first, e2, P);
             // first k >= kself with k = c (mod C)
             const int k0 = kself <= c ? c : c + C * (((kself - c + C - 1) * rcpC) >> 16);
             consume<Law, false>(stage[st], k0, m.nb, C, rcpC, T, 0, e2, P);
+#endif
         }
         PROF_ADD(3, t_m);
         PROF_T(t_l);
