@@ -41,7 +41,7 @@ class AfmmError(RuntimeError):
 class Config(C.Structure):
     _fields_ = [("device", C.c_int), ("rank", C.c_int), ("world", C.c_int), ("G", C.c_float),
                 ("eps2", C.c_float), ("max_leaf", C.c_int), ("stream", C.c_void_p), ("law", C.c_int),
-                ("mu", C.c_float)]
+                ("mu", C.c_float), ("slice_world", C.c_int)]
 
 
 LAW_GRAVITY, LAW_STOKESLET = 0, 1
@@ -310,7 +310,7 @@ class P2P:
     """One afmm_p2p handle (one per rank / GPU)."""
 
     def __init__(self, device=0, rank=0, world=1, G=1.0, eps2=0.0, max_leaf=None, stream=None,
-                 law=LAW_GRAVITY, mu=1.0):
+                 law=LAW_GRAVITY, mu=1.0, slice_world=0):
         cfg = Config()
         _lib.afmm_p2p_config_init(C.byref(cfg))
         cfg.device, cfg.rank, cfg.world = int(device), int(rank), int(world)
@@ -319,6 +319,7 @@ class P2P:
             cfg.max_leaf = int(max_leaf)
         cfg.stream = stream
         cfg.law, cfg.mu = int(law), float(mu)
+        cfg.slice_world = int(slice_world)
         h = _p()
         st = _lib.afmm_p2p_create(C.byref(cfg), C.byref(h))
         if st:

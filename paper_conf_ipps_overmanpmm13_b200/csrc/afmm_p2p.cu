@@ -153,6 +153,8 @@ afmm_status ensure_device(afmm_p2p *h, T **ptr, size_t &cap, size_t count) {
     return AFMM_OK;
 }
 
+int slice_world(const afmm_p2p *h) { return h->cfg.slice_world > 0 ? h->cfg.slice_world : h->cfg.world; }
+
 afmm_status set_device(afmm_p2p *h) {
     CUDA_TRY(h, cudaSetDevice(h->cfg.device));
     return AFMM_OK;
@@ -238,6 +240,7 @@ extern "C" afmm_status afmm_p2p_config_init(afmm_p2p_config *cfg) {
     cfg->stream = nullptr;
     cfg->law = AFMM_LAW_GRAVITY;
     cfg->mu = 1.0f;
+    cfg->slice_world = 0;
     return AFMM_OK;
 }
 
@@ -251,7 +254,7 @@ extern "C" afmm_status afmm_p2p_create(const afmm_p2p_config *cfg, afmm_p2p **ou
     if (cfg->max_leaf < 1 || cfg->world < 1 || cfg->rank < 0 || cfg->rank >= cfg->world ||
         !std::isfinite(cfg->G) || !std::isfinite(cfg->eps2) || !(cfg->eps2 >= 0.0f) ||
         cfg->device < 0 || (cfg->law != AFMM_LAW_GRAVITY && cfg->law != AFMM_LAW_STOKESLET) ||
-        !std::isfinite(cfg->mu) || !(cfg->mu > 0.0f))
+        !std::isfinite(cfg->mu) || !(cfg->mu > 0.0f) || cfg->slice_world < 0)
         return AFMM_EINVAL;
     afmm_p2p *h = new (std::nothrow) afmm_p2p();
     if (!h) return AFMM_ENOMEM;
@@ -593,6 +596,7 @@ extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const
     CUDA_TRY(h, cudaStreamSynchronize(s));
     // 3. this rank's work list
     const int r = h->cfg.rank;
+    const long long cap = afmm::task_cap(h->I_total / slice_world(h), (long long)h->num_sms * h->blocks_per_sm * afmm::kWarps);
     const int lo = (int)h->leaf_split[r], m = (int)(h->leaf_split[r + 1] - h->leaf_split[r]);
     if ((st = dws(h, sNseg, &nseg, (size_t)m + 1)) || (st = dws(h, sNtask, &ntask, (size_t)m + 1)) ||
         (st = dws(h, sNsrc, &nsrc, (size_t)m + 1)) || (st = dws(h, sSegOff, &seg_off, (size_t)m + 1)) ||
@@ -603,7 +607,7 @@ extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const
     CUDA_TRY(h, cudaMemsetAsync(ntask + m, 0, sizeof(int), s));
     if (m > 0) {
         dev::count_kernel<<<grid(m), TH, 0, s>>>(m, lo, leaf_start, leaf_count, u_off, u_idx, I, nseg, ntask, nsrc,
-                                                stats);
+                                                stats, cap);
         CUDA_TRY(h, cudaGetLastError());
     }
     {
@@ -629,7 +633,7 @@ extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const
         return st;
     if (m > 0) {
         dev::write_kernel<<<grid(m), TH, 0, s>>>(m, lo, leaf_start, leaf_count, u_off, u_idx, seg_off, task_off,
-                                                ntask, nsrc, h->d_segs, tasks_u, keys, vals);
+                                                ntask, nsrc, h->d_segs, tasks_u, keys, vals, cap);
         CUDA_TRY(h, cudaGetLastError());
     }
     if (nt > 0) {

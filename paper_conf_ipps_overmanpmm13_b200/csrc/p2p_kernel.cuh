@@ -120,17 +120,30 @@ __host__ __device__ __forceinline__ long long slice_iters(long long nsrc, int m)
     const long long C = slice_copies(m), ns = nsrc > 1 ? nsrc : 1;
     return (ns + C - 1) / C;
 }
-// Leaves of 2 kTaskTargets or more targets first take full kTaskTargets slices
-// (100% lane use) until < 2 kTaskTargets remain (tn % kTaskTargets + kTaskTargets,
-// so the remainder may still merge with one full block); the DP cuts the rest.  Returns the number of DP slices
-// and writes their sizes (each 1..kTaskTargets) to sz[0..k); *n_full = leading full slices.
-__host__ __device__ inline int plan_slices(int tn, long long nsrc, int *n_full, unsigned short *sz) {
+// Task-size cap (strong scaling): a slice may cost at most `cap` warp iterations,
+// so the largest task stays a small fraction of a warp's share of the launch (with
+// few tasks per warp the kernel would otherwise last as long as its largest task).
+// Candidates whose ceil(nsrc / C) exceeds the cap are dropped, except m = kTPT
+// (C = 32), the smallest slice.  Leaves of 2 M or more targets, M the largest
+// allowed candidate, first take full M-target slices until < 2 M remain
+// (tn % M + M, so the remainder may still merge with one full block); the DP cuts
+// the rest.  Returns the number of DP slices and writes their sizes (each
+// 1..kTaskTargets) to sz[0..k); *n_full = leading full slices of *full_m targets.
+__host__ __device__ inline int plan_slices(int tn, long long nsrc, long long cap, int *n_full, int *full_m,
+                                           unsigned short *sz) {
+    bool ok[kSliceCands];
+    int M = slice_cand_m(0);
+    for (int i = 0; i < kSliceCands; ++i) {
+        ok[i] = i == 0 || slice_iters(nsrc, slice_cand_m(i)) <= cap;
+        if (ok[i]) M = slice_cand_m(i);
+    }
     int rest = tn, full = 0;
-    if (tn >= 2 * kTaskTargets) {
-        rest = tn % kTaskTargets + kTaskTargets;
-        full = (tn - rest) / kTaskTargets;
+    if (tn >= 2 * M) {
+        rest = tn % M + M;
+        full = (tn - rest) / M;
     }
     *n_full = full;
+    *full_m = M;
     long long cost[kSliceCands];
     for (int i = 0; i < kSliceCands; ++i) cost[i] = slice_iters(nsrc, slice_cand_m(i)) + kSliceTaskCost;
     constexpr int kRing = kTaskTargets + 1;
@@ -141,6 +154,7 @@ __host__ __device__ inline int plan_slices(int tn, long long nsrc, int *n_full, 
         long long best = -1;
         int bi = 0;
         for (int i = 0; i < kSliceCands; ++i) {
+            if (!ok[i]) continue;
             const int m = slice_cand_m(i), prev = a > m ? a - m : 0;
             const long long v = f[prev % kRing] + cost[i];
             if (best < 0 || v < best) {
@@ -160,8 +174,19 @@ __host__ __device__ inline int plan_slices(int tn, long long nsrc, int *n_full, 
     return k;
 }
 // Size of slice j of a plan (full slices first).
-__host__ __device__ __forceinline__ int plan_size(int j, int n_full, const unsigned short *sz) {
-    return j < n_full ? kTaskTargets : sz[j - n_full];
+__host__ __device__ __forceinline__ int plan_size(int j, int n_full, int full_m, const unsigned short *sz) {
+    return j < n_full ? full_m : sz[j - n_full];
+}
+// Cap for a rank whose tasks total about `inter` interactions on `warps` warps:
+// inter / (32 lanes * kTPT) warp iterations if every lane slot were used, split
+// kCapDiv ways per warp; never below kCapMin.
+#ifndef AFMM_CAP_DIV
+#define AFMM_CAP_DIV 3
+#endif
+constexpr long long kCapMin = 64;
+__host__ __device__ inline long long task_cap(long long inter, long long warps) {
+    const long long c = inter / ((long long)kTaskTargets * (warps > 0 ? warps : 1) * AFMM_CAP_DIV);
+    return c > kCapMin ? c : kCapMin;
 }
 
 // Task: targets [tgt_start, +tgt_count <= 128) of the leaf whose bodies start

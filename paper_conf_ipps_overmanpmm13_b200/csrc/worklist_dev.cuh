@@ -110,10 +110,10 @@ __global__ void weighted_cut_kernel(int L, int G, const double *__restrict__ P, 
     for (int r = g + 1; r <= G; ++r) split[r] = L;
 }
 
-__device__ __forceinline__ int slices_for(int tn, long long nsrc) {
+__device__ __forceinline__ int slices_for(int tn, long long nsrc, long long cap) {
     unsigned short sz[kMaxDpSlices];
-    int n_full = 0;
-    const int k = plan_slices(tn, nsrc, &n_full, sz);
+    int n_full = 0, full_m = 0;
+    const int k = plan_slices(tn, nsrc, cap, &n_full, &full_m, sz);
     return n_full + k;
 }
 
@@ -122,7 +122,8 @@ __device__ __forceinline__ int slices_for(int tn, long long nsrc) {
 __global__ void count_kernel(int m, int lo, const int *__restrict__ ls, const int *__restrict__ lc,
                              const long long *__restrict__ uo, const int *__restrict__ ui,
                              const long long *__restrict__ I, int *__restrict__ nseg, int *__restrict__ ntask,
-                             long long *__restrict__ nsrc, unsigned long long *__restrict__ stats) {
+                             long long *__restrict__ nsrc, unsigned long long *__restrict__ stats,
+                             long long cap) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= m) return;
     const int t = lo + i;
@@ -142,7 +143,7 @@ __global__ void count_kernel(int m, int lo, const int *__restrict__ ls, const in
     }
     nseg[i] = segs + (self ? 1 : 0);
     nsrc[i] = src;
-    ntask[i] = slices_for(lc[t], src);
+    ntask[i] = slices_for(lc[t], src, cap);
     atomicAdd(&stats[0], (unsigned long long)I[t]);
     atomicAdd(&stats[1 + bucket_of_d(lc[t])], (unsigned long long)I[t]);
 }
@@ -153,7 +154,7 @@ __global__ void write_kernel(int m, int lo, const int *__restrict__ ls, const in
                              const int *__restrict__ seg_off, const int *__restrict__ task_off,
                              const int *__restrict__ ntask, const long long *__restrict__ nsrc,
                              Seg *__restrict__ segs, Task *__restrict__ tasks,
-                             unsigned long long *__restrict__ keys, int *__restrict__ vals) {
+                             unsigned long long *__restrict__ keys, int *__restrict__ vals, long long cap) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= m) return;
     const int t = lo + i;
@@ -173,11 +174,11 @@ __global__ void write_kernel(int m, int lo, const int *__restrict__ ls, const in
     }
     const long long src = nsrc[i];
     unsigned short sz[kMaxDpSlices];
-    int n_full = 0;
-    const int k_dp = plan_slices(tn, src, &n_full, sz);   // n_full + k_dp == ntask[i] (same plan as count_kernel)
-    for (int j = 0, a = 0; j < n_full + k_dp; a += plan_size(j, n_full, sz), ++j) {
+    int n_full = 0, full_m = 0;
+    const int k_dp = plan_slices(tn, src, cap, &n_full, &full_m, sz);   // same plan as count_kernel
+    for (int j = 0, a = 0; j < n_full + k_dp; a += plan_size(j, n_full, full_m, sz), ++j) {
         const int q = task_off[i] + j;
-        const int cnt = plan_size(j, n_full, sz);
+        const int cnt = plan_size(j, n_full, full_m, sz);
         tasks[q] = Task{ts + a, cnt, ts, self ? tn : 0, seg_begin, w - seg_begin, (int)src, 0};
         const unsigned long long cost = (unsigned long long)slice_iters(src, cnt);
         keys[q] = ~cost;                              // ascending sort of ~cost = largest cost first

@@ -4,6 +4,9 @@ No arithmetic of the method lives here: these helpers only move the library's
 inputs and outputs between ranks (NCCL over NVLink/NVSwitch on B200; gloo on
 CPU in the tests).
 
+* packed_bodies(h, device)     -- a4: the library's packed body array as a
+                                  tensor: the root packs, one broadcast of it
+                                  replicates the bodies (bench.py N > 1).
 * replicate(tensors, src)      -- a4: "building the data to send to the GPUs"
                                   (PAPER L16 SIII.C): every rank holds all bodies.
 * gather_slices(rows, split)   -- a7: every rank's disjoint output slice to all
@@ -31,6 +34,21 @@ def body_split_from(leaf_split, leaf_start, n):
     ls = np.asarray(leaf_split, np.int64)
     L = len(leaf_start)
     return np.array([n if v >= L else int(leaf_start[v]) for v in ls], np.int64)
+
+
+class _DeviceArray:
+    """A raw device range as a __cuda_array_interface__ object (zero copy)."""
+
+    def __init__(self, ptr, nbytes):
+        self.__cuda_array_interface__ = {"shape": (nbytes // 4,), "typestr": "<f4", "data": (int(ptr), False),
+                                         "version": 3}
+
+
+def packed_bodies(h, device):
+    """The handle's packed {x, y, z, m} body array (afmm_p2p_bodies_buffer) as a
+    float32 CUDA tensor view, for one NCCL broadcast of the packed bodies (a4)."""
+    ptr, nbytes = h.bodies_buffer()
+    return torch.as_tensor(_DeviceArray(ptr, nbytes), device=device)
 
 
 def replicate(tensors, src=0):

@@ -40,9 +40,9 @@ def _setup(n, S, seed, dist_name="plummer"):
     return b, T
 
 
-def _eval(b, T, world, rank, out, eps2=1e-6, windows=None):
+def _eval(b, T, world, rank, out, eps2=1e-6, windows=None, slice_world=0):
     afmm = _afmm()
-    h = afmm.P2P(device=0, rank=rank, world=world, eps2=eps2)
+    h = afmm.P2P(device=0, rank=rank, world=world, eps2=eps2, slice_world=slice_world)
     h.set_bodies(b[0], b[1], b[2], b[3])
     h.set_tree(T["leaf_start"], T["leaf_count"], T["u_off"], T["u_idx"])
     if windows is not None:
@@ -56,7 +56,7 @@ def test_windows_single_process_bit_identical(world):
     n = 60000
     b, T = _setup(n, 64, 5)
     ref = torch.full((4, n), float("nan"), device="cuda")
-    _eval(b, T, 1, 0, ref).close()
+    _eval(b, T, 1, 0, ref, slice_world=world).close()        # the same task slicing as the ranks
     outs = [torch.full((4, n), float("nan"), device="cuda") for _ in range(world)]
     hs = []
     for r in range(world):
@@ -131,7 +131,7 @@ def test_ipc_two_processes_same_gpu():
         outs = [np.load(os.path.join(d, f"out{r}.npy")) for r in range(world)]
     b, T = _setup(n, S, seed)
     ref = torch.full((4, n), float("nan"), device="cuda")
-    _eval(b, T, 1, 0, ref).close()
+    _eval(b, T, 1, 0, ref, slice_world=world).close()
     R = ref.cpu().numpy()
     assert np.isfinite(R).all()
     for r in range(world):

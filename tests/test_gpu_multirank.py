@@ -60,7 +60,7 @@ def _worker(rank, world, port, q):
         split = h.get_partition()[0]
         ref = None
         if rank == 0:
-            h1 = afmm.P2P(device=0, eps2=1e-6)
+            h1 = afmm.P2P(device=0, eps2=1e-6, slice_world=world)   # the ranks' task slicing
             h1.set_bodies(bod[0], bod[1], bod[2], bod[3])
             h1.set_tree(T["leaf_start"], T["leaf_count"], T["u_off"], T["u_idx"])
             o1 = torch.empty((4, n), device=dev)
