@@ -541,8 +541,10 @@ extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const
     const int L = n_leaves, W = h->cfg.world, TH = 256;
     auto grid = [&](long long m) { return (int)std::max<long long>(1, (m + TH - 1) / TH); };
     enum { sI, sP, sW, sPW, sSplit, sErr, sNseg, sNtask, sNsrc, sSegOff, sTaskOff, sStats, sKeys, sVals, sKeys2,
-           sVals2, sTasksU, sCoef, sTmp, sBsplit };
+           sVals2, sTasksU, sCoef, sTmp, sBsplit, sPlan, sPlanHdr };
     long long *I, *P, *split, *nsrc, *bsplit;
+    unsigned short *plan;
+    int4 *plan_hdr;
     int *err, *nseg, *ntask, *seg_off, *task_off, *vals, *vals2;
     unsigned long long *stats, *keys, *keys2;
     if ((st = dws(h, sI, &I, L)) || (st = dws(h, sP, &P, L)) || (st = dws(h, sSplit, &split, W + 1)) ||
@@ -600,14 +602,16 @@ extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const
     const int lo = (int)h->leaf_split[r], m = (int)(h->leaf_split[r + 1] - h->leaf_split[r]);
     if ((st = dws(h, sNseg, &nseg, (size_t)m + 1)) || (st = dws(h, sNtask, &ntask, (size_t)m + 1)) ||
         (st = dws(h, sNsrc, &nsrc, (size_t)m + 1)) || (st = dws(h, sSegOff, &seg_off, (size_t)m + 1)) ||
-        (st = dws(h, sTaskOff, &task_off, (size_t)m + 1)) || (st = dws(h, sStats, &stats, 9)))
+        (st = dws(h, sTaskOff, &task_off, (size_t)m + 1)) || (st = dws(h, sStats, &stats, 9)) ||
+        (st = dws(h, sPlan, &plan, (size_t)(m + 1) * afmm::kMaxDpSlices)) ||
+        (st = dws(h, sPlanHdr, &plan_hdr, (size_t)m + 1)))
         return st;
     CUDA_TRY(h, cudaMemsetAsync(stats, 0, 9 * sizeof(unsigned long long), s));
     CUDA_TRY(h, cudaMemsetAsync(nseg + m, 0, sizeof(int), s));
     CUDA_TRY(h, cudaMemsetAsync(ntask + m, 0, sizeof(int), s));
     if (m > 0) {
         dev::count_kernel<<<grid(m), TH, 0, s>>>(m, lo, leaf_start, leaf_count, u_off, u_idx, I, nseg, ntask, nsrc,
-                                                stats, cap);
+                                                stats, cap, plan, plan_hdr);
         CUDA_TRY(h, cudaGetLastError());
     }
     {
@@ -633,15 +637,17 @@ extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const
         return st;
     if (m > 0) {
         dev::write_kernel<<<grid(m), TH, 0, s>>>(m, lo, leaf_start, leaf_count, u_off, u_idx, seg_off, task_off,
-                                                ntask, nsrc, h->d_segs, tasks_u, keys, vals, cap);
+                                                ntask, nsrc, h->d_segs, tasks_u, keys, vals, plan, plan_hdr);
         CUDA_TRY(h, cudaGetLastError());
     }
     if (nt > 0) {
         size_t tb = 0;
-        CUDA_TRY(h, cub::DeviceRadixSort::SortPairs(nullptr, tb, keys, keys2, vals, vals2, nt, 0, 64, s));
+        CUDA_TRY(h, cub::DeviceRadixSort::SortPairs(nullptr, tb, keys, keys2, vals, vals2, nt, 0, 32, s));
         char *tmp;
         if ((st = dws(h, sTmp, &tmp, tb))) return st;
-        CUDA_TRY(h, cub::DeviceRadixSort::SortPairs(tmp, tb, keys, keys2, vals, vals2, nt, 0, 64, s));
+        // keys = ~cost with cost < 2^31 (a task's warp iterations <= its sources < 2^31):
+        // the high half is constant, so the low 32 bits give the same stable order
+        CUDA_TRY(h, cub::DeviceRadixSort::SortPairs(tmp, tb, keys, keys2, vals, vals2, nt, 0, 32, s));
         dev::gather_tasks_kernel<<<grid(nt), TH, 0, s>>>(nt, vals2, tasks_u, h->d_tasks);
         CUDA_TRY(h, cudaGetLastError());
     }

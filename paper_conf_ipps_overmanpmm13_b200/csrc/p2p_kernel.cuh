@@ -146,28 +146,33 @@ __host__ __device__ inline int plan_slices(int tn, long long nsrc, long long cap
     *full_m = M;
     long long cost[kSliceCands];
     for (int i = 0; i < kSliceCands; ++i) cost[i] = slice_iters(nsrc, slice_cand_m(i)) + kSliceTaskCost;
-    constexpr int kRing = kTaskTargets + 1;
-    long long f[kRing];                         // f(a) for the last kRing values of a (ring)
-    unsigned char arg[2 * kTaskTargets];
+    // Every candidate is a multiple of kTPT, so f(a) -- the best cost of cutting a
+    // targets -- is constant on each block (kTPT(q-1), kTPT q] (induction: a - m
+    // stays in one block), and so is the argmin: the DP runs over blocks q.
+    constexpr int kRing = kTaskTargets / kTPT + 1;
+    long long f[kRing];                         // f(block q) for the last kRing blocks (ring)
+    unsigned char arg[2 * kTaskTargets / kTPT + 1];
     f[0] = 0;
-    for (int a = 1; a <= rest; ++a) {
+    const int nb = (rest + kTPT - 1) / kTPT;
+    for (int q = 1; q <= nb; ++q) {
         long long best = -1;
         int bi = 0;
         for (int i = 0; i < kSliceCands; ++i) {
             if (!ok[i]) continue;
-            const int m = slice_cand_m(i), prev = a > m ? a - m : 0;
+            const int mq = slice_cand_m(i) / kTPT, prev = q > mq ? q - mq : 0;
             const long long v = f[prev % kRing] + cost[i];
             if (best < 0 || v < best) {
                 best = v;
                 bi = i;
             }
         }
-        f[a % kRing] = best;
-        arg[a] = (unsigned char)bi;
+        f[q % kRing] = best;
+        arg[q] = (unsigned char)bi;
     }
     int k = 0;
     for (int a = rest; a > 0;) {
-        const int m = slice_cand_m(arg[a]) < a ? slice_cand_m(arg[a]) : a;
+        const int mc = slice_cand_m(arg[(a + kTPT - 1) / kTPT]);
+        const int m = mc < a ? mc : a;
         sz[k++] = (unsigned short)m;
         a -= m;
     }

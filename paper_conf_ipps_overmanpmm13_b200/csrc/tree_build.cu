@@ -150,48 +150,56 @@ enum { kModeFresh = 0, kModeEnforce = 1, kModeKeep = 2 };
 // (L10 SI.B).  Enforce_S (L20 SVI.A; pv.levels > 0) additionally keeps a node
 // with exactly S bodies split when it was a parent before: Collapse applies only
 // to parents with FEWER than S bodies, PushDown only to leaves with MORE than S.
-// Child ranges by binary search on the octant digit inside [b, e).
+// Child ranges by binary search on the octant digit inside [b, e): eight lanes
+// per node, lane o finds the first position with digit >= o (independent
+// searches, so a level costs one search's latency, not seven in a row).
 __global__ void split_count_kernel(int m, int base, Nodes nd, const unsigned long long *__restrict__ keys,
                                    int S, int mode, PrevTree pv, Edits ed, int *__restrict__ cb,
                                    int *__restrict__ nc) {
-    const int i = blockIdx.x * blockDim.x + threadIdx.x;
-    if (i >= m) return;
-    const int id = base + i;
-    const int b = nd.b[id], e = nd.e[id], lev = nd.level[id];
-    int cnt = 0;
-    bool split;
-    if (mode == kModeKeep)            // structure kept: split iff it was a parent (Collapse/PushDown edits below)
-        split = pv.levels > 0 && prev_internal(pv, lev, nd.prefix[id]);
-    else
-        split = e - b > S || (mode == kModeEnforce && e - b == S && pv.levels > 0 &&
-                              prev_internal(pv, lev, nd.prefix[id]));
-    if (ed.n > 0) {
-        const int a = edit_of(ed, lev, nd.prefix[id]);
-        if (a == 1) split = false;
-        else if (a == 2) split = true;
+    const long long gt = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    const int o = (int)(gt & 7);
+    const int i = (int)(gt >> 3);
+    const bool live = i < m;
+    int b = 0, e = 0, lev = 0;
+    bool split = false;
+    if (live) {
+        const int id = base + i;
+        b = nd.b[id];
+        e = nd.e[id];
+        lev = nd.level[id];
+        if (mode == kModeKeep)        // structure kept: split iff it was a parent (Collapse/PushDown edits below)
+            split = pv.levels > 0 && prev_internal(pv, lev, nd.prefix[id]);
+        else
+            split = e - b > S || (mode == kModeEnforce && e - b == S && pv.levels > 0 &&
+                                  prev_internal(pv, lev, nd.prefix[id]));
+        if (ed.n > 0) {
+            const int a = edit_of(ed, lev, nd.prefix[id]);
+            if (a == 1) split = false;
+            else if (a == 2) split = true;
+        }
+        split = split && lev < kMaxLevel;
     }
-    split = split && lev < kMaxLevel;
-    if (split) {
+    int bound = b;                                   // lane o: first position in [b, e) with digit >= o
+    if (split && o > 0) {
         const int shift = 3 * (kMaxLevel - 1 - lev);
-        int bound[9];
-        bound[0] = b;
-        bound[8] = e;
-        for (int o = 1; o < 8; ++o) {
-            int lo = bound[o - 1], hi = e;            // first position with digit >= o
-            while (lo < hi) {
-                const int mid = lo + ((hi - lo) >> 1);
-                if ((int)((keys[mid] >> shift) & 7ull) < o) lo = mid + 1;
-                else hi = mid;
-            }
-            bound[o] = lo;
+        int lo = b, hi = e;
+        while (lo < hi) {
+            const int mid = lo + ((hi - lo) >> 1);
+            if ((int)((keys[mid] >> shift) & 7ull) < o) lo = mid + 1;
+            else hi = mid;
         }
-        for (int o = 0; o < 8; ++o) {
-            cb[i * 9 + o] = bound[o];
-            cnt += bound[o + 1] > bound[o];
-        }
-        cb[i * 9 + 8] = e;
+        bound = lo;
     }
-    nc[i] = cnt;
+    // next boundary (lane o+1's, or e for o = 7) -> is child o non-empty?
+    int nxt = __shfl_down_sync(0xffffffffu, bound, 1, 8);
+    if (o == 7) nxt = e;
+    const unsigned nonempty = __ballot_sync(0xffffffffu, split && nxt > bound);
+    if (!live) return;
+    if (split) {
+        cb[i * 9 + o] = bound;
+        if (o == 7) cb[i * 9 + 8] = e;
+    }
+    if (o == 0) nc[i] = __popc((nonempty >> (threadIdx.x & 24)) & 0xffu);
 }
 
 __global__ void split_write_kernel(int m, int base, int next_base, Nodes nd, const int *__restrict__ cb,
@@ -284,6 +292,102 @@ __global__ void ulist_kernel(int L, Nodes nd, const int *__restrict__ node_leaf,
         }
     }
     if (counts) counts[t] = cnt;
+}
+
+// U-lists by a warp-cooperative level-order descent (one warp per target leaf):
+// the frontier of nodes whose closed box touches the leaf's box is expanded 32
+// nodes at a time, touching leaves are collected, and the row is put in
+// ascending leaf order (= the per-thread DFS order above) by a rank sort.  Rows
+// go to a fixed-capacity scratch row (kURow); counts[t] = row length.  A leaf
+// whose frontier or row exceeds the capacity raises *overflow and the caller
+// falls back to ulist_kernel for the whole tree (same result).
+constexpr int kURow = 256;                  // max row length kept by the warp path
+constexpr int kUFront = 512;                // max frontier length
+constexpr int kUWarps = 4;                  // warps per block
+__global__ void __launch_bounds__(32 * kUWarps) ulist_warp_kernel(int L, Nodes nd, const int *__restrict__ node_leaf,
+                                                                  const int *__restrict__ leaf_node,
+                                                                  int *__restrict__ rows, long long *__restrict__ counts,
+                                                                  int *__restrict__ overflow) {
+    __shared__ int front[kUWarps][2][kUFront];
+    __shared__ int res[kUWarps][kURow];
+    const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5;
+    const int nwarps = gridDim.x * kUWarps;
+    for (int t = blockIdx.x * kUWarps + wi; t < L; t += nwarps) {
+        const int tn = leaf_node[t];
+        long long At[3], wt;
+        box_of(nd.level[tn], nd.prefix[tn], At, wt);
+        int cur = 0, ncur = 1, nres = 0;
+        bool ovf = false;
+        if (lane == 0) front[wi][0][0] = 0;          // the root
+        __syncwarp();
+        while (ncur > 0 && !ovf) {
+            int nnext = 0;
+            for (int j0 = 0; j0 < ncur; j0 += 32) {
+                const int j = j0 + lane;
+                bool leaf = false;
+                int nch = 0, fc = 0, lid = 0;
+                if (j < ncur) {
+                    const int ni = front[wi][cur][j];
+                    long long As[3], ws;
+                    box_of(nd.level[ni], nd.prefix[ni], As, ws);
+                    bool touch = true;
+#pragma unroll
+                    for (int a = 0; a < 3; ++a) touch &= (At[a] <= As[a] + ws) && (As[a] <= At[a] + wt);
+                    if (touch) {
+                        const int c = nd.nchild[ni];
+                        if (c == 0) {
+                            leaf = true;
+                            lid = node_leaf[ni];
+                        } else {
+                            nch = c;
+                            fc = nd.first_child[ni];
+                        }
+                    }
+                }
+                const unsigned lm = __ballot_sync(0xffffffffu, leaf);
+                const int lpos = nres + __popc(lm & ((1u << lane) - 1));
+                if (leaf && lpos < kURow) res[wi][lpos] = lid;
+                nres += __popc(lm);
+                int inc = nch;                        // exclusive prefix of child counts
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const int u = __shfl_up_sync(0xffffffffu, inc, o);
+                    if (lane >= o) inc += u;
+                }
+                const int cpos = nnext + inc - nch;
+                for (int c = 0; c < nch; ++c)
+                    if (cpos + c < kUFront) front[wi][cur ^ 1][cpos + c] = fc + c;
+                nnext += __shfl_sync(0xffffffffu, inc, 31);
+            }
+            __syncwarp();
+            ovf = nres > kURow || nnext > kUFront;
+            cur ^= 1;
+            ncur = nnext;
+        }
+        if (ovf) {
+            if (lane == 0) *overflow = 1;
+            continue;
+        }
+        // rank sort (leaf ids are distinct): ascending leaf order
+        int *row = rows + (size_t)t * kURow;
+        for (int j = lane; j < nres; j += 32) {
+            const int v = res[wi][j];
+            int rk = 0;
+            for (int k = 0; k < nres; ++k) rk += res[wi][k] < v;
+            row[rk] = v;
+        }
+        if (lane == 0) counts[t] = nres;
+        __syncwarp();
+    }
+}
+
+__global__ void ulist_copy_kernel(int L, const int *__restrict__ rows, const long long *__restrict__ u_off,
+                                  int *__restrict__ u_idx) {
+    const int t = blockIdx.x;                      // one block per leaf
+    if (t >= L) return;
+    const long long o = u_off[t];
+    const int n = (int)(u_off[t + 1] - o);
+    for (int j = threadIdx.x; j < n; j += blockDim.x) u_idx[o + j] = rows[(size_t)t * kURow + j];
 }
 
 __global__ void leaf_node_kernel(int nn, const int *__restrict__ node_leaf, int *__restrict__ leaf_node) {
@@ -467,7 +571,7 @@ afmm_status wsalloc(afmm_tree *t, int slot, T **p, size_t count) {
 enum Slot {
     kPart, kKeys, kIdx, kKeysSorted, kPerm, kSortTmp, kNodeA, kNodeB = kNodeA + 6, kCb = kNodeB + 6, kNc, kOff,
     kScanTmp, kFlag, kLeafAt, kNodeLeaf, kScan2, kLs, kLc, kLl, kLp, kLeafNode, kCounts, kUoff, kScan3, kUidx,
-    kFarfield, kEditPrefix, kEditAction, kEditBase
+    kFarfield, kEditPrefix, kEditAction, kEditBase, kURows, kUOvf
 };
 
 __global__ void root_kernel(Nodes nd, int n) {
@@ -620,8 +724,8 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
                 scan_tmp_bytes = need;
             }
         }
-        split_count_kernel<<<grid_for(m, TH), TH, 0, st>>>((int)m, (int)base, nd, t->keys_sorted, S, mode, pv, ed,
-                                                            cb, nc);
+        split_count_kernel<<<grid_for(8 * m, TH), TH, 0, st>>>((int)m, (int)base, nd, t->keys_sorted, S, mode, pv,
+                                                                ed, cb, nc);
         TCU(t, cudaGetLastError());
         TCU(t, cudaMemsetAsync(nc + m, 0, sizeof(int), st));
         size_t sb = scan_tmp_bytes;
@@ -704,13 +808,28 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     leaf_node_kernel<<<grid_for(nn, TH), TH, 0, st>>>((int)nn, node_leaf, leaf_node);
     TCU(t, cudaGetLastError());
 
-    // 6. U-lists: count, scan, fill
+    // 6. U-lists: warp-cooperative descent into fixed-capacity rows, scan, compact
+    //    (rows longer than kURow or frontiers wider than kUFront: per-thread DFS count + fill)
     long long *counts;
+    int *rows, *ovf;
     if (afmm_status s = wsalloc(t, kCounts, &counts, (size_t)L + 1)) return s;
     if (afmm_status s = wsalloc(t, kUoff, &t->u_off, (size_t)L + 1)) return s;
+    if (afmm_status s = wsalloc(t, kURows, &rows, (size_t)L * kURow)) return s;
+    if (afmm_status s = wsalloc(t, kUOvf, &ovf, 1)) return s;
     TCU(t, cudaMemsetAsync(counts + L, 0, sizeof(long long), st));
-    ulist_kernel<<<grid_for(L, 128), 128, 0, st>>>(L, nd, node_leaf, leaf_node, nullptr, nullptr, counts);
-    TCU(t, cudaGetLastError());
+    TCU(t, cudaMemsetAsync(ovf, 0, sizeof(int), st));
+    {
+        const int blocks = (int)std::min<long long>((L + kUWarps - 1) / kUWarps, 148LL * 16);
+        ulist_warp_kernel<<<blocks, 32 * kUWarps, 0, st>>>(L, nd, node_leaf, leaf_node, rows, counts, ovf);
+        TCU(t, cudaGetLastError());
+    }
+    int hovf = 0;
+    TCU(t, cudaMemcpyAsync(&hovf, ovf, sizeof(int), cudaMemcpyDeviceToHost, st));
+    TCU(t, cudaStreamSynchronize(st));
+    if (hovf) {
+        ulist_kernel<<<grid_for(L, 128), 128, 0, st>>>(L, nd, node_leaf, leaf_node, nullptr, nullptr, counts);
+        TCU(t, cudaGetLastError());
+    }
     {
         size_t sb = 0;
         TCU(t, cub::DeviceScan::ExclusiveSum(nullptr, sb, counts, t->u_off, L + 1, st));
@@ -721,7 +840,10 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     TCU(t, cudaMemcpyAsync(&t->nnz, t->u_off + L, sizeof(long long), cudaMemcpyDeviceToHost, st));
     TCU(t, cudaStreamSynchronize(st));
     if (afmm_status s = wsalloc(t, kUidx, &t->u_idx, (size_t)t->nnz)) return s;
-    ulist_kernel<<<grid_for(L, 128), 128, 0, st>>>(L, nd, node_leaf, leaf_node, t->u_off, t->u_idx, nullptr);
+    if (hovf)
+        ulist_kernel<<<grid_for(L, 128), 128, 0, st>>>(L, nd, node_leaf, leaf_node, t->u_off, t->u_idx, nullptr);
+    else
+        ulist_copy_kernel<<<L, 64, 0, st>>>(L, rows, t->u_off, t->u_idx);
     TCU(t, cudaGetLastError());
     TCU(t, cudaStreamSynchronize(st));
     t->n = n;

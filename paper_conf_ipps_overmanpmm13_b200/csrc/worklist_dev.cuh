@@ -110,12 +110,6 @@ __global__ void weighted_cut_kernel(int L, int G, const double *__restrict__ P, 
     for (int r = g + 1; r <= G; ++r) split[r] = L;
 }
 
-__device__ __forceinline__ int slices_for(int tn, long long nsrc, long long cap) {
-    unsigned short sz[kMaxDpSlices];
-    int n_full = 0, full_m = 0;
-    const int k = plan_slices(tn, nsrc, cap, &n_full, &full_m, sz);
-    return n_full + k;
-}
 
 // pass 1 over this rank's leaves [lo, lo+m): segment and slice counts, nsrc,
 // bucket statistics (int64 atomics: order-independent)
@@ -123,7 +117,7 @@ __global__ void count_kernel(int m, int lo, const int *__restrict__ ls, const in
                              const long long *__restrict__ uo, const int *__restrict__ ui,
                              const long long *__restrict__ I, int *__restrict__ nseg, int *__restrict__ ntask,
                              long long *__restrict__ nsrc, unsigned long long *__restrict__ stats,
-                             long long cap) {
+                             long long cap, unsigned short *__restrict__ plan, int4 *__restrict__ plan_hdr) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= m) return;
     const int t = lo + i;
@@ -143,7 +137,11 @@ __global__ void count_kernel(int m, int lo, const int *__restrict__ ls, const in
     }
     nseg[i] = segs + (self ? 1 : 0);
     nsrc[i] = src;
-    ntask[i] = slices_for(lc[t], src, cap);
+    // the leaf's slice plan, kept for write_kernel (the DP runs once per leaf)
+    int n_full = 0, full_m = 0;
+    const int k = plan_slices(lc[t], src, cap, &n_full, &full_m, plan + (size_t)i * kMaxDpSlices);
+    plan_hdr[i] = make_int4(n_full, full_m, k, 0);
+    ntask[i] = n_full + k;
     atomicAdd(&stats[0], (unsigned long long)I[t]);
     atomicAdd(&stats[1 + bucket_of_d(lc[t])], (unsigned long long)I[t]);
 }
@@ -154,7 +152,8 @@ __global__ void write_kernel(int m, int lo, const int *__restrict__ ls, const in
                              const int *__restrict__ seg_off, const int *__restrict__ task_off,
                              const int *__restrict__ ntask, const long long *__restrict__ nsrc,
                              Seg *__restrict__ segs, Task *__restrict__ tasks,
-                             unsigned long long *__restrict__ keys, int *__restrict__ vals, long long cap) {
+                             unsigned long long *__restrict__ keys, int *__restrict__ vals,
+                             const unsigned short *__restrict__ plan, const int4 *__restrict__ plan_hdr) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= m) return;
     const int t = lo + i;
@@ -173,9 +172,9 @@ __global__ void write_kernel(int m, int lo, const int *__restrict__ ls, const in
         else segs[w++] = Seg{ls[s], lc[s]};
     }
     const long long src = nsrc[i];
-    unsigned short sz[kMaxDpSlices];
-    int n_full = 0, full_m = 0;
-    const int k_dp = plan_slices(tn, src, cap, &n_full, &full_m, sz);   // same plan as count_kernel
+    const unsigned short *sz = plan + (size_t)i * kMaxDpSlices;           // count_kernel's plan
+    const int4 hd = plan_hdr[i];
+    const int n_full = hd.x, full_m = hd.y, k_dp = hd.z;
     for (int j = 0, a = 0; j < n_full + k_dp; a += plan_size(j, n_full, full_m, sz), ++j) {
         const int q = task_off[i] + j;
         const int cnt = plan_size(j, n_full, full_m, sz);
