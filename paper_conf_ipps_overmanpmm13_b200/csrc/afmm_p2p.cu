@@ -884,6 +884,8 @@ static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, flo
     p.eps2 = h->cfg.eps2;
     p.G = h->cfg.law == AFMM_LAW_STOKESLET ? 1.0 / (8.0 * 3.14159265358979323846 * (double)h->cfg.mu)
                                            : (double)h->cfg.G;
+    p.Gf = (float)p.G;
+    p.g_exact = (double)p.Gf == p.G;
     p.done = nullptr;
     CUDA_TRY(h, cudaMemsetAsync(h->d_queue, 0, sizeof(int), h->stream));
     const int ri = (int)(h->n_evals % afmm_p2p::kRing);
@@ -1133,6 +1135,8 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
         prm.n_win = 1;
         prm.eps2 = h->cfg.eps2;
         prm.G = (double)h->cfg.G;
+        prm.Gf = h->cfg.G;
+        prm.g_exact = 1;
         prm.done = done;
         const int grid = std::max(1, std::min((nt + afmm::kWarps - 1) / afmm::kWarps, h->num_sms * h->blocks_per_sm));
         afmm::p2p_kernel_t<afmm::Gravity><<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(prm);

@@ -221,6 +221,8 @@ struct P2PParams {
     int n_win;
     float eps2;
     double G;                // output scale: G (gravity) or 1/(8 pi mu) (Stokeslet)
+    float Gf;                // (float)G, used when g_exact (G is an fp32 value)
+    int g_exact;
     int *done;               // nullptr, or per-piece counters of finished tasks (afmm_p2p_eval_host_pipelined)
 };
 
@@ -314,6 +316,9 @@ struct Gravity {
     __device__ __forceinline__ static float out(int comp, double v, double scale) {
         return (float)(comp == 3 ? -scale * v : scale * v);
     }
+    __device__ __forceinline__ static float outf(int comp, float v, float scale) {
+        return comp == 3 ? -__fmul_rn(scale, v) : __fmul_rn(scale, v);
+    }
 };
 
 // Regularized Stokeslet (reading R26; PAPER L22 SVIII.B "method of regularized
@@ -352,6 +357,9 @@ struct Stokeslet {
     // u = v / (8 pi mu); the fourth output is zero
     __device__ __forceinline__ static float out(int comp, double v, double scale) {
         return comp == 3 ? 0.0f : (float)(scale * v);
+    }
+    __device__ __forceinline__ static float outf(int comp, float v, float scale) {
+        return comp == 3 ? 0.0f : __fmul_rn(scale, v);
     }
 };
 
@@ -700,8 +708,9 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
             // (lanes c*g + l2, c < C): round o adds copy c+o into copy c for c = 0 mod 2o
             // (R17).  If no lane folded (every copy's sources fit one fp32 partial) the
             // tree runs on the fp32 partials, else in fp64 on accumulators + partials.
-            double v[kVals];
+            float o[kVals];                   // outputs (one RN rounding, R18)
             if (__any_sync(0xffffffffu, P.folded)) {
+                double v[kVals];
 #pragma unroll
                 for (int q = 0; q < kPairs; ++q) {
                     const double *a = P.acc + 8 * q * 32;
@@ -715,14 +724,16 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
                     v[8 * q + 6] = (f ? a[6 * 32] : 0.0) + (double)P.az[q].y;
                     v[8 * q + 7] = (f ? a[7 * 32] : 0.0) + (double)P.ph[q].y;
                 }
-                for (int o = 1; o < C; o <<= 1) {
-                    const bool take = (c & (2 * o - 1)) == 0 && c + o < C;
+                for (int ro = 1; ro < C; ro <<= 1) {
+                    const bool take = (c & (2 * ro - 1)) == 0 && c + ro < C;
 #pragma unroll
                     for (int u = 0; u < kVals; ++u) {
-                        const double w = __shfl_down_sync(0xffffffffu, v[u], o * g);
+                        const double w = __shfl_down_sync(0xffffffffu, v[u], ro * g);
                         if (take) v[u] += w;
                     }
                 }
+#pragma unroll
+                for (int u = 0; u < kVals; ++u) o[u] = Law::out(u & 3, v[u], p.G);
             } else {
                 float f[kVals];
 #pragma unroll
@@ -732,16 +743,20 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
                     f[8 * q + 4] = P.ax[q].y; f[8 * q + 5] = P.ay[q].y;
                     f[8 * q + 6] = P.az[q].y; f[8 * q + 7] = P.ph[q].y;
                 }
-                for (int o = 1; o < C; o <<= 1) {
-                    const bool take = (c & (2 * o - 1)) == 0 && c + o < C;
+                for (int ro = 1; ro < C; ro <<= 1) {
+                    const bool take = (c & (2 * ro - 1)) == 0 && c + ro < C;
 #pragma unroll
                     for (int u = 0; u < kVals; ++u) {
-                        const float w = __shfl_down_sync(0xffffffffu, f[u], o * g);
+                        const float w = __shfl_down_sync(0xffffffffu, f[u], ro * g);
                         if (take) f[u] = __fadd_rn(f[u], w);
                     }
                 }
+                // fp32 G: G*f rounded once in fp32 equals the fp64 product rounded
+                // once (the product of two fp32 values is exact in fp64), so this
+                // path skips the conversions with bit-identical outputs
 #pragma unroll
-                for (int u = 0; u < kVals; ++u) v[u] = (double)f[u];
+                for (int u = 0; u < kVals; ++u)
+                    o[u] = p.g_exact ? Law::outf(u & 3, f[u], p.Gf) : Law::out(u & 3, (double)f[u], p.G);
             }
             if (active && c == 0) {
 #pragma unroll
@@ -749,8 +764,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
                     const int tgt = kTPT * l + j;
                     if (tgt < m.tgt_count) {
                         const int u = 8 * (j >> 1) + 4 * (j & 1), i = m.tgt_start + tgt;
-                        const float o0 = Law::out(0, v[u + 0], p.G), o1 = Law::out(1, v[u + 1], p.G);
-                        const float o2 = Law::out(2, v[u + 2], p.G), o3 = Law::out(3, v[u + 3], p.G);
+                        const float o0 = o[u + 0], o1 = o[u + 1], o2 = o[u + 2], o3 = o[u + 3];
                         p.out[0][0][i] = o0;                    // own outputs
                         p.out[0][1][i] = o1;
                         p.out[0][2][i] = o2;
