@@ -38,7 +38,7 @@ sys.path.insert(0, ROOT)
 
 import synth  # noqa: E402  (seeded input generator shared by both arms)
 
-E2E_PIECES = 4             # pieces of the pipelined host-to-host evaluation (e2e)
+E2E_PIECES = 2             # output pieces of the pipelined host-to-host evaluation (e2e; tools/e2e_probe.py)
 FLOPS_PER_INTERACTION = 20
 METRIC = "near-field P2P interactions/s (and % FP32 peak) at 1/2/4/8 B200"
 SWEEP_S = [32, 48, 64, 96, 128, 192, 256, 384, 512]
@@ -472,7 +472,7 @@ def main():
             "clocks": clk.summary(),
             "e2e": {"value": e2e_value, "unit": "interactions/s", "h2d_bytes_per_step": 16 * n,
                     "d2h_bytes_per_step": 16 * n, "steps": Ke,
-                    "path": f"afmm_p2p_eval_host_pipelined ({E2E_PIECES} pieces) from pinned host arrays" if world == 1
+                    "path": f"afmm_p2p_eval_host_pipelined (8 streamed input chunks, {E2E_PIECES} output pieces) from pinned host arrays" if world == 1
                     else "rank 0 H2D + step + D2H"},
             "gpu_launches": 2 * K,
             "rebalanced_in_warmup": rebalanced,

@@ -86,11 +86,13 @@ struct afmm_p2p {
     int pipe_P = 0;
     std::vector<int> pipe_off;                       // P + 1 offsets into d_ptasks
     std::vector<long long> pipe_need, pipe_lo, pipe_hi;   // bodies needed (prefix), output range per piece
+    int pipe_K = 0;                                   // input chunks (streamed H2D)
     afmm::Task *d_ptasks = nullptr;
     size_t ptasks_cap = 0;
     int *d_pqueue = nullptr;                         // kMaxPieces counters
     cudaStream_t s_in = nullptr, s_out = nullptr;
     void *wait_value32 = nullptr;                    // cuStreamWaitValue32 (driver entry point)
+    void *write_value32 = nullptr;                   // cuStreamWriteValue32 (driver entry point)
     cudaEvent_t ev_start = nullptr, ev_in[64] = {}, ev_k[64] = {}, ev_done = nullptr;
 
     // peer output windows (fused gather, afmm_p2p_set_peer_windows)
@@ -887,6 +889,8 @@ static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, flo
     p.Gf = (float)p.G;
     p.g_exact = (double)p.Gf == p.G;
     p.done = nullptr;
+    p.in_ready = nullptr;
+    p.in_err = nullptr;
     CUDA_TRY(h, cudaMemsetAsync(h->d_queue, 0, sizeof(int), h->stream));
     const int ri = (int)(h->n_evals % afmm_p2p::kRing);
     h->ev0 = h->ring0[ri];
@@ -972,6 +976,7 @@ extern "C" afmm_status afmm_p2p_eval_host(afmm_p2p *h, float *ax, float *ay, flo
 // ------------------------------------------------------------------ pipelined host evaluation
 
 static constexpr int kMaxPieces = 64;
+static constexpr int kInChunks = 8;                 // input chunks of the streamed H2D
 
 // Regroup this rank's tasks into P pieces of consecutive targets (equal modelled
 // cost tgt_count * nsrc, cut in tgt_start order); inside a piece the tasks keep
@@ -1021,13 +1026,34 @@ static afmm_status build_pipe(afmm_p2p *h, int P) {
         if (q > 0) h->pipe_need[q] = std::max(h->pipe_need[q], h->pipe_need[q - 1]);
         if (h->pipe_lo[q] > h->pipe_hi[q]) h->pipe_lo[q] = h->pipe_hi[q] = 0;   // empty piece
     }
-    std::vector<afmm::Task> grouped(std::max(nt, 1));
-    std::vector<int> fill(h->pipe_off.begin(), h->pipe_off.end() - 1);
-    for (int i = 0; i < nt; ++i) {                                              // stable: LPT kept
-        afmm::Task x = t[i];
-        x.piece = piece[i];
-        grouped[fill[piece[i]]++] = x;
+    // Input chunks: the bodies in K equal Morton ranges, copied and packed in order while
+    // the kernel runs.  Task order: by the last input chunk the task needs (its sources
+    // and targets), then by output piece, LPT kept inside -- so the kernel starts on the
+    // first chunk and stays behind the copies, and every output piece's stragglers (leaves
+    // whose U-lists reach far in Morton order) run as soon as the last chunk lands.
+    const int K = (int)std::min<long long>(kInChunks, std::max<long long>(1, h->n / 4096));
+    const long long chunk = (h->n + K - 1) / K;
+    std::vector<int> need_chunk(nt, 0);
+    for (int i = 0; i < nt; ++i) {
+        long long need = (long long)t[i].tgt_start + t[i].tgt_count;
+        for (int j = 0; j < t[i].seg_count; ++j) {
+            const afmm::Seg &z = sg[t[i].seg_begin + j];
+            need = std::max(need, (long long)z.gstart + z.len);
+        }
+        need_chunk[i] = (int)std::min<long long>(K - 1, (need - 1) / chunk);
     }
+    std::vector<int> ord2(nt);
+    for (int i = 0; i < nt; ++i) ord2[i] = i;
+    std::stable_sort(ord2.begin(), ord2.end(), [&](int a, int b) {
+        return need_chunk[a] != need_chunk[b] ? need_chunk[a] < need_chunk[b] : piece[a] < piece[b];
+    });
+    std::vector<afmm::Task> grouped(std::max(nt, 1));
+    for (int r = 0; r < nt; ++r) {                                              // stable: LPT kept
+        afmm::Task x = t[ord2[r]];
+        x.piece = piece[ord2[r]] | (need_chunk[ord2[r]] << 16);
+        grouped[r] = x;
+    }
+    h->pipe_K = K;
     afmm_status st = ensure_device(h, &h->d_ptasks, h->ptasks_cap, grouped.size());
     if (st) return st;
     CUDA_TRY(h, cudaMemcpy(h->d_ptasks, grouped.data(), grouped.size() * sizeof(afmm::Task), cudaMemcpyHostToDevice));
@@ -1058,11 +1084,14 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
             CUDA_TRY(h, cudaEventCreateWithFlags(&h->ev_in[i], cudaEventDisableTiming));
             CUDA_TRY(h, cudaEventCreateWithFlags(&h->ev_k[i], cudaEventDisableTiming));
         }
-        CUDA_TRY(h, cudaMalloc(&h->d_pqueue, (kMaxPieces + 1) * sizeof(int)));
+        CUDA_TRY(h, cudaMalloc(&h->d_pqueue, (kMaxPieces + 3) * sizeof(int)));
         cudaDriverEntryPointQueryResult q;
         CUDA_TRY(h, cudaGetDriverEntryPoint("cuStreamWaitValue32", &h->wait_value32, cudaEnableDefault, &q));
         if (q != cudaDriverEntryPointSuccess || !h->wait_value32)
             return fail(h, AFMM_ENOTSUP, "eval_host_pipelined: cuStreamWaitValue32 unavailable");
+        CUDA_TRY(h, cudaGetDriverEntryPoint("cuStreamWriteValue32", &h->write_value32, cudaEnableDefault, &q));
+        if (q != cudaDriverEntryPointSuccess || !h->write_value32)
+            return fail(h, AFMM_ENOTSUP, "eval_host_pipelined: cuStreamWriteValue32 unavailable");
     }
     if (4 * n > h->soa_cap) {
         cudaFree(h->d_soa);
@@ -1092,28 +1121,42 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
     // first (sources of a piece may lie anywhere in the tree order).
     using WaitFn = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
     const WaitFn wait32 = reinterpret_cast<WaitFn>(h->wait_value32);
+    using WriteFn = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+    const WriteFn write32 = reinterpret_cast<WriteFn>(h->write_value32);
     int *queue = h->d_pqueue, *done = h->d_pqueue + 1;
-    CUDA_TRY(h, cudaMemsetAsync(h->d_pqueue, 0, (P + 1) * sizeof(int), h->stream));
+    unsigned *in_ready = reinterpret_cast<unsigned *>(h->d_pqueue + kMaxPieces + 1);
+    int *in_err = h->d_pqueue + kMaxPieces + 2;
+    CUDA_TRY(h, cudaMemsetAsync(h->d_pqueue, 0, (kMaxPieces + 3) * sizeof(int), h->stream));
     CUDA_TRY(h, cudaEventRecord(h->ev_start, h->stream));      // earlier readers of the bodies / outputs
     CUDA_TRY(h, cudaStreamWaitEvent(h->s_in, h->ev_start, 0));
     CUDA_TRY(h, cudaStreamWaitEvent(h->s_out, h->ev_start, 0));
-    const size_t b = (size_t)n * sizeof(float);
-    const long long half = n / 2;
-    for (int part = 0; part < 2; ++part) {                     // two halves: pack of the first overlaps the second copy
-        const long long lo = part ? half : 0, hi = part ? n : half;
-        if (hi <= lo) continue;
-        for (int a = 0; a < 4; ++a)
-            CUDA_TRY(h, cudaMemcpyAsync(dsoa[a] + lo, hin[a] + lo, (size_t)(hi - lo) * sizeof(float),
-                                        cudaMemcpyHostToDevice, h->s_in));
-        const int threads = 256;
-        const int blocks = (int)std::min<long long>((hi - lo + threads - 1) / threads, (long long)h->num_sms * 16);
-        afmm::pack_bodies_kernel<<<blocks, threads, 0, h->s_in>>>(hi - lo, dsoa[0] + lo, dsoa[1] + lo, dsoa[2] + lo,
-                                                                 dsoa[3] + lo, h->d_bodies + lo);
-        CUDA_TRY(h, cudaGetLastError());
+    // inputs streamed in K Morton chunks: copy (4 SoA slices), pack, then publish the
+    // chunk count in device memory (cuStreamWriteValue32 orders the packed bodies
+    // before the flag); the kernel's warps wait per task for the chunk it needs.
+    // The pack kernels run next to the persistent P2P kernel (128 threads, few
+    // registers: they fit in what one P2P CTA leaves free on an SM).  Chunk 0 is in
+    // place before the launch.
+    const int K = h->pipe_K;
+    const long long chunk = (n + K - 1) / K;
+    for (int k = 0; k < K; ++k) {
+        const long long lo = k * chunk, hi = std::min<long long>(n, lo + chunk);
+        if (hi > lo) {
+            for (int a = 0; a < 4; ++a)
+                CUDA_TRY(h, cudaMemcpyAsync(dsoa[a] + lo, hin[a] + lo, (size_t)(hi - lo) * sizeof(float),
+                                            cudaMemcpyHostToDevice, h->s_in));
+            const int threads = 128;
+            const int blocks = (int)std::min<long long>((hi - lo + threads - 1) / threads, (long long)h->num_sms);
+            afmm::pack_chunk_kernel<<<blocks, threads, 0, h->s_in>>>((int)(hi - lo), dsoa[0] + lo, dsoa[1] + lo,
+                                                                    dsoa[2] + lo, dsoa[3] + lo, h->d_bodies + lo);
+            CUDA_TRY(h, cudaGetLastError());
+        }
+        const CUresult r = write32((CUstream)h->s_in, (CUdeviceptr)in_ready, (cuuint32_t)(k + 1), 0);
+        if (r != CUDA_SUCCESS) return fail(h, AFMM_ECUDA, "eval_host_pipelined: cuStreamWriteValue32 failed (%d)", (int)r);
+        if (k == 0) {
+            CUDA_TRY(h, cudaEventRecord(h->ev_in[0], h->s_in));
+            CUDA_TRY(h, cudaStreamWaitEvent(h->stream, h->ev_in[0], 0));
+        }
     }
-    (void)b;
-    CUDA_TRY(h, cudaEventRecord(h->ev_in[0], h->s_in));
-    CUDA_TRY(h, cudaStreamWaitEvent(h->stream, h->ev_in[0], 0));
     const int ri = (int)(h->n_evals % afmm_p2p::kRing);
     h->ev0 = h->ring0[ri];
     h->ev1 = h->ring1[ri];
@@ -1138,6 +1181,8 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
         prm.Gf = h->cfg.G;
         prm.g_exact = 1;
         prm.done = done;
+        prm.in_ready = in_ready;
+        prm.in_err = in_err;
         const int grid = std::max(1, std::min((nt + afmm::kWarps - 1) / afmm::kWarps, h->num_sms * h->blocks_per_sm));
         afmm::p2p_kernel_t<afmm::Gravity><<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(prm);
         CUDA_TRY(h, cudaGetLastError());
@@ -1162,7 +1207,11 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
     h->n_evals++;
     h->evaluated = true;
     h->last.n_launches = nlaunch;
-    return fill_stats(h, stats);
+    if ((st = fill_stats(h, stats))) return st;
+    int herr = 0;
+    CUDA_TRY(h, cudaMemcpy(&herr, in_err, sizeof(int), cudaMemcpyDeviceToHost));
+    if (herr) return fail(h, AFMM_ECUDA, "eval_host_pipelined: input chunks never arrived (kernel wait timed out)");
+    return AFMM_OK;
 }
 
 extern "C" afmm_status afmm_p2p_set_peer_windows(afmm_p2p *h, int count, float *const *ptrs) {

@@ -200,7 +200,8 @@ __host__ __device__ inline long long task_cap(long long inter, long long warps) 
 // [seg_begin, +seg_count) totalling nsrc bodies.
 struct Task {
     int tgt_start, tgt_count, self_start, self_len, seg_begin, seg_count, nsrc;
-    int piece;               // completion counter index (pipelined host evaluation), else 0
+    int piece;               // pipelined host evaluation: output piece (low 16 bits) and the last input
+                             // chunk its sources and targets need (high 16 bits); else 0
 };
 // Segment: bodies [gstart, gstart+len).
 struct Seg {
@@ -224,6 +225,12 @@ struct P2PParams {
     float Gf;                // (float)G, used when g_exact (G is an fp32 value)
     int g_exact;
     int *done;               // nullptr, or per-piece counters of finished tasks (afmm_p2p_eval_host_pipelined)
+    // streamed inputs (afmm_p2p_eval_host_pipelined): nullptr, or the number of input
+    // chunks already packed (written by the copy stream); a task whose sources reach
+    // chunk r = piece >> 16 waits until *in_ready > r.  *in_err is set if the wait
+    // times out (the copy stream never delivered: results invalid, reported as an error)
+    const unsigned *in_ready;
+    int *in_err;
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
@@ -521,6 +528,25 @@ __device__ __forceinline__ void copy_piece(const P2PParams &p, float4 *buf, uint
                     (uint32_t)(b - a) * 16u * kWords, bar);
 }
 
+// Streamed inputs: before a task's first chunk is staged, wait until the input
+// chunk its sources (and targets) reach has been packed.  Every lane acquires the
+// flag; the proxy fence orders the packed bodies before this warp's bulk copies.
+// A wait longer than ~0.5 s sets *in_err and gives up (no hang).
+__device__ __forceinline__ void wait_inputs(const P2PParams &p, int piece) {
+    const unsigned need = (unsigned)piece >> 16;
+    unsigned v;
+    for (int spin = 0;; ++spin) {
+        asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p.in_ready) : "memory");
+        if (v > need) break;
+        if (spin > (1 << 21)) {
+            if ((threadIdx.x & 31) == 0) atomicExch(p.in_err, 1);
+            break;
+        }
+        __nanosleep(256);
+    }
+    asm volatile("fence.proxy.async.global;" ::: "memory");
+}
+
 // Stage the next chunk (<= kWCap bodies) of the stream into `buf`; returns
 // false when no task is left.  Lane 0 posts the byte count, then every lane
 // whose segment overlaps the chunk issues that piece (no warp-serial walk).
@@ -533,6 +559,7 @@ __device__ __forceinline__ bool issue_chunk(const P2PParams &p, Stream &S, float
         S.pre_ok = true;
     }
     const int nb = min(kWCap / kWords, S.t.nsrc - S.staged);
+    if (p.in_ready && S.staged == 0) wait_inputs(p, S.t.piece);
     PROF_T(t_a);
     if (lane == 0) {
         ChunkMeta m;
@@ -784,7 +811,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
             if (p.done) {                 // publish the task's outputs (pipelined copy-back waits on it)
                 __threadfence();
                 __syncwarp();
-                if (lane == 0) atomicAdd(p.done + m.piece, 1);
+                if (lane == 0) atomicAdd(p.done + (m.piece & 0xffff), 1);
             }
         }
         PROF_ADD(4, t_l);
@@ -815,6 +842,16 @@ __global__ void pack_stokeslet_kernel(long long n, const float *__restrict__ x, 
         out[2 * i] = make_float4(x[i], y[i], z[i], fx[i]);
         out[2 * i + 1] = make_float4(fy[i], fz[i], 0.f, 0.f);
     }
+}
+
+// Streamed-input pack (afmm_p2p_eval_host_pipelined): runs NEXT TO the persistent
+// P2P kernel, so it must fit in what a P2P CTA leaves free on an SM (4096
+// registers): 128 threads, <= 24 registers, 32-bit indices.
+__global__ void __launch_bounds__(128, 21) pack_chunk_kernel(int n, const float *__restrict__ x,
+                                                             const float *__restrict__ y, const float *__restrict__ z,
+                                                             const float *__restrict__ m, float4 *__restrict__ out) {
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
+        out[i] = make_float4(x[i], y[i], z[i], m[i]);
 }
 
 __global__ void pack_bodies_kernel(long long n, const float *__restrict__ x, const float *__restrict__ y,
