@@ -153,17 +153,19 @@ enum { kModeFresh = 0, kModeEnforce = 1, kModeKeep = 2 };
 // Child ranges by binary search on the octant digit inside [b, e): eight lanes
 // per node, lane o finds the first position with digit >= o (independent
 // searches, so a level costs one search's latency, not seven in a row).
-__global__ void split_count_kernel(int m, int base, Nodes nd, const unsigned long long *__restrict__ keys,
-                                   int S, int mode, PrevTree pv, Edits ed, int *__restrict__ cb,
-                                   int *__restrict__ nc) {
-    const long long gt = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+// one lane of the 8 of node i = gt >> 3 (lane o = gt & 7); all 32 lanes of the
+// warp call it together (shuffles / ballot), with gt >= 8m for padding lanes
+__device__ __forceinline__ void split_count_lane(long long gt, int m, long long base, const Nodes &nd,
+                                                 const unsigned long long *__restrict__ keys, int S, int mode,
+                                                 const PrevTree &pv, const Edits &ed, int *__restrict__ cb,
+                                                 int *__restrict__ nc) {
     const int o = (int)(gt & 7);
     const int i = (int)(gt >> 3);
     const bool live = i < m;
     int b = 0, e = 0, lev = 0;
     bool split = false;
     if (live) {
-        const int id = base + i;
+        const long long id = base + i;
         b = nd.b[id];
         e = nd.e[id];
         lev = nd.level[id];
@@ -196,26 +198,29 @@ __global__ void split_count_kernel(int m, int base, Nodes nd, const unsigned lon
     const unsigned nonempty = __ballot_sync(0xffffffffu, split && nxt > bound);
     if (!live) return;
     if (split) {
-        cb[i * 9 + o] = bound;
-        if (o == 7) cb[i * 9 + 8] = e;
+        cb[(size_t)i * 9 + o] = bound;
+        if (o == 7) cb[(size_t)i * 9 + 8] = e;
     }
     if (o == 0) nc[i] = __popc((nonempty >> (threadIdx.x & 24)) & 0xffu);
 }
 
-__global__ void split_write_kernel(int m, int base, int next_base, Nodes nd, const int *__restrict__ cb,
-                                   const int *__restrict__ nc, const int *__restrict__ off) {
-    const int i = blockIdx.x * blockDim.x + threadIdx.x;
-    if (i >= m) return;
-    const int id = base + i;
-    const int cnt = nc[i];
+__global__ void split_count_kernel(int m, int base, Nodes nd, const unsigned long long *__restrict__ keys,
+                                   int S, int mode, PrevTree pv, Edits ed, int *__restrict__ cb,
+                                   int *__restrict__ nc) {
+    split_count_lane((long long)blockIdx.x * blockDim.x + threadIdx.x, m, base, nd, keys, S, mode, pv, ed, cb, nc);
+}
+
+__device__ __forceinline__ void split_write_node(int i, long long base, long long next_base, const Nodes &nd,
+                                                 const int *__restrict__ cb, int cnt, int off) {
+    const long long id = base + i;
     nd.nchild[id] = cnt;
-    nd.first_child[id] = cnt ? next_base + off[i] : -1;
+    nd.first_child[id] = cnt ? (int)(next_base + off) : -1;
     if (!cnt) return;
-    int w = next_base + off[i];
+    long long w = next_base + off;
     const unsigned long long pre = nd.prefix[id];
     const int lev = nd.level[id];
     for (int o = 0; o < 8; ++o) {
-        const int b = cb[i * 9 + o], e = cb[i * 9 + o + 1];
+        const int b = cb[(size_t)i * 9 + o], e = cb[(size_t)i * 9 + o + 1];
         if (e > b) {
             nd.b[w] = b;
             nd.e[w] = e;
@@ -225,6 +230,133 @@ __global__ void split_write_kernel(int m, int base, int next_base, Nodes nd, con
             nd.nchild[w] = 0;
             ++w;
         }
+    }
+}
+
+__global__ void split_write_kernel(int m, int base, int next_base, Nodes nd, const int *__restrict__ cb,
+                                   const int *__restrict__ nc, const int *__restrict__ off) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= m) return;
+    split_write_node(i, base, next_base, nd, cb, nc[i], off[i]);
+}
+
+// The whole level loop in ONE cooperative launch (no host round trip per level):
+// per level, (1) split counts (8 lanes per node, grid-stride), grid barrier,
+// (2) every block scans its tile of the child counts and publishes the tile sum,
+// grid barrier, (3) every block adds the sums of the tiles before its own (so no
+// third barrier is needed for the scan), writes its nodes' children, grid barrier.
+// Level starts go to ctl->base[]; a level that would exceed the node capacity
+// sets ctl->overflow and every block stops (the host grows the arrays and reruns).
+struct LevelCtl {
+    long long base[kMaxLevel + 3];  // level starts, base[levels] = total nodes
+    int levels;
+    int overflow;
+    unsigned bar_count, bar_gen;
+};
+
+__device__ __forceinline__ void grid_barrier(LevelCtl *c) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        volatile unsigned *gen = &c->bar_gen;
+        const unsigned g = *gen;
+        __threadfence();
+        if (atomicAdd(&c->bar_count, 1u) == gridDim.x - 1) {
+            c->bar_count = 0;
+            __threadfence();
+            atomicAdd(&c->bar_gen, 1u);
+        } else {
+            while (*gen == g) __nanosleep(32);
+        }
+        __threadfence();
+    }
+    __syncthreads();
+}
+
+constexpr int kLvlThreads = 256;
+__global__ void __launch_bounds__(kLvlThreads) levels_kernel(Nodes nd, const unsigned long long *__restrict__ keys,
+                                                             int S, int mode, PrevTree pv, Edits ed,
+                                                             int *__restrict__ cb, int *__restrict__ nc,
+                                                             int *__restrict__ off, int *__restrict__ tsum,
+                                                             LevelCtl *ctl, long long cap) {
+    __shared__ int wsum[kLvlThreads / 32];
+    __shared__ int carry;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const long long stride = (long long)gridDim.x * kLvlThreads;
+    long long base = 0;
+    int m = 1;
+    int lev = 0;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        ctl->base[0] = 0;
+        ctl->overflow = 0;
+    }
+    while (m > 0) {
+        // (1) split counts
+        for (long long w0 = ((long long)blockIdx.x * kLvlThreads + threadIdx.x) & ~31LL; w0 < 8LL * m; w0 += stride)
+            split_count_lane(w0 + lane, m, base, nd, keys, S, mode, pv, ed, cb, nc);
+        grid_barrier(ctl);
+        // (2) tile scan: block b owns nodes [b*tile, min(m, (b+1)*tile))
+        const int tile = (int)((m + gridDim.x - 1) / gridDim.x);
+        const int t0 = (int)min((long long)blockIdx.x * tile, (long long)m), t1 = min(t0 + tile, m);
+        if (threadIdx.x == 0) carry = 0;
+        __syncthreads();
+        for (int c0 = t0; c0 < t1; c0 += kLvlThreads) {
+            const int i = c0 + threadIdx.x;
+            const int v = i < t1 ? nc[i] : 0;
+            int inc = v;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int u = __shfl_up_sync(0xffffffffu, inc, o);
+                if (lane >= o) inc += u;
+            }
+            if (lane == 31) wsum[wid] = inc;
+            __syncthreads();
+            int wpre = 0;
+            for (int k = 0; k < wid; ++k) wpre += wsum[k];
+            int ctot = 0;
+            for (int k = 0; k < kLvlThreads / 32; ++k) ctot += wsum[k];
+            if (i < t1) off[i] = carry + wpre + inc - v;
+            __syncthreads();
+            if (threadIdx.x == 0) carry += ctot;
+            __syncthreads();
+        }
+        if (threadIdx.x == 0) tsum[blockIdx.x] = carry;
+        grid_barrier(ctl);
+        // (3) tile prefix + total (every block reads all tile sums: no extra barrier)
+        int pre = 0, total = 0;
+        for (int k = threadIdx.x; k < (int)gridDim.x; k += kLvlThreads) {
+            const int v = tsum[k];
+            total += v;
+            if (k < (int)blockIdx.x) pre += v;
+        }
+        for (int o = 16; o > 0; o >>= 1) {
+            pre += __shfl_xor_sync(0xffffffffu, pre, o);
+            total += __shfl_xor_sync(0xffffffffu, total, o);
+        }
+        __syncthreads();
+        if (lane == 0) wsum[wid] = pre;
+        __syncthreads();
+        int bpre = 0;
+        for (int k = 0; k < kLvlThreads / 32; ++k) bpre += wsum[k];
+        __syncthreads();
+        if (lane == 0) wsum[wid] = total;
+        __syncthreads();
+        int btot = 0;
+        for (int k = 0; k < kLvlThreads / 32; ++k) btot += wsum[k];
+        const long long next_base = base + m;
+        if (next_base + btot > cap) {                 // every block sees the same totals
+            if (blockIdx.x == 0 && threadIdx.x == 0) ctl->overflow = 1;
+            return;
+        }
+        for (int i = t0 + threadIdx.x; i < t1; i += kLvlThreads) split_write_node(i, base, next_base, nd, cb, nc[i],
+                                                                                bpre + off[i]);
+        ++lev;
+        if (blockIdx.x == 0 && threadIdx.x == 0) {
+            ctl->base[lev] = next_base;
+            ctl->levels = lev;
+        }
+        base = next_base;
+        m = btot;
+        grid_barrier(ctl);
     }
 }
 
@@ -510,6 +642,7 @@ struct afmm_tree {
     std::vector<void *> ws_ptr;
     std::vector<size_t> ws_cap;
     size_t node_cap = 1024;
+    bool coop_ok = true;             // cooperative launch of levels_kernel available
 };
 
 namespace {
@@ -571,7 +704,7 @@ afmm_status wsalloc(afmm_tree *t, int slot, T **p, size_t count) {
 enum Slot {
     kPart, kKeys, kIdx, kKeysSorted, kPerm, kSortTmp, kNodeA, kNodeB = kNodeA + 6, kCb = kNodeB + 6, kNc, kOff,
     kScanTmp, kFlag, kLeafAt, kNodeLeaf, kScan2, kLs, kLc, kLl, kLp, kLeafNode, kCounts, kUoff, kScan3, kUidx,
-    kFarfield, kEditPrefix, kEditAction, kEditBase, kURows, kUOvf
+    kFarfield, kEditPrefix, kEditAction, kEditBase, kURows, kUOvf, kLvlCtl, kTsum
 };
 
 __global__ void root_kernel(Nodes nd, int n) {
@@ -701,13 +834,69 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
         return AFMM_OK;
     };
     if (afmm_status s = alloc_nodes(cap, nd, node_set)) return s;
-    root_kernel<<<1, 1, 0, st>>>(nd, (int)n);
-    TCU(t, cudaGetLastError());
+    if (!t->coop_ok) {
+        root_kernel<<<1, 1, 0, st>>>(nd, (int)n);
+        TCU(t, cudaGetLastError());
+    }
     PrevTree pv{t->pv_prefix, t->pv_nchild, t->pv_base, mode != kModeFresh ? t->pv_levels : 0};
     std::vector<long long> lvl_base;
     long long base = 0, m = 1;     // current level occupies [base, base+m)
     int level = 0;
     int *cb = nullptr, *nc = nullptr, *off = nullptr;
+    bool done_levels = false;
+    // 4a. all levels in one cooperative launch (grid barriers between phases); the
+    //     node arrays start at >= 2n + 64 nodes and are doubled on overflow
+    if (t->coop_ok) {
+        if (cap < (size_t)(2 * n + 64)) {
+            cap = (size_t)(2 * n + 64);
+            if (afmm_status s = alloc_nodes(cap, nd, node_set)) return s;
+        }
+        LevelCtl *ctl;
+        int *tsum;
+        if (afmm_status s = wsalloc(t, kCb, &cb, (size_t)(n + 1) * 9)) return s;
+        if (afmm_status s = wsalloc(t, kNc, &nc, (size_t)n + 1)) return s;
+        if (afmm_status s = wsalloc(t, kOff, &off, (size_t)n + 1)) return s;
+        if (afmm_status s = wsalloc(t, kLvlCtl, reinterpret_cast<char **>(&ctl), sizeof(LevelCtl))) return s;
+        int per_sm = 0, dev_sms = 0;
+        TCU(t, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, levels_kernel, kLvlThreads, 0));
+        TCU(t, cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, t->device));
+        const int blocks = std::max(1, std::min(per_sm, 2) * dev_sms);
+        if (afmm_status s = wsalloc(t, kTsum, &tsum, (size_t)blocks)) return s;
+        for (int attempt = 0; attempt < 8 && !done_levels; ++attempt) {
+            root_kernel<<<1, 1, 0, st>>>(nd, (int)n);
+            TCU(t, cudaGetLastError());
+            TCU(t, cudaMemsetAsync(ctl, 0, sizeof(LevelCtl), st));
+            long long capll = (long long)cap;
+            void *args[] = {&nd, &t->keys_sorted, &S, &mode, &pv, &ed, &cb, &nc, &off, &tsum, &ctl, &capll};
+            const cudaError_t e = cudaLaunchCooperativeKernel((const void *)levels_kernel, blocks, kLvlThreads, args,
+                                                              0, st);
+            if (e != cudaSuccess) {                   // no cooperative launch here: the per-level host loop
+                cudaGetLastError();
+                t->coop_ok = false;
+                break;
+            }
+            LevelCtl hc;
+            TCU(t, cudaMemcpyAsync(&hc, ctl, sizeof(LevelCtl), cudaMemcpyDeviceToHost, st));
+            TCU(t, cudaStreamSynchronize(st));
+            if (hc.overflow) {                        // grow and rebuild the levels
+                cap *= 2;
+                node_set = node_set == kNodeA ? kNodeB : kNodeA;
+                if (afmm_status s = alloc_nodes(cap, nd, node_set)) return s;
+                continue;
+            }
+            lvl_base.assign(hc.base, hc.base + hc.levels);
+            base = hc.base[hc.levels];
+            t->max_level = hc.levels - 1;
+            done_levels = true;
+        }
+        if (!done_levels && t->coop_ok) return tfail(t, AFMM_ENOMEM, "tree_build: node arrays kept overflowing");
+        if (!done_levels) {
+            root_kernel<<<1, 1, 0, st>>>(nd, (int)n);
+            TCU(t, cudaGetLastError());
+        }
+    }
+    if (!done_levels) {
+    // 4b. per-level host loop (no cooperative launch)
     size_t lvl_cap = 0;
     void *scan_tmp = nullptr;
     size_t scan_tmp_bytes = 0;
@@ -755,6 +944,7 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
         base = next_base;
         m = total;
         ++level;
+    }
     }
     const long long nn = base;     // total nodes
     t->n_nodes = nn;
