@@ -402,6 +402,34 @@ def main():
                 h2.close()
                 tr2.close()
             extra["sweep_S"] = sweep
+            # strong-scaling proxy of the kernel: every rank's work is independent (disjoint
+            # target leaves, replicated sources), so rank r of a world-W partition is timed
+            # alone on this GPU (tools/scaling_proxy.py; one rebalance from measured times)
+            proxy = {}
+            for W in (2, 4, 8):
+                hs = []
+                for r in range(W):
+                    hw = afmm.P2P(device=local, rank=r, world=W, eps2=eps2, stream=stream.cuda_stream)
+                    hw.set_bodies(bod[0], bod[1], bod[2], bod[3])
+                    hw.set_tree(T["leaf_start"], T["leaf_count"], T["u_off"], T["u_idx"])
+                    hs.append(hw)
+                for it in range(2):
+                    ts = []
+                    for hw in hs:
+                        for _ in range(6):
+                            hw.eval(out[0], out[1], out[2], out[3])
+                        ts.append(float(np.median(hw.kernel_times(4))))
+                    if it == 0:
+                        for hw in hs:
+                            hw.rebalance(np.array(ts), 0.02)
+                proxy[str(W)] = {"rank_kernel_ms_max": round(max(ts), 4),
+                                 "E": round(kern_mean / (W * max(ts)), 3)}
+                for hw in hs:
+                    hw.close()
+            extra["strong_scaling_proxy"] = {
+                "method": "kernel only: rank r of a world-W cost-model partition timed alone on one GPU after one "
+                          "rebalance; E = T1 / (W * max_r T_r); no broadcast / gather / launch costs",
+                "T1_ms": round(kern_mean, 4), "worlds": proxy}
 
     if rank == 0 and world == 1 and not args.no_stokeslet:
         # row f4: the regularized-Stokeslet law on its paper workload (C6: 10M uniform sources, L26 SIX.B)

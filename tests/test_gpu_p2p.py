@@ -421,3 +421,19 @@ def test_eval_host_pipelined_errors():
     with pytest.raises(afmm.AfmmError) as e:
         s.eval_host_pipelined(*b)
     s.close()
+
+
+def test_task_cap_splits_for_strong_scaling():
+    """slice_world = 8 caps every task at I_total / 8 / (128 * warps * 3) warp
+    iterations: more, smaller tasks than slice_world = 1, results within R16 of
+    the oracle either way (a leaf's targets may be cut, its sums not)."""
+    x, y, z, m = synth.make("plummer", 300000, 31)
+    T, d = _tree(x, y, z, 128)
+    xs, ys, zs, ms = T.sorted_bodies(x, y, z, m)
+    ref = oracle.p2p(xs, ys, zs, ms, T.leaf_start, T.leaf_count, T.u_off, T.u_idx, 1.0, 1e-6, with_scale=True)
+    items = {}
+    for sw in (1, 8):
+        got, stats = gpu_eval(xs, ys, zs, ms, d, 1e-6, slice_world=sw)
+        _tol.check(list(got), list(ref[:4]), ref[4])
+        items[sw] = stats[0]["n_work_items"]
+    assert items[8] > items[1]
