@@ -118,6 +118,7 @@ _sig("afmm_tree_info", _i, _p, C.POINTER(_i), C.POINTER(_ll), _p, C.POINTER(_i),
      C.POINTER(_ll))
 _sig("afmm_tree_copy_out", _i, _p, _p, _p, _p, _p, _p, _p, _p)
 _sig("afmm_tree_gather", _i, _p, _p, _p)
+_sig("afmm_tree_gather_rows", _i, _p, _i, _p, _p)
 _sig("afmm_tree_scatter", _i, _p, _p, _p)
 _sig("afmm_tree_destroy", None, _p)
 _sig("afmm_tree_last_error", C.c_char_p, _p)
@@ -166,7 +167,8 @@ EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
             "afmm_lb_predicted", "afmm_lb_state", "afmm_lb_destroy", "afmm_tree_copy_out",
             "afmm_tree_gather", "afmm_tree_scatter", "afmm_tree_destroy", "afmm_tree_last_error",
             "afmm_tree_rebuild", "afmm_tree_nodes", "afmm_fine_grained", "afmm_p2p_eval_host_pipelined",
-            "afmm_p2p_set_peer_windows", "afmm_ipc_export", "afmm_ipc_import", "afmm_ipc_close"]
+            "afmm_p2p_set_peer_windows", "afmm_ipc_export", "afmm_ipc_import", "afmm_ipc_close",
+            "afmm_tree_gather_rows"]
 
 
 def ipc_export(dev_ptr):
@@ -581,6 +583,14 @@ class GpuTree:
     def gather(self, src, dst):
         """dst[p] = src[perm[p]] (device tensors)."""
         self._check(_lib.afmm_tree_gather(self._h, _ptr(src), _ptr(dst)), "afmm_tree_gather")
+
+    def gather_rows(self, src, dst):
+        """afmm_tree_gather_rows: every row of a contiguous (rows, n) device tensor
+        into tree order in one kernel."""
+        if src.dim() != 2 or not src.is_contiguous() or not dst.is_contiguous() or dst.shape != src.shape:
+            raise ValueError("gather_rows takes two contiguous (rows, n) tensors of the same shape")
+        self._check(_lib.afmm_tree_gather_rows(self._h, int(src.shape[0]), _ptr(src), _ptr(dst)),
+                    "afmm_tree_gather_rows")
 
     def scatter(self, src, dst):
         self._check(_lib.afmm_tree_scatter(self._h, _ptr(src), _ptr(dst)), "afmm_tree_scatter")

@@ -596,6 +596,14 @@ __global__ void gather_kernel(long long n, const int *__restrict__ perm, const f
          i += (long long)gridDim.x * blockDim.x)
         out[i] = in[perm[i]];
 }
+__global__ void gather_rows_kernel(long long n, int rows, const int *__restrict__ perm, const float *__restrict__ in,
+                                   float *__restrict__ out) {
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n;
+         i += (long long)gridDim.x * blockDim.x) {
+        const long long src = perm[i];
+        for (int r = 0; r < rows; ++r) out[r * n + i] = in[r * n + src];
+    }
+}
 __global__ void scatter_kernel(long long n, const int *__restrict__ perm, const float *__restrict__ in,
                                float *__restrict__ out) {
     for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n;
@@ -1201,6 +1209,15 @@ extern "C" afmm_status afmm_tree_gather(afmm_tree *t, const float *in, float *ou
     if (!t->built) return AFMM_ESTATE;
     TCU(t, cudaSetDevice(t->device));
     gather_kernel<<<grid_for(t->n, 256), 256, 0, t->stream>>>(t->n, t->perm, in, out);
+    TCU(t, cudaGetLastError());
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_tree_gather_rows(afmm_tree *t, int rows, const float *in, float *out) {
+    if (!t || !in || !out || rows < 1) return AFMM_EINVAL;
+    if (!t->built) return AFMM_ESTATE;
+    TCU(t, cudaSetDevice(t->device));
+    gather_rows_kernel<<<grid_for(t->n, 256), 256, 0, t->stream>>>(t->n, rows, t->perm, in, out);
     TCU(t, cudaGetLastError());
     return AFMM_OK;
 }

@@ -203,8 +203,7 @@ class TimeLoop:
         lbrec = self._maintain(s[0], s[1], s[2])
         if hooks and "post_maintain" in hooks:
             hooks["post_maintain"](self, lbrec)
-        for a in range(7):
-            self.tree.gather(s[a], self.tmp[a])
+        self.tree.gather_rows(s, self.tmp)          # all 7 state rows into the new tree order, one kernel
         self.state, self.tmp = self.tmp, self.state
         ev[2].record(self.stream)
         self._load_tree(host_copy=bool(hooks))

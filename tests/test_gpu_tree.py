@@ -83,6 +83,11 @@ def test_gather_scatter_roundtrip():
     t.scatter(out, back)
     torch.cuda.synchronize()
     assert np.array_equal(back.cpu().numpy(), x)
+    rows = torch.stack([_dev(v) for v in (x, y, z, m)])          # afmm_tree_gather_rows
+    rows_out = torch.empty_like(rows)
+    t.gather_rows(rows, rows_out)
+    torch.cuda.synchronize()
+    assert np.array_equal(rows_out.cpu().numpy(), np.stack([x, y, z, m])[:, perm])
     t.close()
 
 
