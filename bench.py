@@ -489,6 +489,8 @@ def main():
                                 "ranks' outputs over CUDA-IPC peer windows (fused gather) + 4-byte all_reduce"),
                        "parallelism": f"leaf-partition x{world} (cost model, PAPER L16)",
                        "gather": gather_mode,
+                       "masses": "equal (1/N, reading R19): the kernel detects it at pack time and runs its "
+                                 "equal-mass pair loop (12 packed FP32 ops per pair, G m applied once; reading R30)",
                        "tree_build_s": round(tree_s, 4), "set_tree_s": round(set_tree_s, 4)},
             "kernel_ms": {"mean": kern_mean, "max_over_ranks": kern_max},
             "gpu_time_interactions_per_s": inter / (kern_max * 1e-3),

@@ -338,7 +338,9 @@ extern "C" void *afmm_p2p_stream(const afmm_p2p *h) { return h ? (void *)h->stre
 static int words_of(const afmm_p2p *h) { return h->cfg.law == AFMM_LAW_STOKESLET ? 2 : 1; }
 
 static afmm_status alloc_bodies(afmm_p2p *h, long long n) {
-    const long long words = n * words_of(h);       // float4 per body: 1 (gravity) or 2 (Stokeslet)
+    // float4 per body: 1 (gravity) or 2 (Stokeslet), plus one trailer float4 holding the
+    // equal-mass flag (travels with the packed array when it is broadcast)
+    const long long words = n * words_of(h) + 1;
     if (words > h->bodies_cap) {
         cudaFree(h->d_bodies);
         h->d_bodies = nullptr;
@@ -352,11 +354,16 @@ static afmm_status alloc_bodies(afmm_p2p *h, long long n) {
     return AFMM_OK;
 }
 
+// the equal-mass flag: first int of the trailer float4 after the packed bodies
+static int *mass_flag(afmm_p2p *h) { return reinterpret_cast<int *>(h->d_bodies + h->n * words_of(h)); }
+
 static afmm_status pack(afmm_p2p *h, const float *x, const float *y, const float *z,
                         const float *m) {
     const int threads = 256;
     long long blocks = std::min<long long>((h->n + threads - 1) / threads, (long long)h->num_sms * 16);
-    afmm::pack_bodies_kernel<<<(int)blocks, threads, 0, h->stream>>>(h->n, x, y, z, m, h->d_bodies);
+    int *flag = mass_flag(h);
+    CUDA_TRY(h, cudaMemsetAsync(flag, 0, sizeof(int), h->stream));
+    afmm::pack_bodies_kernel<<<(int)blocks, threads, 0, h->stream>>>(h->n, x, y, z, m, h->d_bodies, flag);
     CUDA_TRY(h, cudaGetLastError());
     return AFMM_OK;
 }
@@ -372,6 +379,11 @@ extern "C" afmm_status afmm_p2p_set_bodies(afmm_p2p *h, long long n, const float
     if (st) return st;
     if ((st = alloc_bodies(h, n))) return st;
     if (nn == 4) return pack(h, x, y, z, m);
+    // allocate only: the equal-mass flag reads "unequal" until a full-buffer
+    // broadcast (afmm_p2p_bodies_buffer, trailer included) brings the root's
+    static const int one = 1;
+    CUDA_TRY(h, cudaMemcpyAsync(mass_flag(h), &one, sizeof(int), cudaMemcpyHostToDevice, h->stream));
+    CUDA_TRY(h, cudaStreamSynchronize(h->stream));
     return AFMM_OK;
 }
 
@@ -425,7 +437,7 @@ extern "C" afmm_status afmm_p2p_bodies_buffer(afmm_p2p *h, void **dev_ptr, long 
     CHECK_HANDLE(h);
     if (!h->d_bodies || h->n < 1) return fail(h, AFMM_ESTATE, "bodies_buffer: no bodies set");
     if (dev_ptr) *dev_ptr = h->d_bodies;
-    if (bytes) *bytes = h->n * (long long)sizeof(float4) * words_of(h);
+    if (bytes) *bytes = (h->n * words_of(h) + 1) * (long long)sizeof(float4);   // + the flag trailer
     return AFMM_OK;
 }
 
@@ -886,11 +898,13 @@ static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, flo
     p.eps2 = h->cfg.eps2;
     p.G = h->cfg.law == AFMM_LAW_STOKESLET ? 1.0 / (8.0 * 3.14159265358979323846 * (double)h->cfg.mu)
                                            : (double)h->cfg.G;
-    p.Gf = (float)p.G;
-    p.g_exact = (double)p.Gf == p.G;
     p.done = nullptr;
     p.in_ready = nullptr;
     p.in_err = nullptr;
+#ifndef AFMM_EQMASS
+#define AFMM_EQMASS 1
+#endif
+    p.mass_unequal = (AFMM_EQMASS && h->cfg.law == AFMM_LAW_GRAVITY) ? mass_flag(h) : nullptr;
     CUDA_TRY(h, cudaMemsetAsync(h->d_queue, 0, sizeof(int), h->stream));
     const int ri = (int)(h->n_evals % afmm_p2p::kRing);
     h->ev0 = h->ring0[ri];
@@ -1127,6 +1141,7 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
     unsigned *in_ready = reinterpret_cast<unsigned *>(h->d_pqueue + kMaxPieces + 1);
     int *in_err = h->d_pqueue + kMaxPieces + 2;
     CUDA_TRY(h, cudaMemsetAsync(h->d_pqueue, 0, (kMaxPieces + 3) * sizeof(int), h->stream));
+    CUDA_TRY(h, cudaMemsetAsync(mass_flag(h), 0xff, sizeof(int), h->stream));   // bodies replaced: flag "unequal"
     CUDA_TRY(h, cudaEventRecord(h->ev_start, h->stream));      // earlier readers of the bodies / outputs
     CUDA_TRY(h, cudaStreamWaitEvent(h->s_in, h->ev_start, 0));
     CUDA_TRY(h, cudaStreamWaitEvent(h->s_out, h->ev_start, 0));
@@ -1178,8 +1193,7 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
         prm.n_win = 1;
         prm.eps2 = h->cfg.eps2;
         prm.G = (double)h->cfg.G;
-        prm.Gf = h->cfg.G;
-        prm.g_exact = 1;
+        prm.mass_unequal = nullptr;                  // the flag is final only after the last chunk
         prm.done = done;
         prm.in_ready = in_ready;
         prm.in_err = in_err;

@@ -91,9 +91,6 @@ constexpr int kDynSmem = kWarps * (kStageBytesW + kAccBytesW);
 // the second term standing for a task's fixed cost (descriptors, first-chunk
 // latency, copy reduction) in warp iterations.  Integer arithmetic only, so the
 // host and device builders produce identical task lists.
-#ifndef AFMM_ALLMASK
-#define AFMM_ALLMASK 0                            // chunks holding self sources run wholly in the masked loop
-#endif
 #ifndef AFMM_STATIC_FRAC
 #define AFMM_STATIC_FRAC 0.9                      // share of the tasks dealt statically (snake rounds) ...
 #endif
@@ -222,8 +219,6 @@ struct P2PParams {
     int n_win;
     float eps2;
     double G;                // output scale: G (gravity) or 1/(8 pi mu) (Stokeslet)
-    float Gf;                // (float)G, used when g_exact (G is an fp32 value)
-    int g_exact;
     int *done;               // nullptr, or per-piece counters of finished tasks (afmm_p2p_eval_host_pipelined)
     // streamed inputs (afmm_p2p_eval_host_pipelined): nullptr, or the number of input
     // chunks already packed (written by the copy stream); a task whose sources reach
@@ -231,6 +226,10 @@ struct P2PParams {
     // times out (the copy stream never delivered: results invalid, reported as an error)
     const unsigned *in_ready;
     int *in_err;
+    // equal masses: nullptr, or the packed-body trailer word that the pack kernel
+    // sets when some m_j differs from m_0 (0 = all equal -> the 12-op pair loop,
+    // the common mass applied in the epilogue)
+    const int *mass_unequal;
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
@@ -281,7 +280,7 @@ __device__ __forceinline__ float rsqrt_ftz(float x) {
 
 // One source against two targets (FFMA2; 13 packed FP32 ops + 2 MUFU.RSQ).
 // n{x,y,z} hold the NEGATED target coordinates.
-template <bool kMasked>
+template <bool kMasked, bool kEq = false>
 __device__ __forceinline__ void interact2(const float4 q, const float2 nx, const float2 ny,
                                           const float2 nz, const float2 e2, float2 &ax, float2 &ay,
                                           float2 &az, float2 &ph, bool skip0, bool skip1) {
@@ -298,7 +297,9 @@ __device__ __forceinline__ void interact2(const float4 q, const float2 nx, const
         inv.x = skip0 ? 0.0f : inv.x;
         inv.y = skip1 ? 0.0f : inv.y;
     }
-    const float2 t = __fmul2_rn(make_float2(q.w, q.w), inv);   // m_j / r
+    // equal masses (kEq): the common mass m is applied once in the epilogue, so the
+    // pair needs 1/r and 1/r^3 only (12 packed ops instead of 13)
+    const float2 t = kEq ? inv : __fmul2_rn(make_float2(q.w, q.w), inv);   // m_j / r
     ph = __fadd2_rn(ph, t);
     const float2 i2 = __fmul2_rn(inv, inv);
     const float2 s = __fmul2_rn(t, i2);                         // m_j / r^3
@@ -313,11 +314,12 @@ __device__ __forceinline__ void interact2(const float4 q, const float2 nx, const
 struct Gravity {
     static constexpr int kWords = 1;
     static constexpr bool kMaskSelf = true;        // reading R2: the j == i pair is excluded
-    template <bool kMasked>
+    static constexpr bool kHasEq = true;           // an equal-mass variant exists
+    template <bool kMasked, bool kEq>
     __device__ __forceinline__ static void apply(const float4 *__restrict__ src, int k, const float2 nx,
                                                  const float2 ny, const float2 nz, const float2 e2, float2 &a0,
                                                  float2 &a1, float2 &a2, float2 &a3, bool s0, bool s1) {
-        interact2<kMasked>(src[k], nx, ny, nz, e2, a0, a1, a2, a3, s0, s1);
+        interact2<kMasked, kEq>(src[k], nx, ny, nz, e2, a0, a1, a2, a3, s0, s1);
     }
     // a = G v, phi = -G v
     __device__ __forceinline__ static float out(int comp, double v, double scale) {
@@ -336,7 +338,8 @@ struct Gravity {
 struct Stokeslet {
     static constexpr int kWords = 2;
     static constexpr bool kMaskSelf = false;
-    template <bool kMasked>
+    static constexpr bool kHasEq = false;
+    template <bool kMasked, bool kEq>
     __device__ __forceinline__ static void apply(const float4 *__restrict__ src, int k, const float2 nx,
                                                  const float2 ny, const float2 nz, const float2 e2, float2 &ux,
                                                  float2 &uy, float2 &uz, float2 &, bool, bool) {
@@ -436,7 +439,7 @@ __device__ __forceinline__ int2 lane_map(int g) { return kLaneMap.v[g]; }
 // into fp64 before they would exceed kFold sources.  Masks compare k with
 // T.m[j] - moff.  rcpC = ceil(2^16 / C): floor(N rcpC / 2^16) == floor(N / C)
 // exactly for 0 <= N < 2048, C <= 32 (no integer division in the loop setup).
-template <class Law, bool kMasked>
+template <class Law, bool kMasked, bool kEq>
 __device__ __forceinline__ void consume(const float4 *__restrict__ src, int k, int kend, int C, int rcpC,
                                         const Targets &T, int moff, const float2 e2, Partial &P) {
     while (k < kend) {
@@ -447,7 +450,7 @@ __device__ __forceinline__ void consume(const float4 *__restrict__ src, int k, i
         for (int it = 0; it < iters; ++it, k += C) {
 #pragma unroll
             for (int q = 0; q < kPairs; ++q)
-                Law::template apply<kMasked>(src, k, T.nx[q], T.ny[q], T.nz[q], e2, P.ax[q], P.ay[q], P.az[q],
+                Law::template apply<kMasked, kEq>(src, k, T.nx[q], T.ny[q], T.nz[q], e2, P.ax[q], P.ay[q], P.az[q],
                                              P.ph[q], kMasked && k == T.m[2 * q] - moff,
                                              kMasked && k == T.m[2 * q + 1] - moff);
         }
@@ -671,6 +674,10 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
             break;
 
     const float2 e2 = make_float2(p.eps2, p.eps2);
+    const bool eqm = Law::kHasEq && p.mass_unequal != nullptr && *p.mass_unequal == 0;
+    const double scale = eqm ? p.G * (double)p.bodies[0].w : p.G;     // G, or G m for equal masses
+    const float scale_f = (float)scale;
+    const bool scale_exact = (double)scale_f == scale;
     Targets T;
     Partial P;
     P.acc = accw + lane;
@@ -715,18 +722,15 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
         PROF_T(t_m);
         if (active) {
             const int kself = Law::kMaskSelf ? min(max(m.self_len - m.first, 0), m.nb) : 0;
-#if AFMM_ALLMASK
-            if (kself > 0) {             // the whole chunk in the masked loop (one call, one remainder)
-                consume<Law, true>(stage[st], c, m.nb, C, rcpC, T, m.first, e2, P);
-            } else {
-                consume<Law, false>(stage[st], c, m.nb, C, rcpC, T, 0, e2, P);
-            }
-#else
-            if (kself > 0) consume<Law, true>(stage[st], c, kself, C, rcpC, T, m.first, e2, P);
             // first k >= kself with k = c (mod C)
             const int k0 = kself <= c ? c : c + C * (((kself - c + C - 1) * rcpC) >> 16);
-            consume<Law, false>(stage[st], k0, m.nb, C, rcpC, T, 0, e2, P);
-#endif
+            if (Law::kHasEq && eqm) {
+                if (kself > 0) consume<Law, true, true>(stage[st], c, kself, C, rcpC, T, m.first, e2, P);
+                consume<Law, false, true>(stage[st], k0, m.nb, C, rcpC, T, 0, e2, P);
+            } else {
+                if (kself > 0) consume<Law, true, false>(stage[st], c, kself, C, rcpC, T, m.first, e2, P);
+                consume<Law, false, false>(stage[st], k0, m.nb, C, rcpC, T, 0, e2, P);
+            }
         }
         PROF_ADD(3, t_m);
         PROF_T(t_l);
@@ -760,7 +764,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
                     }
                 }
 #pragma unroll
-                for (int u = 0; u < kVals; ++u) o[u] = Law::out(u & 3, v[u], p.G);
+                for (int u = 0; u < kVals; ++u) o[u] = Law::out(u & 3, v[u], scale);
             } else {
                 float f[kVals];
 #pragma unroll
@@ -783,7 +787,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
                 // path skips the conversions with bit-identical outputs
 #pragma unroll
                 for (int u = 0; u < kVals; ++u)
-                    o[u] = p.g_exact ? Law::outf(u & 3, f[u], p.Gf) : Law::out(u & 3, (double)f[u], p.G);
+                    o[u] = scale_exact ? Law::outf(u & 3, f[u], scale_f) : Law::out(u & 3, (double)f[u], scale);
             }
             if (active && c == 0) {
 #pragma unroll
@@ -854,12 +858,21 @@ __global__ void __launch_bounds__(128, 21) pack_chunk_kernel(int n, const float 
         out[i] = make_float4(x[i], y[i], z[i], m[i]);
 }
 
+// SoA -> packed {x, y, z, m}; *unequal |= (some m_i != m_0) (the equal-mass flag)
 __global__ void pack_bodies_kernel(long long n, const float *__restrict__ x, const float *__restrict__ y,
                                    const float *__restrict__ z, const float *__restrict__ m,
-                                   float4 *__restrict__ out) {
+                                   float4 *__restrict__ out, int *__restrict__ unequal) {
+    const float m0 = m[0];
+    bool diff = false;
     for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n;
-         i += (long long)gridDim.x * blockDim.x)
-        out[i] = make_float4(x[i], y[i], z[i], m[i]);
+         i += (long long)gridDim.x * blockDim.x) {
+        const float mi = m[i];
+        out[i] = make_float4(x[i], y[i], z[i], mi);
+        diff |= mi != m0;
+    }
+    if (__any_sync(0xffffffffu, diff) && (threadIdx.x & 31) == 0) atomicOr(unequal, 1);
 }
+
+
 
 }  // namespace afmm

@@ -359,9 +359,12 @@ def test_set_tree_device_rejects_invalid_tree():
 def test_eval_host_pipelined_bit_identical(world, pieces, ingest):
     """afmm_p2p_eval_host_pipelined (H2D / kernel pieces / D2H overlapped) ==
     afmm_p2p_eval on device buffers, bit for bit, on every rank's slice; the
-    handle's bodies afterwards are the host ones (a plain eval agrees too)."""
+    handle's bodies afterwards are the host ones (a plain eval agrees too).
+    Unequal masses: both take the general pair loop (the streamed inputs never
+    use the equal-mass loop, whose flag is final only after the last chunk)."""
     afmm = _afmm()
     x, y, z, m = synth.make("plummer", 200000, 21)
+    m = (m * np.random.default_rng(3).uniform(0.5, 1.5, m.shape[0])).astype(np.float32)
     n = x.shape[0]
     tree = afmm.GpuTree(0)
     X, Y, Z, M = (torch.from_numpy(v).cuda() for v in (x, y, z, m))
@@ -396,6 +399,27 @@ def test_eval_host_pipelined_bit_identical(world, pieces, ingest):
         assert np.array_equal(got[a].numpy(), r_[a])
     assert np.array_equal(again.cpu().numpy(), r_)
     tree.close()
+
+
+def test_eval_host_pipelined_equal_masses_within_tolerance():
+    """Equal masses: eval (equal-mass loop) and eval_host_pipelined (general loop)
+    agree within R16 of the oracle."""
+    afmm = _afmm()
+    x, y, z, m = synth.make("plummer", 60000, 22)
+    T, d = _tree(x, y, z, 64)
+    xs, ys, zs, ms = T.sorted_bodies(x, y, z, m)
+    ref = oracle.p2p(xs, ys, zs, ms, T.leaf_start, T.leaf_count, T.u_off, T.u_idx, 1.0, 1e-6, with_scale=True)
+    dev_out, _ = gpu_eval(xs, ys, zs, ms, d, 1e-6)
+    h = afmm.P2P(eps2=1e-6)
+    h.set_bodies(*[_dev(v) for v in (xs, ys, zs, ms)])
+    h.set_tree(d["leaf_start"], d["leaf_count"], d["u_off"], d["u_idx"])
+    hb = [torch.from_numpy(np.ascontiguousarray(v, np.float32)).pin_memory() for v in (xs, ys, zs, ms)]
+    got = [torch.empty(xs.shape[0]).pin_memory() for _ in range(4)]
+    h.eval_host_pipelined(*hb, *got, pieces=3)
+    h.close()
+    pipe = (got[3].numpy(), got[0].numpy(), got[1].numpy(), got[2].numpy())     # oracle order phi, ax, ay, az
+    _tol.check(list(pipe), list(ref[:4]), ref[4])
+    _tol.check(list(dev_out), list(ref[:4]), ref[4])
 
 
 def test_eval_host_pipelined_errors():
@@ -437,3 +461,30 @@ def test_task_cap_splits_for_strong_scaling():
         _tol.check(list(got), list(ref[:4]), ref[4])
         items[sw] = stats[0]["n_work_items"]
     assert items[8] > items[1]
+
+
+def test_unequal_masses_general_path_and_equal_mass_path():
+    """The synthetic workloads have equal masses (R19), which the kernel detects
+    (pack flag) and evaluates with the 12-op pair loop, applying G m once at the
+    end.  Unequal masses take the general 13-op loop.  Both against the oracle
+    (R16); equal masses scaled by 2^k scale the outputs bit-exactly on both."""
+    x, y, z, m = synth.make("plummer", 120000, 41)
+    T, d = _tree(x, y, z, 96)
+    xs, ys, zs, ms = T.sorted_bodies(x, y, z, m)
+    rng = np.random.default_rng(5)
+    mu = (ms * rng.uniform(0.5, 1.5, ms.shape[0])).astype(np.float32)     # unequal
+    for mm in (ms, mu):
+        ref = oracle.p2p(xs, ys, zs, mm, T.leaf_start, T.leaf_count, T.u_off, T.u_idx, 1.0, 1e-6, with_scale=True)
+        got, _ = gpu_eval(xs, ys, zs, mm, d, 1e-6)
+        _tol.check(list(got), list(ref[:4]), ref[4])
+    # one body's mass differs by one ulp: the general loop, within R16 of the oracle
+    m1 = ms.copy()
+    m1[777] = np.nextafter(m1[777], np.float32(1))
+    ref1 = oracle.p2p(xs, ys, zs, m1, T.leaf_start, T.leaf_count, T.u_off, T.u_idx, 1.0, 1e-6, with_scale=True)
+    g_1, _ = gpu_eval(xs, ys, zs, m1, d, 1e-6)
+    _tol.check(list(g_1), list(ref1[:4]), ref1[4])
+    g_eq, _ = gpu_eval(xs, ys, zs, ms, d, 1e-6)
+    assert not all(np.array_equal(a, b) for a, b in zip(g_eq, g_1))     # the two loops round differently
+    g8, _ = gpu_eval(xs, ys, zs, (ms * 8).astype(np.float32), d, 1e-6)
+    for a, b in zip(g_eq, g8):
+        assert np.array_equal(a * 8, b)
