@@ -38,7 +38,7 @@ sys.path.insert(0, ROOT)
 
 import synth  # noqa: E402  (seeded input generator shared by both arms)
 
-E2E_PIECES = 2             # output pieces of the pipelined host-to-host evaluation (e2e; tools/e2e_probe.py)
+E2E_PIECES = 1             # output pieces of the pipelined host-to-host evaluation (staged mode only; zero-copy: 1 = tasks ordered by input chunk; tools/e2e_probe.py)
 FLOPS_PER_INTERACTION = 20
 METRIC = "near-field P2P interactions/s (and % FP32 peak) at 1/2/4/8 B200"
 SWEEP_S = [32, 48, 64, 96, 128, 192, 256, 384, 512]
@@ -333,10 +333,12 @@ def main():
     ho = [torch.empty(n, dtype=torch.float32).pin_memory() for _ in range(4)]
     Ke = max(3, K // 2)
 
+    e2e_mode = {"zero_copy": 0}
+
     def step_e2e():
         if world == 1:
             # afmm_p2p_eval_host_pipelined: H2D + pack, kernel pieces, D2H overlapped; blocking
-            h.eval_host_pipelined(*hx, *ho, pieces=E2E_PIECES)
+            e2e_mode["zero_copy"] = h.eval_host_pipelined(*hx, *ho, pieces=E2E_PIECES)["zero_copy"]
         else:
             if rank == 0:
                 for a in range(4):
@@ -502,7 +504,11 @@ def main():
             "clocks": clk.summary(),
             "e2e": {"value": e2e_value, "unit": "interactions/s", "h2d_bytes_per_step": 16 * n,
                     "d2h_bytes_per_step": 16 * n, "steps": Ke,
-                    "path": f"afmm_p2p_eval_host_pipelined (8 streamed input chunks, {E2E_PIECES} output pieces) from pinned host arrays" if world == 1
+                    "path": (("afmm_p2p_eval_host_pipelined, zero-copy: 8 input chunks packed from the pinned host "
+                              "arrays over PCIe while the kernel runs, outputs written to the pinned host arrays by "
+                              "the kernel's task epilogue") if e2e_mode["zero_copy"] else
+                             f"afmm_p2p_eval_host_pipelined (8 streamed input chunks, {E2E_PIECES} output pieces) "
+                             "from pinned host arrays") if world == 1
                     else "rank 0 H2D + step + D2H"},
             "gpu_launches": 2 * K,
             "rebalanced_in_warmup": rebalanced,

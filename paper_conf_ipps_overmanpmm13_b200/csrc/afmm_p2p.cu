@@ -78,6 +78,7 @@ struct afmm_p2p {
     cudaEvent_t ring0[kRing] = {}, ring1[kRing] = {};
     long long n_evals = 0;
     bool evaluated = false;
+    bool last_zero_copy = false;                     // last eval_host_pipelined ran zero-copy
     afmm_p2p_stats last{};
 
     // pipelined host evaluation (afmm_p2p_eval_host_pipelined): the rank's tasks
@@ -279,6 +280,9 @@ extern "C" afmm_status afmm_p2p_create(const afmm_p2p_config *cfg, afmm_p2p **ou
         if (e == cudaSuccess)
             e = cudaFuncSetAttribute(afmm::p2p_kernel_t<afmm::Gravity>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                      afmm::kDynSmem);
+        if (e == cudaSuccess)
+            e = cudaFuncSetAttribute(afmm::p2p_kernel_t<afmm::Gravity, true>,
+                                     cudaFuncAttributeMaxDynamicSharedMemorySize, afmm::kDynSmem);
         if (e == cudaSuccess)
             e = cudaFuncSetAttribute(afmm::p2p_kernel_t<afmm::Stokeslet>,
                                      cudaFuncAttributeMaxDynamicSharedMemorySize, afmm::kDynSmem);
@@ -905,6 +909,9 @@ static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, flo
 #define AFMM_EQMASS 1
 #endif
     p.mass_unequal = (AFMM_EQMASS && h->cfg.law == AFMM_LAW_GRAVITY) ? mass_flag(h) : nullptr;
+    p.mass_bits = nullptr;
+    p.out_coalesce = 0;
+    h->last_zero_copy = false;
     CUDA_TRY(h, cudaMemsetAsync(h->d_queue, 0, sizeof(int), h->stream));
     const int ri = (int)(h->n_evals % afmm_p2p::kRing);
     h->ev0 = h->ring0[ri];
@@ -943,6 +950,7 @@ static afmm_status fill_stats(afmm_p2p *h, afmm_p2p_stats *s) {
     o.body_hi = h->body_split[h->cfg.rank + 1];
     o.n_work_items = h->n_tasks;
     o.n_launches = h->last.n_launches;
+    o.zero_copy = h->last_zero_copy ? 1 : 0;
     for (int b = 0; b < 8; ++b) o.bucket_interactions[b] = h->bucket_inter[b];
     h->last = o;
     if (s) *s = o;
@@ -989,8 +997,21 @@ extern "C" afmm_status afmm_p2p_eval_host(afmm_p2p *h, float *ax, float *ay, flo
 
 // ------------------------------------------------------------------ pipelined host evaluation
 
+// A host pointer the device can dereference (page-locked, mapped: pinned memory
+// under unified addressing); *dptr = its device address.  Pageable memory -> false.
+static bool host_mapped(const void *p, void **dptr) {
+    cudaPointerAttributes at{};
+    if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    if (at.type != cudaMemoryTypeHost || !at.devicePointer) return false;
+    *dptr = at.devicePointer;
+    return true;
+}
+
 static constexpr int kMaxPieces = 64;
-static constexpr int kInChunks = 8;                 // input chunks of the streamed H2D
+static constexpr int kInChunks = 8;                 // input chunks of the streamed H2D (<= 32: mass bits)
 
 // Regroup this rank's tasks into P pieces of consecutive targets (equal modelled
 // cost tgt_count * nsrc, cut in tgt_start order); inside a piece the tasks keep
@@ -1045,7 +1066,9 @@ static afmm_status build_pipe(afmm_p2p *h, int P) {
     // and targets), then by output piece, LPT kept inside -- so the kernel starts on the
     // first chunk and stays behind the copies, and every output piece's stragglers (leaves
     // whose U-lists reach far in Morton order) run as soon as the last chunk lands.
-    const int K = (int)std::min<long long>(kInChunks, std::max<long long>(1, h->n / 4096));
+    const char *kenv = getenv("AFMM_E2E_CHUNKS");             // measurements only
+    const int kin = kenv ? std::max(1, std::min(32, atoi(kenv))) : kInChunks;
+    const int K = (int)std::min<long long>(kin, std::max<long long>(1, h->n / 4096));
     const long long chunk = (h->n + K - 1) / K;
     std::vector<int> need_chunk(nt, 0);
     for (int i = 0; i < nt; ++i) {
@@ -1058,7 +1081,13 @@ static afmm_status build_pipe(afmm_p2p *h, int P) {
     }
     std::vector<int> ord2(nt);
     for (int i = 0; i < nt; ++i) ord2[i] = i;
+    static const bool piece_major = [] {
+        const char *e = getenv("AFMM_PIPE_ORDER");
+        return !(e && e[0] == 'c');
+    }();
     std::stable_sort(ord2.begin(), ord2.end(), [&](int a, int b) {
+        if (piece_major)
+            return piece[a] != piece[b] ? piece[a] < piece[b] : need_chunk[a] < need_chunk[b];
         return need_chunk[a] != need_chunk[b] ? need_chunk[a] < need_chunk[b] : piece[a] < piece[b];
     });
     std::vector<afmm::Task> grouped(std::max(nt, 1));
@@ -1098,7 +1127,7 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
             CUDA_TRY(h, cudaEventCreateWithFlags(&h->ev_in[i], cudaEventDisableTiming));
             CUDA_TRY(h, cudaEventCreateWithFlags(&h->ev_k[i], cudaEventDisableTiming));
         }
-        CUDA_TRY(h, cudaMalloc(&h->d_pqueue, (kMaxPieces + 3) * sizeof(int)));
+        CUDA_TRY(h, cudaMalloc(&h->d_pqueue, (kMaxPieces + 4) * sizeof(int)));
         cudaDriverEntryPointQueryResult q;
         CUDA_TRY(h, cudaGetDriverEntryPoint("cuStreamWaitValue32", &h->wait_value32, cudaEnableDefault, &q));
         if (q != cudaDriverEntryPointSuccess || !h->wait_value32)
@@ -1140,7 +1169,27 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
     int *queue = h->d_pqueue, *done = h->d_pqueue + 1;
     unsigned *in_ready = reinterpret_cast<unsigned *>(h->d_pqueue + kMaxPieces + 1);
     int *in_err = h->d_pqueue + kMaxPieces + 2;
-    CUDA_TRY(h, cudaMemsetAsync(h->d_pqueue, 0, (kMaxPieces + 3) * sizeof(int), h->stream));
+    unsigned *mass_bits = reinterpret_cast<unsigned *>(h->d_pqueue + kMaxPieces + 3);
+    CUDA_TRY(h, cudaMemsetAsync(h->d_pqueue, 0, (kMaxPieces + 4) * sizeof(int), h->stream));
+    // Zero-copy when all eight host arrays are page-locked and device-mapped (pinned
+    // memory under unified addressing): the pack kernels read the inputs and the P2P
+    // kernel's epilogue writes the outputs straight over PCIe -- no staging copies,
+    // the output transfer spread over the whole kernel.  Else staged copies.
+    const float *zin[4] = {nullptr, nullptr, nullptr, nullptr};
+    float *zout[4] = {nullptr, nullptr, nullptr, nullptr};
+    // (AFMM_E2E_ZEROCOPY: "0" off; "i" / "o" inputs / outputs only -- for measurements)
+    const char *zenv = getenv("AFMM_E2E_ZEROCOPY");
+    bool zc = !(zenv && zenv[0] == '0');
+    for (int a = 0; a < 4 && zc; ++a) {
+        void *d = nullptr;
+        zc = host_mapped(hin[a], &d);
+        zin[a] = static_cast<const float *>(d);
+        zc = zc && host_mapped(hout[a], &d);
+        zout[a] = static_cast<float *>(d);
+    }
+    const bool zc_in = zc && !(zenv && zenv[0] == 'o'), zc_out = zc && !(zenv && zenv[0] == 'i');
+    h->last_zero_copy = zc;
+    const float m0 = m[0];                          // equal-mass test of the streamed chunks
     CUDA_TRY(h, cudaMemsetAsync(mass_flag(h), 0xff, sizeof(int), h->stream));   // bodies replaced: flag "unequal"
     CUDA_TRY(h, cudaEventRecord(h->ev_start, h->stream));      // earlier readers of the bodies / outputs
     CUDA_TRY(h, cudaStreamWaitEvent(h->s_in, h->ev_start, 0));
@@ -1149,62 +1198,72 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
     // chunk count in device memory (cuStreamWriteValue32 orders the packed bodies
     // before the flag); the kernel's warps wait per task for the chunk it needs.
     // The pack kernels run next to the persistent P2P kernel (128 threads, few
-    // registers: they fit in what one P2P CTA leaves free on an SM).  Chunk 0 is in
-    // place before the launch.
+    // registers: they fit in what one P2P CTA leaves free on an SM).
+    // The P2P launch is enqueued AFTER every input chunk's pack (host order): if the
+    // copy stream and the compute stream share a hardware queue, a pack queued behind
+    // the persistent kernel would never run (the kernel waits for it).  The kernel
+    // does not wait for chunk 0 (its warps wait per task; m_0 comes from the host).
+    int nlaunch = 0;
+    auto launch = [&]() -> afmm_status {
+        const int ri = (int)(h->n_evals % afmm_p2p::kRing);
+        h->ev0 = h->ring0[ri];
+        h->ev1 = h->ring1[ri];
+        CUDA_TRY(h, cudaEventRecord(h->ev0, h->stream));
+        const int nt = h->pipe_off[P];
+        if (nt > 0) {
+            afmm::P2PParams prm;
+            prm.bodies = h->d_bodies;
+            prm.tasks = h->d_ptasks;
+            prm.segs = h->d_segs;
+            prm.n_tasks = nt;
+            prm.queue = queue;
+            prm.static_rounds = 0;                       // pieces complete in claim order
+            for (int a = 0; a < 4; ++a) prm.out[0][a] = zc_out ? zout[a] : dout[a];
+            prm.n_win = 1;
+            prm.out_coalesce = zc_out ? 1 : 0;
+            prm.mass_bits = (AFMM_EQMASS && h->cfg.law == AFMM_LAW_GRAVITY) ? mass_bits : nullptr;
+            prm.eps2 = h->cfg.eps2;
+            prm.G = (double)h->cfg.G;
+            prm.mass_unequal = nullptr;                  // the flag is final only after the last chunk
+            prm.done = zc_out ? nullptr : done;
+            prm.in_ready = in_ready;
+            prm.in_err = in_err;
+            prm.m0 = m0;
+            const int grid = std::max(1, std::min((nt + afmm::kWarps - 1) / afmm::kWarps, h->num_sms * h->blocks_per_sm));
+            afmm::p2p_kernel_t<afmm::Gravity, true><<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(prm);
+            CUDA_TRY(h, cudaGetLastError());
+            nlaunch = 1;
+        }
+        CUDA_TRY(h, cudaEventRecord(h->ev1, h->stream));
+        return AFMM_OK;
+    };
     const int K = h->pipe_K;
     const long long chunk = (n + K - 1) / K;
     for (int k = 0; k < K; ++k) {
         const long long lo = k * chunk, hi = std::min<long long>(n, lo + chunk);
         if (hi > lo) {
-            for (int a = 0; a < 4; ++a)
-                CUDA_TRY(h, cudaMemcpyAsync(dsoa[a] + lo, hin[a] + lo, (size_t)(hi - lo) * sizeof(float),
-                                            cudaMemcpyHostToDevice, h->s_in));
+            const float *src[4];
+            for (int a = 0; a < 4; ++a) {
+                if (zc_in) {
+                    src[a] = zin[a] + lo;
+                } else {
+                    CUDA_TRY(h, cudaMemcpyAsync(dsoa[a] + lo, hin[a] + lo, (size_t)(hi - lo) * sizeof(float),
+                                                cudaMemcpyHostToDevice, h->s_in));
+                    src[a] = dsoa[a] + lo;
+                }
+            }
             const int threads = 128;
             const int blocks = (int)std::min<long long>((hi - lo + threads - 1) / threads, (long long)h->num_sms);
-            afmm::pack_chunk_kernel<<<blocks, threads, 0, h->s_in>>>((int)(hi - lo), dsoa[0] + lo, dsoa[1] + lo,
-                                                                    dsoa[2] + lo, dsoa[3] + lo, h->d_bodies + lo);
+            afmm::pack_chunk_kernel<<<blocks, threads, 0, h->s_in>>>((int)(hi - lo), src[0], src[1], src[2], src[3],
+                                                                    h->d_bodies + lo, m0, mass_bits, k);
             CUDA_TRY(h, cudaGetLastError());
         }
         const CUresult r = write32((CUstream)h->s_in, (CUdeviceptr)in_ready, (cuuint32_t)(k + 1), 0);
         if (r != CUDA_SUCCESS) return fail(h, AFMM_ECUDA, "eval_host_pipelined: cuStreamWriteValue32 failed (%d)", (int)r);
-        if (k == 0) {
-            CUDA_TRY(h, cudaEventRecord(h->ev_in[0], h->s_in));
-            CUDA_TRY(h, cudaStreamWaitEvent(h->stream, h->ev_in[0], 0));
-        }
     }
-    const int ri = (int)(h->n_evals % afmm_p2p::kRing);
-    h->ev0 = h->ring0[ri];
-    h->ev1 = h->ring1[ri];
-    CUDA_TRY(h, cudaEventRecord(h->ev0, h->stream));
-    const int nt = h->pipe_off[P];
-    int nlaunch = 0;
-    if (nt > 0) {
-        afmm::P2PParams prm;
-        prm.bodies = h->d_bodies;
-        prm.tasks = h->d_ptasks;
-        prm.segs = h->d_segs;
-        prm.n_tasks = nt;
-        prm.queue = queue;
-        prm.static_rounds = 0;                       // pieces complete in claim order
-        prm.out[0][0] = dout[0];
-        prm.out[0][1] = dout[1];
-        prm.out[0][2] = dout[2];
-        prm.out[0][3] = dout[3];
-        prm.n_win = 1;
-        prm.eps2 = h->cfg.eps2;
-        prm.G = (double)h->cfg.G;
-        prm.mass_unequal = nullptr;                  // the flag is final only after the last chunk
-        prm.done = done;
-        prm.in_ready = in_ready;
-        prm.in_err = in_err;
-        const int grid = std::max(1, std::min((nt + afmm::kWarps - 1) / afmm::kWarps, h->num_sms * h->blocks_per_sm));
-        afmm::p2p_kernel_t<afmm::Gravity><<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(prm);
-        CUDA_TRY(h, cudaGetLastError());
-        nlaunch = 1;
-    }
-    CUDA_TRY(h, cudaEventRecord(h->ev1, h->stream));
+    if ((st = launch())) return st;
     // the launch must be enqueued before the copy-out stream starts waiting on its counters
-    for (int q = 0; q < P; ++q) {
+    for (int q = 0; q < P && !zc_out; ++q) {
         const long long lo = h->pipe_lo[q], hi = h->pipe_hi[q];
         const int cnt = h->pipe_off[q + 1] - h->pipe_off[q];
         if (hi <= lo || cnt == 0) continue;

@@ -79,6 +79,7 @@ constexpr int kUnroll = AFMM_UNROLL;            // inner-loop unroll (sources)
 constexpr int kStageBytesW = kWStages * kWCap * 16;     // per warp
 constexpr int kAccBytesW = kVals * 32 * 8;              // per warp
 constexpr int kDynSmem = kWarps * (kStageBytesW + kAccBytesW);
+static_assert(4 * kTaskTargets * (int)sizeof(float) <= kAccBytesW, "output staging must fit the accumulator area");
 
 // ---- target slicing (host and device worklist builders share this; SURVEY
 // S8(a) a5 "leaves bucketed by size, so adaptive leaves of 1..S bodies do not
@@ -230,6 +231,16 @@ struct P2PParams {
     // sets when some m_j differs from m_0 (0 = all equal -> the 12-op pair loop,
     // the common mass applied in the epilogue)
     const int *mass_unequal;
+    // streamed inputs only: nullptr, or a word whose bit k the pack of input chunk k
+    // sets when some mass in that chunk differs from m_0; a task whose sources lie in
+    // chunks 0..r (r = piece >> 16) runs the equal-mass loop when bits 0..r are clear
+    // (read after the task's wait_inputs, so every bit it looks at is final)
+    const unsigned *mass_bits;
+    float m0;                // streamed inputs: m_0 (from the host), the equal-mass scale's mass
+    // 1: outputs are written through shared memory as whole runs of consecutive
+    // targets per component (host-mapped output arrays: full PCIe lines, not 4-byte
+    // pieces with byte enables)
+    int out_coalesce;
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
@@ -553,7 +564,7 @@ __device__ __forceinline__ void wait_inputs(const P2PParams &p, int piece) {
 // Stage the next chunk (<= kWCap bodies) of the stream into `buf`; returns
 // false when no task is left.  Lane 0 posts the byte count, then every lane
 // whose segment overlaps the chunk issues that piece (no warp-serial walk).
-template <int kWords>
+template <int kWords, bool kStream>
 __device__ __forceinline__ bool issue_chunk(const P2PParams &p, Stream &S, float4 *buf, uint64_t *bar,
                                             ChunkMeta *meta, int lane, long long *prof = nullptr) {
     if (S.task >= p.n_tasks) return false;
@@ -562,7 +573,7 @@ __device__ __forceinline__ bool issue_chunk(const P2PParams &p, Stream &S, float
         S.pre_ok = true;
     }
     const int nb = min(kWCap / kWords, S.t.nsrc - S.staged);
-    if (p.in_ready && S.staged == 0) wait_inputs(p, S.t.piece);
+    if (kStream && p.in_ready && S.staged == 0) wait_inputs(p, S.t.piece);
     PROF_T(t_a);
     if (lane == 0) {
         ChunkMeta m;
@@ -635,7 +646,10 @@ __device__ __forceinline__ void load_targets(Targets &T, const float4 *__restric
     }
 }
 
-template <class Law>
+// kStream: the streamed host evaluation's features (input-chunk waits, per-task
+// equal-mass test, finished-task counters, coalesced host-mapped output stores);
+// a separate instantiation so the device path carries none of their registers.
+template <class Law, bool kStream = false>
 __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const __grid_constant__ P2PParams p) {
     extern __shared__ __align__(128) unsigned char dsmem[];
     __shared__ __align__(8) uint64_t full_all[kWarps][kWStages];
@@ -669,15 +683,16 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
     S.staged = 0;
     int issued = 0;
     for (; issued < kWStages - 1; ++issued)
-        if (!issue_chunk<Law::kWords>(p, S, stage[issued % kWStages], &full[issued % kWStages],
+        if (!issue_chunk<Law::kWords, kStream>(p, S, stage[issued % kWStages], &full[issued % kWStages],
                                       &meta[issued % kWStages], lane))
             break;
 
     const float2 e2 = make_float2(p.eps2, p.eps2);
-    const bool eqm = Law::kHasEq && p.mass_unequal != nullptr && *p.mass_unequal == 0;
-    const double scale = eqm ? p.G * (double)p.bodies[0].w : p.G;     // G, or G m for equal masses
-    const float scale_f = (float)scale;
-    const bool scale_exact = (double)scale_f == scale;
+    bool eqm = Law::kHasEq && p.mass_unequal != nullptr && *p.mass_unequal == 0;
+    const double scale_eq = p.G * (double)(kStream ? p.m0 : p.bodies[0].w);   // G m for equal masses
+    double scale = eqm ? scale_eq : p.G;                               // else G
+    float scale_f = (float)scale;
+    bool scale_exact = (double)scale_f == scale;
     Targets T;
     Partial P;
     P.acc = accw + lane;
@@ -690,9 +705,9 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
         if (issued == q + kWStages - 1) {
             const int s2 = issued % kWStages;
 #if AFMM_PROF
-            if (issue_chunk<Law::kWords>(p, S, stage[s2], &full[s2], &meta[s2], lane, prof)) ++issued;
+            if (issue_chunk<Law::kWords, kStream>(p, S, stage[s2], &full[s2], &meta[s2], lane, prof)) ++issued;
 #else
-            if (issue_chunk<Law::kWords>(p, S, stage[s2], &full[s2], &meta[s2], lane)) ++issued;
+            if (issue_chunk<Law::kWords, kStream>(p, S, stage[s2], &full[s2], &meta[s2], lane)) ++issued;
 #endif
         }
         PROF_ADD(0, t_is);
@@ -715,6 +730,16 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
             l = lane - c * g;
             active = c < C;
             load_targets<Law::kWords>(T, stage[st], p.bodies, m, l, active);
+            if (kStream && Law::kHasEq && p.mass_bits) {         // streamed inputs: per-task equal-mass test
+                unsigned b;
+                asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(b) : "l"(p.mass_bits) : "memory");
+                const unsigned r = (unsigned)m.piece >> 16;
+                const unsigned mask = r >= 31 ? 0xffffffffu : (2u << r) - 1u;
+                eqm = (b & mask) == 0;
+                scale = eqm ? scale_eq : p.G;
+                scale_f = (float)scale;
+                scale_exact = (double)scale_f == scale;
+            }
             P.clear();
             P.folded = false;
         }
@@ -789,7 +814,24 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
                 for (int u = 0; u < kVals; ++u)
                     o[u] = scale_exact ? Law::outf(u & 3, f[u], scale_f) : Law::out(u & 3, (double)f[u], scale);
             }
-            if (active && c == 0) {
+            if (kStream && p.out_coalesce) {
+                // stage the task's outputs in the (now free) accumulator area as
+                // [component][target], then every lane stores consecutive targets
+                __syncwarp();
+                float *sc = reinterpret_cast<float *>(accw);
+                if (active && c == 0) {
+#pragma unroll
+                    for (int j = 0; j < kTPT; ++j) {
+                        const int u = 8 * (j >> 1) + 4 * (j & 1), tgt = kTPT * l + j;
+#pragma unroll
+                        for (int a = 0; a < 4; ++a) sc[a * kTaskTargets + tgt] = o[u + a];
+                    }
+                }
+                __syncwarp();
+#pragma unroll
+                for (int a = 0; a < 4; ++a)
+                    for (int t = lane; t < m.tgt_count; t += 32) p.out[0][a][m.tgt_start + t] = sc[a * kTaskTargets + t];
+            } else if (active && c == 0) {
 #pragma unroll
                 for (int j = 0; j < kTPT; ++j) {
                     const int tgt = kTPT * l + j;
@@ -812,7 +854,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
                     }
                 }
             }
-            if (p.done) {                 // publish the task's outputs (pipelined copy-back waits on it)
+            if (kStream && p.done) {      // publish the task's outputs (pipelined copy-back waits on it)
                 __threadfence();
                 __syncwarp();
                 if (lane == 0) atomicAdd(p.done + (m.piece & 0xffff), 1);
@@ -850,12 +892,20 @@ __global__ void pack_stokeslet_kernel(long long n, const float *__restrict__ x, 
 
 // Streamed-input pack (afmm_p2p_eval_host_pipelined): runs NEXT TO the persistent
 // P2P kernel, so it must fit in what a P2P CTA leaves free on an SM (4096
-// registers): 128 threads, <= 24 registers, 32-bit indices.
+// registers): 128 threads, <= 24 registers, 32-bit indices.  The SoA inputs are
+// device staging copies or host-mapped pinned arrays (zero-copy: read over PCIe).
+// Sets bit `chunk` of *mass_bits when some mass of the chunk differs from m0.
 __global__ void __launch_bounds__(128, 21) pack_chunk_kernel(int n, const float *__restrict__ x,
                                                              const float *__restrict__ y, const float *__restrict__ z,
-                                                             const float *__restrict__ m, float4 *__restrict__ out) {
-    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
-        out[i] = make_float4(x[i], y[i], z[i], m[i]);
+                                                             const float *__restrict__ m, float4 *__restrict__ out,
+                                                             float m0, unsigned *mass_bits, int chunk) {
+    bool diff = false;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+        const float mi = m[i];
+        out[i] = make_float4(x[i], y[i], z[i], mi);
+        diff |= mi != m0;
+    }
+    if (__any_sync(0xffffffffu, diff) && (threadIdx.x & 31) == 0) atomicOr(mass_bits, 1u << chunk);
 }
 
 // SoA -> packed {x, y, z, m}; *unequal |= (some m_i != m_0) (the equal-mass flag)

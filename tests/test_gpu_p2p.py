@@ -354,14 +354,16 @@ def test_set_tree_device_rejects_invalid_tree():
     h.close()
 
 
-@pytest.mark.parametrize("world,pieces,ingest", [(1, 1, "host"), (1, 8, "host"), (1, 64, "device"), (2, 5, "host"),
-                                                 (3, 8, "device")])
-def test_eval_host_pipelined_bit_identical(world, pieces, ingest):
-    """afmm_p2p_eval_host_pipelined (H2D / kernel pieces / D2H overlapped) ==
+@pytest.mark.parametrize("world,pieces,ingest,zc", [(1, 1, "host", "1"), (1, 8, "host", "0"), (1, 64, "device", "0"),
+                                                    (1, 8, "device", "1"), (2, 5, "host", "0"), (2, 5, "host", "1"),
+                                                    (3, 8, "device", "1")])
+def test_eval_host_pipelined_bit_identical(world, pieces, ingest, zc, monkeypatch):
+    """afmm_p2p_eval_host_pipelined (H2D / kernel pieces / D2H overlapped;
+    zc = "1": zero-copy, the kernels read and write the pinned host arrays) ==
     afmm_p2p_eval on device buffers, bit for bit, on every rank's slice; the
     handle's bodies afterwards are the host ones (a plain eval agrees too).
-    Unequal masses: both take the general pair loop (the streamed inputs never
-    use the equal-mass loop, whose flag is final only after the last chunk)."""
+    Unequal masses: both take the general pair loop."""
+    monkeypatch.setenv("AFMM_E2E_ZEROCOPY", zc)
     afmm = _afmm()
     x, y, z, m = synth.make("plummer", 200000, 21)
     m = (m * np.random.default_rng(3).uniform(0.5, 1.5, m.shape[0])).astype(np.float32)
@@ -390,6 +392,7 @@ def test_eval_host_pipelined_bit_identical(world, pieces, ingest):
         for _ in range(2):                                                  # plan reused on the 2nd call
             st = h.eval_host_pipelined(*hb, *got, pieces=pieces)
         assert st["n_launches"] <= pieces and st["n_launches"] >= 1
+        assert st["zero_copy"] == int(zc)
         h.eval(again[0], again[1], again[2], again[3])
         h.close()
     torch.cuda.synchronize()
@@ -401,9 +404,13 @@ def test_eval_host_pipelined_bit_identical(world, pieces, ingest):
     tree.close()
 
 
-def test_eval_host_pipelined_equal_masses_within_tolerance():
-    """Equal masses: eval (equal-mass loop) and eval_host_pipelined (general loop)
-    agree within R16 of the oracle."""
+@pytest.mark.parametrize("zc", ["0", "1"])
+def test_eval_host_pipelined_equal_masses(zc, monkeypatch):
+    """Equal masses: the streamed chunks are flagged equal-mass, so
+    eval_host_pipelined runs the equal-mass loop like eval: bit-identical to it,
+    and both within R16 of the oracle.  One changed mass in the last chunk sends
+    the tasks that reach it (only those) to the general loop: still within R16."""
+    monkeypatch.setenv("AFMM_E2E_ZEROCOPY", zc)
     afmm = _afmm()
     x, y, z, m = synth.make("plummer", 60000, 22)
     T, d = _tree(x, y, z, 64)
@@ -415,11 +422,24 @@ def test_eval_host_pipelined_equal_masses_within_tolerance():
     h.set_tree(d["leaf_start"], d["leaf_count"], d["u_off"], d["u_idx"])
     hb = [torch.from_numpy(np.ascontiguousarray(v, np.float32)).pin_memory() for v in (xs, ys, zs, ms)]
     got = [torch.empty(xs.shape[0]).pin_memory() for _ in range(4)]
-    h.eval_host_pipelined(*hb, *got, pieces=3)
-    h.close()
-    pipe = (got[3].numpy(), got[0].numpy(), got[1].numpy(), got[2].numpy())     # oracle order phi, ax, ay, az
+    st = h.eval_host_pipelined(*hb, *got, pieces=3)
+    assert st["zero_copy"] == int(zc)
+    pipe = tuple(got[a].numpy().copy() for a in (3, 0, 1, 2))     # oracle order phi, ax, ay, az
+    for a in range(4):
+        assert np.array_equal(pipe[a], dev_out[a])
     _tol.check(list(pipe), list(ref[:4]), ref[4])
     _tol.check(list(dev_out), list(ref[:4]), ref[4])
+    # perturb one mass in the last input chunk (x1.5): general loop for the tasks reaching it
+    n = xs.shape[0]
+    ms2 = ms.copy()
+    ms2[n - 5] *= 1.5
+    hb[3].copy_(torch.from_numpy(np.ascontiguousarray(ms2, np.float32)))
+    ref2 = oracle.p2p(xs, ys, zs, ms2, T.leaf_start, T.leaf_count, T.u_off, T.u_idx, 1.0, 1e-6, with_scale=True)
+    h.eval_host_pipelined(*hb, *got, pieces=3)
+    h.close()
+    pipe2 = (got[3].numpy(), got[0].numpy(), got[1].numpy(), got[2].numpy())
+    _tol.check(list(pipe2), list(ref2[:4]), ref2[4])
+    assert not np.array_equal(pipe2[0], pipe[0])
 
 
 def test_eval_host_pipelined_errors():

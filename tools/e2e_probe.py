@@ -50,7 +50,7 @@ def timeit(fn):
 
 res = {}
 res["host_sequential"] = timeit(lambda: (h.set_bodies(*hx), h.eval(*ho)))
-for P in (1, 2, 4, 8, 16, 32):
+for P in [int(v) for v in os.environ.get("PIECES", "1,2,4,8,16,32").split(",")]:
     res[f"pipelined_{P}"] = timeit(lambda: h.eval_host_pipelined(*hx, *ho, pieces=P))
     res[f"pipelined_{P}_kernel_span_ms"] = h.stats()["kernel_ms"]
 res["kernel_only"] = timeit(lambda: h.eval(*[bod[0], bod[1], bod[2], bod[3]]) if False else

@@ -86,6 +86,61 @@ __device__ __forceinline__ void interact1(const float4 q, float nx, float ny, fl
     az = fmaf(s, dz, az);
 }
 
+
+// Variant 5/6: equal-mass loop (12 packed ops); 6 = the three a-updates as six scalar FFMAs
+// (an FFMA2 reading three distinct register pairs costs 3 pipe cycles, two scalar FFMAs 2)
+template <bool kScalarA>
+__device__ __forceinline__ void interact2_eq(const float4 q, const float2 nx, const float2 ny, const float2 nz,
+                                             const float2 e2, float2 &ax, float2 &ay, float2 &az, float2 &ph) {
+    const float2 dx = __fadd2_rn(make_float2(q.x, q.x), nx);
+    const float2 dy = __fadd2_rn(make_float2(q.y, q.y), ny);
+    const float2 dz = __fadd2_rn(make_float2(q.z, q.z), nz);
+    float2 r2 = __ffma2_rn(dx, dx, e2);
+    r2 = __ffma2_rn(dy, dy, r2);
+    r2 = __ffma2_rn(dz, dz, r2);
+    float2 inv;
+    inv.x = rsqrt_ftz(r2.x);
+    inv.y = rsqrt_ftz(r2.y);
+    ph = __fadd2_rn(ph, inv);
+    const float2 i2 = __fmul2_rn(inv, inv);
+    const float2 s = __fmul2_rn(inv, i2);
+    if (kScalarA) {
+        asm("fma.rn.f32 %0, %1, %2, %0;" : "+f"(ax.x) : "f"(s.x), "f"(dx.x));
+        asm("fma.rn.f32 %0, %1, %2, %0;" : "+f"(ax.y) : "f"(s.y), "f"(dx.y));
+        asm("fma.rn.f32 %0, %1, %2, %0;" : "+f"(ay.x) : "f"(s.x), "f"(dy.x));
+        asm("fma.rn.f32 %0, %1, %2, %0;" : "+f"(ay.y) : "f"(s.y), "f"(dy.y));
+        asm("fma.rn.f32 %0, %1, %2, %0;" : "+f"(az.x) : "f"(s.x), "f"(dz.x));
+        asm("fma.rn.f32 %0, %1, %2, %0;" : "+f"(az.y) : "f"(s.y), "f"(dz.y));
+    } else {
+        ax = __ffma2_rn(s, dx, ax);
+        ay = __ffma2_rn(s, dy, ay);
+        az = __ffma2_rn(s, dz, az);
+    }
+}
+// Variant 7: general masses, scalar a-updates
+__device__ __forceinline__ void interact2_sa(const float4 q, const float2 nx, const float2 ny, const float2 nz,
+                                             const float2 e2, float2 &ax, float2 &ay, float2 &az, float2 &ph) {
+    const float2 dx = __fadd2_rn(make_float2(q.x, q.x), nx);
+    const float2 dy = __fadd2_rn(make_float2(q.y, q.y), ny);
+    const float2 dz = __fadd2_rn(make_float2(q.z, q.z), nz);
+    float2 r2 = __ffma2_rn(dx, dx, e2);
+    r2 = __ffma2_rn(dy, dy, r2);
+    r2 = __ffma2_rn(dz, dz, r2);
+    float2 inv;
+    inv.x = rsqrt_ftz(r2.x);
+    inv.y = rsqrt_ftz(r2.y);
+    const float2 t = __fmul2_rn(make_float2(q.w, q.w), inv);
+    ph = __fadd2_rn(ph, t);
+    const float2 i2 = __fmul2_rn(inv, inv);
+    const float2 s = __fmul2_rn(t, i2);
+    asm("fma.rn.f32 %0, %1, %2, %0;" : "+f"(ax.x) : "f"(s.x), "f"(dx.x));
+    asm("fma.rn.f32 %0, %1, %2, %0;" : "+f"(ax.y) : "f"(s.y), "f"(dx.y));
+    asm("fma.rn.f32 %0, %1, %2, %0;" : "+f"(ay.x) : "f"(s.x), "f"(dy.x));
+    asm("fma.rn.f32 %0, %1, %2, %0;" : "+f"(ay.y) : "f"(s.y), "f"(dy.y));
+    asm("fma.rn.f32 %0, %1, %2, %0;" : "+f"(az.x) : "f"(s.x), "f"(dz.x));
+    asm("fma.rn.f32 %0, %1, %2, %0;" : "+f"(az.y) : "f"(s.y), "f"(dz.y));
+}
+
 template <int kWarpsT, int kU, bool kFoldOn, int kVar>
 __global__ void __launch_bounds__(32 * kWarpsT, 1) loop_kernel(const float4 *__restrict__ g, int reps, float eps2,
                                                               float *out) {
@@ -117,6 +172,12 @@ __global__ void __launch_bounds__(32 * kWarpsT, 1) loop_kernel(const float4 *__r
                         interact2_blk(s[k], nx[q], ny[q], nz[q], e2, ux, uy, uz, ph[q]);
                         ax[q] = u2f(ux); ay[q] = u2f(uy); az[q] = u2f(uz);
                     }
+                    else if (kVar == 5)
+                        interact2_eq<false>(s[k], nx[q], ny[q], nz[q], e2, ax[q], ay[q], az[q], ph[q]);
+                    else if (kVar == 6)
+                        interact2_eq<true>(s[k], nx[q], ny[q], nz[q], e2, ax[q], ay[q], az[q], ph[q]);
+                    else if (kVar == 7)
+                        interact2_sa(s[k], nx[q], ny[q], nz[q], e2, ax[q], ay[q], az[q], ph[q]);
                     else if (kVar == 1 || kVar == 3)
                         interact2_rcp(s[k], nx[q], ny[q], nz[q], e2, ax[q], ay[q], az[q], ph[q]);
                     else {
@@ -182,6 +243,11 @@ int main() {
     }
     cudaMemcpy(g, h, sizeof(h), cudaMemcpyHostToDevice);
     run<12, 4, true>(g, out, sms, "product-like");
+    run<12, 4, true, 7>(g, out, sms, "scalar a-updates");
+    run<12, 4, true, 5>(g, out, sms, "equal mass");
+    run<12, 4, true, 6>(g, out, sms, "equal mass, scalar a");
+    run<16, 4, true, 6>(g, out, sms, "equal mass, scalar a");
+    run<12, 8, true, 6>(g, out, sms, "equal mass, scalar a");
     run<12, 4, false>(g, out, sms, "no fold");
     run<8, 4, true>(g, out, sms, "8 warps");
     run<16, 4, true>(g, out, sms, "16 warps");
