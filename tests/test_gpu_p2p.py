@@ -404,6 +404,47 @@ def test_eval_host_pipelined_bit_identical(world, pieces, ingest, zc, monkeypatc
     tree.close()
 
 
+@pytest.mark.parametrize("offset,n", [(0, 199997), (1, 200000), (3, 99999)])
+def test_eval_host_pipelined_zero_copy_ragged_and_misaligned(offset, n, monkeypatch):
+    """Zero-copy streamed inputs with chunk lengths not a multiple of 4 and host
+    arrays that are not 16-byte aligned (views at an element offset into pinned
+    buffers): the pack kernel's float4 path, its scalar tail and its scalar
+    fallback all give results bit-identical to afmm_p2p_eval on device buffers."""
+    monkeypatch.setenv("AFMM_E2E_ZEROCOPY", "1")
+    afmm = _afmm()
+    x, y, z, m = synth.make("plummer", n, 24)
+    tree = afmm.GpuTree(0)
+    X, Y, Z, M = (torch.from_numpy(v).cuda() for v in (x, y, z, m))
+    tree.build(X, Y, Z, 64)
+    T = tree.copy_out(n)
+    bod = torch.empty((4, n), device="cuda")
+    for a, src in enumerate((X, Y, Z, M)):
+        tree.gather(src, bod[a])
+    hb = []
+    for a in range(4):
+        buf = torch.empty(n + offset).pin_memory()
+        buf[offset:].copy_(bod[a].cpu())
+        hb.append(buf[offset:])
+    got = []
+    for a in range(4):
+        buf = torch.full((n + offset,), float("nan")).pin_memory()
+        got.append(buf[offset:])
+    ref = torch.full((4, n), float("nan"), device="cuda")
+    h = afmm.P2P(eps2=1e-6)
+    h.set_bodies(bod[0], bod[1], bod[2], bod[3])
+    h.set_tree(T["leaf_start"], T["leaf_count"], T["u_off"], T["u_idx"])
+    h.eval(ref[0], ref[1], ref[2], ref[3])
+    h.set_bodies(*[torch.zeros(n, device="cuda") for _ in range(4)])   # stale device bodies
+    st = h.eval_host_pipelined(*hb, *got, pieces=1)
+    assert st["zero_copy"] == 1
+    h.close()
+    tree.close()
+    r_ = ref.cpu().numpy()
+    assert np.isfinite(r_).all()
+    for a in range(4):
+        assert np.array_equal(got[a].numpy(), r_[a])
+
+
 @pytest.mark.parametrize("zc", ["0", "1"])
 def test_eval_host_pipelined_equal_masses(zc, monkeypatch):
     """Equal masses: the streamed chunks are flagged equal-mass, so
