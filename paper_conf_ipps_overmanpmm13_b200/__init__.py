@@ -52,7 +52,8 @@ class Stats(C.Structure):
                 ("interactions_rank", C.c_longlong), ("leaf_lo", C.c_longlong),
                 ("leaf_hi", C.c_longlong), ("body_lo", C.c_longlong), ("body_hi", C.c_longlong),
                 ("n_work_items", C.c_int), ("n_launches", C.c_int),
-                ("bucket_interactions", C.c_longlong * N_BUCKETS), ("zero_copy", C.c_int)]
+                ("bucket_interactions", C.c_longlong * N_BUCKETS), ("zero_copy", C.c_int),
+                ("input_graph", C.c_int)]
 
     def as_dict(self):
         d = {f: getattr(self, f) for f, _ in self._fields_ if f != "bucket_interactions"}

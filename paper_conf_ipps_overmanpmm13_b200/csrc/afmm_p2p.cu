@@ -79,6 +79,7 @@ struct afmm_p2p {
     long long n_evals = 0;
     bool evaluated = false;
     bool last_zero_copy = false;                     // last eval_host_pipelined ran zero-copy
+    bool last_input_graph = false;                   // ... and replayed its input chain from a graph
     afmm_p2p_stats last{};
 
     // pipelined host evaluation (afmm_p2p_eval_host_pipelined): the rank's tasks
@@ -95,6 +96,15 @@ struct afmm_p2p {
     void *wait_value32 = nullptr;                    // cuStreamWaitValue32 (driver entry point)
     void *write_value32 = nullptr;                   // cuStreamWriteValue32 (driver entry point)
     cudaEvent_t ev_start = nullptr, ev_in[64] = {}, ev_k[64] = {}, ev_done = nullptr;
+    // zero-copy input chain (K pack launches + K stream writes) captured once as a
+    // CUDA graph and replayed with one launch; re-captured when its key changes
+    cudaGraphExec_t in_graph = nullptr;
+    bool in_graph_off = false;                       // capture unsupported: direct launches
+    const float *ig_src[4] = {nullptr, nullptr, nullptr, nullptr};
+    long long ig_n = 0;
+    int ig_K = 0;
+    unsigned ig_m0 = 0;
+    const void *ig_bodies = nullptr;
 
     // peer output windows (fused gather, afmm_p2p_set_peer_windows)
     int n_peers = 0;
@@ -314,6 +324,7 @@ extern "C" void afmm_p2p_destroy(afmm_p2p *h) {
     cudaFree(h->d_ptasks);
     cudaFree(h->d_pqueue);
     if (h->s_in) cudaStreamSynchronize(h->s_in), cudaStreamDestroy(h->s_in);
+    if (h->in_graph) cudaGraphExecDestroy(h->in_graph);
     if (h->s_out) cudaStreamSynchronize(h->s_out), cudaStreamDestroy(h->s_out);
 
     for (int i = 0; i < 64; ++i) {
@@ -912,6 +923,7 @@ static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, flo
     p.mass_bits = nullptr;
     p.out_coalesce = 0;
     h->last_zero_copy = false;
+    h->last_input_graph = false;
     CUDA_TRY(h, cudaMemsetAsync(h->d_queue, 0, sizeof(int), h->stream));
     const int ri = (int)(h->n_evals % afmm_p2p::kRing);
     h->ev0 = h->ring0[ri];
@@ -951,6 +963,7 @@ static afmm_status fill_stats(afmm_p2p *h, afmm_p2p_stats *s) {
     o.n_work_items = h->n_tasks;
     o.n_launches = h->last.n_launches;
     o.zero_copy = h->last_zero_copy ? 1 : 0;
+    o.input_graph = h->last_input_graph ? 1 : 0;
     for (int b = 0; b < 8; ++b) o.bucket_interactions[b] = h->bucket_inter[b];
     h->last = o;
     if (s) *s = o;
@@ -1239,27 +1252,82 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
     };
     const int K = h->pipe_K;
     const long long chunk = (n + K - 1) / K;
-    for (int k = 0; k < K; ++k) {
-        const long long lo = k * chunk, hi = std::min<long long>(n, lo + chunk);
-        if (hi > lo) {
-            const float *src[4];
-            for (int a = 0; a < 4; ++a) {
-                if (zc_in) {
-                    src[a] = zin[a] + lo;
-                } else {
-                    CUDA_TRY(h, cudaMemcpyAsync(dsoa[a] + lo, hin[a] + lo, (size_t)(hi - lo) * sizeof(float),
-                                                cudaMemcpyHostToDevice, h->s_in));
-                    src[a] = dsoa[a] + lo;
+    // Enqueue the input chain: pack chunk k, then publish k + 1 (stream write).
+    auto enqueue_inputs = [&](bool capturing) -> afmm_status {
+        for (int k = 0; k < K; ++k) {
+            const long long lo = k * chunk, hi = std::min<long long>(n, lo + chunk);
+            if (hi > lo) {
+                const float *src[4];
+                for (int a = 0; a < 4; ++a) {
+                    if (zc_in) {
+                        src[a] = zin[a] + lo;
+                    } else {
+                        CUDA_TRY(h, cudaMemcpyAsync(dsoa[a] + lo, hin[a] + lo, (size_t)(hi - lo) * sizeof(float),
+                                                    cudaMemcpyHostToDevice, h->s_in));
+                        src[a] = dsoa[a] + lo;
+                    }
+                }
+                const int threads = 128;
+                const int blocks = (int)std::min<long long>((hi - lo + threads - 1) / threads, (long long)h->num_sms);
+                afmm::pack_chunk_kernel<<<blocks, threads, 0, h->s_in>>>((int)(hi - lo), src[0], src[1], src[2],
+                                                                        src[3], h->d_bodies + lo, m0, mass_bits, k);
+                const cudaError_t le = cudaPeekAtLastError();
+                if (le != cudaSuccess) {
+                    if (capturing) return AFMM_ECUDA;
+                    (void)cudaGetLastError();
+                    return fail(h, AFMM_ECUDA, "eval_host_pipelined: pack launch failed: %s", cudaGetErrorString(le));
                 }
             }
-            const int threads = 128;
-            const int blocks = (int)std::min<long long>((hi - lo + threads - 1) / threads, (long long)h->num_sms);
-            afmm::pack_chunk_kernel<<<blocks, threads, 0, h->s_in>>>((int)(hi - lo), src[0], src[1], src[2], src[3],
-                                                                    h->d_bodies + lo, m0, mass_bits, k);
-            CUDA_TRY(h, cudaGetLastError());
+            const CUresult r = write32((CUstream)h->s_in, (CUdeviceptr)in_ready, (cuuint32_t)(k + 1), 0);
+            if (r != CUDA_SUCCESS) {
+                if (capturing) return AFMM_ECUDA;
+                return fail(h, AFMM_ECUDA, "eval_host_pipelined: cuStreamWriteValue32 failed (%d)", (int)r);
+            }
         }
-        const CUresult r = write32((CUstream)h->s_in, (CUdeviceptr)in_ready, (cuuint32_t)(k + 1), 0);
-        if (r != CUDA_SUCCESS) return fail(h, AFMM_ECUDA, "eval_host_pipelined: cuStreamWriteValue32 failed (%d)", (int)r);
+        return AFMM_OK;
+    };
+    // Zero-copy: the chain is the same on every call with the same arrays, so it is
+    // captured once into a graph and replayed by one launch (2K host API calls fewer
+    // before the P2P launch).  AFMM_INPUT_GRAPH=0, or a failed capture: direct launches.
+    const char *genv = getenv("AFMM_INPUT_GRAPH");
+    bool use_graph = zc_in && !h->in_graph_off && !(genv && genv[0] == '0');
+    if (use_graph) {
+        unsigned m0bits;
+        std::memcpy(&m0bits, &m0, sizeof m0bits);
+        const bool same = h->in_graph && h->ig_n == n && h->ig_K == K && h->ig_m0 == m0bits &&
+                          h->ig_bodies == h->d_bodies && h->ig_src[0] == zin[0] && h->ig_src[1] == zin[1] &&
+                          h->ig_src[2] == zin[2] && h->ig_src[3] == zin[3];
+        if (!same) {
+            if (h->in_graph) cudaGraphExecDestroy(h->in_graph);
+            h->in_graph = nullptr;
+            cudaGraph_t g = nullptr;
+            bool ok = cudaStreamBeginCapture(h->s_in, cudaStreamCaptureModeThreadLocal) == cudaSuccess;
+            if (ok) {
+                const afmm_status es = enqueue_inputs(true);
+                const cudaError_t ee = cudaStreamEndCapture(h->s_in, &g);
+                ok = es == AFMM_OK && ee == cudaSuccess && g != nullptr;
+            }
+            if (ok) ok = cudaGraphInstantiate(&h->in_graph, g, 0) == cudaSuccess;
+            if (g) cudaGraphDestroy(g);
+            if (!ok) {
+                (void)cudaGetLastError();
+                if (h->in_graph) cudaGraphExecDestroy(h->in_graph);
+                h->in_graph = nullptr;
+                h->in_graph_off = true;                  // do not try again on this handle
+                use_graph = false;
+            } else {
+                h->ig_n = n;
+                h->ig_K = K;
+                h->ig_m0 = m0bits;
+                h->ig_bodies = h->d_bodies;
+                for (int a = 0; a < 4; ++a) h->ig_src[a] = zin[a];
+            }
+        }
+        if (use_graph) CUDA_TRY(h, cudaGraphLaunch(h->in_graph, h->s_in));
+    }
+    h->last_input_graph = use_graph;
+    if (!use_graph) {
+        if ((st = enqueue_inputs(false))) return st;
     }
     if ((st = launch())) return st;
     // the launch must be enqueued before the copy-out stream starts waiting on its counters

@@ -393,6 +393,7 @@ def test_eval_host_pipelined_bit_identical(world, pieces, ingest, zc, monkeypatc
             st = h.eval_host_pipelined(*hb, *got, pieces=pieces)
         assert st["n_launches"] <= pieces and st["n_launches"] >= 1
         assert st["zero_copy"] == int(zc)
+        assert st["input_graph"] == int(zc)            # zero-copy inputs: the chain replays from a graph
         h.eval(again[0], again[1], again[2], again[3])
         h.close()
     torch.cuda.synchronize()
@@ -436,7 +437,15 @@ def test_eval_host_pipelined_zero_copy_ragged_and_misaligned(offset, n, monkeypa
     h.eval(ref[0], ref[1], ref[2], ref[3])
     h.set_bodies(*[torch.zeros(n, device="cuda") for _ in range(4)])   # stale device bodies
     st = h.eval_host_pipelined(*hb, *got, pieces=1)
-    assert st["zero_copy"] == 1
+    assert st["zero_copy"] == 1 and st["input_graph"] == 1
+    for a in range(4):
+        assert np.array_equal(got[a].numpy(), ref[a].cpu().numpy())
+    # a changed host array (new pointer) re-captures the input chain; same results
+    hb[0] = hb[0].clone().pin_memory()
+    for a in range(4):
+        got[a].fill_(float("nan"))
+    st = h.eval_host_pipelined(*hb, *got, pieces=1)
+    assert st["input_graph"] == 1
     h.close()
     tree.close()
     r_ = ref.cpu().numpy()
