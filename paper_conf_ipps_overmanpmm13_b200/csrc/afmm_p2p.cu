@@ -98,6 +98,7 @@ struct afmm_p2p {
     cudaEvent_t ev_start = nullptr, ev_in[64] = {}, ev_k[64] = {}, ev_done = nullptr;
     // zero-copy input chain (K pack launches + K stream writes) captured once as a
     // CUDA graph and replayed with one launch; re-captured when its key changes
+    int *h_err = nullptr;                            // pinned: the input-wait timeout flag after an eval
     cudaGraphExec_t in_graph = nullptr;
     bool in_graph_off = false;                       // capture unsupported: direct launches
     const float *ig_src[4] = {nullptr, nullptr, nullptr, nullptr};
@@ -325,6 +326,7 @@ extern "C" void afmm_p2p_destroy(afmm_p2p *h) {
     cudaFree(h->d_pqueue);
     if (h->s_in) cudaStreamSynchronize(h->s_in), cudaStreamDestroy(h->s_in);
     if (h->in_graph) cudaGraphExecDestroy(h->in_graph);
+    if (h->h_err) cudaFreeHost(h->h_err);
     if (h->s_out) cudaStreamSynchronize(h->s_out), cudaStreamDestroy(h->s_out);
 
     for (int i = 0; i < 64; ++i) {
@@ -1141,6 +1143,7 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
             CUDA_TRY(h, cudaEventCreateWithFlags(&h->ev_k[i], cudaEventDisableTiming));
         }
         CUDA_TRY(h, cudaMalloc(&h->d_pqueue, (kMaxPieces + 4) * sizeof(int)));
+        CUDA_TRY(h, cudaMallocHost(&h->h_err, sizeof(int)));
         cudaDriverEntryPointQueryResult q;
         CUDA_TRY(h, cudaGetDriverEntryPoint("cuStreamWaitValue32", &h->wait_value32, cudaEnableDefault, &q));
         if (q != cudaDriverEntryPointSuccess || !h->wait_value32)
@@ -1348,10 +1351,12 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
     h->n_evals++;
     h->evaluated = true;
     h->last.n_launches = nlaunch;
+    // the wait-timeout flag rides on the stream into pinned memory: fill_stats'
+    // synchronise covers it (no separate blocking copy)
+    *h->h_err = 0;
+    CUDA_TRY(h, cudaMemcpyAsync(h->h_err, in_err, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
     if ((st = fill_stats(h, stats))) return st;
-    int herr = 0;
-    CUDA_TRY(h, cudaMemcpy(&herr, in_err, sizeof(int), cudaMemcpyDeviceToHost));
-    if (herr) return fail(h, AFMM_ECUDA, "eval_host_pipelined: input chunks never arrived (kernel wait timed out)");
+    if (*(volatile int *)h->h_err) return fail(h, AFMM_ECUDA, "eval_host_pipelined: input chunks never arrived (kernel wait timed out)");
     return AFMM_OK;
 }
 
