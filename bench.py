@@ -333,12 +333,13 @@ def main():
     ho = [torch.empty(n, dtype=torch.float32).pin_memory() for _ in range(4)]
     Ke = max(3, K // 2)
 
-    e2e_mode = {"zero_copy": 0}
+    e2e_mode = {"zero_copy": 0, "input_graph": 0}
 
     def step_e2e():
         if world == 1:
             # afmm_p2p_eval_host_pipelined: H2D + pack, kernel pieces, D2H overlapped; blocking
-            e2e_mode["zero_copy"] = h.eval_host_pipelined(*hx, *ho, pieces=E2E_PIECES)["zero_copy"]
+            st_ = h.eval_host_pipelined(*hx, *ho, pieces=E2E_PIECES)
+            e2e_mode["zero_copy"], e2e_mode["input_graph"] = st_["zero_copy"], st_["input_graph"]
         else:
             if rank == 0:
                 for a in range(4):
@@ -505,7 +506,9 @@ def main():
             "e2e": {"value": e2e_value, "unit": "interactions/s", "h2d_bytes_per_step": 16 * n,
                     "d2h_bytes_per_step": 16 * n, "steps": Ke,
                     "path": (("afmm_p2p_eval_host_pipelined, zero-copy: 8 input chunks packed from the pinned host "
-                              "arrays over PCIe while the kernel runs, outputs written to the pinned host arrays by "
+                              "arrays over PCIe while the kernel runs" +
+                              (" (the pack chain replayed from a captured CUDA graph)" if e2e_mode["input_graph"] else "") +
+                              ", outputs written to the pinned host arrays by "
                               "the kernel's task epilogue") if e2e_mode["zero_copy"] else
                              f"afmm_p2p_eval_host_pipelined (8 streamed input chunks, {E2E_PIECES} output pieces) "
                              "from pinned host arrays") if world == 1
