@@ -71,3 +71,31 @@ def test_interactions_rejects_bad_index():
     import paper_conf_ipps_overmanpmm13_b200 as afmm
     with pytest.raises(afmm.AfmmError):
         afmm.interactions(np.array([1, 1]), np.array([0, 1, 2]), np.array([0, 2]))
+
+
+def test_ctypes_structs_match_the_c_headers(tmp_path):
+    """Every ctypes mirror of a header struct has the C layout: the same size and
+    the same offset for every field (compiled with gcc against include/*.h), so a
+    field added on one side only fails here rather than corrupting calls."""
+    import paper_conf_ipps_overmanpmm13_b200 as afmm
+    pairs = [("afmm_p2p_config", afmm.Config), ("afmm_p2p_stats", afmm.Stats), ("afmm_ipc_handle", afmm.IpcHandle),
+             ("afmm_lb_config", afmm.LbConfig), ("afmm_fg_result", afmm.FgResult)]
+    lines = ['#include <stdio.h>', '#include <stddef.h>', '#include "afmm_balance.h"', "int main(void) {"]
+    for cname, py in pairs:
+        lines.append(f'printf("{cname} size %zu\\n", sizeof({cname}));')
+        for f, _ in py._fields_:
+            lines.append(f'printf("{cname} {f} %zu\\n", offsetof({cname}, {f}));')
+    lines += ["return 0;", "}"]
+    src = tmp_path / "layout.c"
+    src.write_text("\n".join(lines))
+    exe = tmp_path / "layout"
+    import subprocess
+    subprocess.check_call(["gcc", "-std=c11", "-I", os.path.join(ROOT, "include"), str(src), "-o", str(exe)])
+    got = {}
+    for ln in subprocess.check_output([str(exe)], text=True).splitlines():
+        a, b, v = ln.split()
+        got[(a, b)] = int(v)
+    for cname, py in pairs:
+        assert got[(cname, "size")] == ctypes.sizeof(py), cname
+        for f, _ in py._fields_:
+            assert got[(cname, f)] == getattr(py, f).offset, (cname, f)
