@@ -99,6 +99,7 @@ struct afmm_p2p {
     // zero-copy input chain (K pack launches + K stream writes) captured once as a
     // CUDA graph and replayed with one launch; re-captured when its key changes
     int *h_err = nullptr;                            // pinned: the input-wait timeout flag after an eval
+    int *h_ingest_err = nullptr;                     // pinned: set_tree_device's validation flags
     cudaGraphExec_t in_graph = nullptr;
     bool in_graph_off = false;                       // capture unsupported: direct launches
     const float *ig_src[4] = {nullptr, nullptr, nullptr, nullptr};
@@ -327,6 +328,7 @@ extern "C" void afmm_p2p_destroy(afmm_p2p *h) {
     if (h->s_in) cudaStreamSynchronize(h->s_in), cudaStreamDestroy(h->s_in);
     if (h->in_graph) cudaGraphExecDestroy(h->in_graph);
     if (h->h_err) cudaFreeHost(h->h_err);
+    if (h->h_ingest_err) cudaFreeHost(h->h_ingest_err);
     if (h->s_out) cudaStreamSynchronize(h->s_out), cudaStreamDestroy(h->s_out);
 
     for (int i = 0; i < 64; ++i) {
@@ -586,12 +588,13 @@ extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const
     dev::validate_interactions_kernel<<<grid(L), TH, 0, s>>>(L, h->n, h->cfg.max_leaf, leaf_start, leaf_count,
                                                             u_off, u_idx, I, err);
     CUDA_TRY(h, cudaGetLastError());
-    int herr = 0;
-    CUDA_TRY(h, cudaMemcpyAsync(&herr, err, sizeof(int), cudaMemcpyDeviceToHost, s));
-    CUDA_TRY(h, cudaStreamSynchronize(s));
-    if (herr)
-        return fail(h, AFMM_EINVAL, "set_tree_device: invalid tree (flags 0x%x: 1 start, 2 count, 4 cover, "
-                                    "8 u_off, 16 u_idx range, 32 row order)", herr);
+    // the flags ride with the partition's results (one synchronise instead of two): the
+    // partition kernels only touch L- and W-sized arrays, and nothing of the handle's
+    // state changes before the flags are checked
+    if (!h->h_ingest_err) CUDA_TRY(h, cudaMallocHost(&h->h_ingest_err, sizeof(int)));   // pinned: an async copy
+    *h->h_ingest_err = 0;
+    CUDA_TRY(h, cudaMemcpyAsync(h->h_ingest_err, err, sizeof(int), cudaMemcpyDeviceToHost, s));
+    bool clear_user = false;                        // applied once the tree is known valid
     // 2. partition (literal rule, or the per-bucket coefficients of the last step)
     {
         size_t tb = 0;
@@ -614,19 +617,27 @@ extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const
         if ((st = dws(h, sTmp, &tmp, tb))) return st;
         CUDA_TRY(h, cub::DeviceScan::InclusiveSum(tmp, tb, w, pw, L, s));
         dev::weighted_cut_kernel<<<1, 1, 0, s>>>(L, W, pw, split);
-        h->user_partition = false;
+        clear_user = true;
     } else {
         dev::literal_cut_kernel<<<1, 1, 0, s>>>(L, W, P, split);
-        h->user_partition = false;
+        clear_user = true;
     }
     CUDA_TRY(h, cudaGetLastError());
     body_split_kernel<<<1, 64, 0, s>>>(W, L, h->n, split, leaf_start, bsplit);
-    h->leaf_split.assign(W + 1, 0);
-    h->body_split.assign(W + 1, 0);
-    CUDA_TRY(h, cudaMemcpyAsync(h->leaf_split.data(), split, (W + 1) * sizeof(long long), cudaMemcpyDeviceToHost, s));
-    CUDA_TRY(h, cudaMemcpyAsync(h->body_split.data(), bsplit, (W + 1) * sizeof(long long), cudaMemcpyDeviceToHost, s));
-    CUDA_TRY(h, cudaMemcpyAsync(&h->I_total, P + (L - 1), sizeof(long long), cudaMemcpyDeviceToHost, s));
+    std::vector<long long> lsplit(W + 1, 0), bsplit_h(W + 1, 0);
+    long long itot = 0;
+    CUDA_TRY(h, cudaMemcpyAsync(lsplit.data(), split, (W + 1) * sizeof(long long), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(h, cudaMemcpyAsync(bsplit_h.data(), bsplit, (W + 1) * sizeof(long long), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(h, cudaMemcpyAsync(&itot, P + (L - 1), sizeof(long long), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(h, cudaStreamSynchronize(s));
+    const int herr = *(volatile int *)h->h_ingest_err;
+    if (herr)
+        return fail(h, AFMM_EINVAL, "set_tree_device: invalid tree (flags 0x%x: 1 start, 2 count, 4 cover, "
+                                    "8 u_off, 16 u_idx range, 32 row order)", herr);
+    if (clear_user) h->user_partition = false;
+    h->leaf_split = std::move(lsplit);
+    h->body_split = std::move(bsplit_h);
+    h->I_total = itot;
     // 3. this rank's work list
     const int r = h->cfg.rank;
     const long long cap = afmm::task_cap(h->I_total / slice_world(h), (long long)h->num_sms * h->blocks_per_sm * afmm::kWarps);
