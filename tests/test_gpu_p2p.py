@@ -405,13 +405,17 @@ def test_eval_host_pipelined_bit_identical(world, pieces, ingest, zc, monkeypatc
     tree.close()
 
 
-@pytest.mark.parametrize("offset,n", [(0, 199997), (1, 200000), (3, 99999)])
-def test_eval_host_pipelined_zero_copy_ragged_and_misaligned(offset, n, monkeypatch):
+@pytest.mark.parametrize("offset,n,graph", [(0, 199997, "1"), (1, 200000, "1"), (3, 99999, "1"), (0, 200000, "0"),
+                                           (1, 99999, "0")])
+def test_eval_host_pipelined_zero_copy_ragged_and_misaligned(offset, n, graph, monkeypatch):
     """Zero-copy streamed inputs with chunk lengths not a multiple of 4 and host
     arrays that are not 16-byte aligned (views at an element offset into pinned
     buffers): the pack kernel's float4 path, its scalar tail and its scalar
-    fallback all give results bit-identical to afmm_p2p_eval on device buffers."""
+    fallback all give results bit-identical to afmm_p2p_eval on device buffers,
+    with the input chain replayed from its captured graph (graph = "1") or
+    launched directly (AFMM_INPUT_GRAPH=0)."""
     monkeypatch.setenv("AFMM_E2E_ZEROCOPY", "1")
+    monkeypatch.setenv("AFMM_INPUT_GRAPH", graph)
     afmm = _afmm()
     x, y, z, m = synth.make("plummer", n, 24)
     tree = afmm.GpuTree(0)
@@ -437,7 +441,7 @@ def test_eval_host_pipelined_zero_copy_ragged_and_misaligned(offset, n, monkeypa
     h.eval(ref[0], ref[1], ref[2], ref[3])
     h.set_bodies(*[torch.zeros(n, device="cuda") for _ in range(4)])   # stale device bodies
     st = h.eval_host_pipelined(*hb, *got, pieces=1)
-    assert st["zero_copy"] == 1 and st["input_graph"] == 1
+    assert st["zero_copy"] == 1 and st["input_graph"] == int(graph)
     for a in range(4):
         assert np.array_equal(got[a].numpy(), ref[a].cpu().numpy())
     # a changed host array (new pointer) re-captures the input chain; same results
@@ -445,7 +449,7 @@ def test_eval_host_pipelined_zero_copy_ragged_and_misaligned(offset, n, monkeypa
     for a in range(4):
         got[a].fill_(float("nan"))
     st = h.eval_host_pipelined(*hb, *got, pieces=1)
-    assert st["input_graph"] == 1
+    assert st["input_graph"] == int(graph)
     h.close()
     tree.close()
     r_ = ref.cpu().numpy()
