@@ -43,7 +43,11 @@ h1.set_tree(T["leaf_start"], T["leaf_count"], T["u_off"], T["u_idx"])
 h1.eval(out[0], out[1], out[2], out[3])
 hx = [b[a].cpu().pin_memory() for a in range(4)]
 ho = [torch.empty(n).pin_memory() for _ in range(4)]
-h1.eval_host_pipelined(*hx, *ho, pieces=3)
+h1.eval_host_pipelined(*hx, *ho, pieces=3)                 # zero-copy, input chain from its graph
+os.environ["AFMM_INPUT_GRAPH"] = "0"
+h1.eval_host_pipelined(*hx, *ho, pieces=3)                 # zero-copy, direct launches
+os.environ["AFMM_E2E_ZEROCOPY"] = "0"
+h1.eval_host_pipelined(*hx, *ho, pieces=3)                 # staged copies + per-piece copy-back
 fx, fy, fz = (torch.from_numpy(np.ascontiguousarray(v)).to(dev) for v in synth.uniform_with_forces(n, 4)[3:])
 hs = afmm.P2P(eps2=1e-6, law=afmm.LAW_STOKESLET)
 hs.set_bodies_stokeslet(b[0], b[1], b[2], fx, fy, fz)
