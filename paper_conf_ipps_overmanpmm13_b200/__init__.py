@@ -41,7 +41,7 @@ class AfmmError(RuntimeError):
 class Config(C.Structure):
     _fields_ = [("device", C.c_int), ("rank", C.c_int), ("world", C.c_int), ("G", C.c_float),
                 ("eps2", C.c_float), ("max_leaf", C.c_int), ("stream", C.c_void_p), ("law", C.c_int),
-                ("mu", C.c_float), ("slice_world", C.c_int)]
+                ("mu", C.c_float), ("slice_world", C.c_int), ("nccl_id", C.c_void_p), ("comm_sms", C.c_int)]
 
 
 LAW_GRAVITY, LAW_STOKESLET = 0, 1
@@ -53,7 +53,8 @@ class Stats(C.Structure):
                 ("leaf_hi", C.c_longlong), ("body_lo", C.c_longlong), ("body_hi", C.c_longlong),
                 ("n_work_items", C.c_int), ("n_launches", C.c_int),
                 ("bucket_interactions", C.c_longlong * N_BUCKETS), ("zero_copy", C.c_int),
-                ("input_graph", C.c_int)]
+                ("input_graph", C.c_int), ("streamed_inputs", C.c_int), ("chunked_bodies", C.c_int),
+                ("kernel_ms_max", C.c_double)]
 
     def as_dict(self):
         d = {f: getattr(self, f) for f, _ in self._fields_ if f != "bucket_interactions"}
@@ -88,6 +89,10 @@ _sig("afmm_p2p_eval_host", _i, _p, _p, _p, _p, _p, C.POINTER(Stats))
 _sig("afmm_p2p_eval_host_pipelined", _i, _p, _ll, _p, _p, _p, _p, _p, _p, _p, _p, _i, C.POINTER(Stats))
 _sig("afmm_p2p_stats_get", _i, _p, C.POINTER(Stats))
 _sig("afmm_p2p_set_peer_windows", _i, _p, _i, _p)
+_sig("afmm_p2p_nccl_id", _i, _p)
+_sig("afmm_p2p_chunks", _i, _p, C.POINTER(_i), _p, _p)
+_sig("afmm_p2p_eval_chunked", _i, _p, _p, _p, _p, _p)
+_sig("afmm_p2p_publish_chunks", _i, _p, _i, _p)
 
 
 class IpcHandle(C.Structure):
@@ -169,7 +174,8 @@ EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
             "afmm_tree_gather", "afmm_tree_scatter", "afmm_tree_destroy", "afmm_tree_last_error",
             "afmm_tree_rebuild", "afmm_tree_nodes", "afmm_fine_grained", "afmm_p2p_eval_host_pipelined",
             "afmm_p2p_set_peer_windows", "afmm_ipc_export", "afmm_ipc_import", "afmm_ipc_close",
-            "afmm_tree_gather_rows"]
+            "afmm_tree_gather_rows", "afmm_p2p_nccl_id", "afmm_p2p_chunks", "afmm_p2p_eval_chunked",
+            "afmm_p2p_publish_chunks"]
 
 
 def ipc_export(dev_ptr):
@@ -201,6 +207,15 @@ def ipc_close(base):
 
 def version() -> str:
     return _lib.afmm_version().decode()
+
+
+def nccl_id() -> bytes:
+    """afmm_p2p_nccl_id: a new 128-byte ncclUniqueId (rank 0) for P2P(nccl_id=...)."""
+    buf = C.create_string_buffer(128)
+    st = _lib.afmm_p2p_nccl_id(buf)
+    if st:
+        raise AfmmError(st, "afmm_p2p_nccl_id")
+    return buf.raw
 
 
 def _np(a, dt):
@@ -313,7 +328,7 @@ class P2P:
     """One afmm_p2p handle (one per rank / GPU)."""
 
     def __init__(self, device=0, rank=0, world=1, G=1.0, eps2=0.0, max_leaf=None, stream=None,
-                 law=LAW_GRAVITY, mu=1.0, slice_world=0):
+                 law=LAW_GRAVITY, mu=1.0, slice_world=0, nccl_id=None, comm_sms=0):
         cfg = Config()
         _lib.afmm_p2p_config_init(C.byref(cfg))
         cfg.device, cfg.rank, cfg.world = int(device), int(rank), int(world)
@@ -323,6 +338,13 @@ class P2P:
         cfg.stream = stream
         cfg.law, cfg.mu = int(law), float(mu)
         cfg.slice_world = int(slice_world)
+        idbuf = None
+        if nccl_id is not None:
+            if len(nccl_id) != 128:
+                raise ValueError("nccl_id must be the 128-byte id of afmm_p2p_nccl_id")
+            idbuf = C.create_string_buffer(bytes(nccl_id), 128)
+            cfg.nccl_id = C.cast(idbuf, C.c_void_p)
+        cfg.comm_sms = int(comm_sms)
         h = _p()
         st = _lib.afmm_p2p_create(C.byref(cfg), C.byref(h))
         if st:
@@ -460,6 +482,25 @@ class P2P:
         self._check(_lib.afmm_p2p_eval_host_pipelined(self._h, n, *[_ptr(a) for a in arrs], int(pieces), C.byref(s)),
                     "afmm_p2p_eval_host_pipelined")
         return s.as_dict()
+
+    def chunks(self):
+        """afmm_p2p_chunks: (bounds[K+1], order[K]) of the chunked body delivery."""
+        K = _i()
+        self._check(_lib.afmm_p2p_chunks(self._h, C.byref(K), None, None), "afmm_p2p_chunks")
+        b = np.empty(K.value + 1, np.int64)
+        o = np.empty(K.value, np.int32)
+        self._check(_lib.afmm_p2p_chunks(self._h, C.byref(K), _ptr(b), _ptr(o)), "afmm_p2p_chunks")
+        return b, o
+
+    def eval_chunked(self, ax, ay, az, phi):
+        """afmm_p2p_eval_chunked: launch before the bodies arrive (device outputs, async)."""
+        self._check(_lib.afmm_p2p_eval_chunked(self._h, _ptr(ax), _ptr(ay), _ptr(az), _ptr(phi)),
+                    "afmm_p2p_eval_chunked")
+
+    def publish_chunks(self, count, stream=None):
+        """afmm_p2p_publish_chunks: the first `count` chunks of the delivery order are in
+        place once `stream` (cudaStream_t int, None = the handle's stream) reaches this."""
+        self._check(_lib.afmm_p2p_publish_chunks(self._h, int(count), stream), "afmm_p2p_publish_chunks")
 
     def kernel_times(self, max_count=64):
         """Kernel ms of the last <= 64 evals (oldest first); synchronises."""

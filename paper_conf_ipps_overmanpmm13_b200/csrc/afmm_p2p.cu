@@ -20,6 +20,7 @@
 #include <cuda_runtime.h>
 
 #include "../../include/afmm_p2p.h"
+#include "nccl_api.h"
 #include "p2p_kernel.cuh"
 
 using afmm::Seg;
@@ -33,6 +34,7 @@ struct afmm_p2p {
     std::string err;
     int num_sms = 148;
     int blocks_per_sm = 1;
+    bool co_resident_pack = true;    // a pack_chunk_kernel block fits beside a streamed P2P CTA
 
     // bodies
     long long n = 0;
@@ -79,6 +81,7 @@ struct afmm_p2p {
     long long n_evals = 0;
     bool evaluated = false;
     bool last_zero_copy = false;                     // last eval_host_pipelined ran zero-copy
+    bool last_streamed = false;                      // ... and overlapped its input chain with the kernel
     bool last_input_graph = false;                   // ... and replayed its input chain from a graph
     afmm_p2p_stats last{};
 
@@ -95,7 +98,7 @@ struct afmm_p2p {
     cudaStream_t s_in = nullptr, s_out = nullptr;
     void *wait_value32 = nullptr;                    // cuStreamWaitValue32 (driver entry point)
     void *write_value32 = nullptr;                   // cuStreamWriteValue32 (driver entry point)
-    cudaEvent_t ev_start = nullptr, ev_in[64] = {}, ev_k[64] = {}, ev_done = nullptr;
+    cudaEvent_t ev_start = nullptr, ev_in[64] = {}, ev_k[64] = {}, ev_done = nullptr, ev_in_done = nullptr;
     // zero-copy input chain (K pack launches + K stream writes) captured once as a
     // CUDA graph and replayed with one launch; re-captured when its key changes
     int *h_err = nullptr;                            // pinned: the input-wait timeout flag after an eval
@@ -111,6 +114,25 @@ struct afmm_p2p {
     // peer output windows (fused gather, afmm_p2p_set_peer_windows)
     int n_peers = 0;
     float *peers[afmm::kMaxWin - 1][4] = {};
+
+    // library communicator (afmm_p2p_config.nccl_id) and the chunked replication
+    ncclComm_t comm = nullptr;
+    cudaStream_t s_comm = nullptr;                   // NCCL work + chunk publication
+    cudaEvent_t ev_c0 = nullptr, ev_c1 = nullptr, ev_c2 = nullptr, ev_c3 = nullptr;
+    bool bodies_pending = false;                     // set_bodies since the last eval: replicate in the next
+    bool last_chunked = false;
+    // device words: [0] chunk mask (epoch << 16 | mask), [1] wait-timeout flag, then
+    // tspan[2] (u64, %globaltimer), kernel_ms[2] (double: own span, max over ranks)
+    unsigned char *d_words = nullptr;
+    double *h_kms = nullptr;                         // pinned: kernel_ms max over ranks
+    int *h_cerr = nullptr;                           // pinned: the chunked eval's wait-timeout flag
+    unsigned epoch = 0;                              // chunked evals so far (16 bits in the flag word)
+    bool chunk_valid = false;                        // the plan below matches the work list
+    int chunk_K = 0;
+    std::vector<long long> chunk_bounds;             // K + 1 body offsets
+    std::vector<int> chunk_order;                    // delivery order (permutation of 0..K-1)
+    afmm::Task *d_ctasks = nullptr;                  // the work list in delivery order, need masks in piece
+    size_t ctasks_cap = 0;
 };
 
 namespace {
@@ -169,6 +191,43 @@ afmm_status ensure_device(afmm_p2p *h, T **ptr, size_t &cap, size_t count) {
 }
 
 int slice_world(const afmm_p2p *h) { return h->cfg.slice_world > 0 ? h->cfg.slice_world : h->cfg.world; }
+
+// Bound on one in-kernel wait for an input chunk (P2PParams.wait_ns):
+// AFMM_WAIT_MS (default 2000 ms) -- generous, it only matters when a producer died.
+unsigned long long wait_ns(const afmm_p2p *) {
+    static const unsigned long long ns = [] {
+        const char *e = getenv("AFMM_WAIT_MS");
+        const double ms = e ? atof(e) : 2000.0;
+        return (unsigned long long)((ms > 0 ? ms : 2000.0) * 1e6);
+    }();
+    return ns;
+}
+
+// Can one pack_chunk_kernel block (the streamed input chain) run on an SM that
+// holds a streamed P2P CTA?  From the built kernels' attributes: registers
+// (allocated per warp in units of 256), threads, shared memory (+ the per-block
+// reservation) and the block slots of one SM.  AFMM_PACK_CORESIDENT=0 forces "no"
+// (tests of the fallback).
+cudaError_t co_residency(int device, bool *ok) {
+    cudaFuncAttributes fp{}, fk{};
+    cudaError_t e = cudaFuncGetAttributes(&fp, afmm::p2p_kernel_t<afmm::Gravity, true>);
+    if (e == cudaSuccess) e = cudaFuncGetAttributes(&fk, afmm::pack_chunk_kernel);
+    int regs = 0, smem = 0, thr = 0, rsv = 0, blk = 0;
+    if (e == cudaSuccess) e = cudaDeviceGetAttribute(&regs, cudaDevAttrMaxRegistersPerMultiprocessor, device);
+    if (e == cudaSuccess) e = cudaDeviceGetAttribute(&smem, cudaDevAttrMaxSharedMemoryPerMultiprocessor, device);
+    if (e == cudaSuccess) e = cudaDeviceGetAttribute(&thr, cudaDevAttrMaxThreadsPerMultiProcessor, device);
+    if (e == cudaSuccess) e = cudaDeviceGetAttribute(&rsv, cudaDevAttrReservedSharedMemoryPerBlock, device);
+    if (e == cudaSuccess) e = cudaDeviceGetAttribute(&blk, cudaDevAttrMaxBlocksPerMultiprocessor, device);
+    if (e != cudaSuccess) return e;
+    const int kPackThreads = 128;
+    auto warp_regs = [](int r) { return ((r + 7) / 8) * 8 * 32; };
+    const long long rp = (long long)warp_regs(fp.numRegs) * afmm::kWarps, rk = (long long)warp_regs(fk.numRegs) * (kPackThreads / 32);
+    const long long sp = (long long)fp.sharedSizeBytes + afmm::kDynSmem + rsv, sk = (long long)fk.sharedSizeBytes + rsv;
+    const char *env = getenv("AFMM_PACK_CORESIDENT");
+    *ok = rp + rk <= regs && sp + sk <= smem && afmm::kThreads + kPackThreads <= thr && blk >= 2 &&
+          !(env && env[0] == '0');
+    return cudaSuccess;
+}
 
 afmm_status set_device(afmm_p2p *h) {
     CUDA_TRY(h, cudaSetDevice(h->cfg.device));
@@ -256,8 +315,57 @@ extern "C" afmm_status afmm_p2p_config_init(afmm_p2p_config *cfg) {
     cfg->law = AFMM_LAW_GRAVITY;
     cfg->mu = 1.0f;
     cfg->slice_world = 0;
+    cfg->nccl_id = nullptr;
+    cfg->comm_sms = 0;
     return AFMM_OK;
 }
+
+extern "C" afmm_status afmm_p2p_nccl_id(void *out128) {
+    if (!out128) return AFMM_EINVAL;
+    const afmm::NcclApi &nc = afmm::nccl_api();
+    if (!nc.ok) return AFMM_ENOTSUP;
+    ncclUniqueId id;
+    static_assert(sizeof(id) == 128, "ncclUniqueId is 128 bytes");
+    if (nc.GetUniqueId(&id) != ncclSuccess) return AFMM_ENCCL;
+    std::memcpy(out128, &id, sizeof(id));
+    return AFMM_OK;
+}
+
+namespace {
+int comm_sms(const afmm_p2p *h) { return h->cfg.comm_sms > 0 ? h->cfg.comm_sms : 8; }
+
+#define NCCL_TRY(h, call)                                                                    \
+    do {                                                                                     \
+        ncclResult_t r_ = (call);                                                            \
+        if (r_ != ncclSuccess)                                                               \
+            return fail((h), AFMM_ENCCL, "%s failed: %s (%s:%d)", #call,                     \
+                        afmm::nccl_api().GetErrorString(r_), __FILE__, __LINE__);            \
+    } while (0)
+
+// The library communicator (afmm_p2p_config.nccl_id): world ranks, at most
+// comm_sms CTAs per NCCL kernel (ncclConfig_t.maxCTAs, NCCL >= 2.28; earlier
+// versions: ncclCommInitRank and NCCL's own channel count), its own stream.
+afmm_status init_comm(afmm_p2p *h) {
+    const afmm::NcclApi &nc = afmm::nccl_api();
+    if (!nc.ok) return fail(h, AFMM_ENOTSUP, "create: nccl_id given but libnccl.so.2 could not be loaded");
+    ncclUniqueId id;
+    std::memcpy(&id, h->cfg.nccl_id, sizeof(id));
+    if (nc.CommInitRankConfig && nc.version >= 22800) {
+        ncclConfig_t c = NCCL_CONFIG_INITIALIZER;
+        c.blocking = 1;
+        c.minCTAs = 1;
+        c.maxCTAs = comm_sms(h);
+        NCCL_TRY(h, nc.CommInitRankConfig(&h->comm, h->cfg.world, id, h->cfg.rank, &c));
+    } else {
+        NCCL_TRY(h, nc.CommInitRank(&h->comm, h->cfg.world, id, h->cfg.rank));
+    }
+    CUDA_TRY(h, cudaStreamCreateWithFlags(&h->s_comm, cudaStreamNonBlocking));
+    for (cudaEvent_t *e : {&h->ev_c0, &h->ev_c1, &h->ev_c2, &h->ev_c3})
+        CUDA_TRY(h, cudaEventCreateWithFlags(e, cudaEventDisableTiming));
+    CUDA_TRY(h, cudaMallocHost(&h->h_kms, sizeof(double)));
+    return AFMM_OK;
+}
+}  // namespace
 
 extern "C" const char *afmm_version(void) { return "afmm_p2p 0.1 sm_100a"; }
 
@@ -269,7 +377,8 @@ extern "C" afmm_status afmm_p2p_create(const afmm_p2p_config *cfg, afmm_p2p **ou
     if (cfg->max_leaf < 1 || cfg->world < 1 || cfg->rank < 0 || cfg->rank >= cfg->world ||
         !std::isfinite(cfg->G) || !std::isfinite(cfg->eps2) || !(cfg->eps2 >= 0.0f) ||
         cfg->device < 0 || (cfg->law != AFMM_LAW_GRAVITY && cfg->law != AFMM_LAW_STOKESLET) ||
-        !std::isfinite(cfg->mu) || !(cfg->mu > 0.0f) || cfg->slice_world < 0)
+        !std::isfinite(cfg->mu) || !(cfg->mu > 0.0f) || cfg->slice_world < 0 || cfg->comm_sms < 0 ||
+        cfg->comm_sms > 64)
         return AFMM_EINVAL;
     afmm_p2p *h = new (std::nothrow) afmm_p2p();
     if (!h) return AFMM_ENOMEM;
@@ -301,8 +410,17 @@ extern "C" afmm_status afmm_p2p_create(const afmm_p2p_config *cfg, afmm_p2p **ou
         if (e == cudaSuccess)
             e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&h->blocks_per_sm, afmm::p2p_kernel_t<afmm::Gravity>,
                                                               afmm::kThreads, afmm::kDynSmem);
+        if (e == cudaSuccess) e = co_residency(cfg->device, &h->co_resident_pack);
+        if (e == cudaSuccess) e = cudaMalloc(&h->d_words, 64);
+        if (e == cudaSuccess) e = cudaMemset(h->d_words, 0, 64);
+        if (e == cudaSuccess) e = cudaMallocHost(&h->h_cerr, sizeof(int));
         if (e != cudaSuccess) st = fail(h, AFMM_ECUDA, "create: %s", cudaGetErrorString(e));
         if (h->blocks_per_sm < 1) h->blocks_per_sm = 1;
+        if (h->h_cerr) *h->h_cerr = 0;
+        if (st == AFMM_OK && cfg->nccl_id && cfg->law != AFMM_LAW_GRAVITY)
+            st = fail(h, AFMM_ENOTSUP, "create: the library communicator replicates gravity bodies only");
+        if (st == AFMM_OK && cfg->nccl_id) st = init_comm(h);
+        h->cfg.nccl_id = nullptr;                   // the caller's buffer is not kept
     }
     if (st != AFMM_OK) {
         afmm_p2p_destroy(h);
@@ -325,6 +443,15 @@ extern "C" void afmm_p2p_destroy(afmm_p2p *h) {
     cudaFree(h->d_queue);
     cudaFree(h->d_ptasks);
     cudaFree(h->d_pqueue);
+    if (h->s_comm) cudaStreamSynchronize(h->s_comm);
+    if (h->comm) afmm::nccl_api().CommDestroy(h->comm);
+    if (h->s_comm) cudaStreamDestroy(h->s_comm);
+    for (cudaEvent_t e : {h->ev_c0, h->ev_c1, h->ev_c2, h->ev_c3})
+        if (e) cudaEventDestroy(e);
+    cudaFree(h->d_words);
+    cudaFree(h->d_ctasks);
+    if (h->h_kms) cudaFreeHost(h->h_kms);
+    if (h->h_cerr) cudaFreeHost(h->h_cerr);
     if (h->s_in) cudaStreamSynchronize(h->s_in), cudaStreamDestroy(h->s_in);
     if (h->in_graph) cudaGraphExecDestroy(h->in_graph);
     if (h->h_err) cudaFreeHost(h->h_err);
@@ -337,6 +464,7 @@ extern "C" void afmm_p2p_destroy(afmm_p2p *h) {
     }
     if (h->ev_start) cudaEventDestroy(h->ev_start);
     if (h->ev_done) cudaEventDestroy(h->ev_done);
+    if (h->ev_in_done) cudaEventDestroy(h->ev_in_done);
     for (int i = 0; i < afmm_p2p::kRing; ++i) {
         if (h->ring0[i]) cudaEventDestroy(h->ring0[i]);
         if (h->ring1[i]) cudaEventDestroy(h->ring1[i]);
@@ -397,11 +525,12 @@ extern "C" afmm_status afmm_p2p_set_bodies(afmm_p2p *h, long long n, const float
     afmm_status st = set_device(h);
     if (st) return st;
     if ((st = alloc_bodies(h, n))) return st;
+    h->bodies_pending = h->comm != nullptr;          // the next eval replicates them (library communicator)
     if (nn == 4) return pack(h, x, y, z, m);
     // allocate only: the equal-mass flag reads "unequal" until a full-buffer
     // broadcast (afmm_p2p_bodies_buffer, trailer included) brings the root's
-    static const int one = 1;
-    CUDA_TRY(h, cudaMemcpyAsync(mass_flag(h), &one, sizeof(int), cudaMemcpyHostToDevice, h->stream));
+    static const int unequal = -1;
+    CUDA_TRY(h, cudaMemcpyAsync(mass_flag(h), &unequal, sizeof(int), cudaMemcpyHostToDevice, h->stream));
     CUDA_TRY(h, cudaStreamSynchronize(h->stream));
     return AFMM_OK;
 }
@@ -415,6 +544,7 @@ extern "C" afmm_status afmm_p2p_set_bodies_host(afmm_p2p *h, long long n, const 
     afmm_status st = set_device(h);
     if (st) return st;
     if ((st = alloc_bodies(h, n))) return st;
+    h->bodies_pending = h->comm != nullptr;
     if (4 * n > h->soa_cap) {
         cudaFree(h->d_soa);
         h->d_soa = nullptr;
@@ -556,7 +686,7 @@ static afmm_status dws(afmm_p2p *h, int slot, T **p, size_t count) {
 
 __global__ void body_split_kernel(int G, int L, long long n, const long long *__restrict__ split,
                                   const int *__restrict__ ls, long long *__restrict__ bsplit) {
-    const int r = threadIdx.x;
+    const int r = blockIdx.x * blockDim.x + threadIdx.x;
     if (r <= G) bsplit[r] = split[r] >= L ? n : ls[split[r]];
 }
 
@@ -623,7 +753,7 @@ extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const
         clear_user = true;
     }
     CUDA_TRY(h, cudaGetLastError());
-    body_split_kernel<<<1, 64, 0, s>>>(W, L, h->n, split, leaf_start, bsplit);
+    body_split_kernel<<<(W + 1 + 63) / 64, 64, 0, s>>>(W, L, h->n, split, leaf_start, bsplit);
     std::vector<long long> lsplit(W + 1, 0), bsplit_h(W + 1, 0);
     long long itot = 0;
     CUDA_TRY(h, cudaMemcpyAsync(lsplit.data(), split, (W + 1) * sizeof(long long), cudaMemcpyDeviceToHost, s));
@@ -695,6 +825,7 @@ extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const
     }
     h->n_tasks = nt;
     h->pipe_valid = false;
+    h->chunk_valid = false;
     h->L = L;
     h->rank_interactions = (long long)hstats[0];
     for (int b = 0; b < 8; ++b) h->bucket_inter[b] = (long long)hstats[1 + b];
@@ -915,6 +1046,22 @@ static void set_windows(afmm_p2p *h, afmm::P2PParams &p, float *ax, float *ay, f
         for (int a = 0; a < 4; ++a) p.out[w][a] = w <= h->n_peers ? h->peers[w - 1][a] : nullptr;
 }
 
+// the handle's device words (d_words, 64 bytes)
+static unsigned *w_ready(afmm_p2p *h) { return reinterpret_cast<unsigned *>(h->d_words); }
+static int *w_err(afmm_p2p *h) { return reinterpret_cast<int *>(h->d_words + 4); }
+static unsigned long long *w_tspan(afmm_p2p *h) { return reinterpret_cast<unsigned long long *>(h->d_words + 16); }
+static double *w_kms(afmm_p2p *h) { return reinterpret_cast<double *>(h->d_words + 32); }
+
+// tspan = {max, 0}: the kernel's CTAs atomicMin their start, warps atomicMax their end
+static afmm_status reset_tspan(afmm_p2p *h) {
+    CUDA_TRY(h, cudaMemsetAsync(w_tspan(h), 0xff, sizeof(unsigned long long), h->stream));
+    CUDA_TRY(h, cudaMemsetAsync(w_tspan(h) + 1, 0, sizeof(unsigned long long), h->stream));
+    return AFMM_OK;
+}
+
+static afmm_status launch_chunked(afmm_p2p *h, float *ax, float *ay, float *az, float *phi, bool deliver);
+static afmm_status comm_finish(afmm_p2p *h);
+
 static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, float *phi) {
     afmm::P2PParams p;
     p.bodies = h->d_bodies;
@@ -929,6 +1076,15 @@ static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, flo
     p.done = nullptr;
     p.in_ready = nullptr;
     p.in_err = nullptr;
+    p.wait_ns = 0;
+    p.in_epoch = 0;
+    p.m0 = 0.f;
+    p.m0_ptr = nullptr;
+    p.tspan = h->comm ? w_tspan(h) : nullptr;
+    if (h->comm) {
+        afmm_status st = reset_tspan(h);
+        if (st) return st;
+    }
 #ifndef AFMM_EQMASS
 #define AFMM_EQMASS 1
 #endif
@@ -937,6 +1093,8 @@ static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, flo
     p.out_coalesce = 0;
     h->last_zero_copy = false;
     h->last_input_graph = false;
+    h->last_streamed = false;
+    h->last_chunked = false;
     CUDA_TRY(h, cudaMemsetAsync(h->d_queue, 0, sizeof(int), h->stream));
     const int ri = (int)(h->n_evals % afmm_p2p::kRing);
     h->ev0 = h->ring0[ri];
@@ -977,10 +1135,29 @@ static afmm_status fill_stats(afmm_p2p *h, afmm_p2p_stats *s) {
     o.n_launches = h->last.n_launches;
     o.zero_copy = h->last_zero_copy ? 1 : 0;
     o.input_graph = h->last_input_graph ? 1 : 0;
+    o.streamed_inputs = h->last_streamed ? 1 : 0;
+    o.chunked_bodies = h->last_chunked ? 1 : 0;
+    o.kernel_ms_max = h->comm ? *(volatile double *)h->h_kms : (double)ms;
     for (int b = 0; b < 8; ++b) o.bucket_interactions[b] = h->bucket_inter[b];
     h->last = o;
     if (s) *s = o;
+    if (h->last_chunked && *(volatile int *)h->h_cerr)
+        return fail(h, AFMM_ECUDA, "eval: body chunks never arrived (kernel wait timed out, AFMM_WAIT_MS)");
     return AFMM_OK;
+}
+
+// One evaluation on device outputs: the chunked replication when the library
+// communicator has bodies to broadcast, else the plain launch; then (library
+// communicator) the GPU time all-reduce that also completes the fused gather.
+static afmm_status launch_any(afmm_p2p *h, float *ax, float *ay, float *az, float *phi) {
+    afmm_status st;
+    if (h->comm && h->bodies_pending) {
+        if ((st = launch_chunked(h, ax, ay, az, phi, true))) return st;
+        h->bodies_pending = false;
+    } else if ((st = launch_eval(h, ax, ay, az, phi))) {
+        return st;
+    }
+    return h->comm ? comm_finish(h) : AFMM_OK;
 }
 
 extern "C" afmm_status afmm_p2p_eval(afmm_p2p *h, float *ax, float *ay, float *az, float *phi,
@@ -990,7 +1167,7 @@ extern "C" afmm_status afmm_p2p_eval(afmm_p2p *h, float *ax, float *ay, float *a
     if (!ax || !ay || !az || !phi) return fail(h, AFMM_EINVAL, "eval: null output pointer");
     afmm_status st = set_device(h);
     if (st) return st;
-    if ((st = launch_eval(h, ax, ay, az, phi))) return st;
+    if ((st = launch_any(h, ax, ay, az, phi))) return st;
     if (stats) return fill_stats(h, stats);
     return AFMM_OK;
 }
@@ -1011,7 +1188,7 @@ extern "C" afmm_status afmm_p2p_eval_host(afmm_p2p *h, float *ax, float *ay, flo
         h->out_cap = 4 * n;
     }
     float *d[4] = {h->d_out, h->d_out + n, h->d_out + 2 * n, h->d_out + 3 * n};
-    if ((st = launch_eval(h, d[0], d[1], d[2], d[3]))) return st;
+    if ((st = launch_any(h, d[0], d[1], d[2], d[3]))) return st;
     const long long lo = h->body_split[h->cfg.rank], hi = h->body_split[h->cfg.rank + 1];
     float *hp[4] = {ax, ay, az, phi};
     if (hi > lo)
@@ -1036,21 +1213,47 @@ static bool host_mapped(const void *p, void **dptr) {
     return true;
 }
 
+// cuStreamWaitValue32 / cuStreamWriteValue32 through the runtime's driver entry points
+static afmm_status resolve_stream_ops(afmm_p2p *h) {
+    if (h->wait_value32 && h->write_value32) return AFMM_OK;
+    cudaDriverEntryPointQueryResult q;
+    CUDA_TRY(h, cudaGetDriverEntryPoint("cuStreamWaitValue32", &h->wait_value32, cudaEnableDefault, &q));
+    if (q != cudaDriverEntryPointSuccess || !h->wait_value32)
+        return fail(h, AFMM_ENOTSUP, "cuStreamWaitValue32 unavailable");
+    CUDA_TRY(h, cudaGetDriverEntryPoint("cuStreamWriteValue32", &h->write_value32, cudaEnableDefault, &q));
+    if (q != cudaDriverEntryPointSuccess || !h->write_value32)
+        return fail(h, AFMM_ENOTSUP, "cuStreamWriteValue32 unavailable");
+    return AFMM_OK;
+}
+using WriteValueFn = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+
 static constexpr int kMaxPieces = 64;
-static constexpr int kInChunks = 8;                 // input chunks of the streamed H2D (<= 32: mass bits)
+static constexpr int kInChunks = 8;                 // input chunks of the streamed H2D
+static constexpr int kMaxChunks = 16;               // chunk masks ride in the high 16 bits of Task.piece
 
 // Regroup this rank's tasks into P pieces of consecutive targets (equal modelled
 // cost tgt_count * nsrc, cut in tgt_start order); inside a piece the tasks keep
 // the work list's largest-cost-first order.  Per piece: the output body range and
 // the prefix of bodies [0, need) its sources and targets lie in.
-static afmm_status build_pipe(afmm_p2p *h, int P) {
+// Host copy of this rank's work list (tasks in work-list order and the segments
+// they reference), whether it was built on the host or by the device ingest.
+static afmm_status fetch_worklist(afmm_p2p *h, std::vector<afmm::Task> &t, std::vector<afmm::Seg> &sg) {
     const int nt = h->n_tasks;
-    std::vector<afmm::Task> t(nt);
+    t.resize(nt);
+    CUDA_TRY(h, cudaStreamSynchronize(h->stream));
     if (nt) CUDA_TRY(h, cudaMemcpy(t.data(), h->d_tasks, nt * sizeof(afmm::Task), cudaMemcpyDeviceToHost));
     int nseg = 0;
     for (const auto &x : t) nseg = std::max(nseg, x.seg_begin + x.seg_count);
-    std::vector<afmm::Seg> sg(nseg);
+    sg.resize(nseg);
     if (nseg) CUDA_TRY(h, cudaMemcpy(sg.data(), h->d_segs, nseg * sizeof(afmm::Seg), cudaMemcpyDeviceToHost));
+    return AFMM_OK;
+}
+
+static afmm_status build_pipe(afmm_p2p *h, int P) {
+    const int nt = h->n_tasks;
+    std::vector<afmm::Task> t;
+    std::vector<afmm::Seg> sg;
+    if (afmm_status st0 = fetch_worklist(h, t, sg)) return st0;
     std::vector<int> ord(nt);
     for (int i = 0; i < nt; ++i) ord[i] = i;
     std::stable_sort(ord.begin(), ord.end(), [&](int a, int b) { return t[a].tgt_start < t[b].tgt_start; });
@@ -1093,7 +1296,7 @@ static afmm_status build_pipe(afmm_p2p *h, int P) {
     // first chunk and stays behind the copies, and every output piece's stragglers (leaves
     // whose U-lists reach far in Morton order) run as soon as the last chunk lands.
     const char *kenv = getenv("AFMM_E2E_CHUNKS");             // measurements only
-    const int kin = kenv ? std::max(1, std::min(32, atoi(kenv))) : kInChunks;
+    const int kin = kenv ? std::max(1, std::min(kMaxChunks, atoi(kenv))) : kInChunks;
     const int K = (int)std::min<long long>(kin, std::max<long long>(1, h->n / 4096));
     const long long chunk = (h->n + K - 1) / K;
     std::vector<int> need_chunk(nt, 0);
@@ -1119,7 +1322,8 @@ static afmm_status build_pipe(afmm_p2p *h, int P) {
     std::vector<afmm::Task> grouped(std::max(nt, 1));
     for (int r = 0; r < nt; ++r) {                                              // stable: LPT kept
         afmm::Task x = t[ord2[r]];
-        x.piece = piece[ord2[r]] | (need_chunk[ord2[r]] << 16);
+        // need mask: chunks 0..need_chunk (they arrive in Morton order)
+        x.piece = (int)((unsigned)piece[ord2[r]] | (((2u << need_chunk[ord2[r]]) - 1u) << 16));
         grouped[r] = x;
     }
     h->pipe_K = K;
@@ -1149,20 +1353,15 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
         CUDA_TRY(h, cudaStreamCreateWithFlags(&h->s_out, cudaStreamNonBlocking));
         CUDA_TRY(h, cudaEventCreateWithFlags(&h->ev_start, cudaEventDisableTiming));
         CUDA_TRY(h, cudaEventCreateWithFlags(&h->ev_done, cudaEventDisableTiming));
+        CUDA_TRY(h, cudaEventCreateWithFlags(&h->ev_in_done, cudaEventDisableTiming));
         for (int i = 0; i < kMaxPieces; ++i) {
             CUDA_TRY(h, cudaEventCreateWithFlags(&h->ev_in[i], cudaEventDisableTiming));
             CUDA_TRY(h, cudaEventCreateWithFlags(&h->ev_k[i], cudaEventDisableTiming));
         }
         CUDA_TRY(h, cudaMalloc(&h->d_pqueue, (kMaxPieces + 4) * sizeof(int)));
         CUDA_TRY(h, cudaMallocHost(&h->h_err, sizeof(int)));
-        cudaDriverEntryPointQueryResult q;
-        CUDA_TRY(h, cudaGetDriverEntryPoint("cuStreamWaitValue32", &h->wait_value32, cudaEnableDefault, &q));
-        if (q != cudaDriverEntryPointSuccess || !h->wait_value32)
-            return fail(h, AFMM_ENOTSUP, "eval_host_pipelined: cuStreamWaitValue32 unavailable");
-        CUDA_TRY(h, cudaGetDriverEntryPoint("cuStreamWriteValue32", &h->write_value32, cudaEnableDefault, &q));
-        if (q != cudaDriverEntryPointSuccess || !h->write_value32)
-            return fail(h, AFMM_ENOTSUP, "eval_host_pipelined: cuStreamWriteValue32 unavailable");
     }
+    if ((st = resolve_stream_ops(h))) return st;
     if (4 * n > h->soa_cap) {
         cudaFree(h->d_soa);
         h->d_soa = nullptr;
@@ -1217,6 +1416,8 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
     const bool zc_in = zc && !(zenv && zenv[0] == 'o'), zc_out = zc && !(zenv && zenv[0] == 'i');
     h->last_zero_copy = zc;
     const float m0 = m[0];                          // equal-mass test of the streamed chunks
+    h->bodies_pending = false;                      // every body comes from this call's host arrays
+    h->last_chunked = false;
     CUDA_TRY(h, cudaMemsetAsync(mass_flag(h), 0xff, sizeof(int), h->stream));   // bodies replaced: flag "unequal"
     CUDA_TRY(h, cudaEventRecord(h->ev_start, h->stream));      // earlier readers of the bodies / outputs
     CUDA_TRY(h, cudaStreamWaitEvent(h->s_in, h->ev_start, 0));
@@ -1232,6 +1433,10 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
     // does not wait for chunk 0 (its warps wait per task; m_0 comes from the host).
     int nlaunch = 0;
     auto launch = [&]() -> afmm_status {
+        if (h->comm) {
+            const afmm_status s0 = reset_tspan(h);
+            if (s0) return s0;
+        }
         const int ri = (int)(h->n_evals % afmm_p2p::kRing);
         h->ev0 = h->ring0[ri];
         h->ev1 = h->ring1[ri];
@@ -1255,7 +1460,11 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
             prm.done = zc_out ? nullptr : done;
             prm.in_ready = in_ready;
             prm.in_err = in_err;
+            prm.wait_ns = wait_ns(h);
+            prm.in_epoch = 0;                            // the flag word is zeroed per call (epoch 0)
             prm.m0 = m0;
+            prm.m0_ptr = nullptr;
+            prm.tspan = h->comm ? w_tspan(h) : nullptr;
             const int grid = std::max(1, std::min((nt + afmm::kWarps - 1) / afmm::kWarps, h->num_sms * h->blocks_per_sm));
             afmm::p2p_kernel_t<afmm::Gravity, true><<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(prm);
             CUDA_TRY(h, cudaGetLastError());
@@ -1266,6 +1475,11 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
     };
     const int K = h->pipe_K;
     const long long chunk = (n + K - 1) / K;
+    // Without room for a pack block beside a P2P CTA (co_resident_pack) the chain
+    // could not progress under the persistent kernel: pack every chunk first, then
+    // launch (the kernel's chunk waits then pass at once).
+    const bool streamed = h->co_resident_pack;
+    h->last_streamed = streamed;
     // Enqueue the input chain: pack chunk k, then publish k + 1 (stream write).
     auto enqueue_inputs = [&](bool capturing) -> afmm_status {
         for (int k = 0; k < K; ++k) {
@@ -1292,7 +1506,8 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
                     return fail(h, AFMM_ECUDA, "eval_host_pipelined: pack launch failed: %s", cudaGetErrorString(le));
                 }
             }
-            const CUresult r = write32((CUstream)h->s_in, (CUdeviceptr)in_ready, (cuuint32_t)(k + 1), 0);
+            // the delivered-chunk mask: chunks 0..k
+            const CUresult r = write32((CUstream)h->s_in, (CUdeviceptr)in_ready, (cuuint32_t)((2u << k) - 1u), 0);
             if (r != CUDA_SUCCESS) {
                 if (capturing) return AFMM_ECUDA;
                 return fail(h, AFMM_ECUDA, "eval_host_pipelined: cuStreamWriteValue32 failed (%d)", (int)r);
@@ -1343,7 +1558,17 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
     if (!use_graph) {
         if ((st = enqueue_inputs(false))) return st;
     }
+    if (!streamed) {                                  // serial fallback: inputs complete before the launch
+        CUDA_TRY(h, cudaEventRecord(h->ev_in_done, h->s_in));
+        CUDA_TRY(h, cudaStreamWaitEvent(h->stream, h->ev_in_done, 0));
+    }
     if ((st = launch())) return st;
+    // join the input chain into the handle's stream: the kernel waits only for the
+    // chunks its own tasks reach (none at all for a rank without tasks or after a
+    // wait timeout), so without this the call could return -- and the next call
+    // reset the chunk flags -- while pack kernels still read the host inputs
+    CUDA_TRY(h, cudaEventRecord(h->ev_in_done, h->s_in));
+    CUDA_TRY(h, cudaStreamWaitEvent(h->stream, h->ev_in_done, 0));
     // the launch must be enqueued before the copy-out stream starts waiting on its counters
     for (int q = 0; q < P && !zc_out; ++q) {
         const long long lo = h->pipe_lo[q], hi = h->pipe_hi[q];
@@ -1366,8 +1591,220 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
     // synchronise covers it (no separate blocking copy)
     *h->h_err = 0;
     CUDA_TRY(h, cudaMemcpyAsync(h->h_err, in_err, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+    if (h->comm && (st = comm_finish(h))) return st;
     if ((st = fill_stats(h, stats))) return st;
     if (*(volatile int *)h->h_err) return fail(h, AFMM_ECUDA, "eval_host_pipelined: input chunks never arrived (kernel wait timed out)");
+    return AFMM_OK;
+}
+
+// ------------------------------------------------------------------ chunked body replication
+
+// The delivery plan of the packed bodies (afmm_p2p_chunks) and the work list in
+// delivery order: K <= 16 chunks of consecutive bodies; chunk c is owned by the
+// rank whose body slice holds its first body; the delivery order deals the
+// ranks' chunks round robin (every rank's first chunk among the first `world`
+// deliveries, its k-th among the first k*world).  Every task gets the mask of the
+// chunks its targets and source segments touch (high 16 bits of Task.piece) and
+// the tasks are ordered by the delivery position of the last chunk they need
+// (stable: the work list's largest-cost-first order inside each position), so
+// the first tasks a warp claims are the ones the first chunks make runnable.
+static afmm_status build_chunks(afmm_p2p *h) {
+    std::vector<afmm::Task> t;
+    std::vector<afmm::Seg> sg;
+    afmm_status st = fetch_worklist(h, t, sg);
+    if (st) return st;
+    const long long n = h->n;
+    const int K = (int)std::min<long long>(kMaxChunks, std::max<long long>(1, n / 4096));
+    const int W = h->cfg.world;
+    std::vector<long long> b(K + 1);
+    for (int k = 0; k <= K; ++k) b[k] = n * k / K;
+    auto chunk_of = [&](long long i) {            // chunk holding body i
+        return (int)(std::upper_bound(b.begin(), b.end(), i) - b.begin()) - 1;
+    };
+    std::vector<std::vector<int>> owned(W);
+    for (int k = 0; k < K; ++k) {
+        int r = (int)(std::upper_bound(h->body_split.begin(), h->body_split.end(), b[k]) - h->body_split.begin()) - 1;
+        r = std::max(0, std::min(W - 1, r));
+        owned[r].push_back(k);
+    }
+    std::vector<int> order, pos(K);
+    for (size_t j = 0; (int)order.size() < K; ++j)
+        for (int r = 0; r < W; ++r)
+            if (j < owned[r].size()) order.push_back(owned[r][j]);
+    for (int j = 0; j < K; ++j) pos[order[j]] = j;
+    const int nt = (int)t.size();
+    std::vector<unsigned> mask(nt, 0);
+    std::vector<int> ready(nt, 0);
+    for (int i = 0; i < nt; ++i) {
+        unsigned msk = 0;
+        auto add = [&](long long lo, long long len) {
+            if (len <= 0) return;
+            for (int c = chunk_of(lo), e = chunk_of(lo + len - 1); c <= e; ++c) msk |= 1u << c;
+        };
+        add(t[i].tgt_start, t[i].tgt_count);
+        for (int j = 0; j < t[i].seg_count; ++j) add(sg[t[i].seg_begin + j].gstart, sg[t[i].seg_begin + j].len);
+        mask[i] = msk;
+        int rd = 0;
+        for (int c = 0; c < K; ++c)
+            if (msk >> c & 1u) rd = std::max(rd, pos[c]);
+        ready[i] = rd;
+    }
+    std::vector<int> ord(nt);
+    std::iota(ord.begin(), ord.end(), 0);
+    std::stable_sort(ord.begin(), ord.end(), [&](int a, int c) { return ready[a] < ready[c]; });
+    std::vector<afmm::Task> out(std::max(nt, 1));
+    for (int i = 0; i < nt; ++i) {
+        out[i] = t[ord[i]];
+        out[i].piece = (int)(mask[ord[i]] << 16);
+    }
+    if ((st = ensure_device(h, &h->d_ctasks, h->ctasks_cap, out.size()))) return st;
+    CUDA_TRY(h, cudaMemcpy(h->d_ctasks, out.data(), out.size() * sizeof(afmm::Task), cudaMemcpyHostToDevice));
+    h->chunk_K = K;
+    h->chunk_bounds = b;
+    h->chunk_order = order;
+    h->chunk_valid = true;
+    return AFMM_OK;
+}
+
+// The P2P kernel on the chunk-ordered work list, every task waiting for its
+// chunks (epoch-tagged mask word, never reset).  deliver: the library
+// communicator broadcasts the trailer, then the chunks in delivery order on
+// s_comm, publishing the cumulative mask after each (cuStreamWriteValue32 orders
+// the broadcast's writes before the flag); else the caller delivers and
+// publishes (afmm_p2p_publish_chunks).  The kernel leaves comm_sms SMs free for
+// the transport's kernels.
+static afmm_status launch_chunked(afmm_p2p *h, float *ax, float *ay, float *az, float *phi, bool deliver) {
+    afmm_status st;
+    if (h->cfg.law != AFMM_LAW_GRAVITY) return fail(h, AFMM_ENOTSUP, "chunked replication: gravity handles only");
+    if (!h->chunk_valid && (st = build_chunks(h))) return st;
+    if ((st = resolve_stream_ops(h))) return st;
+    const WriteValueFn write32 = reinterpret_cast<WriteValueFn>(h->write_value32);
+    h->epoch = h->epoch % 0xffffu + 1u;                       // 1 .. 65535 (0: the pipelined path)
+    const unsigned tag = h->epoch << 16;
+    CUDA_TRY(h, cudaMemsetAsync(w_err(h), 0, sizeof(int), h->stream));
+    CUDA_TRY(h, cudaMemsetAsync(h->d_queue, 0, sizeof(int), h->stream));
+    if (deliver) {
+        const afmm::NcclApi &nc = afmm::nccl_api();
+        CUDA_TRY(h, cudaEventRecord(h->ev_c0, h->stream));    // the root's pack, earlier readers of the bodies
+        CUDA_TRY(h, cudaStreamWaitEvent(h->s_comm, h->ev_c0, 0));
+        NCCL_TRY(h, nc.Broadcast(mass_flag(h), mass_flag(h), sizeof(float4), ncclChar, 0, h->comm, h->s_comm));
+        unsigned cum = 0;
+        for (int j = 0; j < h->chunk_K; ++j) {
+            const int c = h->chunk_order[j];
+            const long long lo = h->chunk_bounds[c], cnt = h->chunk_bounds[c + 1] - lo;
+            if (cnt > 0)
+                NCCL_TRY(h, nc.Broadcast(h->d_bodies + lo, h->d_bodies + lo, (size_t)cnt * sizeof(float4), ncclChar, 0,
+                                         h->comm, h->s_comm));
+            cum |= 1u << c;
+            const CUresult r = write32((CUstream)h->s_comm, (CUdeviceptr)w_ready(h), (cuuint32_t)(tag | cum), 0);
+            if (r != CUDA_SUCCESS) return fail(h, AFMM_ECUDA, "chunked eval: cuStreamWriteValue32 failed (%d)", (int)r);
+        }
+        CUDA_TRY(h, cudaEventRecord(h->ev_c1, h->s_comm));
+    }
+    afmm::P2PParams p;
+    p.bodies = h->d_bodies;
+    p.tasks = h->d_ctasks;
+    p.segs = h->d_segs;
+    p.n_tasks = h->n_tasks;
+    p.queue = h->d_queue;
+    p.static_rounds = 0;                                       // claims follow the delivery order
+    set_windows(h, p, ax, ay, az, phi);
+    p.eps2 = h->cfg.eps2;
+    p.G = (double)h->cfg.G;
+    p.done = nullptr;
+    p.in_ready = w_ready(h);
+    p.in_err = w_err(h);
+    p.wait_ns = wait_ns(h);
+    p.in_epoch = h->epoch;
+    p.mass_unequal = nullptr;
+    p.mass_bits = (AFMM_EQMASS ? reinterpret_cast<const unsigned *>(mass_flag(h)) : nullptr);   // 0 or all bits
+    p.m0 = 0.f;
+    p.m0_ptr = reinterpret_cast<const float *>(mass_flag(h) + 1);                            // trailer word 1
+    p.out_coalesce = 0;
+    p.tspan = h->comm ? w_tspan(h) : nullptr;
+    if (h->comm && (st = reset_tspan(h))) return st;
+    h->last_zero_copy = false;
+    h->last_input_graph = false;
+    h->last_streamed = false;
+    const int ri = (int)(h->n_evals % afmm_p2p::kRing);
+    h->ev0 = h->ring0[ri];
+    h->ev1 = h->ring1[ri];
+    CUDA_TRY(h, cudaEventRecord(h->ev0, h->stream));
+    int nlaunch = 0;
+    if (p.n_tasks > 0) {
+        const int room = std::max(1, h->num_sms * h->blocks_per_sm - comm_sms(h));
+        const int grid = std::max(1, std::min((p.n_tasks + afmm::kWarps - 1) / afmm::kWarps, room));
+        afmm::p2p_kernel_t<afmm::Gravity, true><<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(p);
+        CUDA_TRY(h, cudaGetLastError());
+        nlaunch = 1;
+    }
+    CUDA_TRY(h, cudaEventRecord(h->ev1, h->stream));
+    *h->h_cerr = 0;
+    CUDA_TRY(h, cudaMemcpyAsync(h->h_cerr, w_err(h), sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+    if (deliver) CUDA_TRY(h, cudaStreamWaitEvent(h->stream, h->ev_c1, 0));   // the broadcast joins the stream
+    h->n_evals++;
+    h->evaluated = true;
+    h->last_chunked = true;
+    h->last.n_launches = nlaunch;
+    return AFMM_OK;
+}
+
+// Library communicator, after every eval: the kernel's device-timer span (ms),
+// all-reduced with MAX on s_comm -> *h_kms (the GPU time of PAPER L20 SVII.A).
+// Every rank's contribution is enqueued after its own kernel, so when the
+// all-reduce completes every rank's kernel -- and its fused-gather stores into
+// the peer windows, fenced system-wide at kernel end -- has completed: the
+// handle's stream waits for it.
+static afmm_status comm_finish(afmm_p2p *h) {
+    const afmm::NcclApi &nc = afmm::nccl_api();
+    afmm::span_ms_kernel<<<1, 1, 0, h->stream>>>(w_tspan(h), w_kms(h));
+    CUDA_TRY(h, cudaGetLastError());
+    CUDA_TRY(h, cudaEventRecord(h->ev_c2, h->stream));
+    CUDA_TRY(h, cudaStreamWaitEvent(h->s_comm, h->ev_c2, 0));
+    NCCL_TRY(h, nc.AllReduce(w_kms(h), w_kms(h) + 1, 1, ncclFloat64, ncclMax, h->comm, h->s_comm));
+    CUDA_TRY(h, cudaMemcpyAsync(h->h_kms, w_kms(h) + 1, sizeof(double), cudaMemcpyDeviceToHost, h->s_comm));
+    CUDA_TRY(h, cudaEventRecord(h->ev_c3, h->s_comm));
+    CUDA_TRY(h, cudaStreamWaitEvent(h->stream, h->ev_c3, 0));
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_p2p_chunks(afmm_p2p *h, int *K, long long *bounds, int *order) {
+    CHECK_HANDLE(h);
+    if (!h->d_bodies || !h->have_tree) return fail(h, AFMM_ESTATE, "chunks: set_bodies and set_tree first");
+    afmm_status st = set_device(h);
+    if (st) return st;
+    if (!h->chunk_valid && (st = build_chunks(h))) return st;
+    if (K) *K = h->chunk_K;
+    if (bounds) std::copy(h->chunk_bounds.begin(), h->chunk_bounds.end(), bounds);
+    if (order) std::copy(h->chunk_order.begin(), h->chunk_order.end(), order);
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_p2p_eval_chunked(afmm_p2p *h, float *ax, float *ay, float *az, float *phi) {
+    CHECK_HANDLE(h);
+    if (!h->d_bodies || !h->have_tree) return fail(h, AFMM_ESTATE, "eval_chunked: set_bodies and set_tree first");
+    if (!ax || !ay || !az || !phi) return fail(h, AFMM_EINVAL, "eval_chunked: null output pointer");
+    afmm_status st = set_device(h);
+    if (st) return st;
+    if ((st = launch_chunked(h, ax, ay, az, phi, false))) return st;
+    h->bodies_pending = false;
+    return h->comm ? comm_finish(h) : AFMM_OK;
+}
+
+extern "C" afmm_status afmm_p2p_publish_chunks(afmm_p2p *h, int count, void *stream) {
+    CHECK_HANDLE(h);
+    if (!h->chunk_valid) return fail(h, AFMM_ESTATE, "publish_chunks: no chunk plan (call eval_chunked first)");
+    if (count < 1 || count > h->chunk_K)
+        return fail(h, AFMM_EINVAL, "publish_chunks: count %d outside [1, %d]", count, h->chunk_K);
+    afmm_status st = set_device(h);
+    if (st) return st;
+    if ((st = resolve_stream_ops(h))) return st;
+    unsigned cum = 0;
+    for (int j = 0; j < count; ++j) cum |= 1u << h->chunk_order[j];
+    const WriteValueFn write32 = reinterpret_cast<WriteValueFn>(h->write_value32);
+    const CUresult r = write32((CUstream)(stream ? static_cast<cudaStream_t>(stream) : h->stream),
+                               (CUdeviceptr)w_ready(h), (cuuint32_t)((h->epoch << 16) | cum), 0);
+    if (r != CUDA_SUCCESS) return fail(h, AFMM_ECUDA, "publish_chunks: cuStreamWriteValue32 failed (%d)", (int)r);
     return AFMM_OK;
 }
 

@@ -224,22 +224,32 @@ struct P2PParams {
     float eps2;
     double G;                // output scale: G (gravity) or 1/(8 pi mu) (Stokeslet)
     int *done;               // nullptr, or per-piece counters of finished tasks (afmm_p2p_eval_host_pipelined)
-    // streamed inputs (afmm_p2p_eval_host_pipelined): nullptr, or the number of input
-    // chunks already packed (written by the copy stream); a task whose sources reach
-    // chunk r = piece >> 16 waits until *in_ready > r.  *in_err is set if the wait
-    // times out (the copy stream never delivered: results invalid, reported as an error)
+    // streamed inputs (afmm_p2p_eval_host_pipelined; the chunked body replication of
+    // afmm_p2p_eval at world > 1): nullptr, or the mask of input chunks already in
+    // place (bit k = chunk k; written by a stream memory operation on the copy /
+    // communication stream); a task whose sources and targets lie in the chunks of
+    // need = piece >> 16 waits until (*in_ready & need) == need.  *in_err is set if
+    // a wait exceeds wait_ns (never delivered: results invalid, reported as an error)
     const unsigned *in_ready;
     int *in_err;
+    unsigned long long wait_ns;
+    unsigned in_epoch;       // *in_ready = (epoch << 16) | mask: a word of an older evaluation (another
+                             // epoch) counts as nothing delivered, so the flag is never reset between evals
+    // nullptr, or {min CTA start, max warp end} in %globaltimer ns (the kernel's
+    // device-timer span: the GPU time all-reduced over ranks, L20 SVII.A)
+    unsigned long long *tspan;
     // equal masses: nullptr, or the packed-body trailer word that the pack kernel
     // sets when some m_j differs from m_0 (0 = all equal -> the 12-op pair loop,
     // the common mass applied in the epilogue)
     const int *mass_unequal;
-    // streamed inputs only: nullptr, or a word whose bit k the pack of input chunk k
-    // sets when some mass in that chunk differs from m_0; a task whose sources lie in
-    // chunks 0..r (r = piece >> 16) runs the equal-mass loop when bits 0..r are clear
-    // (read after the task's wait_inputs, so every bit it looks at is final)
+    // streamed inputs only: nullptr, or a word whose bit k is set when some mass in
+    // input chunk k differs from m_0; a task runs the equal-mass loop when the bits
+    // of its need mask are clear (read after the task's wait_inputs, so every bit it
+    // looks at is final)
     const unsigned *mass_bits;
-    float m0;                // streamed inputs: m_0 (from the host), the equal-mass scale's mass
+    float m0;                // streamed inputs: m_0 (from the host), the equal-mass scale's mass ...
+    const float *m0_ptr;     // ... or, if not null, read from here after the task's wait (the packed
+                             // array's trailer: chunked replication, where the host does not know m_0)
     // 1: outputs are written through shared memory as whole runs of consecutive
     // targets per component (host-mapped output arrays: full PCIe lines, not 4-byte
     // pieces with byte enables)
@@ -545,21 +555,37 @@ __device__ __forceinline__ void copy_piece(const P2PParams &p, float4 *buf, uint
                     (uint32_t)(b - a) * 16u * kWords, bar);
 }
 
-// Streamed inputs: before a task's first chunk is staged, wait until the input
-// chunk its sources (and targets) reach has been packed.  Every lane acquires the
-// flag; the proxy fence orders the packed bodies before this warp's bulk copies.
-// A wait longer than ~0.5 s sets *in_err and gives up (no hang).
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
+// Streamed inputs: before a task's first chunk is staged, wait until every input
+// chunk its sources (and targets) reach has arrived: the task's need mask (high
+// 16 bits of Task.piece) must be contained in *in_ready, the mask of delivered
+// chunks (written by a stream memory operation after each chunk's copy / pack /
+// broadcast).  Every lane acquires the word; the proxy fence orders the delivered
+// bodies before this warp's bulk copies.  No hang: a wait longer than p.wait_ns
+// (globaltimer) sets *in_err, and once *in_err is set every later wait of every
+// warp returns at once (the results are invalid and reported as an error).
 __device__ __forceinline__ void wait_inputs(const P2PParams &p, int piece) {
     const unsigned need = (unsigned)piece >> 16;
+    const auto arrived = [&](unsigned v) { return (v >> 16) == p.in_epoch && (v & need) == need; };
     unsigned v;
-    for (int spin = 0;; ++spin) {
-        asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p.in_ready) : "memory");
-        if (v > need) break;
-        if (spin > (1 << 21)) {
-            if ((threadIdx.x & 31) == 0) atomicExch(p.in_err, 1);
-            break;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p.in_ready) : "memory");
+    if (!arrived(v)) {
+        const unsigned long long t0 = globaltimer_ns();
+        for (;;) {
+            __nanosleep(256);
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p.in_ready) : "memory");
+            if (arrived(v)) break;
+            if (*(volatile int *)p.in_err) break;                 // an earlier wait already timed out
+            if (globaltimer_ns() - t0 > p.wait_ns) {
+                if ((threadIdx.x & 31) == 0) atomicExch(p.in_err, 1);
+                break;
+            }
         }
-        __nanosleep(256);
     }
     asm volatile("fence.proxy.async.global;" ::: "memory");
 }
@@ -649,11 +675,19 @@ __device__ __forceinline__ void load_targets(Targets &T, const float4 *__restric
     }
 }
 
-// kStream: the streamed host evaluation's features (input-chunk waits, per-task
-// equal-mass test, finished-task counters, coalesced host-mapped output stores);
-// a separate instantiation so the device path carries none of their registers.
+// kStream: the streamed features (input-chunk waits, per-task equal-mass test,
+// finished-task counters, coalesced host-mapped output stores); a separate
+// instantiation so the device path carries none of their registers.
+// Register budget pinned at kMaxRegs (= 160: 12 warps x 32 lanes x 160 = 61,440 of
+// the SM's 65,536 registers), so the 4,096 left always hold one 128-thread x
+// 32-register pack_chunk_kernel block beside a P2P CTA (the streamed inputs of
+// afmm_p2p_eval_host_pipelined); afmm_p2p_create re-checks the fit from the
+// built kernels' attributes (co_resident_pack) and the pipelined evaluation falls
+// back to packing every chunk before the launch when it does not hold.
+constexpr int kMaxRegs = 160;
+static_assert(kMinBlocksPerSM == 1 && kMaxRegs * kThreads <= 65536, "register budget: one CTA per SM");
 template <class Law, bool kStream = false>
-__global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const __grid_constant__ P2PParams p) {
+__global__ void __maxnreg__(kMaxRegs) p2p_kernel_t(const __grid_constant__ P2PParams p) {
     extern __shared__ __align__(128) unsigned char dsmem[];
     __shared__ __align__(8) uint64_t full_all[kWarps][kWStages];
     __shared__ ChunkMeta meta_all[kWarps][kWStages];
@@ -665,6 +699,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
     if (lane == 0) {
         for (int s = 0; s < kWStages; ++s) mbar_init(&full[s], 1);
         fence_mbar_init();
+        if (p.tspan && warp == 0) atomicMin(p.tspan, globaltimer_ns());
     }
     __syncwarp();
 #if AFMM_PROF
@@ -692,7 +727,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
 
     const float2 e2 = make_float2(p.eps2, p.eps2);
     bool eqm = Law::kHasEq && p.mass_unequal != nullptr && *p.mass_unequal == 0;
-    const double scale_eq = p.G * (double)(kStream ? p.m0 : p.bodies[0].w);   // G m for equal masses
+    double scale_eq = p.G * (double)(kStream ? p.m0 : p.bodies[0].w);   // G m for equal masses
     double scale = eqm ? scale_eq : p.G;                               // else G
     float scale_f = (float)scale;
     bool scale_exact = (double)scale_f == scale;
@@ -736,9 +771,8 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
             if (kStream && Law::kHasEq && p.mass_bits) {         // streamed inputs: per-task equal-mass test
                 unsigned b;
                 asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(b) : "l"(p.mass_bits) : "memory");
-                const unsigned r = (unsigned)m.piece >> 16;
-                const unsigned mask = r >= 31 ? 0xffffffffu : (2u << r) - 1u;
-                eqm = (b & mask) == 0;
+                eqm = (b & ((unsigned)m.piece >> 16)) == 0;
+                if (p.m0_ptr) scale_eq = p.G * (double)*(const volatile float *)p.m0_ptr;
                 scale = eqm ? scale_eq : p.G;
                 scale_f = (float)scale;
                 scale_exact = (double)scale_f == scale;
@@ -869,6 +903,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const 
         PROF_ADD(5, t_s);
     }
     if (p.n_win > 1) __threadfence_system();   // peer-window stores performed before the kernel completes
+    if (p.tspan && lane == 0) atomicMax(p.tspan + 1, globaltimer_ns());
 #if AFMM_PROF
     PROF_ADD(8, t_all);
     unsigned long long gt1;
@@ -929,11 +964,14 @@ __global__ void __launch_bounds__(128, 16) pack_chunk_kernel(int n, const float 
     if (__any_sync(0xffffffffu, diff) && (threadIdx.x & 31) == 0) atomicOr(mass_bits, 1u << chunk);
 }
 
-// SoA -> packed {x, y, z, m}; *unequal |= (some m_i != m_0) (the equal-mass flag)
+// SoA -> packed {x, y, z, m}; the trailer after the bodies: unequal[0] = -1 (all
+// bits) when some m_i != m_0 (the equal-mass flag, zeroed before), unequal[1] =
+// m_0's bits (the equal-mass scale for ranks that receive the packed array)
 __global__ void pack_bodies_kernel(long long n, const float *__restrict__ x, const float *__restrict__ y,
                                    const float *__restrict__ z, const float *__restrict__ m,
                                    float4 *__restrict__ out, int *__restrict__ unequal) {
     const float m0 = m[0];
+    if (blockIdx.x == 0 && threadIdx.x == 0) unequal[1] = __float_as_int(m0);
     bool diff = false;
     for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n;
          i += (long long)gridDim.x * blockDim.x) {
@@ -941,7 +979,12 @@ __global__ void pack_bodies_kernel(long long n, const float *__restrict__ x, con
         out[i] = make_float4(x[i], y[i], z[i], mi);
         diff |= mi != m0;
     }
-    if (__any_sync(0xffffffffu, diff) && (threadIdx.x & 31) == 0) atomicOr(unequal, 1);
+    if (__any_sync(0xffffffffu, diff) && (threadIdx.x & 31) == 0) atomicOr(unequal, -1);
+}
+
+// kernel_ms[0] = the device-timer span of the last P2P launch in ms (0 if none ran)
+__global__ void span_ms_kernel(const unsigned long long *__restrict__ tspan, double *__restrict__ kernel_ms) {
+    kernel_ms[0] = tspan[1] > tspan[0] ? (double)(tspan[1] - tspan[0]) * 1e-6 : 0.0;
 }
 
 

@@ -21,6 +21,13 @@ CPU in the tests).
                                   (no NCCL gather); complete after a barrier.
 * allgather_scalar(v, device)  -- a8: per-rank kernel times for the GPU time
                                   (max over GPUs, L20 SVII.A) and the rebalance.
+* deliver_chunks(h, stream, src) -- a4 overlapped, caller-driven: after
+                                  h.eval_chunked(...) the packed bodies go out
+                                  chunk by chunk in the library's delivery order
+                                  (afmm_p2p_chunks), each chunk published to the
+                                  running kernel (afmm_p2p_publish_chunks) as soon
+                                  as it is in place.  (With a library communicator,
+                                  P2P(nccl_id=...), eval does this itself over NCCL.)
 """
 from __future__ import annotations
 
@@ -93,6 +100,42 @@ def open_peer_windows(h, out):
         for b in bases:
             ipc_close(b)
     return close
+
+
+def deliver_chunks(h, stream, src=0):
+    """Replicate h's packed body array from rank `src` chunk by chunk, after
+    h.eval_chunked(...) launched the kernel: the 16-byte trailer first, then the
+    chunks in delivery order, each followed by h.publish_chunks(j + 1) on `stream`
+    (a torch.cuda.Stream other than the kernel's).  NCCL: device broadcasts on
+    `stream`; gloo: staged through host memory (tests on one GPU).
+    `stream` must have been ordered after the handle's earlier work (readers of
+    the old bodies) BEFORE eval_chunked was called -- ordering it after the
+    handle's stream now would wait for the kernel, which waits for the chunks."""
+    bounds, order = h.chunks()
+    ptr, nbytes = h.bodies_buffer()
+    dev = torch.device("cuda", torch.cuda.current_device())
+    packed = torch.as_tensor(_DeviceArray(ptr, nbytes), device=dev)    # float32 view, 4 per body + trailer
+    n4 = int(bounds[-1]) * 4
+    gloo = dist.get_backend() == "gloo"
+    rank = dist.get_rank()
+
+    def bcast(view):
+        if not gloo:
+            dist.broadcast(view, src=src)
+            return
+        stream.synchronize()
+        buf = view.cpu() if rank == src else torch.empty(view.shape, dtype=view.dtype)
+        dist.broadcast(buf, src=src)
+        if rank != src:
+            view.copy_(buf, non_blocking=False)
+
+    with torch.cuda.stream(stream):
+        bcast(packed[n4:n4 + 4])
+        for j, c in enumerate(order):
+            lo, hi = int(bounds[c]) * 4, int(bounds[c + 1]) * 4
+            if hi > lo:
+                bcast(packed[lo:hi])
+            h.publish_chunks(j + 1, stream.cuda_stream)
 
 
 def allgather_scalar(v: float, device) -> np.ndarray:
