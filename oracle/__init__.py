@@ -182,6 +182,12 @@ class Tree:
         return tuple(_c(a, np.float32)[self.perm] for a in arrs)
 
 
+def set_threads(n: int) -> None:
+    """OpenMP threads of the oracle's parallel loops (omp_set_num_threads of the
+    libgomp the oracle links; e.g. 1 for a one-core baseline).  No arithmetic."""
+    _L().omp_set_num_threads(int(n))
+
+
 def kick(vx, vy, vz, ax, ay, az, h):
     """Leapfrog kick v <- v + h a (fp64 arithmetic on fp32 state, one rounding)."""
     v = [np.array(a, np.float32) for a in (vx, vy, vz)]

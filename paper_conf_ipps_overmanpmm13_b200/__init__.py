@@ -66,6 +66,8 @@ _p, _i, _ll, _d = C.c_void_p, C.c_int, C.c_longlong, C.c_double
 
 
 def _sig(name, res, *args):
+    if os.environ.get("AFMM_LIB_OVERRIDE") and not hasattr(_lib, name):
+        return None                       # tools/tune: an older build without this entry point
     f = getattr(_lib, name)
     f.restype = res
     f.argtypes = list(args)
@@ -116,6 +118,7 @@ _sig("afmm_kick", _i, _ll, _p, _p, _p, _p, _p, _p, C.c_float, _p)
 _sig("afmm_drift", _i, _ll, _p, _p, _p, _p, _p, _p, C.c_float, _p)
 _sig("afmm_fp32_peak", _i, _i, C.POINTER(_d), C.POINTER(_d), C.POINTER(_d))
 _sig("afmm_version", C.c_char_p)
+_sig("afmm_launch_count", C.c_longlong)
 _sig("afmm_tree_create", _i, _i, _p, C.POINTER(_p))
 _sig("afmm_tree_build", _i, _p, _ll, _p, _p, _p, _i, _i, _p, _i)
 _sig("afmm_tree_enforce", _i, _p, _ll, _p, _p, _p, _i)
@@ -175,7 +178,7 @@ EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
             "afmm_tree_rebuild", "afmm_tree_nodes", "afmm_fine_grained", "afmm_p2p_eval_host_pipelined",
             "afmm_p2p_set_peer_windows", "afmm_ipc_export", "afmm_ipc_import", "afmm_ipc_close",
             "afmm_tree_gather_rows", "afmm_p2p_nccl_id", "afmm_p2p_chunks", "afmm_p2p_eval_chunked",
-            "afmm_p2p_publish_chunks"]
+            "afmm_p2p_publish_chunks", "afmm_launch_count"]
 
 
 def ipc_export(dev_ptr):
@@ -207,6 +210,11 @@ def ipc_close(base):
 
 def version() -> str:
     return _lib.afmm_version().decode()
+
+
+def launch_count() -> int:
+    """afmm_launch_count: this library's kernels launched so far in this process."""
+    return int(_lib.afmm_launch_count())
 
 
 def nccl_id() -> bytes:

@@ -7,6 +7,7 @@
 // cudaEvent timing (PAPER L20 SVII.A).  Rows a4/a7 (replication, gather) are
 // collectives issued by the caller on the buffers this library exposes.
 #include <algorithm>
+#include <atomic>
 #include <climits>
 #include <cmath>
 #include <cstdarg>
@@ -25,6 +26,13 @@
 
 using afmm::Seg;
 using afmm::Task;
+
+// Kernels of this library launched so far (afmm_launch_count): every <<<>>> site
+// below counts itself; CUB's scans / sorts inside the device ingest are not ours
+// and are not counted.  A pipelined eval whose input chain replays from a CUDA
+// graph counts the graph's K pack kernels.
+static std::atomic<long long> g_launches{0};
+#define COUNT_LAUNCH(k) g_launches.fetch_add((k), std::memory_order_relaxed)
 
 struct afmm_p2p {
     afmm_p2p_config cfg{};
@@ -210,7 +218,7 @@ unsigned long long wait_ns(const afmm_p2p *) {
 // (tests of the fallback).
 cudaError_t co_residency(int device, bool *ok) {
     cudaFuncAttributes fp{}, fk{};
-    cudaError_t e = cudaFuncGetAttributes(&fp, afmm::p2p_kernel_t<afmm::Gravity, true>);
+    cudaError_t e = cudaFuncGetAttributes(&fp, afmm::p2p_stream_kernel_t<afmm::Gravity>);
     if (e == cudaSuccess) e = cudaFuncGetAttributes(&fk, afmm::pack_chunk_kernel);
     int regs = 0, smem = 0, thr = 0, rsv = 0, blk = 0;
     if (e == cudaSuccess) e = cudaDeviceGetAttribute(&regs, cudaDevAttrMaxRegistersPerMultiprocessor, device);
@@ -402,7 +410,7 @@ extern "C" afmm_status afmm_p2p_create(const afmm_p2p_config *cfg, afmm_p2p **ou
             e = cudaFuncSetAttribute(afmm::p2p_kernel_t<afmm::Gravity>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                      afmm::kDynSmem);
         if (e == cudaSuccess)
-            e = cudaFuncSetAttribute(afmm::p2p_kernel_t<afmm::Gravity, true>,
+            e = cudaFuncSetAttribute(afmm::p2p_stream_kernel_t<afmm::Gravity>,
                                      cudaFuncAttributeMaxDynamicSharedMemorySize, afmm::kDynSmem);
         if (e == cudaSuccess)
             e = cudaFuncSetAttribute(afmm::p2p_kernel_t<afmm::Stokeslet>,
@@ -511,6 +519,7 @@ static afmm_status pack(afmm_p2p *h, const float *x, const float *y, const float
     int *flag = mass_flag(h);
     CUDA_TRY(h, cudaMemsetAsync(flag, 0, sizeof(int), h->stream));
     afmm::pack_bodies_kernel<<<(int)blocks, threads, 0, h->stream>>>(h->n, x, y, z, m, h->d_bodies, flag);
+    COUNT_LAUNCH(1);
     CUDA_TRY(h, cudaGetLastError());
     return AFMM_OK;
 }
@@ -529,9 +538,7 @@ extern "C" afmm_status afmm_p2p_set_bodies(afmm_p2p *h, long long n, const float
     if (nn == 4) return pack(h, x, y, z, m);
     // allocate only: the equal-mass flag reads "unequal" until a full-buffer
     // broadcast (afmm_p2p_bodies_buffer, trailer included) brings the root's
-    static const int unequal = -1;
-    CUDA_TRY(h, cudaMemcpyAsync(mass_flag(h), &unequal, sizeof(int), cudaMemcpyHostToDevice, h->stream));
-    CUDA_TRY(h, cudaStreamSynchronize(h->stream));
+    CUDA_TRY(h, cudaMemsetAsync(mass_flag(h), 0xff, sizeof(int), h->stream));   // -1: "unequal"
     return AFMM_OK;
 }
 
@@ -578,6 +585,7 @@ extern "C" afmm_status afmm_p2p_set_bodies_stokeslet(afmm_p2p *h, long long n, c
     const int threads = 256;
     long long blocks = std::min<long long>((n + threads - 1) / threads, (long long)h->num_sms * 16);
     afmm::pack_stokeslet_kernel<<<(int)blocks, threads, 0, h->stream>>>(n, x, y, z, fx, fy, fz, h->d_bodies);
+    COUNT_LAUNCH(1);
     CUDA_TRY(h, cudaGetLastError());
     return AFMM_OK;
 }
@@ -604,13 +612,11 @@ static void compute_body_split(afmm_p2p *h) {
 #include "worklist.inc"
 #include "worklist_dev.cuh"
 
-extern "C" afmm_status afmm_p2p_set_tree(afmm_p2p *h, int n_leaves, const int *leaf_start,
-                                         const int *leaf_count, const long long *u_off,
-                                         const int *u_idx) {
-    CHECK_HANDLE(h);
-    if (h->n < 1 || !h->d_bodies) return fail(h, AFMM_ESTATE, "set_tree: call set_bodies first");
-    if (n_leaves < 1 || !leaf_start || !leaf_count || !u_off)
-        return fail(h, AFMM_EINVAL, "set_tree: n_leaves=%d / null pointer", n_leaves);
+// The host work-list builder (worklist.inc): validation, Interactions(t), the
+// partition and this rank's tasks computed on the CPU.  The reference the device
+// ingest is tested against (AFMM_HOST_INGEST=1 selects it for afmm_p2p_set_tree).
+static afmm_status set_tree_host_builder(afmm_p2p *h, int n_leaves, const int *leaf_start, const int *leaf_count,
+                                         const long long *u_off, const int *u_idx) {
     // leaves must tile [0, n) exactly, 1 <= count <= max_leaf
     long long expect = 0;
     for (int t = 0; t < n_leaves; ++t) {
@@ -690,21 +696,21 @@ __global__ void body_split_kernel(int G, int L, long long n, const long long *__
     if (r <= G) bsplit[r] = split[r] >= L ? n : ls[split[r]];
 }
 
-extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const int *leaf_start,
-                                                const int *leaf_count, const long long *u_off,
-                                                const int *u_idx) {
+enum DwsSlot { sI, sP, sW, sPW, sSplit, sErr, sNseg, sNtask, sNsrc, sSegOff, sTaskOff, sStats, sKeys, sVals, sKeys2,
+               sVals2, sTasksU, sCoef, sTmp, sBsplit, sPlan, sPlanHdr, sNnz,
+               sOwnLS, sOwnLC, sOwnUO, sOwnUI };             // the handle's own copy of the tree (re-ingest)
+
+// Device ingest (validation, Interactions(t), partition, this rank's work list)
+// of the tree arrays ls/lc/uo/ui in device memory.  keep: afterwards also copy
+// them into the handle's own buffers (sOwn*), from which set_partition /
+// rebalance re-ingest the same tree (the caller's arrays may be gone by then).
+static afmm_status ingest(afmm_p2p *h, int n_leaves, const int *leaf_start, const int *leaf_count,
+                          const long long *u_off, const int *u_idx, bool keep) {
     using namespace afmm;
-    CHECK_HANDLE(h);
-    if (h->n < 1 || !h->d_bodies) return fail(h, AFMM_ESTATE, "set_tree_device: call set_bodies first");
-    if (n_leaves < 1 || !leaf_start || !leaf_count || !u_off || !u_idx)
-        return fail(h, AFMM_EINVAL, "set_tree_device: n_leaves=%d / null pointer", n_leaves);
-    afmm_status st = set_device(h);
-    if (st) return st;
+    afmm_status st;
     cudaStream_t s = h->stream;
     const int L = n_leaves, W = h->cfg.world, TH = 256;
     auto grid = [&](long long m) { return (int)std::max<long long>(1, (m + TH - 1) / TH); };
-    enum { sI, sP, sW, sPW, sSplit, sErr, sNseg, sNtask, sNsrc, sSegOff, sTaskOff, sStats, sKeys, sVals, sKeys2,
-           sVals2, sTasksU, sCoef, sTmp, sBsplit, sPlan, sPlanHdr };
     long long *I, *P, *split, *nsrc, *bsplit;
     unsigned short *plan;
     int4 *plan_hdr;
@@ -717,6 +723,7 @@ extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const
     CUDA_TRY(h, cudaMemsetAsync(err, 0, sizeof(int), s));
     dev::validate_interactions_kernel<<<grid(L), TH, 0, s>>>(L, h->n, h->cfg.max_leaf, leaf_start, leaf_count,
                                                             u_off, u_idx, I, err);
+    COUNT_LAUNCH(1);
     CUDA_TRY(h, cudaGetLastError());
     // the flags ride with the partition's results (one synchronise instead of two): the
     // partition kernels only touch L- and W-sized arrays, and nothing of the handle's
@@ -741,29 +748,45 @@ extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const
         if ((st = dws(h, sW, &w, L)) || (st = dws(h, sPW, &pw, L)) || (st = dws(h, sCoef, &coef, 8))) return st;
         CUDA_TRY(h, cudaMemcpyAsync(coef, h->coef, 8 * sizeof(double), cudaMemcpyHostToDevice, s));
         dev::weights_kernel<<<grid(L), TH, 0, s>>>(L, leaf_count, I, coef, w);
+        COUNT_LAUNCH(1);
         size_t tb = 0;
         CUDA_TRY(h, cub::DeviceScan::InclusiveSum(nullptr, tb, w, pw, L, s));
         char *tmp;
         if ((st = dws(h, sTmp, &tmp, tb))) return st;
         CUDA_TRY(h, cub::DeviceScan::InclusiveSum(tmp, tb, w, pw, L, s));
         dev::weighted_cut_kernel<<<1, 1, 0, s>>>(L, W, pw, split);
+        COUNT_LAUNCH(1);
         clear_user = true;
     } else {
         dev::literal_cut_kernel<<<1, 1, 0, s>>>(L, W, P, split);
+        COUNT_LAUNCH(1);
         clear_user = true;
     }
     CUDA_TRY(h, cudaGetLastError());
     body_split_kernel<<<(W + 1 + 63) / 64, 64, 0, s>>>(W, L, h->n, split, leaf_start, bsplit);
+    COUNT_LAUNCH(1);
     std::vector<long long> lsplit(W + 1, 0), bsplit_h(W + 1, 0);
-    long long itot = 0;
+    long long itot = 0, nnz = 0;
     CUDA_TRY(h, cudaMemcpyAsync(lsplit.data(), split, (W + 1) * sizeof(long long), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(h, cudaMemcpyAsync(bsplit_h.data(), bsplit, (W + 1) * sizeof(long long), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(h, cudaMemcpyAsync(&itot, P + (L - 1), sizeof(long long), cudaMemcpyDeviceToHost, s));
+    if (keep) CUDA_TRY(h, cudaMemcpyAsync(&nnz, u_off + L, sizeof(long long), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(h, cudaStreamSynchronize(s));
     const int herr = *(volatile int *)h->h_ingest_err;
     if (herr)
-        return fail(h, AFMM_EINVAL, "set_tree_device: invalid tree (flags 0x%x: 1 start, 2 count, 4 cover, "
+        return fail(h, AFMM_EINVAL, "set_tree: invalid tree (flags 0x%x: 1 start, 2 count, 4 cover, "
                                     "8 u_off, 16 u_idx range, 32 row order)", herr);
+    if (keep) {                                    // the handle's own copy, for set_partition / rebalance
+        int *ols, *olc, *oui;
+        long long *ouo;
+        if ((st = dws(h, sOwnLS, &ols, L)) || (st = dws(h, sOwnLC, &olc, L)) || (st = dws(h, sOwnUO, &ouo, L + 1)) ||
+            (st = dws(h, sOwnUI, &oui, (size_t)std::max<long long>(nnz, 1))))
+            return st;
+        CUDA_TRY(h, cudaMemcpyAsync(ols, leaf_start, L * sizeof(int), cudaMemcpyDeviceToDevice, s));
+        CUDA_TRY(h, cudaMemcpyAsync(olc, leaf_count, L * sizeof(int), cudaMemcpyDeviceToDevice, s));
+        CUDA_TRY(h, cudaMemcpyAsync(ouo, u_off, (L + 1) * sizeof(long long), cudaMemcpyDeviceToDevice, s));
+        if (nnz > 0) CUDA_TRY(h, cudaMemcpyAsync(oui, u_idx, nnz * sizeof(int), cudaMemcpyDeviceToDevice, s));
+    }
     if (clear_user) h->user_partition = false;
     h->leaf_split = std::move(lsplit);
     h->body_split = std::move(bsplit_h);
@@ -784,6 +807,7 @@ extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const
     if (m > 0) {
         dev::count_kernel<<<grid(m), TH, 0, s>>>(m, lo, leaf_start, leaf_count, u_off, u_idx, I, nseg, ntask, nsrc,
                                                 stats, cap, plan, plan_hdr);
+        COUNT_LAUNCH(1);
         CUDA_TRY(h, cudaGetLastError());
     }
     {
@@ -810,6 +834,7 @@ extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const
     if (m > 0) {
         dev::write_kernel<<<grid(m), TH, 0, s>>>(m, lo, leaf_start, leaf_count, u_off, u_idx, seg_off, task_off,
                                                 ntask, nsrc, h->d_segs, tasks_u, keys, vals, plan, plan_hdr);
+        COUNT_LAUNCH(1);
         CUDA_TRY(h, cudaGetLastError());
     }
     if (nt > 0) {
@@ -821,6 +846,7 @@ extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const
         // the high half is constant, so the low 32 bits give the same stable order
         CUDA_TRY(h, cub::DeviceRadixSort::SortPairs(tmp, tb, keys, keys2, vals, vals2, nt, 0, 32, s));
         dev::gather_tasks_kernel<<<grid(nt), TH, 0, s>>>(nt, vals2, tasks_u, h->d_tasks);
+        COUNT_LAUNCH(1);
         CUDA_TRY(h, cudaGetLastError());
     }
     h->n_tasks = nt;
@@ -842,12 +868,80 @@ extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const
     return AFMM_OK;
 }
 
+// re-ingest the current tree from the handle's own copy (after a partition change)
+static afmm_status reingest(afmm_p2p *h) {
+    int *ols, *olc, *oui;
+    long long *ouo;
+    afmm_status st;
+    const int L = h->L;
+    if ((st = dws(h, sOwnLS, &ols, L)) || (st = dws(h, sOwnLC, &olc, L)) || (st = dws(h, sOwnUO, &ouo, L + 1)) ||
+        (st = dws(h, sOwnUI, &oui, 1)))
+        return st;
+    return ingest(h, L, ols, olc, ouo, oui, false);
+}
+
+extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const int *leaf_start,
+                                                const int *leaf_count, const long long *u_off,
+                                                const int *u_idx) {
+    CHECK_HANDLE(h);
+    if (h->n < 1 || !h->d_bodies) return fail(h, AFMM_ESTATE, "set_tree_device: call set_bodies first");
+    if (n_leaves < 1 || !leaf_start || !leaf_count || !u_off || !u_idx)
+        return fail(h, AFMM_EINVAL, "set_tree_device: n_leaves=%d / null pointer", n_leaves);
+    afmm_status st = set_device(h);
+    if (st) return st;
+    return ingest(h, n_leaves, leaf_start, leaf_count, u_off, u_idx, true);
+}
+
+// Host tree ingest: the arrays are copied into the handle's own device buffers
+// and ingested there by the kernels of afmm_p2p_set_tree_device (validation,
+// Interactions(t), partition and work list on the GPU; a few scalars come back).
+// AFMM_HOST_INGEST=1: the host builder instead (reference for the tests).
+extern "C" afmm_status afmm_p2p_set_tree(afmm_p2p *h, int n_leaves, const int *leaf_start,
+                                         const int *leaf_count, const long long *u_off,
+                                         const int *u_idx) {
+    CHECK_HANDLE(h);
+    if (h->n < 1 || !h->d_bodies) return fail(h, AFMM_ESTATE, "set_tree: call set_bodies first");
+    if (n_leaves < 1 || !leaf_start || !leaf_count || !u_off)
+        return fail(h, AFMM_EINVAL, "set_tree: n_leaves=%d / null pointer", n_leaves);
+    const long long nnz = u_off[n_leaves];
+    if (nnz < 0 || (nnz > 0 && !u_idx)) return fail(h, AFMM_EINVAL, "set_tree: u_off[n_leaves]=%lld / u_idx null", nnz);
+    afmm_status st = set_device(h);
+    if (st) return st;
+    const char *hb = getenv("AFMM_HOST_INGEST");
+    if (hb && hb[0] == '1') return set_tree_host_builder(h, n_leaves, leaf_start, leaf_count, u_off, u_idx);
+    const int L = n_leaves;
+    int *ols, *olc, *oui;
+    long long *ouo;
+    if ((st = dws(h, sOwnLS, &ols, L)) || (st = dws(h, sOwnLC, &olc, L)) || (st = dws(h, sOwnUO, &ouo, L + 1)) ||
+        (st = dws(h, sOwnUI, &oui, (size_t)std::max<long long>(nnz, 1))))
+        return st;
+    CUDA_TRY(h, cudaMemcpyAsync(ols, leaf_start, L * sizeof(int), cudaMemcpyHostToDevice, h->stream));
+    CUDA_TRY(h, cudaMemcpyAsync(olc, leaf_count, L * sizeof(int), cudaMemcpyHostToDevice, h->stream));
+    CUDA_TRY(h, cudaMemcpyAsync(ouo, u_off, (L + 1) * sizeof(long long), cudaMemcpyHostToDevice, h->stream));
+    if (nnz > 0) CUDA_TRY(h, cudaMemcpyAsync(oui, u_idx, nnz * sizeof(int), cudaMemcpyHostToDevice, h->stream));
+    return ingest(h, L, ols, olc, ouo, oui, false);
+}
+
 extern "C" afmm_status afmm_p2p_set_partition(afmm_p2p *h, const long long *leaf_split) {
     CHECK_HANDLE(h);
-    if (h->tree_on_device && h->have_tree)
-        return fail(h, AFMM_ESTATE, "set_partition: the tree was ingested from device memory; "
-                                    "set the partition before set_tree_device or use set_tree");
     const int W = h->cfg.world;
+    if (h->tree_on_device) {                           // re-ingest the handle's copy of the tree
+        if (!leaf_split) {
+            h->user_partition = false;
+        } else {
+            if (leaf_split[0] != 0) return fail(h, AFMM_EINVAL, "set_partition: leaf_split[0] != 0");
+            for (int r = 0; r < W; ++r)
+                if (leaf_split[r + 1] < leaf_split[r]) return fail(h, AFMM_EINVAL, "set_partition: not monotone");
+            if (h->have_tree && leaf_split[W] != h->L)
+                return fail(h, AFMM_EINVAL, "set_partition: leaf_split[world]=%lld != n_leaves=%d", leaf_split[W], h->L);
+            h->leaf_split.assign(leaf_split, leaf_split + W + 1);
+            h->user_partition = true;
+        }
+        if (!h->have_tree) return AFMM_OK;
+        afmm_status st = set_device(h);
+        if (st) return st;
+        return reingest(h);
+    }
     if (!leaf_split) {
         h->user_partition = false;
         if (!h->have_tree) return AFMM_OK;
@@ -1012,15 +1106,36 @@ extern "C" afmm_status afmm_p2p_rebalance(afmm_p2p *h, const double *rank_ms, do
     CHECK_HANDLE(h);
     if (changed) *changed = 0;
     if (!h->have_tree) return fail(h, AFMM_ESTATE, "rebalance: no tree");
-    if (h->tree_on_device)
-        return fail(h, AFMM_ESTATE, "rebalance: the tree was ingested from device memory; "
-                                    "use afmm_cost_fit + afmm_p2p_set_cost_coef before the next set_tree_device");
     if (!rank_ms) return fail(h, AFMM_EINVAL, "rebalance: rank_ms is null");
     const int W = h->cfg.world;
     std::vector<long long> split(W + 1);
     int ch = 0;
-    afmm_status st = afmm_partition_rebalance(h->L, h->leaf_count.data(), h->I.data(), W,
-                                              h->leaf_split.data(), rank_ms, threshold, split.data(), &ch);
+    afmm_status st;
+    if (h->tree_on_device) {
+        // the work list was built on the GPU: leaf sizes and Interactions(t) of the
+        // current tree come back from the handle's buffers, the new cut re-ingests it
+        if ((st = set_device(h))) return st;
+        std::vector<int> lc(h->L);
+        std::vector<long long> I(h->L);
+        int *olc;
+        long long *dI;
+        if ((st = dws(h, sOwnLC, &olc, h->L)) || (st = dws(h, sI, &dI, h->L))) return st;
+        CUDA_TRY(h, cudaMemcpyAsync(lc.data(), olc, h->L * sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+        CUDA_TRY(h, cudaMemcpyAsync(I.data(), dI, h->L * sizeof(long long), cudaMemcpyDeviceToHost, h->stream));
+        CUDA_TRY(h, cudaStreamSynchronize(h->stream));
+        st = afmm_partition_rebalance(h->L, lc.data(), I.data(), W, h->leaf_split.data(), rank_ms, threshold,
+                                      split.data(), &ch);
+        if (st) return fail(h, st, "rebalance: invalid rank_ms or partition");
+        if (ch) {
+            h->leaf_split = split;
+            h->user_partition = true;
+            if ((st = reingest(h))) return st;
+            if (changed) *changed = 1;
+        }
+        return AFMM_OK;
+    }
+    st = afmm_partition_rebalance(h->L, h->leaf_count.data(), h->I.data(), W,
+                                  h->leaf_split.data(), rank_ms, threshold, split.data(), &ch);
     if (st) return fail(h, st, "rebalance: invalid rank_ms or partition");
     if (ch) {
         h->leaf_split = split;
@@ -1109,6 +1224,7 @@ static afmm_status launch_eval(afmm_p2p *h, float *ax, float *ay, float *az, flo
             afmm::p2p_kernel_t<afmm::Stokeslet><<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(p);
         else
             afmm::p2p_kernel_t<afmm::Gravity><<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(p);
+        COUNT_LAUNCH(1);
         CUDA_TRY(h, cudaGetLastError());
         nlaunch = 1;
     }
@@ -1466,7 +1582,8 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
             prm.m0_ptr = nullptr;
             prm.tspan = h->comm ? w_tspan(h) : nullptr;
             const int grid = std::max(1, std::min((nt + afmm::kWarps - 1) / afmm::kWarps, h->num_sms * h->blocks_per_sm));
-            afmm::p2p_kernel_t<afmm::Gravity, true><<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(prm);
+            afmm::p2p_stream_kernel_t<afmm::Gravity><<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(prm);
+            COUNT_LAUNCH(1);
             CUDA_TRY(h, cudaGetLastError());
             nlaunch = 1;
         }
@@ -1499,6 +1616,7 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
                 const int blocks = (int)std::min<long long>((hi - lo + threads - 1) / threads, (long long)h->num_sms);
                 afmm::pack_chunk_kernel<<<blocks, threads, 0, h->s_in>>>((int)(hi - lo), src[0], src[1], src[2],
                                                                         src[3], h->d_bodies + lo, m0, mass_bits, k);
+                if (!capturing) COUNT_LAUNCH(1);          // a captured chain counts when its graph replays
                 const cudaError_t le = cudaPeekAtLastError();
                 if (le != cudaSuccess) {
                     if (capturing) return AFMM_ECUDA;
@@ -1552,7 +1670,10 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
                 for (int a = 0; a < 4; ++a) h->ig_src[a] = zin[a];
             }
         }
-        if (use_graph) CUDA_TRY(h, cudaGraphLaunch(h->in_graph, h->s_in));
+        if (use_graph) {
+            CUDA_TRY(h, cudaGraphLaunch(h->in_graph, h->s_in));
+            COUNT_LAUNCH(K);
+        }
     }
     h->last_input_graph = use_graph;
     if (!use_graph) {
@@ -1734,7 +1855,8 @@ static afmm_status launch_chunked(afmm_p2p *h, float *ax, float *ay, float *az, 
     if (p.n_tasks > 0) {
         const int room = std::max(1, h->num_sms * h->blocks_per_sm - comm_sms(h));
         const int grid = std::max(1, std::min((p.n_tasks + afmm::kWarps - 1) / afmm::kWarps, room));
-        afmm::p2p_kernel_t<afmm::Gravity, true><<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(p);
+        afmm::p2p_stream_kernel_t<afmm::Gravity><<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(p);
+        COUNT_LAUNCH(1);
         CUDA_TRY(h, cudaGetLastError());
         nlaunch = 1;
     }
@@ -1758,6 +1880,7 @@ static afmm_status launch_chunked(afmm_p2p *h, float *ax, float *ay, float *az, 
 static afmm_status comm_finish(afmm_p2p *h) {
     const afmm::NcclApi &nc = afmm::nccl_api();
     afmm::span_ms_kernel<<<1, 1, 0, h->stream>>>(w_tspan(h), w_kms(h));
+    COUNT_LAUNCH(1);
     CUDA_TRY(h, cudaGetLastError());
     CUDA_TRY(h, cudaEventRecord(h->ev_c2, h->stream));
     CUDA_TRY(h, cudaStreamWaitEvent(h->s_comm, h->ev_c2, 0));
@@ -1876,6 +1999,8 @@ extern "C" afmm_status afmm_ipc_close(void *base) {
     }
     return AFMM_OK;
 }
+
+extern "C" long long afmm_launch_count(void) { return g_launches.load(std::memory_order_relaxed); }
 
 extern "C" afmm_status afmm_p2p_stats_get(afmm_p2p *h, afmm_p2p_stats *stats) {
     CHECK_HANDLE(h);

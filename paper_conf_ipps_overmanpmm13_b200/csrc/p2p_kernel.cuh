@@ -53,6 +53,9 @@ namespace afmm {
 #ifndef AFMM_PACK_WIDE
 #define AFMM_PACK_WIDE 1                          // pack_chunk_kernel: float4 reads when aligned
 #endif
+#ifndef AFMM_TSPAN
+#define AFMM_TSPAN 1                              // device-timer span of the launch (P2PParams.tspan)
+#endif
 #ifndef AFMM_PROF
 #define AFMM_PROF 0                               // per-warp cycle breakdown (tools/prof_breakdown.py)
 #endif
@@ -686,8 +689,10 @@ __device__ __forceinline__ void load_targets(Targets &T, const float4 *__restric
 // back to packing every chunk before the launch when it does not hold.
 constexpr int kMaxRegs = 160;
 static_assert(kMinBlocksPerSM == 1 && kMaxRegs * kThreads <= 65536, "register budget: one CTA per SM");
-template <class Law, bool kStream = false>
-__global__ void __maxnreg__(kMaxRegs) p2p_kernel_t(const __grid_constant__ P2PParams p) {
+// (The device-path kernel keeps __launch_bounds__: the same 158 registers, but
+// its code under __maxnreg__ measured 1.2 % slower, profiles/r2_ab_regs.txt.)
+template <class Law, bool kStream>
+__device__ __forceinline__ void p2p_body(const P2PParams &p) {
     extern __shared__ __align__(128) unsigned char dsmem[];
     __shared__ __align__(8) uint64_t full_all[kWarps][kWStages];
     __shared__ ChunkMeta meta_all[kWarps][kWStages];
@@ -699,7 +704,7 @@ __global__ void __maxnreg__(kMaxRegs) p2p_kernel_t(const __grid_constant__ P2PPa
     if (lane == 0) {
         for (int s = 0; s < kWStages; ++s) mbar_init(&full[s], 1);
         fence_mbar_init();
-        if (p.tspan && warp == 0) atomicMin(p.tspan, globaltimer_ns());
+        if (AFMM_TSPAN && p.tspan && warp == 0) atomicMin(p.tspan, globaltimer_ns());
     }
     __syncwarp();
 #if AFMM_PROF
@@ -903,7 +908,7 @@ __global__ void __maxnreg__(kMaxRegs) p2p_kernel_t(const __grid_constant__ P2PPa
         PROF_ADD(5, t_s);
     }
     if (p.n_win > 1) __threadfence_system();   // peer-window stores performed before the kernel completes
-    if (p.tspan && lane == 0) atomicMax(p.tspan + 1, globaltimer_ns());
+    if (AFMM_TSPAN && p.tspan && lane == 0) atomicMax(p.tspan + 1, globaltimer_ns());
 #if AFMM_PROF
     PROF_ADD(8, t_all);
     unsigned long long gt1;
@@ -914,6 +919,15 @@ __global__ void __maxnreg__(kMaxRegs) p2p_kernel_t(const __grid_constant__ P2PPa
     if (lane == 0)
         for (int k = 0; k < kProfSlots; ++k) afmm_prof_buf[(blockIdx.x * kWarps + warp) * kProfSlots + k] = prof[k];
 #endif
+}
+
+template <class Law>
+__global__ void __launch_bounds__(kThreads, kMinBlocksPerSM) p2p_kernel_t(const __grid_constant__ P2PParams p) {
+    p2p_body<Law, false>(p);
+}
+template <class Law>
+__global__ void __maxnreg__(kMaxRegs) p2p_stream_kernel_t(const __grid_constant__ P2PParams p) {
+    p2p_body<Law, true>(p);
 }
 
 // Stokeslet bodies: {x, y, z, fx}, {fy, fz, 0, 0}

@@ -38,9 +38,9 @@ __global__ void validate_interactions_kernel(int L, long long n, int max_leaf, c
     if (t + 1 < L && ls[t + 1] != ls[t] + c) e |= kErrStart;
     if (t + 1 == L && (long long)ls[t] + c != n) e |= kErrCover;
     if (t == 0 && uo[0] != 0) e |= kErrOff;
-    const long long b = uo[t], en = uo[t + 1];
+    const long long b = uo[t], en = uo[t + 1], nnz = uo[L];
     long long src = 0;
-    if (en < b) {
+    if (en < b || b < 0 || en > nnz) {               // (reads stay inside u_idx[0, u_off[L]))
         e |= kErrOff;
     } else {
         int prev = -1;

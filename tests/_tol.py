@@ -26,6 +26,7 @@ def check(gpu, ref, A, rel=REL):
     well = kappa <= KAPPA
     ea = np.where(na > 0, da / np.where(na > 0, na, 1.0), 0.0)
     stats = {"phi_max_rel": float(ephi.max()), "a_global_rel": float(glob),
+             "a_max_rel_all": float(ea.max()) if ea.size else 0.0,      # strict per-body max
              "a_max_rel_well": float(ea[well].max()) if well.any() else 0.0,
              "a_p999_rel": float(np.quantile(ea, 0.999)), "n_ill": int((~well).sum()),
              "a_max_abs_over_A_ill": float((da[~well] / np.maximum(A[~well], 1e-300)).max()) if (~well).any() else 0.0}

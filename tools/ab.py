@@ -70,7 +70,12 @@ def main():
     table = {}
     for rep in range(a.reps):
         for lib in a.libs:
-            env = dict(os.environ, AFMM_LIB_OVERRIDE=os.path.abspath(lib))
+            # "path.so::K=V,K2=V2" runs that library with extra environment variables
+            path, _, kv = lib.partition("::")
+            env = dict(os.environ, AFMM_LIB_OVERRIDE=os.path.abspath(path))
+            for item in filter(None, kv.split(",")):
+                k, _, v = item.partition("=")
+                env[k] = v
             r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=600)
             line = [ln for ln in r.stdout.splitlines() if ln.startswith("RESULT")]
             if not line:

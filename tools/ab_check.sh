@@ -10,4 +10,4 @@ for d in build/var_*/; do
   echo "$d parity: $r"
   case "$r" in *failed*|*error*) ;; *) libs="$libs $d/libafmm_p2p.so";; esac
 done
-python tools/ab.py --reps ${REPS:-2} --S ${SLIST:-32,128,512} $libs
+python tools/ab.py --reps ${REPS:-2} --S ${SLIST:-32,128,512} $libs $EXTRA_LIBS
