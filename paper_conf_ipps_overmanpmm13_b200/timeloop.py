@@ -52,7 +52,7 @@ CPU_COEF_DEFAULT = (0.5e-9, 1.0e-9, 1.0e-9, 1.0e-9, 0.5e-9)
 
 class TimeLoop:
     def __init__(self, x, y, z, m, vx, vy, vz, S, eps2, dt, domain, device=0, rank=0, world=1, G=1.0,
-                 lb=None, cpu_coef=CPU_COEF_DEFAULT, fine_group=0.05, fine_max_groups=16):
+                 lb=None, cpu_coef=CPU_COEF_DEFAULT, fine_group=0.05, fine_max_groups=16, slice_world=0):
         self.dev = torch.device("cuda", device)
         self.stream = torch.cuda.Stream(self.dev)
         torch.cuda.set_stream(self.stream)
@@ -74,7 +74,10 @@ class TimeLoop:
         self.tree.build(src[0], src[1], src[2], self.S, domain=domain)
         for a in range(7):
             self.tree.gather(src[a], self.state[a])
-        self.h = P2P(device=device, rank=rank, world=world, G=G, eps2=eps2, stream=self.stream.cuda_stream)
+        # slice_world (afmm_p2p_config): the task slicing; equal slice_world gives bit-identical
+        # accelerations -- hence trajectories -- at any world size and partition (DESIGN R17)
+        self.h = P2P(device=device, rank=rank, world=world, G=G, eps2=eps2, stream=self.stream.cuda_stream,
+                     slice_world=slice_world)
         self.step_no = 0
         self.log = []
         self._load_tree(host_copy=True)
