@@ -144,6 +144,7 @@ _sig("afmm_lb_create", _i, C.POINTER(LbConfig), C.POINTER(_p))
 _sig("afmm_lb_step", _i, _p, _d, _d, C.POINTER(_i), C.POINTER(_i))
 _sig("afmm_lb_predicted", _i, _p, _d, C.POINTER(_i))
 _sig("afmm_lb_state", _i, _p, C.POINTER(_i), C.POINTER(_i), C.POINTER(_d))
+_sig("afmm_lb_predict", _i, _p, _p, C.POINTER(_d), C.POINTER(_d), C.POINTER(_d))
 _sig("afmm_lb_destroy", None, _p)
 
 
@@ -178,7 +179,7 @@ EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
             "afmm_tree_rebuild", "afmm_tree_nodes", "afmm_fine_grained", "afmm_p2p_eval_host_pipelined",
             "afmm_p2p_set_peer_windows", "afmm_ipc_export", "afmm_ipc_import", "afmm_ipc_close",
             "afmm_tree_gather_rows", "afmm_p2p_nccl_id", "afmm_p2p_chunks", "afmm_p2p_eval_chunked",
-            "afmm_p2p_publish_chunks", "afmm_launch_count"]
+            "afmm_p2p_publish_chunks", "afmm_launch_count", "afmm_lb_predict"]
 
 
 def ipc_export(dev_ptr):
@@ -647,6 +648,19 @@ class GpuTree:
 
 
 # ------------------------------------------------------------------ load balancer (row f3)
+
+def lb_predict(counts, coef):
+    """afmm_lb_predict (L18 SIV.D): (t_cpu, t_gpu, t) = (sum of the five far-field C_op M(op),
+    C_P2P M(P2P), their max) from counts[6] (P2M, M2M, M2L, L2L, L2P, P2P) and coef[6]."""
+    m, c = _np(counts, np.int64), _np(coef, np.float64)
+    if m.shape != (6,) or c.shape != (6,):
+        raise ValueError("counts and coef hold 6 values (P2M, M2M, M2L, L2L, L2P, P2P)")
+    tc, tg, t = _d(), _d(), _d()
+    st = _lib.afmm_lb_predict(_ptr(m), _ptr(c), C.byref(tc), C.byref(tg), C.byref(t))
+    if st:
+        raise AfmmError(st, "afmm_lb_predict")
+    return tc.value, tg.value, t.value
+
 
 class LoadBalancer:
     """afmm_lb: the paper's Search / Incremental / Observation controller (L18 SV, L20-L22)."""

@@ -134,9 +134,7 @@ extern "C" afmm_status afmm_lb_step(afmm_lb *lb, double t_cpu, double t_gpu, int
             lb->fine_from_incremental = false;
             lb->pending = AFMM_LB_ENFORCE;
             *action = AFMM_LB_ENFORCE;
-        } else {
-            lb->best = std::min(lb->best, compute);
-        }
+        }                                     // else "nothing is done" (L22): the best stays as recorded
         break;
     }
     }
@@ -160,12 +158,27 @@ extern "C" afmm_status afmm_lb_predicted(afmm_lb *lb, double t_pred, int *action
         }
     } else {                                   // after FineGrainedOptimize
         lb->pending = AFMM_LB_KEEP;
-        if (ok || lb->fine_from_incremental) {
-            lb->fine_from_incremental = false;
-            lb->rebest = true;
+        if (lb->fine_from_incremental) {       // at the transitional S: "upon return from this function the load
+            lb->fine_from_incremental = false; //  balancer enters the observation state" with the best recorded
+        } else if (ok) {                       //  before it (L20 SVII.B)
+            lb->rebest = true;                 // after Enforce_S: the next step's compute time is the best (L24-L26)
         } else {
             lb->to_incremental = true;         // "moves into the incremental state again on the following time step"
         }
     }
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_lb_predict(const long long *counts, const double *coef, double *t_cpu, double *t_gpu,
+                                       double *t) {
+    if (!counts || !coef) return AFMM_EINVAL;
+    for (int i = 0; i < 6; ++i)
+        if (counts[i] < 0 || !(coef[i] >= 0.0) || !std::isfinite(coef[i])) return AFMM_EINVAL;
+    double cpu = 0.0;
+    for (int i = 0; i < 5; ++i) cpu += coef[i] * (double)counts[i];       // T_cpu = sum_op C_op M(op)
+    const double gpu = coef[5] * (double)counts[5];                       // T_gpu = C_P2P M(P2P)
+    if (t_cpu) *t_cpu = cpu;
+    if (t_gpu) *t_gpu = gpu;
+    if (t) *t = std::max(cpu, gpu);                                       // compute time (L20 SVII.A)
     return AFMM_OK;
 }

@@ -240,15 +240,22 @@ __global__ void split_write_kernel(int m, int base, int next_base, Nodes nd, con
     split_write_node(i, base, next_base, nd, cb, nc[i], off[i]);
 }
 
-// The whole level loop in ONE cooperative launch (no host round trip per level):
-// per level, (1) split counts (8 lanes per node, grid-stride), grid barrier,
-// (2) every block scans its tile of the child counts and publishes the tile sum,
-// grid barrier, (3) every block adds the sums of the tiles before its own (so no
-// third barrier is needed for the scan), writes its nodes' children, grid barrier.
-// Level starts go to ctl->base[]; a level that would exceed the node capacity
-// sets ctl->overflow and every block stops (the host grows the arrays and reruns).
+// The whole level loop in ONE cooperative launch (no host round trip per level),
+// ONE grid barrier per level: block b owns the tile [t0, t1) of the level's nodes;
+// it (1) computes their split counts (8 lanes per node), (2) scans its tile's child
+// counts, (3) gets the children of all earlier tiles by a chained scan with
+// decoupled look-back (every block publishes its tile's aggregate, then its
+// inclusive prefix, in a status word tagged with the launch epoch and the level,
+// so nothing is reset between levels or builds), (4) writes its nodes' children,
+// then the grid barrier; the level's total is the last tile's inclusive prefix.
+// Level starts go to ctl->base[]; a level that would exceed the node capacity sets
+// ctl->overflow (each block checks its own writes) and every block stops after the
+// barrier (the host grows the arrays and reruns).  (Round 1 had three barriers per
+// level: counts, tile sums, writes.)
 struct LevelCtl {
     long long base[kMaxLevel + 3];  // level starts, base[levels] = total nodes
+    int count[kMaxLevel + 3];       // nodes of level l + 1 (the last tile's inclusive prefix of level l): a
+                                    // slot per level, so no block reads a word the next level overwrites
     int levels;
     int overflow;
     unsigned bar_count, bar_gen;
@@ -272,31 +279,38 @@ __device__ __forceinline__ void grid_barrier(LevelCtl *c) {
     __syncthreads();
 }
 
+// status word of a tile: high 32 bits = epoch << 8 | level << 2 | flag (1 = aggregate,
+// 2 = inclusive prefix), low 32 bits = the value
+__device__ __forceinline__ unsigned long long tile_status(unsigned epoch, int lev, unsigned flag, unsigned v) {
+    return ((unsigned long long)((epoch << 8) | ((unsigned)lev << 2) | flag) << 32) | v;
+}
+
 constexpr int kLvlThreads = 256;
 __global__ void __launch_bounds__(kLvlThreads) levels_kernel(Nodes nd, const unsigned long long *__restrict__ keys,
                                                              int S, int mode, PrevTree pv, Edits ed,
                                                              int *__restrict__ cb, int *__restrict__ nc,
-                                                             int *__restrict__ off, int *__restrict__ tsum,
+                                                             int *__restrict__ off,
+                                                             unsigned long long *__restrict__ tstat, unsigned epoch,
                                                              LevelCtl *ctl, long long cap) {
     __shared__ int wsum[kLvlThreads / 32];
-    __shared__ int carry;
+    __shared__ int carry, s_excl;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    const long long stride = (long long)gridDim.x * kLvlThreads;
+    const int G = (int)gridDim.x, bid = (int)blockIdx.x;
     long long base = 0;
     int m = 1;
     int lev = 0;
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
+    if (bid == 0 && threadIdx.x == 0) {
         ctl->base[0] = 0;
         ctl->overflow = 0;
     }
     while (m > 0) {
-        // (1) split counts
-        for (long long w0 = ((long long)blockIdx.x * kLvlThreads + threadIdx.x) & ~31LL; w0 < 8LL * m; w0 += stride)
-            split_count_lane(w0 + lane, m, base, nd, keys, S, mode, pv, ed, cb, nc);
-        grid_barrier(ctl);
-        // (2) tile scan: block b owns nodes [b*tile, min(m, (b+1)*tile))
-        const int tile = (int)((m + gridDim.x - 1) / gridDim.x);
-        const int t0 = (int)min((long long)blockIdx.x * tile, (long long)m), t1 = min(t0 + tile, m);
+        const int tile = (m + G - 1) / G;
+        const int t0 = min(bid * tile, m), t1 = min(t0 + tile, m);
+        // (1) split counts of the tile's nodes (8 lanes per node; whole warps, padding lanes not live)
+        for (int w0 = threadIdx.x & ~31; 8 * t0 + w0 < 8 * t1; w0 += kLvlThreads)
+            split_count_lane(8LL * t0 + w0 + lane, t1, base, nd, keys, S, mode, pv, ed, cb, nc);
+        __syncthreads();
+        // (2) tile scan of the child counts -> off[i] (exclusive, tile-local), carry = tile sum
         if (threadIdx.x == 0) carry = 0;
         __syncthreads();
         for (int c0 = t0; c0 < t1; c0 += kLvlThreads) {
@@ -319,44 +333,50 @@ __global__ void __launch_bounds__(kLvlThreads) levels_kernel(Nodes nd, const uns
             if (threadIdx.x == 0) carry += ctot;
             __syncthreads();
         }
-        if (threadIdx.x == 0) tsum[blockIdx.x] = carry;
-        grid_barrier(ctl);
-        // (3) tile prefix + total (every block reads all tile sums: no extra barrier)
-        int pre = 0, total = 0;
-        for (int k = threadIdx.x; k < (int)gridDim.x; k += kLvlThreads) {
-            const int v = tsum[k];
-            total += v;
-            if (k < (int)blockIdx.x) pre += v;
+        // (3) chained scan over the tiles (decoupled look-back)
+        if (threadIdx.x == 0) {
+            const unsigned agg = (unsigned)carry;
+            unsigned excl = 0;
+            if (bid == 0) {
+                atomicExch(&tstat[0], tile_status(epoch, lev, 2u, agg));
+            } else {
+                atomicExch(&tstat[bid], tile_status(epoch, lev, 1u, agg));
+                for (int k = bid - 1; k >= 0;) {
+                    const unsigned long long sw = *(volatile unsigned long long *)&tstat[k];
+                    const unsigned hi = (unsigned)(sw >> 32);
+                    if ((hi >> 2) != ((epoch << 6) | (unsigned)lev)) {   // not yet published this level
+                        __nanosleep(20);
+                        continue;
+                    }
+                    excl += (unsigned)sw;
+                    if ((hi & 3u) == 2u) break;
+                    --k;
+                }
+                atomicExch(&tstat[bid], tile_status(epoch, lev, 2u, excl + agg));
+            }
+            if (bid == G - 1) ctl->count[lev] = (int)(excl + agg);    // read by every block after the barrier
+            s_excl = (int)excl;
         }
-        for (int o = 16; o > 0; o >>= 1) {
-            pre += __shfl_xor_sync(0xffffffffu, pre, o);
-            total += __shfl_xor_sync(0xffffffffu, total, o);
-        }
         __syncthreads();
-        if (lane == 0) wsum[wid] = pre;
-        __syncthreads();
-        int bpre = 0;
-        for (int k = 0; k < kLvlThreads / 32; ++k) bpre += wsum[k];
-        __syncthreads();
-        if (lane == 0) wsum[wid] = total;
-        __syncthreads();
-        int btot = 0;
-        for (int k = 0; k < kLvlThreads / 32; ++k) btot += wsum[k];
+        const int excl = s_excl;
         const long long next_base = base + m;
-        if (next_base + btot > cap) {                 // every block sees the same totals
-            if (blockIdx.x == 0 && threadIdx.x == 0) ctl->overflow = 1;
-            return;
+        // (4) children of the tile's nodes (the block's own writes checked against the capacity)
+        if (next_base + excl + carry > cap) {
+            if (threadIdx.x == 0) ctl->overflow = 1;
+        } else {
+            for (int i = t0 + threadIdx.x; i < t1; i += kLvlThreads)
+                split_write_node(i, base, next_base, nd, cb, nc[i], excl + off[i]);
         }
-        for (int i = t0 + threadIdx.x; i < t1; i += kLvlThreads) split_write_node(i, base, next_base, nd, cb, nc[i],
-                                                                                bpre + off[i]);
+        grid_barrier(ctl);
+        if (*(volatile int *)&ctl->overflow) return;
+        const int total = *(volatile int *)&ctl->count[lev];
         ++lev;
-        if (blockIdx.x == 0 && threadIdx.x == 0) {
+        if (bid == 0 && threadIdx.x == 0) {
             ctl->base[lev] = next_base;
             ctl->levels = lev;
         }
         base = next_base;
-        m = btot;
-        grid_barrier(ctl);
+        m = total;
     }
 }
 
@@ -651,6 +671,7 @@ struct afmm_tree {
     std::vector<size_t> ws_cap;
     size_t node_cap = 1024;
     bool coop_ok = true;             // cooperative launch of levels_kernel available
+    unsigned lvl_epoch = 0;          // launches of levels_kernel (tags its tile status words)
 };
 
 namespace {
@@ -860,7 +881,7 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
             if (afmm_status s = alloc_nodes(cap, nd, node_set)) return s;
         }
         LevelCtl *ctl;
-        int *tsum;
+        unsigned long long *tstat;
         if (afmm_status s = wsalloc(t, kCb, &cb, (size_t)(n + 1) * 9)) return s;
         if (afmm_status s = wsalloc(t, kNc, &nc, (size_t)n + 1)) return s;
         if (afmm_status s = wsalloc(t, kOff, &off, (size_t)n + 1)) return s;
@@ -868,14 +889,19 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
         int per_sm = 0, dev_sms = 0;
         TCU(t, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, levels_kernel, kLvlThreads, 0));
         TCU(t, cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, t->device));
-        const int blocks = std::max(1, std::min(per_sm, 2) * dev_sms);
-        if (afmm_status s = wsalloc(t, kTsum, &tsum, (size_t)blocks)) return s;
+        const int blocks = std::max(1, std::min(per_sm, 1) * dev_sms);     // one per SM: cheaper grid barriers
+        if (afmm_status s = wsalloc(t, kTsum, &tstat, (size_t)blocks)) return s;
         for (int attempt = 0; attempt < 8 && !done_levels; ++attempt) {
             root_kernel<<<1, 1, 0, st>>>(nd, (int)n);
             TCU(t, cudaGetLastError());
             TCU(t, cudaMemsetAsync(ctl, 0, sizeof(LevelCtl), st));
             long long capll = (long long)cap;
-            void *args[] = {&nd, &t->keys_sorted, &S, &mode, &pv, &ed, &cb, &nc, &off, &tsum, &ctl, &capll};
+            unsigned epoch = ++t->lvl_epoch & 0x3fffffu;                 // status words of this launch
+            if (epoch <= 1) {                  // first launch (fresh buffer) or the 22-bit tag wrapped: clear
+                TCU(t, cudaMemsetAsync(tstat, 0, (size_t)blocks * sizeof(unsigned long long), st));
+                if (epoch == 0) epoch = ++t->lvl_epoch & 0x3fffffu;
+            }
+            void *args[] = {&nd, &t->keys_sorted, &S, &mode, &pv, &ed, &cb, &nc, &off, &tstat, &epoch, &ctl, &capll};
             const cudaError_t e = cudaLaunchCooperativeKernel((const void *)levels_kernel, blocks, kLvlThreads, args,
                                                               0, st);
             if (e != cudaSuccess) {                   // no cooperative launch here: the per-level host loop

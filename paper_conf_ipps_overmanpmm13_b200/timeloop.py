@@ -40,7 +40,7 @@ import numpy as np
 import torch
 
 from . import (LB_ENFORCE, LB_FINE, LB_KEEP, LB_REBUILD, TREE_KEEP, GpuTree, P2P, cost_fit, drift,
-               kick)
+               kick, lb_predict)
 
 # Default modelled far-field costs (seconds per operation: P2M, M2M, M2L, L2L,
 # L2P), reading R29: translation operators of an order-p expansion cost
@@ -138,14 +138,14 @@ class TimeLoop:
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ms = float(t.item())
         c = self.tree.farfield_counts()
-        return float(np.dot(self.cpu_coef, c[:5])), 1e-3 * ms, c
+        return lb_predict(c, self._coef6())[0], 1e-3 * ms, c
 
     def _coef6(self):
         return np.concatenate([self.cpu_coef, [self.c_p2p or 0.0]])
 
     def _predict(self):
-        c = self.tree.farfield_counts()
-        return max(float(np.dot(self.cpu_coef, c[:5])), (self.c_p2p or 0.0) * float(c[5]))
+        """The predicted compute time of the current tree (afmm_lb_predict, L18 SIV.D)."""
+        return lb_predict(self.tree.farfield_counts(), self._coef6())[2]
 
     def _maintain(self, x, y, z):
         """Tree maintenance of this step (step 4): Enforce_S without a balancer,
