@@ -497,7 +497,10 @@ struct ChunkMeta {
 // lane can issue the bulk copy of its own segment's part of a chunk.
 struct Stream {
     int task, nxt;                // task ids (>= n_tasks: none)
-    Task t, tn;                   // descriptors (warp-uniform)
+    Task t;                       // the current task's descriptor (warp-uniform); the next one's is
+                                  // prefetched into shared memory (desc[slot], cp.async)
+    Task *desc;                   // this warp's two descriptor slots
+    int slot;                     // the slot holding (or receiving) task nxt's descriptor
     Seg sg;                       // this lane's segment of t
     int pre;                      // sum of the lengths of t's segments before this lane's (seg_count <= 32)
     bool pre_ok;                  // pre computed (deferred to t's first chunk issue)
@@ -528,7 +531,24 @@ __device__ __forceinline__ int claim(const P2PParams &p, int &seq, int lane) {
     return p.static_rounds * W + __shfl_sync(0xffffffffu, it, 0);
 }
 __device__ __forceinline__ void load_desc(const P2PParams &p, int id, Task &t) {
-    if (id < p.n_tasks) t = p.tasks[id];
+    t = p.tasks[min(id, p.n_tasks - 1)];                 // a past-the-end id reads the last task, never used
+}
+// The next task's descriptor goes to shared memory by cp.async (lanes 0 and 1,
+// 16 bytes each) and is read back when the task becomes current -- a task
+// later.  (Held in registers, round 1's prefetched descriptor was merged into the
+// loop-carried registers right after its load, so every task advance waited for
+// the load: ncu source page, C2 S = 32, 5 % of the samples on one MOV.)
+__device__ __forceinline__ void prefetch_desc(const P2PParams &p, int id, Task *slot, int lane) {
+    if (lane < 2) {
+        const char *src = reinterpret_cast<const char *>(p.tasks + min(id, p.n_tasks - 1)) + 16 * lane;
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 16;\n\tcp.async.commit_group;"
+                     ::"r"(smem_u32(reinterpret_cast<char *>(slot) + 16 * lane)), "l"(src) : "memory");
+    }
+}
+__device__ __forceinline__ void take_desc(Task &t, const Task *slot, int lane) {
+    if (lane < 2) asm volatile("cp.async.wait_group 0;" ::: "memory");
+    __syncwarp();
+    t = *slot;
 }
 // this lane's segment of task t (issued when t becomes current; its prefix is
 // taken one chunk later, so the load's latency hides behind a chunk of math)
@@ -643,12 +663,13 @@ __device__ __forceinline__ bool issue_chunk(const P2PParams &p, Stream &S, float
     PROF_T(t_c);
     if (S.staged >= S.t.nsrc) {                           // advance to the prefetched task
         S.task = S.nxt;
-        S.t = S.tn;
+        take_desc(S.t, S.desc + S.slot, lane);
         S.sg = load_seg(p, S.task, S.t, lane);
         S.pre_ok = false;
         S.staged = 0;
         S.nxt = claim(p, S.seq, lane);                    // and prefetch the one after
-        load_desc(p, S.nxt, S.tn);
+        S.slot ^= 1;
+        prefetch_desc(p, S.nxt, S.desc + S.slot, lane);
     }
     PROF_ADD(14, t_c);
     return true;
@@ -696,6 +717,7 @@ __device__ __forceinline__ void p2p_body(const P2PParams &p) {
     extern __shared__ __align__(128) unsigned char dsmem[];
     __shared__ __align__(8) uint64_t full_all[kWarps][kWStages];
     __shared__ ChunkMeta meta_all[kWarps][kWStages];
+    __shared__ __align__(16) Task desc_all[kWarps][2];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     float4 (*stage)[kWCap] = reinterpret_cast<float4 (*)[kWCap]>(dsmem + warp * kStageBytesW);
     double *accw = reinterpret_cast<double *>(dsmem + kWarps * kStageBytesW + warp * kAccBytesW);
@@ -717,12 +739,14 @@ __device__ __forceinline__ void p2p_body(const P2PParams &p) {
     // ---- start the stream: claim two tasks, fill the ring but one stage
     Stream S;
     S.seq = 0;
+    S.desc = desc_all[warp];
+    S.slot = 0;
     S.task = claim(p, S.seq, lane);
     load_desc(p, S.task, S.t);
     S.sg = load_seg(p, S.task, S.t, lane);
     S.pre_ok = false;
     S.nxt = claim(p, S.seq, lane);
-    load_desc(p, S.nxt, S.tn);
+    prefetch_desc(p, S.nxt, S.desc + S.slot, lane);
     S.staged = 0;
     int issued = 0;
     for (; issued < kWStages - 1; ++issued)
