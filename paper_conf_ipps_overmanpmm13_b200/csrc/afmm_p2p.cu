@@ -19,6 +19,7 @@
 
 #include <cuda.h>               // driver types for cuStreamWaitValue32 (resolved at run time)
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>   // NVTX ranges (header-only; no-ops unless a profiler is attached)
 
 #include "../../include/afmm_p2p.h"
 #include "nccl_api.h"
@@ -26,6 +27,13 @@
 
 using afmm::Seg;
 using afmm::Task;
+
+// NVTX range for the duration of a scope ("afmm.<entry point>"): nsys / ncu
+// timelines show the library's host-side phases (SURVEY S5 tracing).
+struct NvtxScope {
+    explicit NvtxScope(const char *name) { nvtxRangePushA(name); }
+    ~NvtxScope() { nvtxRangePop(); }
+};
 
 // Kernels of this library launched so far (afmm_launch_count): every <<<>>> site
 // below counts itself; CUB's scans / sorts inside the device ingest are not ours
@@ -526,6 +534,7 @@ static afmm_status pack(afmm_p2p *h, const float *x, const float *y, const float
 
 extern "C" afmm_status afmm_p2p_set_bodies(afmm_p2p *h, long long n, const float *x,
                                            const float *y, const float *z, const float *m) {
+    NvtxScope nvtx_("afmm.set_bodies");
     CHECK_HANDLE(h);
     if (h->cfg.law != AFMM_LAW_GRAVITY) return fail(h, AFMM_EINVAL, "set_bodies: handle law is not gravity");
     if (n < 1 || n >= (1LL << 31)) return fail(h, AFMM_EINVAL, "set_bodies: n=%lld out of [1, 2^31)", n);
@@ -544,6 +553,7 @@ extern "C" afmm_status afmm_p2p_set_bodies(afmm_p2p *h, long long n, const float
 
 extern "C" afmm_status afmm_p2p_set_bodies_host(afmm_p2p *h, long long n, const float *x,
                                                 const float *y, const float *z, const float *m) {
+    NvtxScope nvtx_("afmm.set_bodies_host");
     CHECK_HANDLE(h);
     if (h->cfg.law != AFMM_LAW_GRAVITY) return fail(h, AFMM_EINVAL, "set_bodies_host: handle law is not gravity");
     if (n < 1 || n >= (1LL << 31)) return fail(h, AFMM_EINVAL, "set_bodies_host: n=%lld out of [1, 2^31)", n);
@@ -883,6 +893,7 @@ static afmm_status reingest(afmm_p2p *h) {
 extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const int *leaf_start,
                                                 const int *leaf_count, const long long *u_off,
                                                 const int *u_idx) {
+    NvtxScope nvtx_("afmm.set_tree_device");
     CHECK_HANDLE(h);
     if (h->n < 1 || !h->d_bodies) return fail(h, AFMM_ESTATE, "set_tree_device: call set_bodies first");
     if (n_leaves < 1 || !leaf_start || !leaf_count || !u_off || !u_idx)
@@ -899,6 +910,7 @@ extern "C" afmm_status afmm_p2p_set_tree_device(afmm_p2p *h, int n_leaves, const
 extern "C" afmm_status afmm_p2p_set_tree(afmm_p2p *h, int n_leaves, const int *leaf_start,
                                          const int *leaf_count, const long long *u_off,
                                          const int *u_idx) {
+    NvtxScope nvtx_("afmm.set_tree");
     CHECK_HANDLE(h);
     if (h->n < 1 || !h->d_bodies) return fail(h, AFMM_ESTATE, "set_tree: call set_bodies first");
     if (n_leaves < 1 || !leaf_start || !leaf_count || !u_off)
@@ -1103,6 +1115,7 @@ extern "C" afmm_status afmm_partition_rebalance(int n_leaves, const int *leaf_co
 
 extern "C" afmm_status afmm_p2p_rebalance(afmm_p2p *h, const double *rank_ms, double threshold,
                                           int *changed) {
+    NvtxScope nvtx_("afmm.rebalance");
     CHECK_HANDLE(h);
     if (changed) *changed = 0;
     if (!h->have_tree) return fail(h, AFMM_ESTATE, "rebalance: no tree");
@@ -1278,6 +1291,7 @@ static afmm_status launch_any(afmm_p2p *h, float *ax, float *ay, float *az, floa
 
 extern "C" afmm_status afmm_p2p_eval(afmm_p2p *h, float *ax, float *ay, float *az, float *phi,
                                      afmm_p2p_stats *stats) {
+    NvtxScope nvtx_("afmm.eval");
     CHECK_HANDLE(h);
     if (!h->d_bodies || !h->have_tree) return fail(h, AFMM_ESTATE, "eval: set_bodies and set_tree first");
     if (!ax || !ay || !az || !phi) return fail(h, AFMM_EINVAL, "eval: null output pointer");
@@ -1290,6 +1304,7 @@ extern "C" afmm_status afmm_p2p_eval(afmm_p2p *h, float *ax, float *ay, float *a
 
 extern "C" afmm_status afmm_p2p_eval_host(afmm_p2p *h, float *ax, float *ay, float *az, float *phi,
                                           afmm_p2p_stats *stats) {
+    NvtxScope nvtx_("afmm.eval_host");
     CHECK_HANDLE(h);
     if (!h->d_bodies || !h->have_tree) return fail(h, AFMM_ESTATE, "eval_host: set_bodies and set_tree first");
     if (!ax || !ay || !az || !phi) return fail(h, AFMM_EINVAL, "eval_host: null output pointer");
@@ -1454,6 +1469,7 @@ static afmm_status build_pipe(afmm_p2p *h, int P) {
 extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, const float *x, const float *y,
                                                     const float *z, const float *m, float *ax, float *ay,
                                                     float *az, float *phi, int n_pieces, afmm_p2p_stats *stats) {
+    NvtxScope nvtx_("afmm.eval_host_pipelined");
     CHECK_HANDLE(h);
     if (h->cfg.law != AFMM_LAW_GRAVITY) return fail(h, AFMM_EINVAL, "eval_host_pipelined: gravity handles only");
     if (!h->have_tree || !h->d_bodies) return fail(h, AFMM_ESTATE, "eval_host_pipelined: set_bodies and set_tree first");
@@ -1904,6 +1920,7 @@ extern "C" afmm_status afmm_p2p_chunks(afmm_p2p *h, int *K, long long *bounds, i
 }
 
 extern "C" afmm_status afmm_p2p_eval_chunked(afmm_p2p *h, float *ax, float *ay, float *az, float *phi) {
+    NvtxScope nvtx_("afmm.eval_chunked");
     CHECK_HANDLE(h);
     if (!h->d_bodies || !h->have_tree) return fail(h, AFMM_ESTATE, "eval_chunked: set_bodies and set_tree first");
     if (!ax || !ay || !az || !phi) return fail(h, AFMM_EINVAL, "eval_chunked: null output pointer");
@@ -2003,6 +2020,7 @@ extern "C" afmm_status afmm_ipc_close(void *base) {
 extern "C" long long afmm_launch_count(void) { return g_launches.load(std::memory_order_relaxed); }
 
 extern "C" afmm_status afmm_p2p_stats_get(afmm_p2p *h, afmm_p2p_stats *stats) {
+    NvtxScope nvtx_("afmm.stats_get");
     CHECK_HANDLE(h);
     if (!h->evaluated) return fail(h, AFMM_ESTATE, "stats_get: no eval yet");
     afmm_status st = set_device(h);

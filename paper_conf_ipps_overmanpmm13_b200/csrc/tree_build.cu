@@ -18,6 +18,7 @@
 
 #include <cub/cub.cuh>
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include "../../include/afmm_tree.h"
 
@@ -788,6 +789,8 @@ extern "C" const char *afmm_tree_last_error(const afmm_tree *t) { return t ? t->
 static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const float *y, const float *z,
                               int S, int fixed_domain, const double *lo_in, int k_in, int mode,
                               Edits ed = Edits{nullptr, nullptr, nullptr, 0}) {
+    nvtxRangePushA(mode == kModeFresh ? "afmm.tree_build" : mode == kModeEnforce ? "afmm.tree_enforce" : "afmm.tree_rebuild");
+    struct Pop { ~Pop() { nvtxRangePop(); } } pop_;
     if (!t) return AFMM_EINVAL;
     if (t->poisoned) return AFMM_ESTATE;
     if (n < 1 || n >= (1LL << 31)) return tfail(t, AFMM_EINVAL, "tree_build: n=%lld out of range", n);
