@@ -154,6 +154,53 @@ enum { kModeFresh = 0, kModeEnforce = 1, kModeKeep = 2 };
 // Child ranges by binary search on the octant digit inside [b, e): eight lanes
 // per node, lane o finds the first position with digit >= o (independent
 // searches, so a level costs one search's latency, not seven in a row).
+// Does node id split (the rule above, edits applied)?  b, e, lev: its body range and level.
+__device__ __forceinline__ bool node_splits(long long id, const Nodes &nd, int S, int mode, const PrevTree &pv,
+                                            const Edits &ed, int &b, int &e, int &lev) {
+    b = nd.b[id];
+    e = nd.e[id];
+    lev = nd.level[id];
+    bool split;
+    if (mode == kModeKeep)            // structure kept: split iff it was a parent (Collapse/PushDown edits below)
+        split = pv.levels > 0 && prev_internal(pv, lev, nd.prefix[id]);
+    else
+        split = e - b > S || (mode == kModeEnforce && e - b == S && pv.levels > 0 && prev_internal(pv, lev, nd.prefix[id]));
+    if (ed.n > 0) {
+        const int a = edit_of(ed, lev, nd.prefix[id]);
+        if (a == 1) split = false;
+        else if (a == 2) split = true;
+    }
+    return split && lev < kMaxLevel;
+}
+
+// First position in [b, e) whose octant digit (key bits shift..shift+2) is >= o,
+// searched by the W lanes of a group together (lane k of the group = kk): every
+// round each lane reads one of W evenly spaced positions and a ballot (mask gmask,
+// group bits at gshift) narrows the range W-fold -- log_W(e - b) rounds of one
+// load instead of log_2 dependent loads.  All 32 lanes of the warp call it.
+__device__ __forceinline__ int kary_bound(const unsigned long long *__restrict__ keys, int b, int e, int o, int shift,
+                                          int W, int kk, int gshift, bool live) {
+    int lo = b, hi = e;                                       // the answer lies in [lo, hi]
+    while (__any_sync(0xffffffffu, live && hi > lo)) {
+        const bool act = live && hi > lo;
+        const int span = hi - lo;
+        const int pk = lo + (int)(((long long)kk * span) / W);
+        const bool ge = act && (int)((keys[pk] >> shift) & 7ull) >= o;
+        const unsigned bal = (__ballot_sync(0xffffffffu, ge) >> gshift) & (W == 32 ? 0xffffffffu : ((1u << W) - 1u));
+        if (act) {
+            const int kf = bal ? __ffs(bal) - 1 : W;          // first sample with digit >= o
+            if (kf == 0) {
+                hi = lo;                                       // p_0 = lo qualifies
+            } else {
+                const int pprev = lo + (int)(((long long)(kf - 1) * span) / W);
+                if (kf < W) hi = lo + (int)(((long long)kf * span) / W);
+                lo = pprev + 1;
+            }
+        }
+    }
+    return lo;
+}
+
 // one lane of the 8 of node i = gt >> 3 (lane o = gt & 7); all 32 lanes of the
 // warp call it together (shuffles / ballot), with gt >= 8m for padding lanes
 __device__ __forceinline__ void split_count_lane(long long gt, int m, long long base, const Nodes &nd,
@@ -244,11 +291,13 @@ __global__ void split_write_kernel(int m, int base, int next_base, Nodes nd, con
 // The whole level loop in ONE cooperative launch (no host round trip per level),
 // ONE grid barrier per level: block b owns the tile [t0, t1) of the level's nodes;
 // it (1) computes their split counts (8 lanes per node), (2) scans its tile's child
-// counts, (3) gets the children of all earlier tiles by a chained scan with
-// decoupled look-back (every block publishes its tile's aggregate, then its
-// inclusive prefix, in a status word tagged with the launch epoch and the level,
-// so nothing is reset between levels or builds), (4) writes its nodes' children,
-// then the grid barrier; the level's total is the last tile's inclusive prefix.
+// counts, (3) publishes its tile's total in a status word tagged with the launch
+// epoch and the level (so nothing is reset between levels or builds) and sums the
+// totals of all earlier tiles in ONE parallel round (thread k waits for tile k's
+// word; a block reduction -- the grid has <= 256 blocks), (4) writes its nodes'
+// children, then the grid barrier; the level's total is written by the last tile.
+// (A chained decoupled look-back walked the predecessors one L2 round trip at a
+// time: the kernel issued on 2 % of its cycles, ncu.)
 // Level starts go to ctl->base[]; a level that would exceed the node capacity sets
 // ctl->overflow (each block checks its own writes) and every block stops after the
 // barrier (the host grows the arrays and reruns).  (Round 1 had three barriers per
@@ -295,6 +344,7 @@ __global__ void __launch_bounds__(kLvlThreads) levels_kernel(Nodes nd, const uns
                                                              LevelCtl *ctl, long long cap) {
     __shared__ int wsum[kLvlThreads / 32];
     __shared__ int carry, s_excl;
+    __shared__ int sbound[9];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const int G = (int)gridDim.x, bid = (int)blockIdx.x;
     long long base = 0;
@@ -307,9 +357,60 @@ __global__ void __launch_bounds__(kLvlThreads) levels_kernel(Nodes nd, const uns
     while (m > 0) {
         const int tile = (m + G - 1) / G;
         const int t0 = min(bid * tile, m), t1 = min(t0 + tile, m);
-        // (1) split counts of the tile's nodes (8 lanes per node; whole warps, padding lanes not live)
-        for (int w0 = threadIdx.x & ~31; 8 * t0 + w0 < 8 * t1; w0 += kLvlThreads)
-            split_count_lane(8LL * t0 + w0 + lane, t1, base, nd, keys, S, mode, pv, ed, cb, nc);
+        // (1) split counts of the tile's nodes.  The few huge nodes of the top levels
+        //     are every level's critical path (all blocks wait for them), so small
+        //     tiles search wide: one node -> the whole block (warp o-1 finds octant
+        //     boundary o, 33-ary), up to 8 nodes -> a warp per node (4 lanes per
+        //     boundary, 5-ary); else 8 lanes per node (binary, split_count_lane).
+        const int ntile = t1 - t0;
+        if (ntile <= 1) {
+            int b = 0, e = 0, nlev = 0;
+            const bool split = ntile == 1 && node_splits(base + t0, nd, S, mode, pv, ed, b, e, nlev);
+            const int shift = 3 * (kMaxLevel - 1 - nlev);
+            if (wid < 7) {
+                const int bound = kary_bound(keys, b, e, wid + 1, shift, 32, lane, 0, split);
+                if (lane == 0) sbound[wid + 1] = bound;
+            }
+            __syncthreads();
+            if (threadIdx.x == 0 && ntile == 1) {
+                int cnt = 0;
+                if (split) {
+                    sbound[0] = b;
+                    sbound[8] = e;
+                    for (int o = 0; o < 8; ++o) {
+                        cb[(size_t)t0 * 9 + o] = sbound[o];
+                        cnt += sbound[o + 1] > sbound[o];
+                    }
+                    cb[(size_t)t0 * 9 + 8] = e;
+                }
+                nc[t0] = cnt;
+            }
+        } else if (ntile <= kLvlThreads / 32) {
+            const int i = t0 + wid;
+            int b = 0, e = 0, nlev = 0;
+            const bool split = wid < ntile && node_splits(base + i, nd, S, mode, pv, ed, b, e, nlev);
+            const int shift = 3 * (kMaxLevel - 1 - nlev);
+            const int o = lane / 4 + 1, kk = lane & 3;
+            const int bound = kary_bound(keys, b, e, o, shift, 4, kk, 4 * (o - 1) & 31, split && lane < 28);
+            int bo[9];
+            bo[0] = b;
+            bo[8] = e;
+#pragma unroll
+            for (int oo = 1; oo < 8; ++oo) bo[oo] = __shfl_sync(0xffffffffu, bound, 4 * (oo - 1));
+            if (lane == 0 && wid < ntile) {
+                int cnt = 0;
+                if (split) {
+#pragma unroll
+                    for (int oo = 0; oo < 9; ++oo) cb[(size_t)i * 9 + oo] = bo[oo];
+#pragma unroll
+                    for (int oo = 0; oo < 8; ++oo) cnt += bo[oo + 1] > bo[oo];
+                }
+                nc[i] = cnt;
+            }
+        } else {
+            for (int w0 = threadIdx.x & ~31; 8 * t0 + w0 < 8 * t1; w0 += kLvlThreads)
+                split_count_lane(8LL * t0 + w0 + lane, t1, base, nd, keys, S, mode, pv, ed, cb, nc);
+        }
         __syncthreads();
         // (2) tile scan of the child counts -> off[i] (exclusive, tile-local), carry = tile sum
         if (threadIdx.x == 0) carry = 0;
@@ -334,29 +435,28 @@ __global__ void __launch_bounds__(kLvlThreads) levels_kernel(Nodes nd, const uns
             if (threadIdx.x == 0) carry += ctot;
             __syncthreads();
         }
-        // (3) chained scan over the tiles (decoupled look-back)
-        if (threadIdx.x == 0) {
-            const unsigned agg = (unsigned)carry;
-            unsigned excl = 0;
-            if (bid == 0) {
-                atomicExch(&tstat[0], tile_status(epoch, lev, 2u, agg));
-            } else {
-                atomicExch(&tstat[bid], tile_status(epoch, lev, 1u, agg));
-                for (int k = bid - 1; k >= 0;) {
-                    const unsigned long long sw = *(volatile unsigned long long *)&tstat[k];
-                    const unsigned hi = (unsigned)(sw >> 32);
-                    if ((hi >> 2) != ((epoch << 6) | (unsigned)lev)) {   // not yet published this level
-                        __nanosleep(20);
-                        continue;
-                    }
-                    excl += (unsigned)sw;
-                    if ((hi & 3u) == 2u) break;
-                    --k;
-                }
-                atomicExch(&tstat[bid], tile_status(epoch, lev, 2u, excl + agg));
+        // (3) publish this tile's total; sum the earlier tiles' totals in one parallel round
+        if (threadIdx.x == 0) atomicExch(&tstat[bid], tile_status(epoch, lev, 1u, (unsigned)carry));
+        unsigned part = 0;
+        for (int k = threadIdx.x; k < bid; k += kLvlThreads) {
+            unsigned long long sw;
+            for (;;) {
+                sw = *(volatile unsigned long long *)&tstat[k];
+                if ((unsigned)(sw >> 34) == ((epoch << 6) | (unsigned)lev)) break;     // this level's word
+                __nanosleep(20);
             }
-            if (bid == G - 1) ctl->count[lev] = (int)(excl + agg);    // read by every block after the barrier
-            s_excl = (int)excl;
+            part += (unsigned)sw;
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
+        __syncthreads();                                          // wsum reuse after the tile scan
+        if (lane == 0) wsum[wid] = (int)part;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            int e = 0;
+            for (int k = 0; k < kLvlThreads / 32; ++k) e += wsum[k];
+            s_excl = e;
+            if (bid == G - 1) ctl->count[lev] = e + carry;       // read by every block after the barrier
         }
         __syncthreads();
         const int excl = s_excl;
