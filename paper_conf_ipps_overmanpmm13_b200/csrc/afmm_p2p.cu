@@ -807,11 +807,11 @@ static afmm_status ingest(afmm_p2p *h, int n_leaves, const int *leaf_start, cons
     const int lo = (int)h->leaf_split[r], m = (int)(h->leaf_split[r + 1] - h->leaf_split[r]);
     if ((st = dws(h, sNseg, &nseg, (size_t)m + 1)) || (st = dws(h, sNtask, &ntask, (size_t)m + 1)) ||
         (st = dws(h, sNsrc, &nsrc, (size_t)m + 1)) || (st = dws(h, sSegOff, &seg_off, (size_t)m + 1)) ||
-        (st = dws(h, sTaskOff, &task_off, (size_t)m + 1)) || (st = dws(h, sStats, &stats, 9)) ||
+        (st = dws(h, sTaskOff, &task_off, (size_t)m + 1)) || (st = dws(h, sStats, &stats, 10)) ||
         (st = dws(h, sPlan, &plan, (size_t)(m + 1) * afmm::kMaxDpSlices)) ||
         (st = dws(h, sPlanHdr, &plan_hdr, (size_t)m + 1)))
         return st;
-    CUDA_TRY(h, cudaMemsetAsync(stats, 0, 9 * sizeof(unsigned long long), s));
+    CUDA_TRY(h, cudaMemsetAsync(stats, 0, 10 * sizeof(unsigned long long), s));
     CUDA_TRY(h, cudaMemsetAsync(nseg + m, 0, sizeof(int), s));
     CUDA_TRY(h, cudaMemsetAsync(ntask + m, 0, sizeof(int), s));
     if (m > 0) {
@@ -829,7 +829,7 @@ static afmm_status ingest(afmm_p2p *h, int n_leaves, const int *leaf_start, cons
         CUDA_TRY(h, cub::DeviceScan::ExclusiveSum(tmp, tb, ntask, task_off, m + 1, s));
     }
     int totals[2] = {0, 0};
-    unsigned long long hstats[9];
+    unsigned long long hstats[10];
     CUDA_TRY(h, cudaMemcpyAsync(&totals[0], seg_off + m, sizeof(int), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(h, cudaMemcpyAsync(&totals[1], task_off + m, sizeof(int), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(h, cudaMemcpyAsync(hstats, stats, sizeof(hstats), cudaMemcpyDeviceToHost, s));
@@ -843,18 +843,18 @@ static afmm_status ingest(afmm_p2p *h, int n_leaves, const int *leaf_start, cons
         return st;
     if (m > 0) {
         dev::write_kernel<<<grid(m), TH, 0, s>>>(m, lo, leaf_start, leaf_count, u_off, u_idx, seg_off, task_off,
-                                                ntask, nsrc, h->d_segs, tasks_u, keys, vals, plan, plan_hdr);
+                                                ntask, nsrc, h->d_segs, tasks_u, keys, vals, plan, plan_hdr, hstats[9]);
         COUNT_LAUNCH(1);
         CUDA_TRY(h, cudaGetLastError());
     }
     if (nt > 0) {
         size_t tb = 0;
-        CUDA_TRY(h, cub::DeviceRadixSort::SortPairs(nullptr, tb, keys, keys2, vals, vals2, nt, 0, 32, s));
+        // keys = cmax - cost < 2^nb: only those bits are sorted (stable: the same order)
+        const int nb = std::max(1, 64 - __builtin_clzll(std::max<unsigned long long>(hstats[9], 1ull)));
+        CUDA_TRY(h, cub::DeviceRadixSort::SortPairs(nullptr, tb, keys, keys2, vals, vals2, nt, 0, nb, s));
         char *tmp;
         if ((st = dws(h, sTmp, &tmp, tb))) return st;
-        // keys = ~cost with cost < 2^31 (a task's warp iterations <= its sources < 2^31):
-        // the high half is constant, so the low 32 bits give the same stable order
-        CUDA_TRY(h, cub::DeviceRadixSort::SortPairs(tmp, tb, keys, keys2, vals, vals2, nt, 0, 32, s));
+        CUDA_TRY(h, cub::DeviceRadixSort::SortPairs(tmp, tb, keys, keys2, vals, vals2, nt, 0, nb, s));
         dev::gather_tasks_kernel<<<grid(nt), TH, 0, s>>>(nt, vals2, tasks_u, h->d_tasks);
         COUNT_LAUNCH(1);
         CUDA_TRY(h, cudaGetLastError());

@@ -554,11 +554,24 @@ __global__ void ulist_kernel(int L, Nodes nd, const int *__restrict__ node_leaf,
 // go to a fixed-capacity scratch row (kURow); counts[t] = row length.  A leaf
 // whose frontier or row exceeds the capacity raises *overflow and the caller
 // falls back to ulist_kernel for the whole tree (same result).
+// Every node's box anchor packed as ax | ay << 21 | az << 42 (level-21 units),
+// computed once per build so the descent below tests a node with one 8-byte load
+// and a few shifts instead of three Morton compactions per node (the descent was
+// instruction-bound, ncu: 69 % issue active).
+__global__ void anchors_kernel(int nn, Nodes nd, unsigned long long *__restrict__ anc) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= nn) return;
+    long long A[3], w;
+    box_of(nd.level[i], nd.prefix[i], A, w);
+    anc[i] = (unsigned long long)A[0] | ((unsigned long long)A[1] << 21) | ((unsigned long long)A[2] << 42);
+}
+
 constexpr int kURow = 256;                  // max row length kept by the warp path
 constexpr int kUFront = 512;                // max frontier length
 constexpr int kUWarps = 4;                  // warps per block
 __global__ void __launch_bounds__(32 * kUWarps) ulist_warp_kernel(int L, Nodes nd, const int *__restrict__ node_leaf,
                                                                   const int *__restrict__ leaf_node,
+                                                                  const unsigned long long *__restrict__ anc,
                                                                   int *__restrict__ rows, long long *__restrict__ counts,
                                                                   int *__restrict__ overflow) {
     __shared__ int front[kUWarps][2][kUFront];
@@ -581,11 +594,14 @@ __global__ void __launch_bounds__(32 * kUWarps) ulist_warp_kernel(int L, Nodes n
                 int nch = 0, fc = 0, lid = 0;
                 if (j < ncur) {
                     const int ni = front[wi][cur][j];
-                    long long As[3], ws;
-                    box_of(nd.level[ni], nd.prefix[ni], As, ws);
+                    const unsigned long long an = anc[ni];
+                    const int ws = 1 << (kMaxLevel - nd.level[ni]);
                     bool touch = true;
 #pragma unroll
-                    for (int a = 0; a < 3; ++a) touch &= (At[a] <= As[a] + ws) && (As[a] <= At[a] + wt);
+                    for (int a = 0; a < 3; ++a) {
+                        const int As = (int)((an >> (21 * a)) & 0x1fffffull);
+                        touch &= (At[a] <= As + ws) && (As <= At[a] + wt);
+                    }
                     if (touch) {
                         const int c = nd.nchild[ni];
                         if (c == 0) {
@@ -636,11 +652,11 @@ __global__ void __launch_bounds__(32 * kUWarps) ulist_warp_kernel(int L, Nodes n
 
 __global__ void ulist_copy_kernel(int L, const int *__restrict__ rows, const long long *__restrict__ u_off,
                                   int *__restrict__ u_idx) {
-    const int t = blockIdx.x;                      // one block per leaf
+    const int t = (int)((blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5);   // one warp per leaf
     if (t >= L) return;
     const long long o = u_off[t];
     const int n = (int)(u_off[t + 1] - o);
-    for (int j = threadIdx.x; j < n; j += blockDim.x) u_idx[o + j] = rows[(size_t)t * kURow + j];
+    for (int j = threadIdx.x & 31; j < n; j += 32) u_idx[o + j] = rows[(size_t)t * kURow + j];
 }
 
 __global__ void leaf_node_kernel(int nn, const int *__restrict__ node_leaf, int *__restrict__ leaf_node) {
@@ -834,7 +850,7 @@ afmm_status wsalloc(afmm_tree *t, int slot, T **p, size_t count) {
 enum Slot {
     kPart, kKeys, kIdx, kKeysSorted, kPerm, kSortTmp, kNodeA, kNodeB = kNodeA + 6, kCb = kNodeB + 6, kNc, kOff,
     kScanTmp, kFlag, kLeafAt, kNodeLeaf, kScan2, kLs, kLc, kLl, kLp, kLeafNode, kCounts, kUoff, kScan3, kUidx,
-    kFarfield, kEditPrefix, kEditAction, kEditBase, kURows, kUOvf, kLvlCtl, kTsum
+    kFarfield, kEditPrefix, kEditAction, kEditBase, kURows, kUOvf, kLvlCtl, kTsum, kAnc
 };
 
 __global__ void root_kernel(Nodes nd, int n) {
@@ -1147,30 +1163,41 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     TCU(t, cudaMemsetAsync(ovf, 0, sizeof(int), st));
     {
         const int blocks = (int)std::min<long long>((L + kUWarps - 1) / kUWarps, 148LL * 16);
-        ulist_warp_kernel<<<blocks, 32 * kUWarps, 0, st>>>(L, nd, node_leaf, leaf_node, rows, counts, ovf);
+        unsigned long long *anc;
+        if (afmm_status s = wsalloc(t, kAnc, &anc, (size_t)nn)) return s;
+        anchors_kernel<<<grid_for(nn, TH), TH, 0, st>>>((int)nn, nd, anc);
+        ulist_warp_kernel<<<blocks, 32 * kUWarps, 0, st>>>(L, nd, node_leaf, leaf_node, anc, rows, counts, ovf);
         TCU(t, cudaGetLastError());
     }
-    int hovf = 0;
-    TCU(t, cudaMemcpyAsync(&hovf, ovf, sizeof(int), cudaMemcpyDeviceToHost, st));
-    TCU(t, cudaStreamSynchronize(st));
-    if (hovf) {
-        ulist_kernel<<<grid_for(L, 128), 128, 0, st>>>(L, nd, node_leaf, leaf_node, nullptr, nullptr, counts);
-        TCU(t, cudaGetLastError());
-    }
-    {
+    // row offsets by a scan of the counts, read back together with the overflow flag
+    // (one synchronise); on overflow the per-thread DFS recounts and the scan reruns
+    auto scan_counts = [&]() -> afmm_status {
         size_t sb = 0;
         TCU(t, cub::DeviceScan::ExclusiveSum(nullptr, sb, counts, t->u_off, L + 1, st));
         char *sbuf;
         if (afmm_status s = wsalloc(t, kScan3, &sbuf, sb)) return s;
         TCU(t, cub::DeviceScan::ExclusiveSum(sbuf, sb, counts, t->u_off, L + 1, st));
-    }
-    TCU(t, cudaMemcpyAsync(&t->nnz, t->u_off + L, sizeof(long long), cudaMemcpyDeviceToHost, st));
+        TCU(t, cudaMemcpyAsync(&t->nnz, t->u_off + L, sizeof(long long), cudaMemcpyDeviceToHost, st));
+        return AFMM_OK;
+    };
+    int hovf = 0;
+    if (afmm_status s = scan_counts()) return s;
+    TCU(t, cudaMemcpyAsync(&hovf, ovf, sizeof(int), cudaMemcpyDeviceToHost, st));
     TCU(t, cudaStreamSynchronize(st));
+    const char *dfs = getenv("AFMM_ULIST_DFS");                   // tests: force the fallback path
+    if (dfs && dfs[0] == '1') hovf = 1;
+    if (hovf) {
+        ulist_kernel<<<grid_for(L, 128), 128, 0, st>>>(L, nd, node_leaf, leaf_node, nullptr, nullptr, counts);
+        TCU(t, cudaGetLastError());
+        TCU(t, cudaMemsetAsync(counts + L, 0, sizeof(long long), st));
+        if (afmm_status s = scan_counts()) return s;
+        TCU(t, cudaStreamSynchronize(st));
+    }
     if (afmm_status s = wsalloc(t, kUidx, &t->u_idx, (size_t)t->nnz)) return s;
     if (hovf)
         ulist_kernel<<<grid_for(L, 128), 128, 0, st>>>(L, nd, node_leaf, leaf_node, t->u_off, t->u_idx, nullptr);
     else
-        ulist_copy_kernel<<<L, 64, 0, st>>>(L, rows, t->u_off, t->u_idx);
+        ulist_copy_kernel<<<(int)(((long long)L * 32 + 255) / 256), 256, 0, st>>>(L, rows, t->u_off, t->u_idx);
     TCU(t, cudaGetLastError());
     TCU(t, cudaStreamSynchronize(st));
     t->n = n;

@@ -144,6 +144,14 @@ __global__ void count_kernel(int m, int lo, const int *__restrict__ ls, const in
     ntask[i] = n_full + k;
     atomicAdd(&stats[0], (unsigned long long)I[t]);
     atomicAdd(&stats[1 + bucket_of_d(lc[t])], (unsigned long long)I[t]);
+    // the largest task cost (stats[9]): the sort keys need only its bits
+    unsigned long long cmax = 0;
+    for (int j = 0; j < n_full + k; ++j) {
+        const unsigned long long c = (unsigned long long)slice_iters(src, plan_size(j, n_full, full_m,
+                                                                                  plan + (size_t)i * kMaxDpSlices));
+        cmax = c > cmax ? c : cmax;
+    }
+    atomicMax(&stats[9], cmax);
 }
 
 // pass 2: write segments (self first) and tasks with their LPT cost keys
@@ -153,7 +161,8 @@ __global__ void write_kernel(int m, int lo, const int *__restrict__ ls, const in
                              const int *__restrict__ ntask, const long long *__restrict__ nsrc,
                              Seg *__restrict__ segs, Task *__restrict__ tasks,
                              unsigned long long *__restrict__ keys, int *__restrict__ vals,
-                             const unsigned short *__restrict__ plan, const int4 *__restrict__ plan_hdr) {
+                             const unsigned short *__restrict__ plan, const int4 *__restrict__ plan_hdr,
+                             unsigned long long cmax) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= m) return;
     const int t = lo + i;
@@ -180,7 +189,7 @@ __global__ void write_kernel(int m, int lo, const int *__restrict__ ls, const in
         const int cnt = plan_size(j, n_full, full_m, sz);
         tasks[q] = Task{ts + a, cnt, ts, self ? tn : 0, seg_begin, w - seg_begin, (int)src, 0};
         const unsigned long long cost = (unsigned long long)slice_iters(src, cnt);
-        keys[q] = ~cost;                              // ascending sort of ~cost = largest cost first
+        keys[q] = cmax - cost;                        // ascending = largest cost first; < 2^bits(cmax)
         vals[q] = q;
     }
 }

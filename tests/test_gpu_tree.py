@@ -130,3 +130,23 @@ def test_c4_end_to_end_sampled():
 
 def test_c3_end_to_end_sampled():
     _end_to_end("C3", 4096, seed=3)
+
+
+def test_ulist_dfs_fallback_matches_warp_descent(monkeypatch):
+    """The U-list fallback (per-thread DFS count + fill, taken when a row or frontier
+    overflows the warp descent's buffers) gives the same CSR as the warp descent
+    (forced with AFMM_ULIST_DFS=1), and both equal the oracle's."""
+    import paper_conf_ipps_overmanpmm13_b200 as afmm
+    x, y, z, m = synth.make("plummer", 70000, 31)
+    To = oracle.Tree(x, y, z, 24)
+    X, Y, Z = (torch.from_numpy(v).cuda() for v in (x, y, z))
+    outs = []
+    for flag in ("0", "1"):
+        monkeypatch.setenv("AFMM_ULIST_DFS", flag)
+        t = afmm.GpuTree(0)
+        t.build(X, Y, Z, 24)
+        outs.append(t.copy_out(70000))
+        t.close()
+    for k in ("u_off", "u_idx", "leaf_start", "leaf_count"):
+        assert np.array_equal(outs[0][k], outs[1][k]), k
+        assert np.array_equal(outs[1][k], getattr(To, k)), k
