@@ -621,7 +621,8 @@ def main():
                 "masses": "equal (1/N, reading R19): detected at pack time, equal-mass pair loop (12 packed FP32 "
                           "ops per pair, G m applied once; reading R30)",
                 "tree_build_s": round(tree_s, 4), "set_tree_device_s": round(set_tree_s, 4)},
-            "kernel_ms": {"mean": kern_mean, "max_over_ranks": kern_max,
+            "kernel_ms": {"mean": kern_mean, "median": float(np.median(kern_ms)), "best": float(np.min(kern_ms)),
+                          "max_over_ranks": kern_max,
                           "kernel_ms_max_device_timer": st["kernel_ms_max"] if comm_mode == "library" else None},
             "gpu_time_interactions_per_s": inter / (kern_max * 1e-3),
             "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
