@@ -358,6 +358,29 @@ def extras_n1(args, afmm, torch, dev, stream, peak, kern_mean_main, main_dev_tre
                       "rebalance; E = T1 / (W * max_r T_r); no broadcast / gather / launch costs",
             "T1_ms": round(kern_mean_main, 4), "worlds": proxy}
 
+    if not args.no_sweep:
+        # row f1: the C5 dynamic workload (BASELINE configs[4]: 1M colliding bodies, leapfrog KDK with Enforce_S tree
+        # maintenance and device ingest every step; fixed S = 128), 60 steps after 5 warm-up steps, one GPU
+        from paper_conf_ipps_overmanpmm13_b200.timeloop import TimeLoop
+        c5 = synth.CONFIGS["C5"]
+        x5, y5, z5, m5, vx5, vy5, vz5 = synth.colliding_with_velocities(c5["n"], c5["seed"])
+        loop = TimeLoop(x5, y5, z5, m5, vx5, vy5, vz5, c5["S"], c5["eps2"], 0.05, synth.c5_domain(x5, y5, z5),
+                        device=dev.index)
+        for _ in range(5):
+            loop.step()
+        recs = [loop.step() for _ in range(60)]
+        keys = ("step_ms", "kernel_ms", "eval_ms", "enforce_ms", "set_tree_ms", "kick_drift_ms")
+        mean = {k: round(float(np.mean([r[k] for r in recs])), 4) for k in keys}
+        inter = float(np.mean([r["interactions"] for r in recs]))
+        extra["c5"] = {"workload": "C5: 1M colliding bodies, KDK dt=0.05, Enforce_S + device ingest every step, S=128, "
+                                   "eps2=1e-4, 60 timed steps (BASELINE configs[4], one GPU)",
+                       "mean_ms": mean, "interactions_per_step": inter,
+                       "kernel_interactions_per_s": inter / (mean["kernel_ms"] * 1e-3),
+                       "step_interactions_per_s": inter / (mean["step_ms"] * 1e-3),
+                       "note": "step_ms is host wall time per step (the loop synchronises once per step)"}
+        loop.close()
+        torch.cuda.set_stream(stream)
+
     if not args.no_stokeslet:
         # row f4: the regularized-Stokeslet law on its paper workload (C6: 10M uniform sources, L26 SIX.B)
         c6 = synth.CONFIGS["C6"]
