@@ -105,6 +105,174 @@ struct Nodes {
     unsigned long long *prefix;
 };
 
+// ---- bucket sort of the keys by the previous build's leaf cells (rebuilds in the
+// same domain: Enforce_S every C5 step).  The previous leaves are disjoint cells
+// in Morton order, so bucket 2j+1 = the keys inside leaf j's cell, bucket 2j+2 =
+// the keys between leaf j's cell and leaf j+1's (emptied space), bucket 0 = before
+// leaf 0: the buckets' key ranges are disjoint and increasing, so sorting every
+// bucket by (key, input index) and concatenating them in bucket order IS the
+// stable sort by (key, index) (round 1: CUB's 8-pass 63-bit radix sort).  Most
+// bodies stay in their leaf's cell between steps (≈ 74 % on C5), the buckets hold
+// about a leaf each, and a warp sorts one (bitonic, <= kBucketCap keys).
+constexpr int kBucketCap = 512;
+__global__ void cell_range_kernel(int L, const int *__restrict__ ll, const unsigned long long *__restrict__ lp,
+                                  unsigned long long *__restrict__ clo, unsigned long long *__restrict__ chi) {
+    const int j = blockIdx.x * blockDim.x + threadIdx.x;
+    if (j >= L) return;
+    const int sh = 3 * (kMaxLevel - ll[j]);
+    clo[j] = lp[j] << sh;
+    chi[j] = (lp[j] + 1ull) << sh;
+}
+// keys (as keys_kernel) + the bucket of each key: the first previous leaf whose cell
+// starts above the key, by a binary search over every kSampleStride-th cell start
+// staged in shared memory, then over the <= stride leaves it leaves open; the
+// bucket's counter is bumped once per warp and bucket (bodies arrive nearly in
+// key order, so a warp's keys mostly share one bucket)
+constexpr int kMaxSamples = 1024, kKeysThreads = 512;
+__global__ void __launch_bounds__(kKeysThreads) keys_bucket_kernel(
+    long long n, const float *__restrict__ x, const float *__restrict__ y, const float *__restrict__ z, double lx,
+    double ly, double lz, double scale, unsigned long long *__restrict__ keys, int L, int stride,
+    const unsigned long long *__restrict__ clo, const unsigned long long *__restrict__ chi, int *__restrict__ bucket,
+    int *__restrict__ slot, int *__restrict__ bcount) {
+    __shared__ unsigned long long smp[kMaxSamples];
+    const int ns = (L + stride - 1) / stride;
+    for (int s = threadIdx.x; s < ns; s += blockDim.x) smp[s] = clo[(long long)s * stride];
+    __syncthreads();
+    const int lane = threadIdx.x & 31;
+    for (long long base = (long long)blockIdx.x * blockDim.x; base < n; base += (long long)gridDim.x * blockDim.x) {
+        const long long i = base + threadIdx.x;
+        const bool act = i < n;
+        const unsigned am = __ballot_sync(0xffffffffu, act);
+        if (!act) continue;
+        const unsigned long long k = spread3(quantize(x[i], lx, scale)) | (spread3(quantize(y[i], ly, scale)) << 1) |
+                                     (spread3(quantize(z[i], lz, scale)) << 2);
+        keys[i] = k;
+        int a = 0, b = ns;                                    // first sample above k
+        while (a < b) {
+            const int mid = (a + b) >> 1;
+            if (smp[mid] <= k) a = mid + 1;
+            else b = mid;
+        }
+        int lo = a == 0 ? 0 : (a - 1) * stride + 1, hi = a == ns ? L : a * stride;
+        while (lo < hi) {                                     // first leaf above k
+            const int mid = (lo + hi) >> 1;
+            if (clo[mid] <= k) lo = mid + 1;
+            else hi = mid;
+        }
+        const int j = lo - 1;
+        const int bk = j < 0 ? 0 : (k < chi[j] ? 2 * j + 1 : 2 * j + 2);
+        bucket[i] = bk;
+        const unsigned same = __match_any_sync(am, bk);
+        const int leader = __ffs(same) - 1;
+        int first = 0;
+        if (lane == leader) first = atomicAdd(&bcount[bk], __popc(same));
+        first = __shfl_sync(same, first, leader);
+        slot[i] = first + __popc(same & ((1u << lane) - 1u));  // order inside a bucket: fixed by its sort
+    }
+}
+__global__ void bucket_scatter_kernel(long long n, const unsigned long long *__restrict__ keys,
+                                      const int *__restrict__ bucket, const int *__restrict__ slot,
+                                      const int *__restrict__ boff, unsigned long long *__restrict__ bkeys,
+                                      int *__restrict__ bidx) {
+    const long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const int pos = boff[bucket[i]] + slot[i];
+    bkeys[pos] = keys[i];
+    bidx[pos] = (int)i;
+}
+// one warp sorts one bucket of <= 32 R keys by (key, input index): a bitonic
+// network on registers, element e = r * 32 + lane; partners 32 or more apart are
+// in the same lane (register swap), nearer ones one shuffle away
+__device__ __forceinline__ bool pair_gt(unsigned long long ka, int ia, unsigned long long kb, int ib) {
+    return ka > kb || (ka == kb && ia > ib);
+}
+template <int R, int k, int j>
+__device__ __forceinline__ void bitonic_stage(unsigned long long (&K)[R], int (&I)[R], int lane) {
+    if constexpr (j >= 32) {                                  // same lane, registers r and r ^ (j / 32)
+        constexpr int jr = j >> 5;
+#pragma unroll
+        for (int r = 0; r < R; ++r)
+            if ((r & jr) == 0) {
+                const int rp = r | jr;
+                const bool up = ((r * 32 + lane) & k) == 0;
+                const bool sw = pair_gt(K[r], I[r], K[rp], I[rp]) == up;
+                const unsigned long long ka = K[r], kb = K[rp];
+                const int ia = I[r], ib = I[rp];
+                K[r] = sw ? kb : ka;
+                K[rp] = sw ? ka : kb;
+                I[r] = sw ? ib : ia;
+                I[rp] = sw ? ia : ib;
+            }
+    } else {                                                  // lanes lane and lane ^ j
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            const unsigned long long ok = __shfl_xor_sync(0xffffffffu, K[r], j);
+            const int oi = __shfl_xor_sync(0xffffffffu, I[r], j);
+            const bool up = ((r * 32 + lane) & k) == 0;
+            const bool keep_min = ((lane & j) == 0) == up;
+            const bool take = pair_gt(K[r], I[r], ok, oi) == keep_min;
+            K[r] = take ? ok : K[r];
+            I[r] = take ? oi : I[r];
+        }
+    }
+    if constexpr (j > 1) bitonic_stage<R, k, j / 2>(K, I, lane);
+}
+template <int R, int k>
+__device__ __forceinline__ void bitonic_merge_all(unsigned long long (&K)[R], int (&I)[R], int lane) {
+    bitonic_stage<R, k, k / 2>(K, I, lane);
+    if constexpr (k < 32 * R) bitonic_merge_all<R, 2 * k>(K, I, lane);
+}
+template <int R>
+__device__ __forceinline__ void warp_bitonic(int o, int cnt, const unsigned long long *__restrict__ bkeys,
+                                             const int *__restrict__ bidx, unsigned long long *__restrict__ okeys,
+                                             int *__restrict__ oidx, int lane) {
+    unsigned long long K[R];
+    int I[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const int e = r * 32 + lane;
+        K[r] = e < cnt ? bkeys[o + e] : ~0ull;
+        I[r] = e < cnt ? bidx[o + e] : 0x7fffffff;
+    }
+    bitonic_merge_all<R, 2>(K, I, lane);
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const int e = r * 32 + lane;
+        if (e < cnt) {
+            okeys[o + e] = K[r];
+            oidx[o + e] = I[r];
+        }
+    }
+}
+constexpr int kBucketWarps = 4;
+__global__ void __launch_bounds__(32 * kBucketWarps) bucket_sort_kernel(int nb, const int *__restrict__ boff,
+                                                                        const unsigned long long *__restrict__ bkeys,
+                                                                        const int *__restrict__ bidx,
+                                                                        unsigned long long *__restrict__ okeys,
+                                                                        int *__restrict__ oidx,
+                                                                        int *__restrict__ overflow) {
+    const int lane = threadIdx.x & 31;
+    const int b = blockIdx.x * kBucketWarps + (threadIdx.x >> 5);
+    if (b >= nb) return;                                      // whole warps
+    const int o = boff[b], cnt = boff[b + 1] - o;
+    if (cnt <= 1) {
+        if (cnt == 1 && lane == 0) {
+            okeys[o] = bkeys[o];
+            oidx[o] = bidx[o];
+        }
+        return;
+    }
+    if (cnt > kBucketCap) {                                   // rare: the caller falls back to a full sort
+        if (lane == 0) atomicExch(overflow, 1);
+        return;
+    }
+    if (cnt <= 32) warp_bitonic<1>(o, cnt, bkeys, bidx, okeys, oidx, lane);
+    else if (cnt <= 64) warp_bitonic<2>(o, cnt, bkeys, bidx, okeys, oidx, lane);
+    else if (cnt <= 128) warp_bitonic<4>(o, cnt, bkeys, bidx, okeys, oidx, lane);
+    else if (cnt <= 256) warp_bitonic<8>(o, cnt, bkeys, bidx, okeys, oidx, lane);
+    else warp_bitonic<16>(o, cnt, bkeys, bidx, okeys, oidx, lane);
+}
+
 // Internal nodes of the previous build, for Enforce_S: per level, node prefixes
 // in ascending order ([base[l], base[l+1])) and their child counts.
 struct PrevTree {
@@ -309,6 +477,7 @@ struct LevelCtl {
     int levels;
     int overflow;
     unsigned bar_count, bar_gen;
+    int sort_overflow;              // the bucket sort's flag, copied in before the launch (not the kernel's)
 };
 
 __device__ __forceinline__ void grid_barrier(LevelCtl *c) {
@@ -789,6 +958,7 @@ struct afmm_tree {
     size_t node_cap = 1024;
     bool coop_ok = true;             // cooperative launch of levels_kernel available
     unsigned lvl_epoch = 0;          // launches of levels_kernel (tags its tile status words)
+    long long sort_fallbacks = 0;    // bucket sorts that overflowed into the full radix sort
 };
 
 namespace {
@@ -850,7 +1020,8 @@ afmm_status wsalloc(afmm_tree *t, int slot, T **p, size_t count) {
 enum Slot {
     kPart, kKeys, kIdx, kKeysSorted, kPerm, kSortTmp, kNodeA, kNodeB = kNodeA + 6, kCb = kNodeB + 6, kNc, kOff,
     kScanTmp, kFlag, kLeafAt, kNodeLeaf, kScan2, kLs, kLc, kLl, kLp, kLeafNode, kCounts, kUoff, kScan3, kUidx,
-    kFarfield, kEditPrefix, kEditAction, kEditBase, kURows, kUOvf, kLvlCtl, kTsum, kAnc
+    kFarfield, kEditPrefix, kEditAction, kEditBase, kURows, kUOvf, kLvlCtl, kTsum, kAnc,
+    kCellLo, kCellHi, kBucket, kSlot, kBCount, kBOff, kBKeys, kBIdx, kBScan, kBOvf
 };
 
 __global__ void root_kernel(Nodes nd, int n) {
@@ -916,6 +1087,10 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
                          !std::isfinite(lo_in[2]) || k_in < -1000 || k_in > 1000))
         return tfail(t, AFMM_EINVAL, "tree_build: bad fixed domain");
     TCU(t, cudaSetDevice(t->device));
+    // the previous build's domain and leaves (for the bucket sort of step 3)
+    const bool had_prev = t->built && t->L > 0 && t->n == n;
+    const double prev_lo[3] = {t->lo[0], t->lo[1], t->lo[2]};
+    const int prev_k = t->k, prev_L = t->L;
     t->built = false;
     cudaStream_t st = t->stream;
     const int TH = 256;
@@ -956,9 +1131,9 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     if (afmm_status s = wsalloc(t, kIdx, &idx, n)) return s;
     if (afmm_status s = wsalloc(t, kKeysSorted, &t->keys_sorted, n)) return s;
     if (afmm_status s = wsalloc(t, kPerm, &t->perm, n)) return s;
-    keys_kernel<<<grid_for(n, TH), TH, 0, st>>>(n, x, y, z, t->lo[0], t->lo[1], t->lo[2], scale, keys, idx);
-    TCU(t, cudaGetLastError());
-    {
+    auto full_sort = [&]() -> afmm_status {                   // first build / new domain / bucket overflow
+        keys_kernel<<<grid_for(n, TH), TH, 0, st>>>(n, x, y, z, t->lo[0], t->lo[1], t->lo[2], scale, keys, idx);
+        TCU(t, cudaGetLastError());
         size_t tb = 0;
         TCU(t, cub::DeviceRadixSort::SortPairs(nullptr, tb, keys, t->keys_sorted, idx, t->perm, (int)n, 0,
                                                3 * kMaxLevel, st));
@@ -966,6 +1141,46 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
         if (afmm_status s = wsalloc(t, kSortTmp, reinterpret_cast<char **>(&tbuf), tb)) return s;
         TCU(t, cub::DeviceRadixSort::SortPairs(tbuf, tb, keys, t->keys_sorted, idx, t->perm, (int)n, 0,
                                                3 * kMaxLevel, st));
+        return AFMM_OK;
+    };
+    const char *cub_env = getenv("AFMM_TREE_FULL_SORT");
+    const bool buckets = had_prev && t->coop_ok && prev_k == t->k && prev_lo[0] == t->lo[0] &&
+                         prev_lo[1] == t->lo[1] && prev_lo[2] == t->lo[2] && !(cub_env && cub_env[0] == '1');
+    int *bovf = nullptr;
+    if (buckets) {                                            // by the previous leaves' cells (see bucket_sort_kernel)
+        const int Lp = prev_L, nb = 2 * Lp + 1;
+        unsigned long long *clo, *chi, *bkeys;
+        int *bucket, *slot, *bcount, *boff, *bidx;
+        if (afmm_status s = wsalloc(t, kCellLo, &clo, Lp)) return s;
+        if (afmm_status s = wsalloc(t, kCellHi, &chi, Lp)) return s;
+        if (afmm_status s = wsalloc(t, kBucket, &bucket, n)) return s;
+        if (afmm_status s = wsalloc(t, kSlot, &slot, n)) return s;
+        if (afmm_status s = wsalloc(t, kBCount, &bcount, (size_t)nb + 1)) return s;
+        if (afmm_status s = wsalloc(t, kBOff, &boff, (size_t)nb + 1)) return s;
+        if (afmm_status s = wsalloc(t, kBKeys, &bkeys, n)) return s;
+        if (afmm_status s = wsalloc(t, kBIdx, &bidx, n)) return s;
+        if (afmm_status s = wsalloc(t, kBOvf, &bovf, 1)) return s;
+        TCU(t, cudaMemsetAsync(bcount, 0, ((size_t)nb + 1) * sizeof(int), st));
+        TCU(t, cudaMemsetAsync(bovf, 0, sizeof(int), st));
+        cell_range_kernel<<<grid_for(Lp, TH), TH, 0, st>>>(Lp, t->ll, t->lp, clo, chi);
+        const int stride = (Lp + kMaxSamples - 1) / kMaxSamples;
+        int kb_grid = 0, dev_sms = 0;
+        TCU(t, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&kb_grid, keys_bucket_kernel, kKeysThreads, 0));
+        TCU(t, cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, t->device));
+        kb_grid = (int)std::min<long long>((n + kKeysThreads - 1) / kKeysThreads, (long long)std::max(1, kb_grid) * dev_sms);
+        keys_bucket_kernel<<<kb_grid, kKeysThreads, 0, st>>>(n, x, y, z, t->lo[0], t->lo[1], t->lo[2], scale, keys, Lp,
+                                                             stride, clo, chi, bucket, slot, bcount);
+        size_t sb = 0;
+        TCU(t, cub::DeviceScan::ExclusiveSum(nullptr, sb, bcount, boff, nb + 1, st));
+        char *sbuf;
+        if (afmm_status s = wsalloc(t, kBScan, &sbuf, sb)) return s;
+        TCU(t, cub::DeviceScan::ExclusiveSum(sbuf, sb, bcount, boff, nb + 1, st));
+        bucket_scatter_kernel<<<grid_for(n, TH), TH, 0, st>>>(n, keys, bucket, slot, boff, bkeys, bidx);
+        bucket_sort_kernel<<<(nb + kBucketWarps - 1) / kBucketWarps, 32 * kBucketWarps, 0, st>>>(
+            nb, boff, bkeys, bidx, t->keys_sorted, t->perm, bovf);
+        TCU(t, cudaGetLastError());
+    } else if (afmm_status s = full_sort()) {
+        return s;
     }
 
     // 4. level-synchronous split into one node array (level-major)
@@ -1014,6 +1229,8 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
             root_kernel<<<1, 1, 0, st>>>(nd, (int)n);
             TCU(t, cudaGetLastError());
             TCU(t, cudaMemsetAsync(ctl, 0, sizeof(LevelCtl), st));
+            if (bovf)                         // read back with the levels' LevelCtl: no extra sync
+                TCU(t, cudaMemcpyAsync(&ctl->sort_overflow, bovf, sizeof(int), cudaMemcpyDeviceToDevice, st));
             long long capll = (long long)cap;
             unsigned epoch = ++t->lvl_epoch & 0x3fffffu;                 // status words of this launch
             if (epoch <= 1) {                  // first launch (fresh buffer) or the 22-bit tag wrapped: clear
@@ -1026,11 +1243,22 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
             if (e != cudaSuccess) {                   // no cooperative launch here: the per-level host loop
                 cudaGetLastError();
                 t->coop_ok = false;
+                if (bovf) {                           // the bucket sort's overflow is not checked there
+                    bovf = nullptr;
+                    if (afmm_status s = full_sort()) return s;
+                }
                 break;
             }
             LevelCtl hc;
             TCU(t, cudaMemcpyAsync(&hc, ctl, sizeof(LevelCtl), cudaMemcpyDeviceToHost, st));
             TCU(t, cudaStreamSynchronize(st));
+            if (hc.sort_overflow) {                   // a bucket exceeded kBucketCap: sort in full, redo the levels
+                bovf = nullptr;
+                ++t->sort_fallbacks;
+                if (getenv("AFMM_TREE_DEBUG")) fprintf(stderr, "afmm tree: bucket sort overflow %lld\n", t->sort_fallbacks);
+                if (afmm_status s = full_sort()) return s;
+                continue;
+            }
             if (hc.overflow) {                        // grow and rebuild the levels
                 cap *= 2;
                 node_set = node_set == kNodeA ? kNodeB : kNodeA;

@@ -150,3 +150,32 @@ def test_ulist_dfs_fallback_matches_warp_descent(monkeypatch):
     for k in ("u_off", "u_idx", "leaf_start", "leaf_count"):
         assert np.array_equal(outs[0][k], outs[1][k]), k
         assert np.array_equal(outs[1][k], getattr(To, k)), k
+
+
+def test_rebuild_bucket_sort_bit_exact(monkeypatch):
+    """Rebuilds in the previous build's domain sort the keys by the previous leaves'
+    cells (bucket_sort_kernel) instead of the full radix sort: small motions (most
+    bodies stay in their cell), a large jump, and a collapse into one cell (buckets
+    over the warp sort's capacity -> the full-sort fallback) all give the oracle's
+    tree, as does the forced full sort (AFMM_TREE_FULL_SORT=1)."""
+    import paper_conf_ipps_overmanpmm13_b200 as afmm
+    rng = np.random.default_rng(41)
+    n, S = 60000, 48
+    x, y, z, m = synth.make("plummer", n, 41)
+    dom = (np.array([-16.0, -16.0, -16.0]), 5)
+    seq = [(x, y, z)]
+    for scale in (1e-3, 1e-2, 0.5):                    # drift, larger drift, a big jump
+        x = (x + scale * rng.standard_normal(n)).astype(np.float32)
+        y = (y + scale * rng.standard_normal(n)).astype(np.float32)
+        z = (z + scale * rng.standard_normal(n)).astype(np.float32)
+        seq.append((x, y, z))
+    c = np.float32(0.3)                                # everything collapses into one leaf's cell
+    seq.append(tuple((c + np.float32(1e-4) * rng.standard_normal(n)).astype(np.float32) for _ in range(3)))
+    seq.append(seq[1])                                  # and back
+    for flag in ("0", "1"):
+        monkeypatch.setenv("AFMM_TREE_FULL_SORT", flag)
+        t = afmm.GpuTree(0)
+        for (px, py, pz) in seq:
+            t.build(_dev(px), _dev(py), _dev(pz), S, domain=dom)
+            assert_same_tree(t.copy_out(n), oracle.Tree(px, py, pz, S, domain=dom))
+        t.close()
