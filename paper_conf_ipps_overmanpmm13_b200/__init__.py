@@ -93,6 +93,7 @@ _sig("afmm_p2p_stats_get", _i, _p, C.POINTER(Stats))
 _sig("afmm_p2p_set_peer_windows", _i, _p, _i, _p)
 _sig("afmm_p2p_nccl_id", _i, _p)
 _sig("afmm_p2p_chunks", _i, _p, C.POINTER(_i), _p, _p)
+_sig("afmm_p2p_worklist", _i, _p, _p, _ll, C.POINTER(_ll), _p, _ll, C.POINTER(_ll))
 _sig("afmm_p2p_eval_chunked", _i, _p, _p, _p, _p, _p)
 _sig("afmm_p2p_publish_chunks", _i, _p, _i, _p)
 
@@ -179,7 +180,7 @@ EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
             "afmm_tree_rebuild", "afmm_tree_nodes", "afmm_fine_grained", "afmm_p2p_eval_host_pipelined",
             "afmm_p2p_set_peer_windows", "afmm_ipc_export", "afmm_ipc_import", "afmm_ipc_close",
             "afmm_tree_gather_rows", "afmm_p2p_nccl_id", "afmm_p2p_chunks", "afmm_p2p_eval_chunked",
-            "afmm_p2p_publish_chunks", "afmm_launch_count", "afmm_lb_predict"]
+            "afmm_p2p_publish_chunks", "afmm_launch_count", "afmm_lb_predict", "afmm_p2p_worklist"]
 
 
 def ipc_export(dev_ptr):
@@ -500,6 +501,16 @@ class P2P:
         o = np.empty(K.value, np.int32)
         self._check(_lib.afmm_p2p_chunks(self._h, C.byref(K), _ptr(b), _ptr(o)), "afmm_p2p_chunks")
         return b, o
+
+    def worklist(self):
+        """afmm_p2p_worklist: (tasks[nt, 8], segs[ns, 2]) int32, in dispatch order."""
+        nt, ns = _ll(), _ll()
+        self._check(_lib.afmm_p2p_worklist(self._h, None, 0, C.byref(nt), None, 0, C.byref(ns)), "afmm_p2p_worklist")
+        t = np.empty((nt.value, 8), np.int32)
+        s = np.empty((ns.value, 2), np.int32)
+        self._check(_lib.afmm_p2p_worklist(self._h, _ptr(t), nt.value, C.byref(nt), _ptr(s), ns.value, C.byref(ns)),
+                    "afmm_p2p_worklist")
+        return t, s
 
     def eval_chunked(self, ax, ay, az, phi):
         """afmm_p2p_eval_chunked: launch before the bodies arrive (device outputs, async)."""

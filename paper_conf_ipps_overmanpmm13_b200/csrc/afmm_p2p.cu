@@ -104,6 +104,8 @@ struct afmm_p2p {
     // pipelined host evaluation (afmm_p2p_eval_host_pipelined): the rank's tasks
     // regrouped into P Morton-contiguous pieces, LPT order kept inside each
     bool pipe_valid = false;
+    unsigned sort_epoch = 0;         // task_sort_kernel launches (tags its status words)
+    bool sort_ready = false;         // its status words and barrier were cleared
     int pipe_P = 0;
     std::vector<int> pipe_off;                       // P + 1 offsets into d_ptasks
     std::vector<long long> pipe_need, pipe_lo, pipe_hi;   // bodies needed (prefix), output range per piece
@@ -118,7 +120,8 @@ struct afmm_p2p {
     // zero-copy input chain (K pack launches + K stream writes) captured once as a
     // CUDA graph and replayed with one launch; re-captured when its key changes
     int *h_err = nullptr;                            // pinned: the input-wait timeout flag after an eval
-    int *h_ingest_err = nullptr;                     // pinned: set_tree_device's validation flags
+    long long *h_rb = nullptr;                       // pinned: set_tree_device's one readback (RbSlot)
+    size_t h_rb_len = 0;
     cudaGraphExec_t in_graph = nullptr;
     bool in_graph_off = false;                       // capture unsupported: direct launches
     const float *ig_src[4] = {nullptr, nullptr, nullptr, nullptr};
@@ -471,7 +474,7 @@ extern "C" void afmm_p2p_destroy(afmm_p2p *h) {
     if (h->s_in) cudaStreamSynchronize(h->s_in), cudaStreamDestroy(h->s_in);
     if (h->in_graph) cudaGraphExecDestroy(h->in_graph);
     if (h->h_err) cudaFreeHost(h->h_err);
-    if (h->h_ingest_err) cudaFreeHost(h->h_ingest_err);
+    if (h->h_rb) cudaFreeHost(h->h_rb);
     if (h->s_out) cudaStreamSynchronize(h->s_out), cudaStreamDestroy(h->s_out);
 
     for (int i = 0; i < 64; ++i) {
@@ -699,6 +702,9 @@ static afmm_status dws(afmm_p2p *h, int slot, T **p, size_t count) {
     *p = static_cast<T *>(h->dws_ptr[slot]);
     return AFMM_OK;
 }
+static size_t slot_capacity(const afmm_p2p *h, int slot) {
+    return (size_t)slot < h->dws_cap.size() ? h->dws_cap[slot] : 0;
+}
 
 __global__ void body_split_kernel(int G, int L, long long n, const long long *__restrict__ split,
                                   const int *__restrict__ ls, long long *__restrict__ bsplit) {
@@ -708,39 +714,101 @@ __global__ void body_split_kernel(int G, int L, long long n, const long long *__
 
 enum DwsSlot { sI, sP, sW, sPW, sSplit, sErr, sNseg, sNtask, sNsrc, sSegOff, sTaskOff, sStats, sKeys, sVals, sKeys2,
                sVals2, sTasksU, sCoef, sTmp, sBsplit, sPlan, sPlanHdr, sNnz,
-               sOwnLS, sOwnLC, sOwnUO, sOwnUI };             // the handle's own copy of the tree (re-ingest)
+               sOwnLS, sOwnLC, sOwnUO, sOwnUI,               // the handle's own copy of the tree (re-ingest)
+               sSortStat, sSortCtl, sNsegAll, sNsrcAll, sRb, sNtEff };              // task_sort_kernel's digit totals, status words, barrier
 
 // Device ingest (validation, Interactions(t), partition, this rank's work list)
 // of the tree arrays ls/lc/uo/ui in device memory.  keep: afterwards also copy
 // them into the handle's own buffers (sOwn*), from which set_partition /
 // rebalance re-ingest the same tree (the caller's arrays may be gone by then).
+//
+// Everything is enqueued back to back and the host synchronises ONCE, at the end
+// (round 1: nine host round trips).  The kernels read what the host used to read
+// back -- this rank's leaf range (split), the task cap (from the total P[L-1]),
+// the list sizes -- on the device; a failed validation gates every later kernel
+// (no read through an invalid index), and the work list is written into the
+// current capacities: when it does not fit (first ingest, a grown tree), the
+// host grows them after the sync and enqueues the list writing again.
+enum RbSlot { rbErr, rbOverflow, rbNsegs, rbNt, rbItot, rbNnz, rbStats, rbSplit = rbStats + 10 };
+enum : long long { kOvSegs = 1, kOvTasks = 2, kOvOwnUI = 4 };
+namespace dev_ingest {
+__global__ void collect_kernel(int L, int W, int r, const long long *__restrict__ split,
+                               const long long *__restrict__ bsplit, const long long *__restrict__ P,
+                               const long long *__restrict__ uo, const int *__restrict__ seg_off,
+                               const int *__restrict__ task_off, const unsigned long long *__restrict__ stats,
+                               const int *__restrict__ err, long long segs_cap, long long tasks_cap,
+                               long long *__restrict__ rb, int *__restrict__ nt_eff) {
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    const int e = *err;
+    const long long m = split[r + 1] - split[r];
+    const long long nsegs = e ? 0 : seg_off[m], nt = e ? 0 : task_off[m];
+    const long long ov = (nsegs > segs_cap ? kOvSegs : 0) | (nt > tasks_cap ? kOvTasks : 0);
+    rb[rbErr] = e;
+    rb[rbOverflow] = ov;
+    rb[rbNsegs] = nsegs;
+    rb[rbNt] = nt;
+    rb[rbItot] = P[L - 1];
+    rb[rbNnz] = uo[L];
+    for (int k = 0; k < 10; ++k) rb[rbStats + k] = (long long)stats[k];
+    for (int k = 0; k <= W; ++k) {
+        rb[rbSplit + k] = split[k];
+        rb[rbSplit + W + 1 + k] = bsplit[k];
+    }
+    *nt_eff = (e || ov) ? 0 : (int)nt;                      // gates write_kernel and the sort
+}
+// the U-list indices into the handle's own buffer (capacity cap; nnz = uo[L] on the device)
+__global__ void copy_ui_kernel(int L, const long long *__restrict__ uo, const int *__restrict__ src,
+                               int *__restrict__ dst, long long cap, const int *__restrict__ err,
+                               long long *__restrict__ rb) {
+    if (*err) return;
+    const long long nnz = uo[L];
+    if (nnz > cap) {
+        if (blockIdx.x == 0 && threadIdx.x == 0) atomicOr((unsigned long long *)&rb[rbOverflow], (unsigned long long)kOvOwnUI);
+        return;
+    }
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < nnz; i += (long long)gridDim.x * blockDim.x)
+        dst[i] = src[i];
+}
+}  // namespace dev_ingest
+
 static afmm_status ingest(afmm_p2p *h, int n_leaves, const int *leaf_start, const int *leaf_count,
                           const long long *u_off, const int *u_idx, bool keep) {
     using namespace afmm;
     afmm_status st;
     cudaStream_t s = h->stream;
-    const int L = n_leaves, W = h->cfg.world, TH = 256;
+    const int L = n_leaves, W = h->cfg.world, r = h->cfg.rank, TH = 256;
     auto grid = [&](long long m) { return (int)std::max<long long>(1, (m + TH - 1) / TH); };
-    long long *I, *P, *split, *nsrc, *bsplit;
+    long long *I, *P, *split, *nsrc, *bsplit, *nsrc_all, *rb;
     unsigned short *plan;
     int4 *plan_hdr;
-    int *err, *nseg, *ntask, *seg_off, *task_off, *vals, *vals2;
-    unsigned long long *stats, *keys, *keys2;
+    int *err, *nseg, *ntask, *seg_off, *task_off, *nseg_all, *nt_eff;
+    unsigned long long *stats;
+    const size_t rb_len = (size_t)rbSplit + 2 * (W + 1);
     if ((st = dws(h, sI, &I, L)) || (st = dws(h, sP, &P, L)) || (st = dws(h, sSplit, &split, W + 1)) ||
-        (st = dws(h, sErr, &err, 1)) || (st = dws(h, sBsplit, &bsplit, W + 1)))
+        (st = dws(h, sErr, &err, 1)) || (st = dws(h, sBsplit, &bsplit, W + 1)) ||
+        (st = dws(h, sNsegAll, &nseg_all, L)) || (st = dws(h, sNsrcAll, &nsrc_all, L)) ||
+        (st = dws(h, sNseg, &nseg, (size_t)L + 1)) || (st = dws(h, sNtask, &ntask, (size_t)L + 1)) ||
+        (st = dws(h, sNsrc, &nsrc, (size_t)L + 1)) || (st = dws(h, sSegOff, &seg_off, (size_t)L + 1)) ||
+        (st = dws(h, sTaskOff, &task_off, (size_t)L + 1)) || (st = dws(h, sStats, &stats, 10)) ||
+        (st = dws(h, sPlan, &plan, (size_t)(L + 1) * afmm::kMaxDpSlices)) ||
+        (st = dws(h, sPlanHdr, &plan_hdr, (size_t)L + 1)) || (st = dws(h, sRb, &rb, rb_len)) ||
+        (st = dws(h, sNtEff, &nt_eff, 1)))
         return st;
-    // 1. validation + Interactions(t)
+    if (h->h_rb_len < rb_len) {                     // pinned: the one readback is an async copy
+        if (h->h_rb) cudaFreeHost(h->h_rb);
+        h->h_rb = nullptr;
+        h->h_rb_len = 0;
+        CUDA_TRY(h, cudaMallocHost(&h->h_rb, rb_len * sizeof(long long)));
+        h->h_rb_len = rb_len;
+    }
+    // 1. validation + Interactions(t) + per-leaf segment counts and source totals
     CUDA_TRY(h, cudaMemsetAsync(err, 0, sizeof(int), s));
-    dev::validate_interactions_kernel<<<grid(L), TH, 0, s>>>(L, h->n, h->cfg.max_leaf, leaf_start, leaf_count,
-                                                            u_off, u_idx, I, err);
+    CUDA_TRY(h, cudaMemsetAsync(stats, 0, 10 * sizeof(unsigned long long), s));
+    dev::validate_interactions_kernel<<<grid(32LL * L), TH, 0, s>>>(L, h->n, h->cfg.max_leaf, leaf_start,
+                                                                   leaf_count, u_off, u_idx, I, nseg_all, nsrc_all,
+                                                                   err);
     COUNT_LAUNCH(1);
     CUDA_TRY(h, cudaGetLastError());
-    // the flags ride with the partition's results (one synchronise instead of two): the
-    // partition kernels only touch L- and W-sized arrays, and nothing of the handle's
-    // state changes before the flags are checked
-    if (!h->h_ingest_err) CUDA_TRY(h, cudaMallocHost(&h->h_ingest_err, sizeof(int)));   // pinned: an async copy
-    *h->h_ingest_err = 0;
-    CUDA_TRY(h, cudaMemcpyAsync(h->h_ingest_err, err, sizeof(int), cudaMemcpyDeviceToHost, s));
     bool clear_user = false;                        // applied once the tree is known valid
     // 2. partition (literal rule, or the per-bucket coefficients of the last step)
     {
@@ -775,96 +843,115 @@ static afmm_status ingest(afmm_p2p *h, int n_leaves, const int *leaf_start, cons
     CUDA_TRY(h, cudaGetLastError());
     body_split_kernel<<<(W + 1 + 63) / 64, 64, 0, s>>>(W, L, h->n, split, leaf_start, bsplit);
     COUNT_LAUNCH(1);
-    std::vector<long long> lsplit(W + 1, 0), bsplit_h(W + 1, 0);
-    long long itot = 0, nnz = 0;
-    CUDA_TRY(h, cudaMemcpyAsync(lsplit.data(), split, (W + 1) * sizeof(long long), cudaMemcpyDeviceToHost, s));
-    CUDA_TRY(h, cudaMemcpyAsync(bsplit_h.data(), bsplit, (W + 1) * sizeof(long long), cudaMemcpyDeviceToHost, s));
-    CUDA_TRY(h, cudaMemcpyAsync(&itot, P + (L - 1), sizeof(long long), cudaMemcpyDeviceToHost, s));
-    if (keep) CUDA_TRY(h, cudaMemcpyAsync(&nnz, u_off + L, sizeof(long long), cudaMemcpyDeviceToHost, s));
-    CUDA_TRY(h, cudaStreamSynchronize(s));
-    const int herr = *(volatile int *)h->h_ingest_err;
-    if (herr)
-        return fail(h, AFMM_EINVAL, "set_tree: invalid tree (flags 0x%x: 1 start, 2 count, 4 cover, "
-                                    "8 u_off, 16 u_idx range, 32 row order)", herr);
-    if (keep) {                                    // the handle's own copy, for set_partition / rebalance
-        int *ols, *olc, *oui;
+    // 3. this rank's segment / slice counts (leaves split[r] .. split[r+1], read on the device)
+    dev::count_kernel<<<grid((long long)L + 1), TH, 0, s>>>(L, r, split, P, slice_world(h),
+                                                           (long long)h->num_sms * h->blocks_per_sm * afmm::kWarps,
+                                                           err, leaf_count, nseg_all, nsrc_all, I, nseg, ntask, nsrc,
+                                                           stats, plan, plan_hdr);
+    COUNT_LAUNCH(1);
+    CUDA_TRY(h, cudaGetLastError());
+    {
+        size_t tb = 0;
+        CUDA_TRY(h, cub::DeviceScan::ExclusiveSum(nullptr, tb, nseg, seg_off, L + 1, s));
+        char *tmp;
+        if ((st = dws(h, sTmp, &tmp, tb))) return st;
+        CUDA_TRY(h, cub::DeviceScan::ExclusiveSum(tmp, tb, nseg, seg_off, L + 1, s));
+        CUDA_TRY(h, cub::DeviceScan::ExclusiveSum(tmp, tb, ntask, task_off, L + 1, s));
+    }
+    // 4. the lists, into the current capacities (a first guess from L when there are none)
+    if ((st = ensure_device(h, &h->d_segs, h->segs_cap, std::max<size_t>(h->segs_cap, (size_t)12 * L))) ||
+        (st = ensure_device(h, &h->d_tasks, h->tasks_cap, std::max<size_t>(h->tasks_cap, (size_t)4 * L))))
+        return st;
+    auto write_lists = [&]() -> afmm_status {
+        const size_t tcap = h->tasks_cap;
+        Task *tasks_u;
+        unsigned long long *keys, *keys2;
+        int *vals, *vals2;
+        afmm_status s2;
+        if ((s2 = dws(h, sTasksU, &tasks_u, tcap)) || (s2 = dws(h, sKeys, &keys, tcap)) ||
+            (s2 = dws(h, sVals, &vals, tcap)) || (s2 = dws(h, sKeys2, &keys2, tcap)) ||
+            (s2 = dws(h, sVals2, &vals2, tcap)))
+            return s2;
+        dev_ingest::collect_kernel<<<1, 1, 0, s>>>(L, W, r, split, bsplit, P, u_off, seg_off, task_off, stats, err,
+                                                   (long long)h->segs_cap, (long long)tcap, rb, nt_eff);
+        COUNT_LAUNCH(1);
+        dev::write_kernel<<<grid(32LL * L), TH, 0, s>>>(r, split, nt_eff, leaf_start, leaf_count, u_off, u_idx,
+                                                       seg_off, task_off, nsrc, h->d_segs, tasks_u, keys, vals, plan,
+                                                       plan_hdr, stats + 9);
+        COUNT_LAUNCH(1);
+        CUDA_TRY(h, cudaGetLastError());
+        // keys = cmax - cost < 2^bits(cmax): stable sort, ascending (task_sort_kernel)
+        const int G = std::max(1, h->num_sms);
+        unsigned long long *sstat;
+        dev::SortCtl *sctl;
+        if ((s2 = dws(h, sSortStat, &sstat, (size_t)G * dev::kRadix)) || (s2 = dws(h, sSortCtl, &sctl, 1))) return s2;
+        unsigned epoch = ++h->sort_epoch & 0x7ffffffu;
+        if (!h->sort_ready || epoch == 0) {      // fresh status words (the tags must not match stale ones)
+            CUDA_TRY(h, cudaMemsetAsync(sstat, 0, (size_t)G * dev::kRadix * sizeof(unsigned long long), s));
+            CUDA_TRY(h, cudaMemsetAsync(sctl, 0, sizeof(dev::SortCtl), s));
+            h->sort_ready = true;
+            if (epoch == 0) epoch = ++h->sort_epoch & 0x7ffffffu;
+        }
+        const int *ntp = nt_eff;
+        const unsigned long long *cmax_ptr = stats + 9;
+        Task *out = h->d_tasks;
+        void *args[] = {&ntp, &cmax_ptr, &keys, &vals, &keys2, &vals2, &tasks_u, &out, &sstat, &epoch, &sctl};
+        CUDA_TRY(h, cudaLaunchCooperativeKernel((const void *)dev::task_sort_kernel, G, dev::kSortThreads, args, 0, s));
+        COUNT_LAUNCH(1);
+        return AFMM_OK;
+    };
+    if ((st = write_lists())) return st;
+    // 5. the handle's own copy of the tree (set_partition / rebalance re-ingest it)
+    int *oui = nullptr;
+    auto copy_ui = [&](size_t cap) -> afmm_status {
+        if (afmm_status s2 = dws(h, sOwnUI, &oui, cap)) return s2;
+        dev_ingest::copy_ui_kernel<<<h->num_sms * 4, TH, 0, s>>>(L, u_off, u_idx, oui, (long long)cap, err, rb);
+        COUNT_LAUNCH(1);
+        CUDA_TRY(h, cudaGetLastError());
+        return AFMM_OK;
+    };
+    if (keep) {
+        int *ols, *olc;
         long long *ouo;
-        if ((st = dws(h, sOwnLS, &ols, L)) || (st = dws(h, sOwnLC, &olc, L)) || (st = dws(h, sOwnUO, &ouo, L + 1)) ||
-            (st = dws(h, sOwnUI, &oui, (size_t)std::max<long long>(nnz, 1))))
+        if ((st = dws(h, sOwnLS, &ols, L)) || (st = dws(h, sOwnLC, &olc, L)) || (st = dws(h, sOwnUO, &ouo, L + 1)))
             return st;
         CUDA_TRY(h, cudaMemcpyAsync(ols, leaf_start, L * sizeof(int), cudaMemcpyDeviceToDevice, s));
         CUDA_TRY(h, cudaMemcpyAsync(olc, leaf_count, L * sizeof(int), cudaMemcpyDeviceToDevice, s));
         CUDA_TRY(h, cudaMemcpyAsync(ouo, u_off, (L + 1) * sizeof(long long), cudaMemcpyDeviceToDevice, s));
-        if (nnz > 0) CUDA_TRY(h, cudaMemcpyAsync(oui, u_idx, nnz * sizeof(int), cudaMemcpyDeviceToDevice, s));
+        const size_t have = slot_capacity(h, sOwnUI) / sizeof(int);
+        if ((st = copy_ui(std::max<size_t>(have, (size_t)32 * L)))) return st;
+    }
+    // 6. the one readback
+    long long *hb = h->h_rb;
+    CUDA_TRY(h, cudaMemcpyAsync(hb, rb, rb_len * sizeof(long long), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(h, cudaStreamSynchronize(s));
+    if (hb[rbErr])
+        return fail(h, AFMM_EINVAL, "set_tree: invalid tree (flags 0x%x: 1 start, 2 count, 4 cover, "
+                                    "8 u_off, 16 u_idx range, 32 row order)", (int)hb[rbErr]);
+    if (hb[rbOverflow] & (kOvSegs | kOvTasks)) {   // the lists did not fit: grow, write them again
+        if ((st = ensure_device(h, &h->d_segs, h->segs_cap, (size_t)hb[rbNsegs])) ||
+            (st = ensure_device(h, &h->d_tasks, h->tasks_cap, (size_t)hb[rbNt])))
+            return st;
+        const long long own_ov = hb[rbOverflow] & kOvOwnUI;
+        if ((st = write_lists())) return st;
+        if (keep && own_ov && (st = copy_ui((size_t)hb[rbNnz]))) return st;
+        CUDA_TRY(h, cudaMemcpyAsync(hb, rb, rb_len * sizeof(long long), cudaMemcpyDeviceToHost, s));
+        CUDA_TRY(h, cudaStreamSynchronize(s));
+        if (hb[rbOverflow] & (kOvSegs | kOvTasks))
+            return fail(h, AFMM_ECUDA, "set_tree: work list still overflowing after growth");
+    } else if (keep && (hb[rbOverflow] & kOvOwnUI)) {
+        if ((st = copy_ui((size_t)hb[rbNnz]))) return st;  // (ordered before any later use)
     }
     if (clear_user) h->user_partition = false;
-    h->leaf_split = std::move(lsplit);
-    h->body_split = std::move(bsplit_h);
-    h->I_total = itot;
-    // 3. this rank's work list
-    const int r = h->cfg.rank;
-    const long long cap = afmm::task_cap(h->I_total / slice_world(h), (long long)h->num_sms * h->blocks_per_sm * afmm::kWarps);
-    const int lo = (int)h->leaf_split[r], m = (int)(h->leaf_split[r + 1] - h->leaf_split[r]);
-    if ((st = dws(h, sNseg, &nseg, (size_t)m + 1)) || (st = dws(h, sNtask, &ntask, (size_t)m + 1)) ||
-        (st = dws(h, sNsrc, &nsrc, (size_t)m + 1)) || (st = dws(h, sSegOff, &seg_off, (size_t)m + 1)) ||
-        (st = dws(h, sTaskOff, &task_off, (size_t)m + 1)) || (st = dws(h, sStats, &stats, 10)) ||
-        (st = dws(h, sPlan, &plan, (size_t)(m + 1) * afmm::kMaxDpSlices)) ||
-        (st = dws(h, sPlanHdr, &plan_hdr, (size_t)m + 1)))
-        return st;
-    CUDA_TRY(h, cudaMemsetAsync(stats, 0, 10 * sizeof(unsigned long long), s));
-    CUDA_TRY(h, cudaMemsetAsync(nseg + m, 0, sizeof(int), s));
-    CUDA_TRY(h, cudaMemsetAsync(ntask + m, 0, sizeof(int), s));
-    if (m > 0) {
-        dev::count_kernel<<<grid(m), TH, 0, s>>>(m, lo, leaf_start, leaf_count, u_off, u_idx, I, nseg, ntask, nsrc,
-                                                stats, cap, plan, plan_hdr);
-        COUNT_LAUNCH(1);
-        CUDA_TRY(h, cudaGetLastError());
-    }
-    {
-        size_t tb = 0;
-        CUDA_TRY(h, cub::DeviceScan::ExclusiveSum(nullptr, tb, nseg, seg_off, m + 1, s));
-        char *tmp;
-        if ((st = dws(h, sTmp, &tmp, tb))) return st;
-        CUDA_TRY(h, cub::DeviceScan::ExclusiveSum(tmp, tb, nseg, seg_off, m + 1, s));
-        CUDA_TRY(h, cub::DeviceScan::ExclusiveSum(tmp, tb, ntask, task_off, m + 1, s));
-    }
-    int totals[2] = {0, 0};
-    unsigned long long hstats[10];
-    CUDA_TRY(h, cudaMemcpyAsync(&totals[0], seg_off + m, sizeof(int), cudaMemcpyDeviceToHost, s));
-    CUDA_TRY(h, cudaMemcpyAsync(&totals[1], task_off + m, sizeof(int), cudaMemcpyDeviceToHost, s));
-    CUDA_TRY(h, cudaMemcpyAsync(hstats, stats, sizeof(hstats), cudaMemcpyDeviceToHost, s));
-    CUDA_TRY(h, cudaStreamSynchronize(s));
-    const int nsegs = totals[0], nt = totals[1];
-    if ((st = ensure_device(h, &h->d_segs, h->segs_cap, (size_t)nsegs))) return st;
-    if ((st = ensure_device(h, &h->d_tasks, h->tasks_cap, (size_t)nt))) return st;
-    Task *tasks_u;
-    if ((st = dws(h, sTasksU, &tasks_u, nt)) || (st = dws(h, sKeys, &keys, nt)) || (st = dws(h, sVals, &vals, nt)) ||
-        (st = dws(h, sKeys2, &keys2, nt)) || (st = dws(h, sVals2, &vals2, nt)))
-        return st;
-    if (m > 0) {
-        dev::write_kernel<<<grid(m), TH, 0, s>>>(m, lo, leaf_start, leaf_count, u_off, u_idx, seg_off, task_off,
-                                                ntask, nsrc, h->d_segs, tasks_u, keys, vals, plan, plan_hdr, hstats[9]);
-        COUNT_LAUNCH(1);
-        CUDA_TRY(h, cudaGetLastError());
-    }
-    if (nt > 0) {
-        size_t tb = 0;
-        // keys = cmax - cost < 2^nb: only those bits are sorted (stable: the same order)
-        const int nb = std::max(1, 64 - __builtin_clzll(std::max<unsigned long long>(hstats[9], 1ull)));
-        CUDA_TRY(h, cub::DeviceRadixSort::SortPairs(nullptr, tb, keys, keys2, vals, vals2, nt, 0, nb, s));
-        char *tmp;
-        if ((st = dws(h, sTmp, &tmp, tb))) return st;
-        CUDA_TRY(h, cub::DeviceRadixSort::SortPairs(tmp, tb, keys, keys2, vals, vals2, nt, 0, nb, s));
-        dev::gather_tasks_kernel<<<grid(nt), TH, 0, s>>>(nt, vals2, tasks_u, h->d_tasks);
-        COUNT_LAUNCH(1);
-        CUDA_TRY(h, cudaGetLastError());
-    }
-    h->n_tasks = nt;
+    h->leaf_split.assign(hb + rbSplit, hb + rbSplit + W + 1);
+    h->body_split.assign(hb + rbSplit + W + 1, hb + rbSplit + 2 * (W + 1));
+    h->I_total = hb[rbItot];
+    h->n_tasks = (int)hb[rbNt];
     h->pipe_valid = false;
     h->chunk_valid = false;
     h->L = L;
-    h->rank_interactions = (long long)hstats[0];
-    for (int b = 0; b < 8; ++b) h->bucket_inter[b] = (long long)hstats[1 + b];
+    h->rank_interactions = hb[rbStats + 0];
+    for (int b = 0; b < 8; ++b) h->bucket_inter[b] = hb[rbStats + 1 + b];
     h->tree_on_device = true;
     h->have_tree = true;
     h->h_tasks.clear();
@@ -1916,6 +2003,23 @@ extern "C" afmm_status afmm_p2p_chunks(afmm_p2p *h, int *K, long long *bounds, i
     if (K) *K = h->chunk_K;
     if (bounds) std::copy(h->chunk_bounds.begin(), h->chunk_bounds.end(), bounds);
     if (order) std::copy(h->chunk_order.begin(), h->chunk_order.end(), order);
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_p2p_worklist(afmm_p2p *h, int *tasks, long long cap_tasks, long long *n_tasks, int *segs,
+                                         long long cap_segs, long long *n_segs) {
+    CHECK_HANDLE(h);
+    if (!h->have_tree) return fail(h, AFMM_ESTATE, "worklist: set_tree first");
+    afmm_status st = set_device(h);
+    if (st) return st;
+    std::vector<afmm::Task> t;
+    std::vector<afmm::Seg> sg;
+    if ((st = fetch_worklist(h, t, sg))) return st;
+    static_assert(sizeof(afmm::Task) == 8 * sizeof(int) && sizeof(afmm::Seg) == 2 * sizeof(int), "layout");
+    if (n_tasks) *n_tasks = (long long)t.size();
+    if (n_segs) *n_segs = (long long)sg.size();
+    if (tasks && cap_tasks >= (long long)t.size() && !t.empty()) std::memcpy(tasks, t.data(), t.size() * sizeof(afmm::Task));
+    if (segs && cap_segs >= (long long)sg.size() && !sg.empty()) std::memcpy(segs, sg.data(), sg.size() * sizeof(afmm::Seg));
     return AFMM_OK;
 }
 

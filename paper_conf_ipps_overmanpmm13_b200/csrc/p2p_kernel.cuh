@@ -132,11 +132,14 @@ __host__ __device__ __forceinline__ long long slice_iters(long long nsrc, int m)
 // allowed candidate, first take full M-target slices until < 2 M remain
 // (tn % M + M, so the remainder may still merge with one full block); the DP cuts
 // the rest.  Returns the number of DP slices and writes their sizes (each
-// 1..kTaskTargets) to sz[0..k); *n_full = leading full slices of *full_m targets.
+// 1..kTaskTargets) to sz[0..k); *n_full = leading full slices of *full_m targets;
+// *max_m (optional) = the largest slice, which has the largest cost (slice_iters is
+// nondecreasing in m).
 __host__ __device__ inline int plan_slices(int tn, long long nsrc, long long cap, int *n_full, int *full_m,
-                                           unsigned short *sz) {
+                                           unsigned short *sz, int *max_m = nullptr) {
     bool ok[kSliceCands];
     int M = slice_cand_m(0);
+#pragma unroll
     for (int i = 0; i < kSliceCands; ++i) {
         ok[i] = i == 0 || slice_iters(nsrc, slice_cand_m(i)) <= cap;
         if (ok[i]) M = slice_cand_m(i);
@@ -149,37 +152,45 @@ __host__ __device__ inline int plan_slices(int tn, long long nsrc, long long cap
     *n_full = full;
     *full_m = M;
     long long cost[kSliceCands];
+#pragma unroll
     for (int i = 0; i < kSliceCands; ++i) cost[i] = slice_iters(nsrc, slice_cand_m(i)) + kSliceTaskCost;
     // Every candidate is a multiple of kTPT, so f(a) -- the best cost of cutting a
     // targets -- is constant on each block (kTPT(q-1), kTPT q] (induction: a - m
-    // stays in one block), and so is the argmin: the DP runs over blocks q.
-    constexpr int kRing = kTaskTargets / kTPT + 1;
-    long long f[kRing];                         // f(block q) for the last kRing blocks (ring)
+    // stays in one block), and so is the argmin: the DP runs over blocks q.  The
+    // last kHist values of f are a shift register (fh[j] = f(q - 1 - j), f = 0 at
+    // and before block 0), so every candidate reads a fixed register.
+    constexpr int kHist = kTaskTargets / kTPT;
+    long long fh[kHist];
+#pragma unroll
+    for (int j = 0; j < kHist; ++j) fh[j] = 0;
     unsigned char arg[2 * kTaskTargets / kTPT + 1];
-    f[0] = 0;
     const int nb = (rest + kTPT - 1) / kTPT;
     for (int q = 1; q <= nb; ++q) {
         long long best = -1;
         int bi = 0;
+#pragma unroll
         for (int i = 0; i < kSliceCands; ++i) {
             if (!ok[i]) continue;
-            const int mq = slice_cand_m(i) / kTPT, prev = q > mq ? q - mq : 0;
-            const long long v = f[prev % kRing] + cost[i];
+            const long long v = fh[slice_cand_m(i) / kTPT - 1] + cost[i];
             if (best < 0 || v < best) {
                 best = v;
                 bi = i;
             }
         }
-        f[q % kRing] = best;
+#pragma unroll
+        for (int j = kHist - 1; j > 0; --j) fh[j] = fh[j - 1];
+        fh[0] = best;
         arg[q] = (unsigned char)bi;
     }
-    int k = 0;
+    int k = 0, mx = full > 0 ? M : 0;
     for (int a = rest; a > 0;) {
         const int mc = slice_cand_m(arg[(a + kTPT - 1) / kTPT]);
         const int m = mc < a ? mc : a;
         sz[k++] = (unsigned short)m;
+        mx = m > mx ? m : mx;
         a -= m;
     }
+    if (max_m) *max_m = mx;
     return k;
 }
 // Size of slice j of a plan (full slices first).

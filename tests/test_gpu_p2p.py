@@ -298,11 +298,11 @@ def test_set_tree_device_matches_host_ingest(world, coef, monkeypatch):
     bod = torch.empty((4, n), device="cuda")
     for a, src in enumerate((X, Y, Z, M)):
         tree.gather(src, bod[a])
-    outs = []
+    outs, worklists = [], []
     for mode in ("host", "device", "host-arrays"):
         monkeypatch.setenv("AFMM_HOST_INGEST", "1" if mode == "host" else "0")
         out = torch.full((4, n), float("nan"), device="cuda")
-        splits, stats = [], []
+        splits, stats, wls = [], [], []
         for r in range(world):
             h = afmm.P2P(rank=r, world=world, eps2=1e-6)
             h.set_bodies(bod[0], bod[1], bod[2], bod[3])
@@ -314,10 +314,19 @@ def test_set_tree_device_matches_host_ingest(world, coef, monkeypatch):
                 h.set_tree_device(info["n_leaves"], d["leaf_start"], d["leaf_count"], d["u_off"], d["u_idx"])
             stats.append(h.eval(out[0], out[1], out[2], out[3], stats=True))
             splits.append(h.get_partition())
+            wls.append(h.worklist())
             h.close()
         torch.cuda.synchronize()
         outs.append((out.cpu().numpy(), splits, stats))
+        worklists.append(wls)
     (oh, sh, th), (od, sd, td), (oa, sa, ta) = outs
+    if coef is None:                            # the same work list, task for task (dispatch order included)
+        for (tw, sw), (tdv, sdv), (ta_, sa_) in zip(*worklists):
+            assert tw.shape[0] > 0
+            assert np.array_equal(tw, tdv) and np.array_equal(sw, sdv)
+            assert np.array_equal(ta_, tdv) and np.array_equal(sa_, sdv)
+            cost = -(-np.maximum(tdv[:, 6], 1) // (32 // (-(-tdv[:, 1] // 4))))
+            assert (np.diff(cost) <= 0).all()     # largest modelled cost first
     assert np.array_equal(oh, od) and np.isfinite(od).all()
     assert np.array_equal(oa, od)
     for a, b in zip(sa, sd):
