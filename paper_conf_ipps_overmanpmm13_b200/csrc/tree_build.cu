@@ -650,6 +650,268 @@ __global__ void __launch_bounds__(kLvlThreads) levels_kernel(Nodes nd, const uns
     }
 }
 
+// ---- Direct construction from the sorted keys (fresh builds and Enforce_S
+// without edits; the level loop above stays for KEEP / FineGrainedOptimize edits).
+// The split rule of R7 / R22 restated on the sorted keys: the node at level l that
+// holds body i has MORE than S bodies iff some window of S + 1 consecutive sorted
+// keys containing i shares its first l octal digits (such a window lies inside the
+// node; conversely a node of >= S + 1 bodies holds such a window around i).  With
+// w_j = lcp(key_j, key_{j+S}) in digits and M_i = max w_j over the windows that
+// contain i, body i's leaf is at level min(M_i + 1, 21) (M_i = -1: the root); Enforce_S
+// then descends further while the node holds exactly S bodies (M'_i, windows of S)
+// and was a parent before.  Leaves start where lcp(key_{i-1}, key_i) < that level.
+// The internal nodes are the leaves' ancestors: the level-l ancestor of leaf j
+// starts at leaf j iff lcp with the previous leaf's first key < l, so every node is
+// (leaf j, level l) with lo_j <= l <= level_j; its rank inside its level is a prefix
+// count over the leaves, its children are the level l+1 nodes starting at leaves
+// [j, j_end).  Output: the same level-major Nodes arrays as levels_kernel, plus
+// the leaf arrays (bit-identical; tests compare both paths).
+__device__ __forceinline__ int lcp_digits(unsigned long long a, unsigned long long b) {
+    return a == b ? kMaxLevel : (__clzll((long long)(a ^ b)) - 1) / 3;
+}
+constexpr int kDirTile = 2048;              // positions per block of leaf_level_kernel
+constexpr int kDirThreads = 256;
+constexpr int kDirMaxS = 2048;              // larger S: the level loop
+constexpr int kDirLevels = kMaxLevel + 1;   // levels 0..21
+struct DirCtl {
+    long long base[kDirLevels + 1];         // level starts; base[levels] = nodes
+    long long nn;
+    int levels;
+    int L;
+    int sort_overflow;                      // the bucket sort's flag, copied in before the readback
+};
+
+__global__ void __launch_bounds__(kDirThreads) leaf_level_kernel(long long n, const unsigned long long *__restrict__ keys,
+                                                                 int S, int mode, PrevTree pv,
+                                                                 unsigned char *__restrict__ lvl, int *__restrict__ flag) {
+    // [buffer][array][pos]: array 0 = windows of S + 1 (w), 1 = windows of S (v);
+    // position a <-> window start j = t0 - S + a; -1 = no such window
+    __shared__ signed char win[2][2][kDirTile + kDirMaxS];
+    const long long t0 = (long long)blockIdx.x * kDirTile;
+    const int len = kDirTile + S;
+    for (int a = threadIdx.x; a < len; a += blockDim.x) {
+        const long long j = t0 - S + a;
+        signed char w = -1, v = -1;
+        if (j >= 0) {
+            const unsigned long long kj = j < n ? keys[j] : 0ull;
+            if (j + S < n) w = (signed char)lcp_digits(kj, keys[j + S]);
+            if (j + S - 1 < n) v = (signed char)lcp_digits(kj, keys[j + S - 1]);
+        }
+        win[0][0][a] = w;
+        win[0][1][a] = v;
+    }
+    // doubling: after the pass of step h, X[a] = max over [a, a + 2h)
+    int HA = 1, HB = 1;                      // largest powers of two <= S + 1 and <= S
+    while (2 * HA <= S + 1) HA *= 2;
+    while (2 * HB <= S) HB *= 2;
+    int cur = 0;
+    for (int h = 1; h < HA; h *= 2) {
+        __syncthreads();
+        for (int a = threadIdx.x; a < len; a += blockDim.x) {
+            const signed char x = win[cur][0][a], y = a + h < len ? win[cur][0][a + h] : (signed char)-1;
+            win[cur ^ 1][0][a] = x > y ? x : y;
+            const signed char p = win[cur][1][a], q = a + h < len ? win[cur][1][a + h] : (signed char)-1;
+            win[cur ^ 1][1][a] = h < HB ? (p > q ? p : q) : p;
+        }
+        cur ^= 1;
+    }
+    __syncthreads();
+    for (int a0 = threadIdx.x; a0 < kDirTile; a0 += blockDim.x) {
+        const long long i = t0 + a0;
+        if (i >= n) break;
+        // windows of S + 1 containing i: j in [i - S, i] -> a in [a0, a0 + S]
+        const int m1 = max((int)win[cur][0][a0], (int)win[cur][0][a0 + S + 1 - HA]);
+        // windows of S containing i: j in [i - S + 1, i] -> a in [a0 + 1, a0 + S]
+        const int m2 = max((int)win[cur][1][a0 + 1], (int)win[cur][1][a0 + 1 + S - HB]);
+        const unsigned long long ki = keys[i];
+        int l = m1 < 0 ? 0 : min(m1 + 1, kMaxLevel);
+        if (mode == kModeEnforce && pv.levels > 0)
+            while (l < kMaxLevel && l <= m2 && prev_internal(pv, l, ki >> (3 * (kMaxLevel - l)))) ++l;
+        lvl[i] = (unsigned char)l;
+        flag[i] = (i == 0 || lcp_digits(keys[i - 1], ki) < l) ? 1 : 0;
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) flag[n] = 0;
+}
+
+// Leaf j (first body i): start, level, prefix, first key, and lo_j = the first level
+// whose node starts at this leaf (lcp with the previous body + 1; 0 for leaf 0).
+__global__ void leaf_info_kernel(long long n, const unsigned long long *__restrict__ keys,
+                                 const unsigned char *__restrict__ lvl, const int *__restrict__ flag,
+                                 const int *__restrict__ leaf_at, int *__restrict__ ls, int *__restrict__ ll,
+                                 unsigned long long *__restrict__ lp, unsigned long long *__restrict__ fk,
+                                 unsigned char *__restrict__ llo) {
+    const long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (i >= n || !flag[i]) return;
+    const int id = leaf_at[i], l = lvl[i];
+    const unsigned long long k = keys[i];
+    ls[id] = (int)i;
+    ll[id] = l;
+    lp[id] = k >> (3 * (kMaxLevel - l));
+    fk[id] = k;
+    llo[id] = (unsigned char)(i == 0 ? 0 : lcp_digits(keys[i - 1], k) + 1);
+}
+
+// Per block of 256 leaves: how many nodes of each level start at its leaves (and
+// the leaf counts).  Grid over an upper bound of L; L = leaf_at[n] on the device.
+constexpr int kDirLeafBlock = 256;
+__global__ void __launch_bounds__(kDirLeafBlock) node_count_kernel(long long n, const int *__restrict__ leaf_at,
+                                                                   const int *__restrict__ ls,
+                                                                   const int *__restrict__ ll,
+                                                                   const unsigned char *__restrict__ llo,
+                                                                   int *__restrict__ lc, int *__restrict__ chunk_cnt) {
+    __shared__ int cnt[kDirLevels];
+    const int L = leaf_at[n];
+    if ((long long)blockIdx.x * kDirLeafBlock >= L) return;
+    if (threadIdx.x < kDirLevels) cnt[threadIdx.x] = 0;
+    __syncthreads();
+    const int j = blockIdx.x * kDirLeafBlock + threadIdx.x;
+    int lo = 1, hi = 0;
+    if (j < L) {
+        lo = llo[j];
+        hi = ll[j];
+        lc[j] = (j + 1 < L ? ls[j + 1] : (int)n) - ls[j];
+    }
+    for (int l = 0; l < kDirLevels; ++l) {
+        const unsigned m = __ballot_sync(0xffffffffu, lo <= l && l <= hi);
+        if ((threadIdx.x & 31) == 0 && m) atomicAdd(&cnt[l], __popc(m));
+    }
+    __syncthreads();
+    if (threadIdx.x < kDirLevels) chunk_cnt[(size_t)blockIdx.x * kDirLevels + threadIdx.x] = cnt[threadIdx.x];
+}
+
+// One block, a warp per level: exclusive scan of the chunk counts over the chunks
+// (chunk_base), level totals -> level starts, node total, levels; L.
+__global__ void __launch_bounds__(32 * kDirLevels) node_scan_kernel(long long n, const int *__restrict__ leaf_at,
+                                                                    const int *__restrict__ chunk_cnt,
+                                                                    int *__restrict__ chunk_base,
+                                                                    int *__restrict__ level_cnt, DirCtl *ctl) {
+    __shared__ long long tot[kDirLevels];
+    const int L = leaf_at[n];
+    const int nchunk = (L + kDirLeafBlock - 1) / kDirLeafBlock;
+    const int l = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    int carry = 0;
+    for (int c0 = 0; c0 < nchunk; c0 += 32) {
+        const int c = c0 + lane;
+        const int v = c < nchunk ? chunk_cnt[(size_t)c * kDirLevels + l] : 0;
+        int inc = v;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int u = __shfl_up_sync(0xffffffffu, inc, o);
+            if (lane >= o) inc += u;
+        }
+        if (c < nchunk) chunk_base[(size_t)c * kDirLevels + l] = carry + inc - v;
+        carry += __shfl_sync(0xffffffffu, inc, 31);
+    }
+    if (lane == 0) {
+        tot[l] = carry;
+        level_cnt[l] = carry;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        long long b = 0;
+        int levels = 0;
+        for (int k = 0; k < kDirLevels; ++k) {
+            ctl->base[k] = b;
+            b += tot[k];
+            if (tot[k] > 0) levels = k + 1;
+        }
+        ctl->base[kDirLevels] = b;
+        ctl->nn = b;
+        ctl->levels = levels;
+        ctl->L = L;
+    }
+}
+
+// Per leaf: its rank among the nodes of every level (rank[l][j] = nodes of level l
+// starting at leaves < j; row length L + 1, rank[l][L] = the level's node count) and
+// the nodes that start at it: b, level, prefix; for the leaf itself also e, no
+// children, and the leaf <-> node maps.
+__global__ void __launch_bounds__(kDirLeafBlock) node_rank_kernel(const DirCtl *__restrict__ ctl,
+                                                                  const int *__restrict__ chunk_base,
+                                                                  const int *__restrict__ level_cnt,
+                                                                  const int *__restrict__ ls,
+                                                                  const int *__restrict__ lc,
+                                                                  const int *__restrict__ ll,
+                                                                  const unsigned char *__restrict__ llo,
+                                                                  const unsigned long long *__restrict__ fk,
+                                                                  int *__restrict__ rank, Nodes nd,
+                                                                  int *__restrict__ node_leaf,
+                                                                  int *__restrict__ leaf_node) {
+    __shared__ int wcnt[kDirLeafBlock / 32][kDirLevels];
+    const int L = ctl->L;
+    if ((long long)blockIdx.x * kDirLeafBlock >= L) return;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int j = blockIdx.x * kDirLeafBlock + threadIdx.x;
+    int lo = 1, hi = 0;
+    if (j < L) {
+        lo = llo[j];
+        hi = ll[j];
+    }
+    unsigned below[kDirLevels];
+#pragma unroll
+    for (int l = 0; l < kDirLevels; ++l) {
+        const unsigned m = __ballot_sync(0xffffffffu, lo <= l && l <= hi);
+        below[l] = __popc(m & ((1u << lane) - 1u));
+        if (lane == 0) wcnt[wid][l] = __popc(m);
+    }
+    __syncthreads();
+    if (j < L) {
+        const size_t row = (size_t)L + 1;
+        const int bj = ls[j];
+        const unsigned long long k = fk[j];
+        int r[kDirLevels];
+#pragma unroll
+        for (int l = 0; l < kDirLevels; ++l) {
+            r[l] = chunk_base[(size_t)blockIdx.x * kDirLevels + l] + (int)below[l];
+            for (int w = 0; w < wid; ++w) r[l] += wcnt[w][l];
+            rank[l * row + j] = r[l];
+        }
+#pragma unroll
+        for (int l = 0; l < kDirLevels; ++l) {
+            if (lo <= l && l <= hi) {
+                const long long id = ctl->base[l] + r[l];
+                nd.b[id] = bj;
+                nd.level[id] = l;
+                nd.prefix[id] = k >> (3 * (kMaxLevel - l));
+                if (l == hi) {
+                    nd.e[id] = bj + lc[j];
+                    nd.nchild[id] = 0;
+                    nd.first_child[id] = -1;
+                    node_leaf[id] = j;
+                    leaf_node[j] = (int)id;
+                } else {                          // internal: its first child starts at this leaf too
+                    nd.first_child[id] = (int)(ctl->base[l + 1] + r[l < kDirLevels - 1 ? l + 1 : l]);
+                    node_leaf[id] = -1;
+                }
+            }
+        }
+        if (j == L - 1) {
+#pragma unroll
+            for (int l = 0; l < kDirLevels; ++l) rank[l * row + L] = level_cnt[l];
+        }
+    }
+}
+
+// Internal nodes, from the side where they end: the level-l ancestors of leaf
+// j' - 1 that do not hold leaf j' (llo[j'] <= l < level of leaf j' - 1; every level
+// for j' = L) end at leaf j': e = its first body (n), and the children are the level
+// l + 1 nodes up to there (first_child was written by node_rank_kernel).  O(1) per node.
+__global__ void node_links_kernel(long long n, const DirCtl *__restrict__ ctl, const int *__restrict__ ls,
+                                  const int *__restrict__ ll, const unsigned char *__restrict__ llo,
+                                  const int *__restrict__ rank, Nodes nd) {
+    const int L = ctl->L;
+    const int j = blockIdx.x * blockDim.x + threadIdx.x + 1;     // j' in [1, L]
+    if (j > L) return;
+    const int lo = j < L ? llo[j] : 0, hi = ll[j - 1];
+    const size_t row = (size_t)L + 1;
+    const int e = j < L ? ls[j] : (int)n;
+    for (int l = lo; l < hi; ++l) {
+        const long long id = ctl->base[l] + rank[l * row + j] - 1;
+        nd.e[id] = e;
+        nd.nchild[id] = (int)(ctl->base[l + 1] + rank[(l + 1) * row + j] - nd.first_child[id]);
+    }
+}
+
 __global__ void leaf_flag_kernel(int nn, Nodes nd, int *__restrict__ flag) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= nn) return;
@@ -727,12 +989,25 @@ __global__ void ulist_kernel(int L, Nodes nd, const int *__restrict__ node_leaf,
 // computed once per build so the descent below tests a node with one 8-byte load
 // and a few shifts instead of three Morton compactions per node (the descent was
 // instruction-bound, ncu: 69 % issue active).
-__global__ void anchors_kernel(int nn, Nodes nd, unsigned long long *__restrict__ anc) {
+// One 16-byte record per node for the descent: {anchor, level | nchild << 8, first
+// child (internal) or leaf id (leaf)} -- one LDG.128 per visited node instead of
+// five loads from the separate node arrays.
+struct __align__(16) NodeRec {
+    unsigned long long anc;
+    int meta;
+    int link;
+};
+__global__ void anchors_kernel(int nn, Nodes nd, const int *__restrict__ node_leaf, NodeRec *__restrict__ rec) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= nn) return;
     long long A[3], w;
-    box_of(nd.level[i], nd.prefix[i], A, w);
-    anc[i] = (unsigned long long)A[0] | ((unsigned long long)A[1] << 21) | ((unsigned long long)A[2] << 42);
+    const int lev = nd.level[i], nc = nd.nchild[i];
+    box_of(lev, nd.prefix[i], A, w);
+    NodeRec r;
+    r.anc = (unsigned long long)A[0] | ((unsigned long long)A[1] << 21) | ((unsigned long long)A[2] << 42);
+    r.meta = lev | (nc << 8);
+    r.link = nc ? nd.first_child[i] : node_leaf[i];
+    rec[i] = r;
 }
 
 constexpr int kURow = 256;                  // max row length kept by the warp path
@@ -740,7 +1015,7 @@ constexpr int kUFront = 512;                // max frontier length
 constexpr int kUWarps = 4;                  // warps per block
 __global__ void __launch_bounds__(32 * kUWarps) ulist_warp_kernel(int L, Nodes nd, const int *__restrict__ node_leaf,
                                                                   const int *__restrict__ leaf_node,
-                                                                  const unsigned long long *__restrict__ anc,
+                                                                  const NodeRec *__restrict__ rec,
                                                                   int *__restrict__ rows, long long *__restrict__ counts,
                                                                   int *__restrict__ overflow) {
     __shared__ int front[kUWarps][2][kUFront];
@@ -763,22 +1038,22 @@ __global__ void __launch_bounds__(32 * kUWarps) ulist_warp_kernel(int L, Nodes n
                 int nch = 0, fc = 0, lid = 0;
                 if (j < ncur) {
                     const int ni = front[wi][cur][j];
-                    const unsigned long long an = anc[ni];
-                    const int ws = 1 << (kMaxLevel - nd.level[ni]);
+                    const NodeRec r = rec[ni];
+                    const int ws = 1 << (kMaxLevel - (r.meta & 255));
                     bool touch = true;
 #pragma unroll
                     for (int a = 0; a < 3; ++a) {
-                        const int As = (int)((an >> (21 * a)) & 0x1fffffull);
+                        const int As = (int)((r.anc >> (21 * a)) & 0x1fffffull);
                         touch &= (At[a] <= As + ws) && (As <= At[a] + wt);
                     }
                     if (touch) {
-                        const int c = nd.nchild[ni];
+                        const int c = r.meta >> 8;
                         if (c == 0) {
                             leaf = true;
-                            lid = node_leaf[ni];
+                            lid = r.link;
                         } else {
                             nch = c;
-                            fc = nd.first_child[ni];
+                            fc = r.link;
                         }
                     }
                 }
@@ -1021,7 +1296,8 @@ enum Slot {
     kPart, kKeys, kIdx, kKeysSorted, kPerm, kSortTmp, kNodeA, kNodeB = kNodeA + 6, kCb = kNodeB + 6, kNc, kOff,
     kScanTmp, kFlag, kLeafAt, kNodeLeaf, kScan2, kLs, kLc, kLl, kLp, kLeafNode, kCounts, kUoff, kScan3, kUidx,
     kFarfield, kEditPrefix, kEditAction, kEditBase, kURows, kUOvf, kLvlCtl, kTsum, kAnc,
-    kCellLo, kCellHi, kBucket, kSlot, kBCount, kBOff, kBKeys, kBIdx, kBScan, kBOvf
+    kCellLo, kCellHi, kBucket, kSlot, kBCount, kBOff, kBKeys, kBIdx, kBScan, kBOvf,
+    kDirLvl, kDirFk, kDirLlo, kDirChunkCnt, kDirChunkBase, kDirLevelCnt, kDirCtl, kDirRank
 };
 
 __global__ void root_kernel(Nodes nd, int n) {
@@ -1207,9 +1483,82 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     int level = 0;
     int *cb = nullptr, *nc = nullptr, *off = nullptr;
     bool done_levels = false;
+    // 4d. direct construction from the sorted keys (fresh / Enforce_S, no edits, S <= kDirMaxS):
+    //     leaves and nodes by a handful of flat kernels, one host readback (L, node
+    //     count, level starts, the bucket sort's overflow flag)
+    int *flag = nullptr, *leaf_at = nullptr, *node_leaf = nullptr, *leaf_node = nullptr;
+    int L = 0;
+    const char *lv_env = getenv("AFMM_TREE_LEVELS");                 // tests / A-B: force the level loop
+    const bool direct = mode != kModeKeep && ed.n == 0 && S <= kDirMaxS && !(lv_env && lv_env[0] == '1');
+    for (int attempt = 0; direct && attempt < 3 && !done_levels; ++attempt) {
+        unsigned char *lvl, *llo;
+        unsigned long long *fk;
+        int *chunk_cnt, *chunk_base, *level_cnt, *rank;
+        DirCtl *dctl;
+        const long long nchunk = (n + kDirLeafBlock - 1) / kDirLeafBlock;
+        if (afmm_status s = wsalloc(t, kFlag, &flag, n + 1)) return s;
+        if (afmm_status s = wsalloc(t, kLeafAt, &leaf_at, n + 1)) return s;
+        if (afmm_status s = wsalloc(t, kDirLvl, &lvl, n)) return s;
+        if (afmm_status s = wsalloc(t, kLs, &t->ls, n)) return s;
+        if (afmm_status s = wsalloc(t, kLc, &t->lc, n)) return s;
+        if (afmm_status s = wsalloc(t, kLl, &t->ll, n)) return s;
+        if (afmm_status s = wsalloc(t, kLp, &t->lp, n)) return s;
+        if (afmm_status s = wsalloc(t, kDirFk, &fk, n)) return s;
+        if (afmm_status s = wsalloc(t, kDirLlo, &llo, n)) return s;
+        if (afmm_status s = wsalloc(t, kDirChunkCnt, &chunk_cnt, (size_t)nchunk * kDirLevels)) return s;
+        if (afmm_status s = wsalloc(t, kDirChunkBase, &chunk_base, (size_t)nchunk * kDirLevels)) return s;
+        if (afmm_status s = wsalloc(t, kDirLevelCnt, &level_cnt, kDirLevels)) return s;
+        if (afmm_status s = wsalloc(t, kDirCtl, reinterpret_cast<char **>(&dctl), sizeof(DirCtl))) return s;
+        leaf_level_kernel<<<(int)((n + kDirTile - 1) / kDirTile), kDirThreads, 0, st>>>(n, t->keys_sorted, S, mode,
+                                                                                       pv, lvl, flag);
+        TCU(t, cudaGetLastError());
+        {
+            size_t sb = 0;
+            TCU(t, cub::DeviceScan::ExclusiveSum(nullptr, sb, flag, leaf_at, (int)(n + 1), st));
+            char *sbuf;
+            if (afmm_status s = wsalloc(t, kScan2, &sbuf, sb)) return s;
+            TCU(t, cub::DeviceScan::ExclusiveSum(sbuf, sb, flag, leaf_at, (int)(n + 1), st));
+        }
+        leaf_info_kernel<<<grid_for(n, TH), TH, 0, st>>>(n, t->keys_sorted, lvl, flag, leaf_at, t->ls, t->ll, t->lp,
+                                                         fk, llo);
+        node_count_kernel<<<(int)nchunk, kDirLeafBlock, 0, st>>>(n, leaf_at, t->ls, t->ll, llo, t->lc, chunk_cnt);
+        node_scan_kernel<<<1, 32 * kDirLevels, 0, st>>>(n, leaf_at, chunk_cnt, chunk_base, level_cnt, dctl);
+        TCU(t, cudaGetLastError());
+        if (bovf) TCU(t, cudaMemcpyAsync(&dctl->sort_overflow, bovf, sizeof(int), cudaMemcpyDeviceToDevice, st));
+        else TCU(t, cudaMemsetAsync(&dctl->sort_overflow, 0, sizeof(int), st));
+        DirCtl hc;
+        TCU(t, cudaMemcpyAsync(&hc, dctl, sizeof(DirCtl), cudaMemcpyDeviceToHost, st));
+        TCU(t, cudaStreamSynchronize(st));
+        if (hc.sort_overflow) {                       // a bucket exceeded kBucketCap: sort in full, redo
+            bovf = nullptr;
+            ++t->sort_fallbacks;
+            if (getenv("AFMM_TREE_DEBUG")) fprintf(stderr, "afmm tree: bucket sort overflow %lld\n", t->sort_fallbacks);
+            if (afmm_status s = full_sort()) return s;
+            continue;
+        }
+        L = hc.L;
+        if ((long long)cap < hc.nn) {
+            cap = std::max<size_t>((size_t)hc.nn, (size_t)(2 * n + 64));
+            node_set = node_set == kNodeA ? kNodeB : kNodeA;
+            if (afmm_status s = alloc_nodes(cap, nd, node_set)) return s;
+        }
+        if (afmm_status s = wsalloc(t, kNodeLeaf, &node_leaf, (size_t)hc.nn)) return s;
+        if (afmm_status s = wsalloc(t, kLeafNode, &leaf_node, (size_t)L)) return s;
+        if (afmm_status s = wsalloc(t, kDirRank, &rank, (size_t)kDirLevels * ((size_t)L + 1))) return s;
+        node_rank_kernel<<<(L + kDirLeafBlock - 1) / kDirLeafBlock, kDirLeafBlock, 0, st>>>(
+            dctl, chunk_base, level_cnt, t->ls, t->lc, t->ll, llo, fk, rank, nd, node_leaf, leaf_node);
+        node_links_kernel<<<grid_for(L, TH), TH, 0, st>>>(n, dctl, t->ls, t->ll, llo, rank, nd);
+        TCU(t, cudaGetLastError());
+        lvl_base.assign(hc.base, hc.base + hc.levels);
+        base = hc.nn;
+        t->max_level = hc.levels - 1;
+        done_levels = true;
+    }
+    const bool direct_done = done_levels;
+    if (direct && !done_levels) return tfail(t, AFMM_ECUDA, "tree_build: bucket sort kept overflowing");
     // 4a. all levels in one cooperative launch (grid barriers between phases); the
     //     node arrays start at >= 2n + 64 nodes and are doubled on overflow
-    if (t->coop_ok) {
+    if (!done_levels && t->coop_ok) {
         if (cap < (size_t)(2 * n + 64)) {
             cap = (size_t)(2 * n + 64);
             if (afmm_status s = alloc_nodes(cap, nd, node_set)) return s;
@@ -1349,8 +1698,8 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
                            cudaMemcpyHostToDevice, st));
     t->pv_levels = (int)lvl_base.size() - 1;
 
-    // 5. leaves in Morton order: flag first bodies, scan
-    int *flag, *leaf_at, *node_leaf;
+    // 5. leaves in Morton order: flag first bodies, scan (the direct path has them)
+    if (!direct_done) {
     if (afmm_status s = wsalloc(t, kFlag, &flag, n + 1)) return s;
     if (afmm_status s = wsalloc(t, kLeafAt, &leaf_at, n + 1)) return s;
     if (afmm_status s = wsalloc(t, kNodeLeaf, &node_leaf, nn)) return s;
@@ -1364,20 +1713,19 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
         if (afmm_status s = wsalloc(t, kScan2, &sbuf, sb)) return s;
         TCU(t, cub::DeviceScan::ExclusiveSum(sbuf, sb, flag, leaf_at, (int)(n + 1), st));
     }
-    int L = 0;
     TCU(t, cudaMemcpyAsync(&L, leaf_at + n, sizeof(int), cudaMemcpyDeviceToHost, st));
     TCU(t, cudaStreamSynchronize(st));
-    t->L = L;
     if (afmm_status s = wsalloc(t, kLs, &t->ls, L)) return s;
     if (afmm_status s = wsalloc(t, kLc, &t->lc, L)) return s;
     if (afmm_status s = wsalloc(t, kLl, &t->ll, L)) return s;
     if (afmm_status s = wsalloc(t, kLp, &t->lp, L)) return s;
     leaf_write_kernel<<<grid_for(nn, TH), TH, 0, st>>>((int)nn, nd, leaf_at, node_leaf, t->ls, t->lc, t->ll, t->lp);
     TCU(t, cudaGetLastError());
-    int *leaf_node;
     if (afmm_status s = wsalloc(t, kLeafNode, &leaf_node, L)) return s;
     leaf_node_kernel<<<grid_for(nn, TH), TH, 0, st>>>((int)nn, node_leaf, leaf_node);
     TCU(t, cudaGetLastError());
+    }
+    t->L = L;
 
     // 6. U-lists: warp-cooperative descent into fixed-capacity rows, scan, compact
     //    (rows longer than kURow or frontiers wider than kUFront: per-thread DFS count + fill)
@@ -1391,10 +1739,10 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     TCU(t, cudaMemsetAsync(ovf, 0, sizeof(int), st));
     {
         const int blocks = (int)std::min<long long>((L + kUWarps - 1) / kUWarps, 148LL * 16);
-        unsigned long long *anc;
-        if (afmm_status s = wsalloc(t, kAnc, &anc, (size_t)nn)) return s;
-        anchors_kernel<<<grid_for(nn, TH), TH, 0, st>>>((int)nn, nd, anc);
-        ulist_warp_kernel<<<blocks, 32 * kUWarps, 0, st>>>(L, nd, node_leaf, leaf_node, anc, rows, counts, ovf);
+        NodeRec *rec;
+        if (afmm_status s = wsalloc(t, kAnc, &rec, (size_t)nn)) return s;
+        anchors_kernel<<<grid_for(nn, TH), TH, 0, st>>>((int)nn, nd, node_leaf, rec);
+        ulist_warp_kernel<<<blocks, 32 * kUWarps, 0, st>>>(L, nd, node_leaf, leaf_node, rec, rows, counts, ovf);
         TCU(t, cudaGetLastError());
     }
     // row offsets by a scan of the counts, read back together with the overflow flag

@@ -179,3 +179,56 @@ def test_rebuild_bucket_sort_bit_exact(monkeypatch):
             t.build(_dev(px), _dev(py), _dev(pz), S, domain=dom)
             assert_same_tree(t.copy_out(n), oracle.Tree(px, py, pz, S, domain=dom))
         t.close()
+
+
+def _tree_and_nodes(t, n):
+    G = t.copy_out(n)
+    G.update({"node_" + k: v for k, v in t.nodes().items()})
+    G.update({"info_" + k: v for k, v in t.info().items() if not isinstance(v, np.ndarray)})
+    return G
+
+
+def test_direct_construction_matches_level_loop(monkeypatch):
+    """The direct construction (leaf levels from sliding windows over the sorted
+    keys, nodes as the leaves' ancestors; tree_build.cu section 4d) and the
+    level-synchronous split loop (AFMM_TREE_LEVELS=1) give identical trees AND
+    identical node arrays (the next Enforce_S reads them): fresh builds incl. S = 1,
+    n <= S, duplicate keys (level-21 leaves above S), and Enforce_S chains where
+    nodes hold exactly S bodies (the 'was a parent' rule), incl. at the root."""
+    afmm = _afmm()
+    cases = []
+    x, y, z, m = synth.make("plummer", 40000, 7)
+    cases.append(("plummer", (x, y, z), [("build", 16), ("enforce", 16), ("enforce", 24), ("enforce", 8)]))
+    x, y, z, m = synth.make("uniform", 600, 3)
+    idx = np.arange(600) % 40
+    cases.append(("dups", (x[idx], y[idx], z[idx]), [("build", 4), ("enforce", 15), ("enforce", 16), ("build", 1)]))
+    x, y, z, m = synth.lattice(8)
+    cases.append(("lattice", (x, y, z), [("build", 1), ("enforce", 2), ("enforce", 8), ("enforce", 1)]))
+    x, y, z, m = synth.make("uniform", 64, 9)
+    cases.append(("root==S", (x, y, z), [("build", 32), ("enforce", 64), ("enforce", 64), ("build", 64),
+                                         ("enforce", 100)]))
+    x, y, z, m = synth.make("uniform", 1, 5)
+    cases.append(("n=1", (x, y, z), [("build", 1), ("enforce", 1)]))
+    rng = np.random.default_rng(3)
+    for name, (x, y, z), ops in cases:
+        n = x.shape[0]
+        res = {}
+        for flag in ("0", "1"):
+            monkeypatch.setenv("AFMM_TREE_LEVELS", flag)
+            t = afmm.GpuTree(0)
+            px, py, pz = x, y, z
+            out = []
+            for step, (op, S) in enumerate(ops):
+                if step > 0 and op == "enforce":        # small deterministic motion between Enforce_S calls
+                    d = np.random.default_rng(step).standard_normal((3, n)).astype(np.float32) * np.float32(1e-3)
+                    px, py, pz = px + d[0], py + d[1], pz + d[2]
+                fn = t.build if op == "build" else t.enforce
+                fn(_dev(px), _dev(py), _dev(pz), S)
+                out.append(_tree_and_nodes(t, n))
+            t.close()
+            res[flag] = out
+        for step, (a, b) in enumerate(zip(res["0"], res["1"])):
+            assert a.keys() == b.keys()
+            for k in a:
+                assert np.array_equal(np.asarray(a[k]), np.asarray(b[k])), (name, step, k)
+    del rng
