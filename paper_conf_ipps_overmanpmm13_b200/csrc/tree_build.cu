@@ -676,10 +676,17 @@ constexpr int kDirLevels = kMaxLevel + 1;   // levels 0..21
 struct DirCtl {
     long long base[kDirLevels + 1];         // level starts; base[levels] = nodes
     long long nn;
+    long long nnz;                          // U-list entries (u_off[L])
     int levels;
     int L;
     int sort_overflow;                      // the bucket sort's flag, copied in before the readback
+    int cap_overflow;                       // nodes > node capacity or leaves > leaf capacity: nothing written
+    int ulist_overflow;                     // a warp-descent row / frontier overflowed: per-thread DFS fallback
+    int nnz_overflow;                       // U-list entries > their capacity: u_idx not written
 };
+__device__ __forceinline__ bool dir_bad(const DirCtl *c) {
+    return c->sort_overflow | c->cap_overflow | c->ulist_overflow | c->nnz_overflow;
+}
 
 __global__ void __launch_bounds__(kDirThreads) leaf_level_kernel(long long n, const unsigned long long *__restrict__ keys,
                                                                  int S, int mode, PrevTree pv,
@@ -826,7 +833,7 @@ __global__ void __launch_bounds__(32 * kDirLevels) node_scan_kernel(long long n,
 // starting at leaves < j; row length L + 1, rank[l][L] = the level's node count) and
 // the nodes that start at it: b, level, prefix; for the leaf itself also e, no
 // children, and the leaf <-> node maps.
-__global__ void __launch_bounds__(kDirLeafBlock) node_rank_kernel(const DirCtl *__restrict__ ctl,
+__global__ void __launch_bounds__(kDirLeafBlock) node_rank_kernel(DirCtl *__restrict__ ctl,
                                                                   const int *__restrict__ chunk_base,
                                                                   const int *__restrict__ level_cnt,
                                                                   const int *__restrict__ ls,
@@ -836,9 +843,14 @@ __global__ void __launch_bounds__(kDirLeafBlock) node_rank_kernel(const DirCtl *
                                                                   const unsigned long long *__restrict__ fk,
                                                                   int *__restrict__ rank, Nodes nd,
                                                                   int *__restrict__ node_leaf,
-                                                                  int *__restrict__ leaf_node) {
+                                                                  int *__restrict__ leaf_node,
+                                                                  long long node_cap, int leaf_cap) {
     __shared__ int wcnt[kDirLeafBlock / 32][kDirLevels];
     const int L = ctl->L;
+    if (ctl->nn > node_cap || L > leaf_cap) {                  // every block returns; the host grows and reruns
+        if (blockIdx.x == 0 && threadIdx.x == 0) ctl->cap_overflow = 1;
+        return;
+    }
     if ((long long)blockIdx.x * kDirLeafBlock >= L) return;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const int j = blockIdx.x * kDirLeafBlock + threadIdx.x;
@@ -898,10 +910,10 @@ __global__ void __launch_bounds__(kDirLeafBlock) node_rank_kernel(const DirCtl *
 // l + 1 nodes up to there (first_child was written by node_rank_kernel).  O(1) per node.
 __global__ void node_links_kernel(long long n, const DirCtl *__restrict__ ctl, const int *__restrict__ ls,
                                   const int *__restrict__ ll, const unsigned char *__restrict__ llo,
-                                  const int *__restrict__ rank, Nodes nd) {
+                                  const int *__restrict__ rank, Nodes nd, long long node_cap, int leaf_cap) {
+    if (ctl->nn > node_cap || ctl->L > leaf_cap) return;
     const int L = ctl->L;
-    const int j = blockIdx.x * blockDim.x + threadIdx.x + 1;     // j' in [1, L]
-    if (j > L) return;
+    for (int j = blockIdx.x * blockDim.x + threadIdx.x + 1; j <= L; j += gridDim.x * blockDim.x) {   // j' in [1, L]
     const int lo = j < L ? llo[j] : 0, hi = ll[j - 1];
     const size_t row = (size_t)L + 1;
     const int e = j < L ? ls[j] : (int)n;
@@ -909,6 +921,26 @@ __global__ void node_links_kernel(long long n, const DirCtl *__restrict__ ctl, c
         const long long id = ctl->base[l] + rank[l * row + j] - 1;
         nd.e[id] = e;
         nd.nchild[id] = (int)(ctl->base[l + 1] + rank[(l + 1) * row + j] - nd.first_child[id]);
+    }
+    }
+}
+
+// The direct build's tail, after the U-lists: unless something overflowed, keep
+// the node arrays as the next Enforce_S's previous tree (prefix, nchild, level
+// starts) and the U-list total -- on the device, no host round trip.
+__global__ void dir_finish_kernel(DirCtl *ctl, Nodes nd, const long long *__restrict__ u_off,
+                                  unsigned long long *__restrict__ pv_prefix, int *__restrict__ pv_nchild,
+                                  long long *__restrict__ pv_base) {
+    if (dir_bad(ctl)) return;
+    const long long nn = ctl->nn;
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < nn; i += (long long)gridDim.x * blockDim.x) {
+        pv_prefix[i] = nd.prefix[i];
+        pv_nchild[i] = nd.nchild[i];
+    }
+    if (blockIdx.x == 0 && threadIdx.x <= kDirLevels) {
+        const int l = threadIdx.x;
+        if (l <= ctl->levels) pv_base[l] = l < ctl->levels ? ctl->base[l] : nn;
+        if (l == 0) ctl->nnz = u_off[ctl->L];
     }
 }
 
@@ -997,7 +1029,12 @@ struct __align__(16) NodeRec {
     int meta;
     int link;
 };
-__global__ void anchors_kernel(int nn, Nodes nd, const int *__restrict__ node_leaf, NodeRec *__restrict__ rec) {
+__global__ void anchors_kernel(int nn, Nodes nd, const int *__restrict__ node_leaf, NodeRec *__restrict__ rec,
+                               const DirCtl *__restrict__ ctl = nullptr) {
+    if (ctl) {                                   // direct build: the node count is on the device
+        if (dir_bad(ctl)) return;
+        nn = (int)ctl->nn;
+    }
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= nn) return;
     long long A[3], w;
@@ -1017,11 +1054,19 @@ __global__ void __launch_bounds__(32 * kUWarps) ulist_warp_kernel(int L, Nodes n
                                                                   const int *__restrict__ leaf_node,
                                                                   const NodeRec *__restrict__ rec,
                                                                   int *__restrict__ rows, long long *__restrict__ counts,
-                                                                  int *__restrict__ overflow) {
+                                                                  int *__restrict__ overflow,
+                                                                  DirCtl *ctl = nullptr, int leaf_cap = 0) {
     __shared__ int front[kUWarps][2][kUFront];
     __shared__ int res[kUWarps][kURow];
     const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5;
     const int nwarps = gridDim.x * kUWarps;
+    if (ctl) {                                   // direct build: L on the device; counts past L zeroed (the scan
+        if (dir_bad(ctl)) return;                // runs over the leaf capacity)
+        L = ctl->L;
+        overflow = &ctl->ulist_overflow;
+        for (int j = L + 1 + blockIdx.x * blockDim.x + threadIdx.x; j <= leaf_cap; j += gridDim.x * blockDim.x)
+            counts[j] = 0;
+    }
     for (int t = blockIdx.x * kUWarps + wi; t < L; t += nwarps) {
         const int tn = leaf_node[t];
         long long At[3], wt;
@@ -1095,7 +1140,18 @@ __global__ void __launch_bounds__(32 * kUWarps) ulist_warp_kernel(int L, Nodes n
 }
 
 __global__ void ulist_copy_kernel(int L, const int *__restrict__ rows, const long long *__restrict__ u_off,
-                                  int *__restrict__ u_idx) {
+                                  int *__restrict__ u_idx, DirCtl *ctl = nullptr, long long nnz_cap = 0) {
+    if (ctl) {                                   // direct build: L and the entry total on the device
+        if (dir_bad(ctl)) return;
+        L = ctl->L;
+        if (u_off[L] > nnz_cap) {
+            if (blockIdx.x == 0 && threadIdx.x == 0) {
+                ctl->nnz = u_off[L];                  // the size to grow to
+                ctl->nnz_overflow = 1;
+            }
+            return;
+        }
+    }
     const int t = (int)((blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5);   // one warp per leaf
     if (t >= L) return;
     const long long o = u_off[t];
@@ -1225,6 +1281,9 @@ struct afmm_tree {
     int *pv_nchild = nullptr;
     long long *pv_base = nullptr;
     size_t pv_cap = 0;
+    unsigned long long *pvw_prefix = nullptr;   // write buffers of the direct build's copy
+    int *pvw_nchild = nullptr;
+    size_t pvw_cap = 0;
     int pv_levels = 0;
     // workspace arena: one grow-only device buffer per call site (no cudaMalloc
     // in steady state -- the tree is rebuilt every time step in C5)
@@ -1234,6 +1293,8 @@ struct afmm_tree {
     bool coop_ok = true;             // cooperative launch of levels_kernel available
     unsigned lvl_epoch = 0;          // launches of levels_kernel (tags its tile status words)
     long long sort_fallbacks = 0;    // bucket sorts that overflowed into the full radix sort
+    long long dir_leaf_cap = 0;      // direct build: leaf / U-list entry capacities (grow-only, checked on the
+    long long dir_nnz_cap = 0;       // device; an overflow grows them and reruns)
 };
 
 namespace {
@@ -1342,6 +1403,8 @@ extern "C" void afmm_tree_destroy(afmm_tree *t) {
     free_all(t);
     cudaFree(t->pv_prefix);
     cudaFree(t->pv_nchild);
+    cudaFree(t->pvw_prefix);
+    cudaFree(t->pvw_nchild);
     cudaFree(t->pv_base);
     if (t->own_stream && t->stream) cudaStreamDestroy(t->stream);
     delete t;
@@ -1484,18 +1547,33 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     int *cb = nullptr, *nc = nullptr, *off = nullptr;
     bool done_levels = false;
     // 4d. direct construction from the sorted keys (fresh / Enforce_S, no edits, S <= kDirMaxS):
-    //     leaves and nodes by a handful of flat kernels, one host readback (L, node
-    //     count, level starts, the bucket sort's overflow flag)
+    //     leaves, nodes and U-lists by flat kernels that read their sizes on the device,
+    //     into grow-only capacities checked on the device; ONE host readback at the end
+    //     (sizes + overflow flags; an overflow grows the capacities and reruns, a warp
+    //     U-list overflow continues on the host-driven path below)
     int *flag = nullptr, *leaf_at = nullptr, *node_leaf = nullptr, *leaf_node = nullptr;
     int L = 0;
     const char *lv_env = getenv("AFMM_TREE_LEVELS");                 // tests / A-B: force the level loop
+    const char *dfs_env = getenv("AFMM_ULIST_DFS");                  // tests: force the DFS U-list fallback
     const bool direct = mode != kModeKeep && ed.n == 0 && S <= kDirMaxS && !(lv_env && lv_env[0] == '1');
-    for (int attempt = 0; direct && attempt < 3 && !done_levels; ++attempt) {
+    for (int attempt = 0; direct && attempt < 8 && !done_levels; ++attempt) {
         unsigned char *lvl, *llo;
         unsigned long long *fk;
-        int *chunk_cnt, *chunk_base, *level_cnt, *rank;
+        int *chunk_cnt, *chunk_base, *level_cnt, *rank, *rows;
+        long long *counts;
+        NodeRec *rec;
         DirCtl *dctl;
         const long long nchunk = (n + kDirLeafBlock - 1) / kDirLeafBlock;
+        const char *small_env = getenv("AFMM_TREE_SMALL_CAPS");        // tests: start every capacity tiny
+        const bool small = small_env && small_env[0] == '1';
+        if (t->dir_leaf_cap == 0)                                    // first guess: ~ 4 n / S leaves
+            t->dir_leaf_cap = small ? 1 : std::min<long long>(n, 1024 + 4 * n / std::max(1, S));
+        if (t->dir_nnz_cap == 0) t->dir_nnz_cap = small ? 1 : 64 * t->dir_leaf_cap;
+        if (!small && (long long)cap < 2 * n + 64) {
+            cap = (size_t)(2 * n + 64);
+            if (afmm_status s = alloc_nodes(cap, nd, node_set)) return s;
+        }
+        const int lcap = (int)t->dir_leaf_cap;
         if (afmm_status s = wsalloc(t, kFlag, &flag, n + 1)) return s;
         if (afmm_status s = wsalloc(t, kLeafAt, &leaf_at, n + 1)) return s;
         if (afmm_status s = wsalloc(t, kDirLvl, &lvl, n)) return s;
@@ -1509,6 +1587,27 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
         if (afmm_status s = wsalloc(t, kDirChunkBase, &chunk_base, (size_t)nchunk * kDirLevels)) return s;
         if (afmm_status s = wsalloc(t, kDirLevelCnt, &level_cnt, kDirLevels)) return s;
         if (afmm_status s = wsalloc(t, kDirCtl, reinterpret_cast<char **>(&dctl), sizeof(DirCtl))) return s;
+        if (afmm_status s = wsalloc(t, kNodeLeaf, &node_leaf, cap)) return s;
+        if (afmm_status s = wsalloc(t, kLeafNode, &leaf_node, n)) return s;
+        if (afmm_status s = wsalloc(t, kDirRank, &rank, (size_t)kDirLevels * ((size_t)lcap + 1))) return s;
+        if (afmm_status s = wsalloc(t, kAnc, &rec, cap)) return s;
+        if (afmm_status s = wsalloc(t, kCounts, &counts, (size_t)lcap + 1)) return s;
+        if (afmm_status s = wsalloc(t, kUoff, &t->u_off, (size_t)lcap + 1)) return s;
+        if (afmm_status s = wsalloc(t, kURows, &rows, (size_t)lcap * kURow)) return s;
+        if (afmm_status s = wsalloc(t, kUidx, &t->u_idx, (size_t)t->dir_nnz_cap)) return s;
+        if (cap > t->pvw_cap) {                       // this build's node copy goes to the write buffers (the
+            cudaFree(t->pvw_prefix);                  // previous tree stays readable); swapped in on success
+            cudaFree(t->pvw_nchild);
+            t->pvw_prefix = nullptr;
+            t->pvw_nchild = nullptr;
+            t->pvw_cap = 0;
+            TCU(t, cudaMalloc(&t->pvw_prefix, cap * sizeof(unsigned long long)));
+            TCU(t, cudaMalloc(&t->pvw_nchild, cap * sizeof(int)));
+            t->pvw_cap = cap;
+        }
+        if (!t->pv_base) TCU(t, cudaMalloc(&t->pv_base, (kMaxLevel + 2) * sizeof(long long)));
+        TCU(t, cudaMemsetAsync(dctl, 0, sizeof(DirCtl), st));
+        if (bovf) TCU(t, cudaMemcpyAsync(&dctl->sort_overflow, bovf, sizeof(int), cudaMemcpyDeviceToDevice, st));
         leaf_level_kernel<<<(int)((n + kDirTile - 1) / kDirTile), kDirThreads, 0, st>>>(n, t->keys_sorted, S, mode,
                                                                                        pv, lvl, flag);
         TCU(t, cudaGetLastError());
@@ -1523,9 +1622,28 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
                                                          fk, llo);
         node_count_kernel<<<(int)nchunk, kDirLeafBlock, 0, st>>>(n, leaf_at, t->ls, t->ll, llo, t->lc, chunk_cnt);
         node_scan_kernel<<<1, 32 * kDirLevels, 0, st>>>(n, leaf_at, chunk_cnt, chunk_base, level_cnt, dctl);
+        node_rank_kernel<<<(lcap + kDirLeafBlock - 1) / kDirLeafBlock, kDirLeafBlock, 0, st>>>(
+            dctl, chunk_base, level_cnt, t->ls, t->lc, t->ll, llo, fk, rank, nd, node_leaf, leaf_node,
+            (long long)cap, lcap);
+        node_links_kernel<<<grid_for(std::min<long long>(lcap, 148LL * 64 * 4), TH), TH, 0, st>>>(
+            n, dctl, t->ls, t->ll, llo, rank, nd, (long long)cap, lcap);
+        anchors_kernel<<<grid_for((long long)cap, TH), TH, 0, st>>>((int)cap, nd, node_leaf, rec, dctl);
+        {
+            const int blocks = (int)std::min<long long>((lcap + kUWarps - 1) / kUWarps, 148LL * 16);
+            ulist_warp_kernel<<<blocks, 32 * kUWarps, 0, st>>>(lcap, nd, node_leaf, leaf_node, rec, rows, counts,
+                                                                nullptr, dctl, lcap);
+            size_t sb = 0;
+            TCU(t, cub::DeviceScan::ExclusiveSum(nullptr, sb, counts, t->u_off, lcap + 1, st));
+            char *sbuf;
+            if (afmm_status s = wsalloc(t, kScan3, &sbuf, sb)) return s;
+            TCU(t, cub::DeviceScan::ExclusiveSum(sbuf, sb, counts, t->u_off, lcap + 1, st));
+            ulist_copy_kernel<<<(int)(((long long)lcap * 32 + 255) / 256), 256, 0, st>>>(lcap, rows, t->u_off,
+                                                                                        t->u_idx, dctl,
+                                                                                        t->dir_nnz_cap);
+        }
+        dir_finish_kernel<<<(int)std::min<long long>(grid_for((long long)cap, TH), 148LL * 8), TH, 0, st>>>(
+            dctl, nd, t->u_off, t->pvw_prefix, t->pvw_nchild, t->pv_base);
         TCU(t, cudaGetLastError());
-        if (bovf) TCU(t, cudaMemcpyAsync(&dctl->sort_overflow, bovf, sizeof(int), cudaMemcpyDeviceToDevice, st));
-        else TCU(t, cudaMemsetAsync(&dctl->sort_overflow, 0, sizeof(int), st));
         DirCtl hc;
         TCU(t, cudaMemcpyAsync(&hc, dctl, sizeof(DirCtl), cudaMemcpyDeviceToHost, st));
         TCU(t, cudaStreamSynchronize(st));
@@ -1536,26 +1654,43 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
             if (afmm_status s = full_sort()) return s;
             continue;
         }
-        L = hc.L;
-        if ((long long)cap < hc.nn) {
-            cap = std::max<size_t>((size_t)hc.nn, (size_t)(2 * n + 64));
-            node_set = node_set == kNodeA ? kNodeB : kNodeA;
-            if (afmm_status s = alloc_nodes(cap, nd, node_set)) return s;
+        if (hc.cap_overflow) {                        // grow the node / leaf capacities, redo
+            if (hc.nn > (long long)cap) {
+                cap = (size_t)(hc.nn + hc.nn / 4);
+                if (afmm_status s = alloc_nodes(cap, nd, node_set)) return s;
+            }
+            if (hc.L > t->dir_leaf_cap) t->dir_leaf_cap = std::min<long long>(n, hc.L + hc.L / 4);
+            continue;
         }
-        if (afmm_status s = wsalloc(t, kNodeLeaf, &node_leaf, (size_t)hc.nn)) return s;
-        if (afmm_status s = wsalloc(t, kLeafNode, &leaf_node, (size_t)L)) return s;
-        if (afmm_status s = wsalloc(t, kDirRank, &rank, (size_t)kDirLevels * ((size_t)L + 1))) return s;
-        node_rank_kernel<<<(L + kDirLeafBlock - 1) / kDirLeafBlock, kDirLeafBlock, 0, st>>>(
-            dctl, chunk_base, level_cnt, t->ls, t->lc, t->ll, llo, fk, rank, nd, node_leaf, leaf_node);
-        node_links_kernel<<<grid_for(L, TH), TH, 0, st>>>(n, dctl, t->ls, t->ll, llo, rank, nd);
-        TCU(t, cudaGetLastError());
-        lvl_base.assign(hc.base, hc.base + hc.levels);
-        base = hc.nn;
+        L = hc.L;
         t->max_level = hc.levels - 1;
-        done_levels = true;
+        if (hc.ulist_overflow || (dfs_env && dfs_env[0] == '1')) {
+            // the host-driven path below recounts the U-lists per thread (nodes and
+            // leaves are complete; the previous-tree copy is made there)
+            lvl_base.assign(hc.base, hc.base + hc.levels);
+            base = hc.nn;
+            done_levels = true;
+            break;
+        }
+        if (hc.nnz_overflow) {                        // grow the U-list entry capacity, redo
+            t->dir_nnz_cap = hc.nnz + hc.nnz / 4 + 64;
+            continue;
+        }
+        // complete: sizes for the host, done
+        t->nnz = hc.nnz;
+        t->n_nodes = hc.nn;
+        t->node_cap = cap;
+        t->pv_levels = hc.levels;
+        std::swap(t->pv_prefix, t->pvw_prefix);
+        std::swap(t->pv_nchild, t->pvw_nchild);
+        std::swap(t->pv_cap, t->pvw_cap);
+        t->L = L;
+        t->n = n;
+        t->built = true;
+        return AFMM_OK;
     }
     const bool direct_done = done_levels;
-    if (direct && !done_levels) return tfail(t, AFMM_ECUDA, "tree_build: bucket sort kept overflowing");
+    if (direct && !done_levels) return tfail(t, AFMM_ECUDA, "tree_build: direct construction kept overflowing");
     // 4a. all levels in one cooperative launch (grid barriers between phases); the
     //     node arrays start at >= 2n + 64 nodes and are doubled on overflow
     if (!done_levels && t->coop_ok) {

@@ -192,7 +192,8 @@ def test_direct_construction_matches_level_loop(monkeypatch):
     """The direct construction (leaf levels from sliding windows over the sorted
     keys, nodes as the leaves' ancestors; tree_build.cu section 4d) and the
     level-synchronous split loop (AFMM_TREE_LEVELS=1) give identical trees AND
-    identical node arrays (the next Enforce_S reads them): fresh builds incl. S = 1,
+    identical node arrays (the next Enforce_S reads them), also when every device
+    capacity starts tiny (AFMM_TREE_SMALL_CAPS=1: overflow, grow, rerun): fresh builds incl. S = 1,
     n <= S, duplicate keys (level-21 leaves above S), and Enforce_S chains where
     nodes hold exactly S bodies (the 'was a parent' rule), incl. at the root."""
     afmm = _afmm()
@@ -213,8 +214,9 @@ def test_direct_construction_matches_level_loop(monkeypatch):
     for name, (x, y, z), ops in cases:
         n = x.shape[0]
         res = {}
-        for flag in ("0", "1"):
+        for flag, small in (("0", "0"), ("1", "0"), ("0", "1")):   # direct, level loop, direct from tiny capacities
             monkeypatch.setenv("AFMM_TREE_LEVELS", flag)
+            monkeypatch.setenv("AFMM_TREE_SMALL_CAPS", small)
             t = afmm.GpuTree(0)
             px, py, pz = x, y, z
             out = []
@@ -226,9 +228,10 @@ def test_direct_construction_matches_level_loop(monkeypatch):
                 fn(_dev(px), _dev(py), _dev(pz), S)
                 out.append(_tree_and_nodes(t, n))
             t.close()
-            res[flag] = out
-        for step, (a, b) in enumerate(zip(res["0"], res["1"])):
-            assert a.keys() == b.keys()
-            for k in a:
-                assert np.array_equal(np.asarray(a[k]), np.asarray(b[k])), (name, step, k)
+            res[flag + small] = out
+        for other in ("10", "01"):
+            for step, (a, b) in enumerate(zip(res["00"], res[other])):
+                assert a.keys() == b.keys()
+                for k in a:
+                    assert np.array_equal(np.asarray(a[k]), np.asarray(b[k])), (name, other, step, k)
     del rng
