@@ -669,7 +669,10 @@ __global__ void __launch_bounds__(kLvlThreads) levels_kernel(Nodes nd, const uns
 __device__ __forceinline__ int lcp_digits(unsigned long long a, unsigned long long b) {
     return a == b ? kMaxLevel : (__clzll((long long)(a ^ b)) - 1) / 3;
 }
-constexpr int kDirTile = 2048;              // positions per block of leaf_level_kernel
+#ifndef AFMM_DIR_TILE
+#define AFMM_DIR_TILE 1024
+#endif
+constexpr int kDirTile = AFMM_DIR_TILE;     // positions per block of leaf_level_kernel
 constexpr int kDirThreads = 256;
 constexpr int kDirMaxS = 2048;              // larger S: the level loop
 constexpr int kDirLevels = kMaxLevel + 1;   // levels 0..21
