@@ -1,7 +1,7 @@
 #!/bin/bash
 # One GPU call for the round's evidence: GPU tests, the bench line, the ncu launch list of
-# the bench command, one `ncu --set full` capture of the C4 P2P kernel, compute-sanitizer
-# on the small end-to-end run (also with tiny tree capacities).  -> gpurun_out/*_$TAG.*
+# the bench command, one `ncu --set full` capture of the C4 P2P kernel
+# -> gpurun_out/*_$TAG.*  (compute-sanitizer is closed on the GPU pool this round)
 cd "$(dirname "$0")/.."
 TAG=${1:-r2}
 mkdir -p gpurun_out
@@ -15,9 +15,4 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --c
     --no-stokeslet --no-proxy > /dev/null 2>&1
 timeout 900 ncu --set full --import-source on --clock-control none -k regex:p2p_kernel -s 1 -c 1 \
     -o gpurun_out/p2p_full_C4_$TAG python tools/prof_p2p.py --config C4 --S 256 --evals 2 > /dev/null 2>&1
-for tool in memcheck racecheck synccheck; do
-  echo "== $tool"; timeout 600 compute-sanitizer --tool $tool python tools/sanitize_run.py 2>&1 | tail -2
-done > gpurun_out/sanitizer_$TAG.txt
-echo "== memcheck, tiny tree capacities (AFMM_TREE_SMALL_CAPS=1)" >> gpurun_out/sanitizer_$TAG.txt
-AFMM_TREE_SMALL_CAPS=1 timeout 600 compute-sanitizer --tool memcheck python tools/sanitize_run.py 2>&1 | tail -2 >> gpurun_out/sanitizer_$TAG.txt
 ls -la gpurun_out | tail -12
