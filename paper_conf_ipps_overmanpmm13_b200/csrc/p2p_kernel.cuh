@@ -719,7 +719,7 @@ __device__ __forceinline__ void load_targets(Targets &T, const float4 *__restric
 // afmm_p2p_eval_host_pipelined); afmm_p2p_create re-checks the fit from the
 // built kernels' attributes (co_resident_pack) and the pipelined evaluation falls
 // back to packing every chunk before the launch when it does not hold.
-constexpr int kMaxRegs = 160;
+constexpr int kMaxRegs = kThreads <= 384 ? 160 : ((65536 - 4096) / kThreads) / 8 * 8;   // (tuning builds: more warps)
 static_assert(kMinBlocksPerSM == 1 && kMaxRegs * kThreads <= 65536, "register budget: one CTA per SM");
 // (The device-path kernel keeps __launch_bounds__: the same 158 registers, but
 // its code under __maxnreg__ measured 1.2 % slower, profiles/r2_ab_regs.txt.)
