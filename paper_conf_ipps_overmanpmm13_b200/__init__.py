@@ -126,6 +126,7 @@ _sig("afmm_tree_enforce", _i, _p, _ll, _p, _p, _p, _i)
 _sig("afmm_tree_farfield_counts", _i, _p, _p)
 _sig("afmm_tree_info", _i, _p, C.POINTER(_i), C.POINTER(_ll), _p, C.POINTER(_i), C.POINTER(_i),
      C.POINTER(_ll))
+_sig("afmm_tree_counters", _i, _p, C.POINTER(_ll), C.POINTER(_ll))
 _sig("afmm_tree_copy_out", _i, _p, _p, _p, _p, _p, _p, _p, _p)
 _sig("afmm_tree_gather", _i, _p, _p, _p)
 _sig("afmm_tree_gather_rows", _i, _p, _i, _p, _p)
@@ -173,7 +174,7 @@ EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
             "afmm_partition_literal", "afmm_partition_weighted", "afmm_partition_rebalance",
             "afmm_cost_fit", "afmm_p2p_set_cost_coef", "afmm_kick", "afmm_drift",
             "afmm_fp32_peak", "afmm_version",
-            "afmm_tree_create", "afmm_tree_build", "afmm_tree_enforce", "afmm_tree_info",
+            "afmm_tree_create", "afmm_tree_build", "afmm_tree_enforce", "afmm_tree_info", "afmm_tree_counters",
             "afmm_tree_farfield_counts", "afmm_lb_config_init", "afmm_lb_create", "afmm_lb_step",
             "afmm_lb_predicted", "afmm_lb_state", "afmm_lb_destroy", "afmm_tree_copy_out",
             "afmm_tree_gather", "afmm_tree_scatter", "afmm_tree_destroy", "afmm_tree_last_error",
@@ -614,6 +615,12 @@ class GpuTree:
                                         C.byref(ml), C.byref(nn)), "afmm_tree_info")
         return {"n_leaves": L.value, "nnz": nnz.value, "lo": lo, "k": k.value,
                 "max_level": ml.value, "n_nodes": nn.value}
+
+    def counters(self):
+        """{'graph_launches', 'sort_fallbacks'} of this handle (afmm_tree_counters)."""
+        g, f = _ll(), _ll()
+        self._check(_lib.afmm_tree_counters(self._h, C.byref(g), C.byref(f)), "afmm_tree_counters")
+        return {"graph_launches": g.value, "sort_fallbacks": f.value}
 
     def copy_out(self, n):
         inf = self.info()

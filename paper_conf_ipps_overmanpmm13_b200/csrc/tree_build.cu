@@ -115,8 +115,10 @@ struct Nodes {
 // bodies stay in their leaf's cell between steps (≈ 74 % on C5), the buckets hold
 // about a leaf each, and a warp sorts one (bitonic, <= kBucketCap keys).
 constexpr int kBucketCap = 512;
-__global__ void cell_range_kernel(int L, const int *__restrict__ ll, const unsigned long long *__restrict__ lp,
-                                  unsigned long long *__restrict__ clo, unsigned long long *__restrict__ chi) {
+__global__ void cell_range_kernel(const int *__restrict__ Ldev, const int *__restrict__ ll,
+                                  const unsigned long long *__restrict__ lp, unsigned long long *__restrict__ clo,
+                                  unsigned long long *__restrict__ chi) {
+    const int L = *Ldev;                          // the previous build's leaf count (device word: graph-stable)
     const int j = blockIdx.x * blockDim.x + threadIdx.x;
     if (j >= L) return;
     const int sh = 3 * (kMaxLevel - ll[j]);
@@ -131,10 +133,11 @@ __global__ void cell_range_kernel(int L, const int *__restrict__ ll, const unsig
 constexpr int kMaxSamples = 1024, kKeysThreads = 512;
 __global__ void __launch_bounds__(kKeysThreads) keys_bucket_kernel(
     long long n, const float *__restrict__ x, const float *__restrict__ y, const float *__restrict__ z, double lx,
-    double ly, double lz, double scale, unsigned long long *__restrict__ keys, int L, int stride,
+    double ly, double lz, double scale, unsigned long long *__restrict__ keys, const int *__restrict__ Ldev,
     const unsigned long long *__restrict__ clo, const unsigned long long *__restrict__ chi, int *__restrict__ bucket,
     int *__restrict__ slot, int *__restrict__ bcount) {
     __shared__ unsigned long long smp[kMaxSamples];
+    const int L = *Ldev, stride = (L + kMaxSamples - 1) / kMaxSamples;
     const int ns = (L + stride - 1) / stride;
     for (int s = threadIdx.x; s < ns; s += blockDim.x) smp[s] = clo[(long long)s * stride];
     __syncthreads();
@@ -245,13 +248,15 @@ __device__ __forceinline__ void warp_bitonic(int o, int cnt, const unsigned long
     }
 }
 constexpr int kBucketWarps = 4;
-__global__ void __launch_bounds__(32 * kBucketWarps) bucket_sort_kernel(int nb, const int *__restrict__ boff,
+__global__ void __launch_bounds__(32 * kBucketWarps) bucket_sort_kernel(const int *__restrict__ Ldev,
+                                                                        const int *__restrict__ boff,
                                                                         const unsigned long long *__restrict__ bkeys,
                                                                         const int *__restrict__ bidx,
                                                                         unsigned long long *__restrict__ okeys,
                                                                         int *__restrict__ oidx,
                                                                         int *__restrict__ overflow) {
     const int lane = threadIdx.x & 31;
+    const int nb = 2 * *Ldev + 1;
     const int b = blockIdx.x * kBucketWarps + (threadIdx.x >> 5);
     if (b >= nb) return;                                      // whole warps
     const int o = boff[b], cnt = boff[b + 1] - o;
@@ -693,7 +698,9 @@ __device__ __forceinline__ bool dir_bad(const DirCtl *c) {
 
 __global__ void __launch_bounds__(kDirThreads) leaf_level_kernel(long long n, const unsigned long long *__restrict__ keys,
                                                                  int S, int mode, PrevTree pv,
+                                                                 const int *__restrict__ pv_levels,
                                                                  unsigned char *__restrict__ lvl, int *__restrict__ flag) {
+    if (pv_levels) pv.levels = mode == kModeEnforce ? *pv_levels : 0;   // the previous build's (device word)
     // [buffer][array][pos]: array 0 = windows of S + 1 (w), 1 = windows of S (v);
     // position a <-> window start j = t0 - S + a; -1 = no such window
     __shared__ signed char win[2][2][kDirTile + kDirMaxS];
@@ -933,8 +940,8 @@ __global__ void node_links_kernel(long long n, const DirCtl *__restrict__ ctl, c
 // starts) and the U-list total -- on the device, no host round trip.
 __global__ void dir_finish_kernel(DirCtl *ctl, Nodes nd, const long long *__restrict__ u_off,
                                   unsigned long long *__restrict__ pv_prefix, int *__restrict__ pv_nchild,
-                                  long long *__restrict__ pv_base) {
-    if (dir_bad(ctl)) return;
+                                  long long *__restrict__ pv_base, int *__restrict__ dstate) {
+    if (dir_bad(ctl)) return;                     // (a failed attempt leaves the previous tree for the rerun)
     const long long nn = ctl->nn;
     for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < nn; i += (long long)gridDim.x * blockDim.x) {
         pv_prefix[i] = nd.prefix[i];
@@ -943,7 +950,11 @@ __global__ void dir_finish_kernel(DirCtl *ctl, Nodes nd, const long long *__rest
     if (blockIdx.x == 0 && threadIdx.x <= kDirLevels) {
         const int l = threadIdx.x;
         if (l <= ctl->levels) pv_base[l] = l < ctl->levels ? ctl->base[l] : nn;
-        if (l == 0) ctl->nnz = u_off[ctl->L];
+        if (l == 0) {
+            ctl->nnz = u_off[ctl->L];
+            dstate[0] = ctl->L;                   // read by the next build's bucket sort / Enforce_S
+            dstate[1] = ctl->levels;
+        }
     }
 }
 
@@ -1258,6 +1269,24 @@ int grid_for(long long n, int threads) {
 
 }  // namespace
 
+// What a captured direct build depends on besides device-side state: the inputs,
+// S, the mode, the domain and every buffer (ws_gen changes whenever one moves).
+struct GraphKey {
+    const float *x, *y, *z;
+    long long n;
+    int S, mode;
+    unsigned long long gen;
+    size_t cap;
+    long long lcap, nnz_cap;
+    double lo[3];
+    int k;
+    bool operator==(const GraphKey &o) const {
+        return x == o.x && y == o.y && z == o.z && n == o.n && S == o.S && mode == o.mode && gen == o.gen &&
+               cap == o.cap && lcap == o.lcap && nnz_cap == o.nnz_cap && lo[0] == o.lo[0] && lo[1] == o.lo[1] &&
+               lo[2] == o.lo[2] && k == o.k;
+    }
+};
+
 struct afmm_tree {
     int device = 0;
     cudaStream_t stream = nullptr;
@@ -1284,9 +1313,6 @@ struct afmm_tree {
     int *pv_nchild = nullptr;
     long long *pv_base = nullptr;
     size_t pv_cap = 0;
-    unsigned long long *pvw_prefix = nullptr;   // write buffers of the direct build's copy
-    int *pvw_nchild = nullptr;
-    size_t pvw_cap = 0;
     int pv_levels = 0;
     // workspace arena: one grow-only device buffer per call site (no cudaMalloc
     // in steady state -- the tree is rebuilt every time step in C5)
@@ -1296,6 +1322,16 @@ struct afmm_tree {
     bool coop_ok = true;             // cooperative launch of levels_kernel available
     unsigned lvl_epoch = 0;          // launches of levels_kernel (tags its tile status words)
     long long sort_fallbacks = 0;    // bucket sorts that overflowed into the full radix sort
+    // device words read by the next build: [0] = leaf count, [1] = levels of the last build (the
+    // bucket sort and Enforce_S read them on the device, so a captured graph stays valid)
+    int *d_state = nullptr;
+    DirCtl *h_ctl = nullptr;         // pinned readback of the direct build
+    unsigned long long ws_gen = 0;   // bumped whenever a workspace buffer is reallocated (graph key)
+    cudaGraphExec_t tg_exec[2] = {nullptr, nullptr};   // captured direct builds (two alternating input sets)
+    GraphKey tg_key[2] = {};
+    int tg_next = 0;
+    bool graph_broken = false;
+    long long graph_launches = 0;
     long long dir_leaf_cap = 0;      // direct build: leaf / U-list entry capacities (grow-only, checked on the
     long long dir_nnz_cap = 0;       // device; an overflow grows them and reruns)
 };
@@ -1349,6 +1385,7 @@ afmm_status wsalloc(afmm_tree *t, int slot, T **p, size_t count) {
         t->ws_ptr[slot] = nullptr;
         t->ws_cap[slot] = 0;
         const size_t want = bytes + bytes / 2;
+        ++t->ws_gen;
         TCU(t, cudaMalloc(&t->ws_ptr[slot], want));
         t->ws_cap[slot] = want;
     }
@@ -1391,7 +1428,13 @@ extern "C" afmm_status afmm_tree_create(int device, void *stream, afmm_tree **ou
             t->own_stream = (e == cudaSuccess);
         }
     }
+    if (e == cudaSuccess) e = cudaMalloc(&t->d_state, 2 * sizeof(int));
+    if (e == cudaSuccess) e = cudaMemset(t->d_state, 0, 2 * sizeof(int));
+    if (e == cudaSuccess) e = cudaMallocHost(&t->h_ctl, sizeof(DirCtl));
     if (e != cudaSuccess) {
+        cudaFree(t->d_state);
+        if (t->h_ctl) cudaFreeHost(t->h_ctl);
+        if (t->own_stream && t->stream) cudaStreamDestroy(t->stream);
         delete t;
         return AFMM_ECUDA;
     }
@@ -1406,9 +1449,11 @@ extern "C" void afmm_tree_destroy(afmm_tree *t) {
     free_all(t);
     cudaFree(t->pv_prefix);
     cudaFree(t->pv_nchild);
-    cudaFree(t->pvw_prefix);
-    cudaFree(t->pvw_nchild);
     cudaFree(t->pv_base);
+    cudaFree(t->d_state);
+    if (t->h_ctl) cudaFreeHost(t->h_ctl);
+    for (auto &g : t->tg_exec)
+        if (g) cudaGraphExecDestroy(g);
     if (t->own_stream && t->stream) cudaStreamDestroy(t->stream);
     delete t;
 }
@@ -1488,41 +1533,64 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     const char *cub_env = getenv("AFMM_TREE_FULL_SORT");
     const bool buckets = had_prev && t->coop_ok && prev_k == t->k && prev_lo[0] == t->lo[0] &&
                          prev_lo[1] == t->lo[1] && prev_lo[2] == t->lo[2] && !(cub_env && cub_env[0] == '1');
+    const char *lv_env = getenv("AFMM_TREE_LEVELS");                 // tests / A-B: force the level loop
+    const char *dfs_env = getenv("AFMM_ULIST_DFS");                  // tests: force the DFS U-list fallback
+    const char *gr_env = getenv("AFMM_TREE_GRAPH");                  // 0: no CUDA graph for the direct build
+    const bool direct = mode != kModeKeep && ed.n == 0 && S <= kDirMaxS && !(lv_env && lv_env[0] == '1');
+    if (direct) {
+        const char *small_env = getenv("AFMM_TREE_SMALL_CAPS");        // tests: start every capacity tiny
+        const bool small = small_env && small_env[0] == '1';
+        if (t->dir_leaf_cap == 0)                                    // first guess: ~ 4 n / S leaves
+            t->dir_leaf_cap = small ? 1 : std::min<long long>(n, 1024 + 4 * n / std::max(1, S));
+        if (t->dir_nnz_cap == 0) t->dir_nnz_cap = small ? 1 : 64 * t->dir_leaf_cap;
+    }
+    if (buckets && prev_L > t->dir_leaf_cap) t->dir_leaf_cap = prev_L;   // the bucket arrays hold the previous leaves
+    // bucket sort by the previous leaves' cells (see bucket_sort_kernel): buffers sized by the leaf
+    // capacity, the previous leaf count read on the device (so a captured graph stays valid)
     int *bovf = nullptr;
-    if (buckets) {                                            // by the previous leaves' cells (see bucket_sort_kernel)
-        const int Lp = prev_L, nb = 2 * Lp + 1;
-        unsigned long long *clo, *chi, *bkeys;
-        int *bucket, *slot, *bcount, *boff, *bidx;
-        if (afmm_status s = wsalloc(t, kCellLo, &clo, Lp)) return s;
-        if (afmm_status s = wsalloc(t, kCellHi, &chi, Lp)) return s;
-        if (afmm_status s = wsalloc(t, kBucket, &bucket, n)) return s;
-        if (afmm_status s = wsalloc(t, kSlot, &slot, n)) return s;
-        if (afmm_status s = wsalloc(t, kBCount, &bcount, (size_t)nb + 1)) return s;
-        if (afmm_status s = wsalloc(t, kBOff, &boff, (size_t)nb + 1)) return s;
-        if (afmm_status s = wsalloc(t, kBKeys, &bkeys, n)) return s;
-        if (afmm_status s = wsalloc(t, kBIdx, &bidx, n)) return s;
+    unsigned long long *b_clo = nullptr, *b_chi = nullptr, *b_keys = nullptr;
+    int *b_bucket = nullptr, *b_slot = nullptr, *b_count = nullptr, *b_off = nullptr, *b_idx = nullptr;
+    char *b_sbuf = nullptr;
+    size_t b_sb = 0;
+    int kb_grid = 0;
+    const long long bcap = std::max<long long>(t->dir_leaf_cap, 1), nbcap = 2 * bcap + 1;
+    if (buckets) {
+        if (afmm_status s = wsalloc(t, kCellLo, &b_clo, bcap)) return s;
+        if (afmm_status s = wsalloc(t, kCellHi, &b_chi, bcap)) return s;
+        if (afmm_status s = wsalloc(t, kBucket, &b_bucket, n)) return s;
+        if (afmm_status s = wsalloc(t, kSlot, &b_slot, n)) return s;
+        if (afmm_status s = wsalloc(t, kBCount, &b_count, (size_t)nbcap + 1)) return s;
+        if (afmm_status s = wsalloc(t, kBOff, &b_off, (size_t)nbcap + 1)) return s;
+        if (afmm_status s = wsalloc(t, kBKeys, &b_keys, n)) return s;
+        if (afmm_status s = wsalloc(t, kBIdx, &b_idx, n)) return s;
         if (afmm_status s = wsalloc(t, kBOvf, &bovf, 1)) return s;
-        TCU(t, cudaMemsetAsync(bcount, 0, ((size_t)nb + 1) * sizeof(int), st));
-        TCU(t, cudaMemsetAsync(bovf, 0, sizeof(int), st));
-        cell_range_kernel<<<grid_for(Lp, TH), TH, 0, st>>>(Lp, t->ll, t->lp, clo, chi);
-        const int stride = (Lp + kMaxSamples - 1) / kMaxSamples;
-        int kb_grid = 0, dev_sms = 0;
+        TCU(t, cub::DeviceScan::ExclusiveSum(nullptr, b_sb, b_count, b_off, (int)(nbcap + 1), st));
+        if (afmm_status s = wsalloc(t, kBScan, &b_sbuf, b_sb)) return s;
+        int dev_sms = 0;
         TCU(t, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&kb_grid, keys_bucket_kernel, kKeysThreads, 0));
         TCU(t, cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, t->device));
         kb_grid = (int)std::min<long long>((n + kKeysThreads - 1) / kKeysThreads, (long long)std::max(1, kb_grid) * dev_sms);
-        keys_bucket_kernel<<<kb_grid, kKeysThreads, 0, st>>>(n, x, y, z, t->lo[0], t->lo[1], t->lo[2], scale, keys, Lp,
-                                                             stride, clo, chi, bucket, slot, bcount);
-        size_t sb = 0;
-        TCU(t, cub::DeviceScan::ExclusiveSum(nullptr, sb, bcount, boff, nb + 1, st));
-        char *sbuf;
-        if (afmm_status s = wsalloc(t, kBScan, &sbuf, sb)) return s;
-        TCU(t, cub::DeviceScan::ExclusiveSum(sbuf, sb, bcount, boff, nb + 1, st));
-        bucket_scatter_kernel<<<grid_for(n, TH), TH, 0, st>>>(n, keys, bucket, slot, boff, bkeys, bidx);
-        bucket_sort_kernel<<<(nb + kBucketWarps - 1) / kBucketWarps, 32 * kBucketWarps, 0, st>>>(
-            nb, boff, bkeys, bidx, t->keys_sorted, t->perm, bovf);
+    }
+    auto enq_buckets = [&]() -> afmm_status {
+        TCU(t, cudaMemsetAsync(b_count, 0, ((size_t)nbcap + 1) * sizeof(int), st));
+        TCU(t, cudaMemsetAsync(bovf, 0, sizeof(int), st));
+        cell_range_kernel<<<grid_for(bcap, TH), TH, 0, st>>>(t->d_state, t->ll, t->lp, b_clo, b_chi);
+        keys_bucket_kernel<<<kb_grid, kKeysThreads, 0, st>>>(n, x, y, z, t->lo[0], t->lo[1], t->lo[2], scale, keys,
+                                                             t->d_state, b_clo, b_chi, b_bucket, b_slot, b_count);
+        size_t sb = b_sb;
+        TCU(t, cub::DeviceScan::ExclusiveSum(b_sbuf, sb, b_count, b_off, (int)(nbcap + 1), st));
+        bucket_scatter_kernel<<<grid_for(n, TH), TH, 0, st>>>(n, keys, b_bucket, b_slot, b_off, b_keys, b_idx);
+        bucket_sort_kernel<<<(int)((nbcap + kBucketWarps - 1) / kBucketWarps), 32 * kBucketWarps, 0, st>>>(
+            t->d_state, b_off, b_keys, b_idx, t->keys_sorted, t->perm, bovf);
         TCU(t, cudaGetLastError());
-    } else if (afmm_status s = full_sort()) {
-        return s;
+        return AFMM_OK;
+    };
+    if (!direct) {                                            // the level loop checks the bucket sort's flag itself
+        if (buckets) {
+            if (afmm_status s = enq_buckets()) return s;
+        } else if (afmm_status s = full_sort()) {
+            return s;
+        }
     }
 
     // 4. level-synchronous split into one node array (level-major)
@@ -1553,12 +1621,14 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     //     leaves, nodes and U-lists by flat kernels that read their sizes on the device,
     //     into grow-only capacities checked on the device; ONE host readback at the end
     //     (sizes + overflow flags; an overflow grows the capacities and reruns, a warp
-    //     U-list overflow continues on the host-driven path below)
+    //     U-list overflow continues on the host-driven path below).  With the bucket
+    //     sort (a rebuild in the previous build's domain: every C5 step) the whole
+    //     sequence -- sort, leaves, nodes, U-lists, previous-tree copy, readback -- is
+    //     captured once into a CUDA graph and replayed (re-captured when the inputs,
+    //     S, the mode or any buffer change): one launch instead of ~25 per build.
     int *flag = nullptr, *leaf_at = nullptr, *node_leaf = nullptr, *leaf_node = nullptr;
     int L = 0;
-    const char *lv_env = getenv("AFMM_TREE_LEVELS");                 // tests / A-B: force the level loop
-    const char *dfs_env = getenv("AFMM_ULIST_DFS");                  // tests: force the DFS U-list fallback
-    const bool direct = mode != kModeKeep && ed.n == 0 && S <= kDirMaxS && !(lv_env && lv_env[0] == '1');
+    bool use_buckets = buckets, need_sort = !buckets;
     for (int attempt = 0; direct && attempt < 8 && !done_levels; ++attempt) {
         unsigned char *lvl, *llo;
         unsigned long long *fk;
@@ -1567,12 +1637,8 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
         NodeRec *rec;
         DirCtl *dctl;
         const long long nchunk = (n + kDirLeafBlock - 1) / kDirLeafBlock;
-        const char *small_env = getenv("AFMM_TREE_SMALL_CAPS");        // tests: start every capacity tiny
-        const bool small = small_env && small_env[0] == '1';
-        if (t->dir_leaf_cap == 0)                                    // first guess: ~ 4 n / S leaves
-            t->dir_leaf_cap = small ? 1 : std::min<long long>(n, 1024 + 4 * n / std::max(1, S));
-        if (t->dir_nnz_cap == 0) t->dir_nnz_cap = small ? 1 : 64 * t->dir_leaf_cap;
-        if (!small && (long long)cap < 2 * n + 64) {
+        const char *small_env = getenv("AFMM_TREE_SMALL_CAPS");
+        if (!(small_env && small_env[0] == '1') && (long long)cap < 2 * n + 64) {
             cap = (size_t)(2 * n + 64);
             if (afmm_status s = alloc_nodes(cap, nd, node_set)) return s;
         }
@@ -1598,71 +1664,131 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
         if (afmm_status s = wsalloc(t, kUoff, &t->u_off, (size_t)lcap + 1)) return s;
         if (afmm_status s = wsalloc(t, kURows, &rows, (size_t)lcap * kURow)) return s;
         if (afmm_status s = wsalloc(t, kUidx, &t->u_idx, (size_t)t->dir_nnz_cap)) return s;
-        if (cap > t->pvw_cap) {                       // this build's node copy goes to the write buffers (the
-            cudaFree(t->pvw_prefix);                  // previous tree stays readable); swapped in on success
-            cudaFree(t->pvw_nchild);
-            t->pvw_prefix = nullptr;
-            t->pvw_nchild = nullptr;
-            t->pvw_cap = 0;
-            TCU(t, cudaMalloc(&t->pvw_prefix, cap * sizeof(unsigned long long)));
-            TCU(t, cudaMalloc(&t->pvw_nchild, cap * sizeof(int)));
-            t->pvw_cap = cap;
+        size_t sb2 = 0, sb3 = 0;
+        char *sbuf2, *sbuf3;
+        TCU(t, cub::DeviceScan::ExclusiveSum(nullptr, sb2, flag, leaf_at, (int)(n + 1), st));
+        if (afmm_status s = wsalloc(t, kScan2, &sbuf2, sb2)) return s;
+        TCU(t, cub::DeviceScan::ExclusiveSum(nullptr, sb3, counts, t->u_off, lcap + 1, st));
+        if (afmm_status s = wsalloc(t, kScan3, &sbuf3, sb3)) return s;
+        if (cap > t->pv_cap) {                        // the previous tree's copy grows, keeping its contents (a rerun
+            unsigned long long *np = nullptr;         // of this build reads them); this build overwrites it on success
+            int *nc2 = nullptr;
+            TCU(t, cudaMalloc(&np, cap * sizeof(unsigned long long)));
+            TCU(t, cudaMalloc(&nc2, cap * sizeof(int)));
+            if (t->pv_prefix && t->n_nodes > 0) {
+                TCU(t, cudaMemcpyAsync(np, t->pv_prefix, (size_t)t->n_nodes * sizeof(unsigned long long),
+                                       cudaMemcpyDeviceToDevice, st));
+                TCU(t, cudaMemcpyAsync(nc2, t->pv_nchild, (size_t)t->n_nodes * sizeof(int), cudaMemcpyDeviceToDevice, st));
+                TCU(t, cudaStreamSynchronize(st));
+            }
+            cudaFree(t->pv_prefix);
+            cudaFree(t->pv_nchild);
+            t->pv_prefix = np;
+            t->pv_nchild = nc2;
+            t->pv_cap = cap;
+            pv.prefix = np;
+            pv.nchild = nc2;
+            ++t->ws_gen;
         }
-        if (!t->pv_base) TCU(t, cudaMalloc(&t->pv_base, (kMaxLevel + 2) * sizeof(long long)));
-        TCU(t, cudaMemsetAsync(dctl, 0, sizeof(DirCtl), st));
-        if (bovf) TCU(t, cudaMemcpyAsync(&dctl->sort_overflow, bovf, sizeof(int), cudaMemcpyDeviceToDevice, st));
-        leaf_level_kernel<<<(int)((n + kDirTile - 1) / kDirTile), kDirThreads, 0, st>>>(n, t->keys_sorted, S, mode,
-                                                                                       pv, lvl, flag);
-        TCU(t, cudaGetLastError());
-        {
-            size_t sb = 0;
-            TCU(t, cub::DeviceScan::ExclusiveSum(nullptr, sb, flag, leaf_at, (int)(n + 1), st));
-            char *sbuf;
-            if (afmm_status s = wsalloc(t, kScan2, &sbuf, sb)) return s;
-            TCU(t, cub::DeviceScan::ExclusiveSum(sbuf, sb, flag, leaf_at, (int)(n + 1), st));
+        if (!t->pv_base) {
+            TCU(t, cudaMalloc(&t->pv_base, (kMaxLevel + 2) * sizeof(long long)));
+            ++t->ws_gen;
         }
-        leaf_info_kernel<<<grid_for(n, TH), TH, 0, st>>>(n, t->keys_sorted, lvl, flag, leaf_at, t->ls, t->ll, t->lp,
-                                                         fk, llo);
-        node_count_kernel<<<(int)nchunk, kDirLeafBlock, 0, st>>>(n, leaf_at, t->ls, t->ll, llo, t->lc, chunk_cnt);
-        node_scan_kernel<<<1, 32 * kDirLevels, 0, st>>>(n, leaf_at, chunk_cnt, chunk_base, level_cnt, dctl);
-        node_rank_kernel<<<(lcap + kDirLeafBlock - 1) / kDirLeafBlock, kDirLeafBlock, 0, st>>>(
-            dctl, chunk_base, level_cnt, t->ls, t->lc, t->ll, llo, fk, rank, nd, node_leaf, leaf_node,
-            (long long)cap, lcap);
-        node_links_kernel<<<grid_for(std::min<long long>(lcap, 148LL * 64 * 4), TH), TH, 0, st>>>(
-            n, dctl, t->ls, t->ll, llo, rank, nd, (long long)cap, lcap);
-        anchors_kernel<<<grid_for((long long)cap, TH), TH, 0, st>>>((int)cap, nd, node_leaf, rec, dctl);
-        {
-            const int blocks = (int)std::min<long long>((lcap + kUWarps - 1) / kUWarps, 148LL * 16);
-            ulist_warp_kernel<<<blocks, 32 * kUWarps, 0, st>>>(lcap, nd, node_leaf, leaf_node, rec, rows, counts,
-                                                                nullptr, dctl, lcap);
-            size_t sb = 0;
-            TCU(t, cub::DeviceScan::ExclusiveSum(nullptr, sb, counts, t->u_off, lcap + 1, st));
-            char *sbuf;
-            if (afmm_status s = wsalloc(t, kScan3, &sbuf, sb)) return s;
-            TCU(t, cub::DeviceScan::ExclusiveSum(sbuf, sb, counts, t->u_off, lcap + 1, st));
+        auto enq_direct = [&]() -> afmm_status {
+            TCU(t, cudaMemsetAsync(dctl, 0, sizeof(DirCtl), st));
+            if (use_buckets) TCU(t, cudaMemcpyAsync(&dctl->sort_overflow, bovf, sizeof(int), cudaMemcpyDeviceToDevice, st));
+            leaf_level_kernel<<<(int)((n + kDirTile - 1) / kDirTile), kDirThreads, 0, st>>>(
+                n, t->keys_sorted, S, mode, pv, t->d_state + 1, lvl, flag);
+            TCU(t, cudaGetLastError());
+            size_t sb = sb2;
+            TCU(t, cub::DeviceScan::ExclusiveSum(sbuf2, sb, flag, leaf_at, (int)(n + 1), st));
+            leaf_info_kernel<<<grid_for(n, TH), TH, 0, st>>>(n, t->keys_sorted, lvl, flag, leaf_at, t->ls, t->ll,
+                                                             t->lp, fk, llo);
+            node_count_kernel<<<(int)nchunk, kDirLeafBlock, 0, st>>>(n, leaf_at, t->ls, t->ll, llo, t->lc, chunk_cnt);
+            node_scan_kernel<<<1, 32 * kDirLevels, 0, st>>>(n, leaf_at, chunk_cnt, chunk_base, level_cnt, dctl);
+            node_rank_kernel<<<(lcap + kDirLeafBlock - 1) / kDirLeafBlock, kDirLeafBlock, 0, st>>>(
+                dctl, chunk_base, level_cnt, t->ls, t->lc, t->ll, llo, fk, rank, nd, node_leaf, leaf_node,
+                (long long)cap, lcap);
+            node_links_kernel<<<grid_for(std::min<long long>(lcap, 148LL * 64 * 4), TH), TH, 0, st>>>(
+                n, dctl, t->ls, t->ll, llo, rank, nd, (long long)cap, lcap);
+            anchors_kernel<<<grid_for((long long)cap, TH), TH, 0, st>>>((int)cap, nd, node_leaf, rec, dctl);
+            const int ublocks = (int)std::min<long long>((lcap + kUWarps - 1) / kUWarps, 148LL * 16);
+            ulist_warp_kernel<<<ublocks, 32 * kUWarps, 0, st>>>(lcap, nd, node_leaf, leaf_node, rec, rows, counts,
+                                                                 nullptr, dctl, lcap);
+            sb = sb3;
+            TCU(t, cub::DeviceScan::ExclusiveSum(sbuf3, sb, counts, t->u_off, lcap + 1, st));
             ulist_copy_kernel<<<(int)(((long long)lcap * 32 + 255) / 256), 256, 0, st>>>(lcap, rows, t->u_off,
                                                                                         t->u_idx, dctl,
                                                                                         t->dir_nnz_cap);
+            dir_finish_kernel<<<(int)std::min<long long>(grid_for((long long)cap, TH), 148LL * 8), TH, 0, st>>>(
+                dctl, nd, t->u_off, t->pv_prefix, t->pv_nchild, t->pv_base, t->d_state);
+            TCU(t, cudaGetLastError());
+            TCU(t, cudaMemcpyAsync(t->h_ctl, dctl, sizeof(DirCtl), cudaMemcpyDeviceToHost, st));
+            return AFMM_OK;
+        };
+        const bool graph = use_buckets && !(gr_env && gr_env[0] == '0') && !t->graph_broken;
+        if (graph) {
+            const GraphKey key{x, y, z, n, S, mode, t->ws_gen, cap, (long long)lcap, t->dir_nnz_cap,
+                               {t->lo[0], t->lo[1], t->lo[2]}, t->k};
+            int slot = -1;
+            for (int g = 0; g < 2; ++g)
+                if (t->tg_exec[g] && t->tg_key[g] == key) slot = g;
+            if (slot < 0) {                           // capture (the C5 loop alternates two state buffers: 2 slots)
+                slot = t->tg_next;
+                t->tg_next ^= 1;
+                if (t->tg_exec[slot]) cudaGraphExecDestroy(t->tg_exec[slot]);
+                t->tg_exec[slot] = nullptr;
+                cudaGraph_t gph = nullptr;
+                cudaError_t e = cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal);
+                afmm_status s1 = AFMM_OK, s2 = AFMM_OK;
+                if (e == cudaSuccess) {
+                    s1 = enq_buckets();
+                    s2 = s1 ? s1 : enq_direct();
+                    e = cudaStreamEndCapture(st, &gph);
+                }
+                if (s1 || s2) return s1 ? s1 : s2;
+                if (e == cudaSuccess) e = cudaGraphInstantiate(&t->tg_exec[slot], gph, 0);
+                if (gph) cudaGraphDestroy(gph);
+                if (e != cudaSuccess) {               // no graph here: launch directly from now on
+                    cudaGetLastError();
+                    t->tg_exec[slot] = nullptr;
+                    t->graph_broken = true;
+                } else {
+                    t->tg_key[slot] = key;
+                }
+            }
+            if (t->tg_exec[slot]) {
+                TCU(t, cudaGraphLaunch(t->tg_exec[slot], st));
+                ++t->graph_launches;
+            } else {
+                if (afmm_status s = enq_buckets()) return s;
+                if (afmm_status s = enq_direct()) return s;
+            }
+        } else {
+            if (use_buckets) {
+                if (afmm_status s = enq_buckets()) return s;
+            } else if (need_sort) {
+                if (afmm_status s = full_sort()) return s;
+                need_sort = false;
+            }
+            if (afmm_status s = enq_direct()) return s;
         }
-        dir_finish_kernel<<<(int)std::min<long long>(grid_for((long long)cap, TH), 148LL * 8), TH, 0, st>>>(
-            dctl, nd, t->u_off, t->pvw_prefix, t->pvw_nchild, t->pv_base);
-        TCU(t, cudaGetLastError());
-        DirCtl hc;
-        TCU(t, cudaMemcpyAsync(&hc, dctl, sizeof(DirCtl), cudaMemcpyDeviceToHost, st));
         TCU(t, cudaStreamSynchronize(st));
+        const DirCtl hc = *t->h_ctl;
         if (hc.sort_overflow) {                       // a bucket exceeded kBucketCap: sort in full, redo
-            bovf = nullptr;
+            use_buckets = false;
+            need_sort = true;
             ++t->sort_fallbacks;
             if (getenv("AFMM_TREE_DEBUG")) fprintf(stderr, "afmm tree: bucket sort overflow %lld\n", t->sort_fallbacks);
-            if (afmm_status s = full_sort()) return s;
             continue;
         }
-        if (hc.cap_overflow) {                        // grow the node / leaf capacities, redo
+        if (hc.cap_overflow) {                        // grow the node / leaf capacities, redo (the sort stands)
             if (hc.nn > (long long)cap) {
                 cap = (size_t)(hc.nn + hc.nn / 4);
                 if (afmm_status s = alloc_nodes(cap, nd, node_set)) return s;
             }
             if (hc.L > t->dir_leaf_cap) t->dir_leaf_cap = std::min<long long>(n, hc.L + hc.L / 4);
+            use_buckets = false;
             continue;
         }
         L = hc.L;
@@ -1675,8 +1801,9 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
             done_levels = true;
             break;
         }
-        if (hc.nnz_overflow) {                        // grow the U-list entry capacity, redo
+        if (hc.nnz_overflow) {                        // grow the U-list entry capacity, redo (the sort stands)
             t->dir_nnz_cap = hc.nnz + hc.nnz / 4 + 64;
+            use_buckets = false;
             continue;
         }
         // complete: sizes for the host, done
@@ -1684,9 +1811,6 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
         t->n_nodes = hc.nn;
         t->node_cap = cap;
         t->pv_levels = hc.levels;
-        std::swap(t->pv_prefix, t->pvw_prefix);
-        std::swap(t->pv_nchild, t->pvw_nchild);
-        std::swap(t->pv_cap, t->pvw_cap);
         t->L = L;
         t->n = n;
         t->built = true;
@@ -1913,6 +2037,10 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     else
         ulist_copy_kernel<<<(int)(((long long)L * 32 + 255) / 256), 256, 0, st>>>(L, rows, t->u_off, t->u_idx);
     TCU(t, cudaGetLastError());
+    {                                             // the next build's device-side view of this one
+        const int hs[2] = {L, t->pv_levels};
+        TCU(t, cudaMemcpyAsync(t->d_state, hs, sizeof(hs), cudaMemcpyHostToDevice, st));
+    }
     TCU(t, cudaStreamSynchronize(st));
     t->n = n;
     t->built = true;
@@ -1999,6 +2127,13 @@ extern "C" afmm_status afmm_tree_nodes(afmm_tree *t, int *level, unsigned long l
     if (level)
         for (int l = 0; l < t->pv_levels; ++l)
             for (long long i = base[l]; i < base[l + 1]; ++i) level[i] = l;
+    return AFMM_OK;
+}
+
+extern "C" afmm_status afmm_tree_counters(const afmm_tree *t, long long *graph_launches, long long *sort_fallbacks) {
+    if (!t) return AFMM_EINVAL;
+    if (graph_launches) *graph_launches = t->graph_launches;
+    if (sort_fallbacks) *sort_fallbacks = t->sort_fallbacks;
     return AFMM_OK;
 }
 

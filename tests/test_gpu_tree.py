@@ -235,3 +235,43 @@ def test_direct_construction_matches_level_loop(monkeypatch):
                 for k in a:
                     assert np.array_equal(np.asarray(a[k]), np.asarray(b[k])), (name, other, step, k)
     del rng
+
+
+def test_enforce_graph_replay_matches_direct_launches(monkeypatch):
+    """Enforce_S along a trajectory with the positions in two alternating device
+    buffers (as the C5 loop holds them): the direct build captured into CUDA graphs
+    and replayed (AFMM_TREE_GRAPH default) gives the same trees and node arrays as
+    launching the same kernels directly (AFMM_TREE_GRAPH=0), and replays happen; the
+    trees also equal the oracle's Collapse / PushDown chain."""
+    afmm = _afmm()
+    x, y, z, m, vx, vy, vz = synth.colliding_with_velocities(50000, 6)
+    dom = synth.c5_domain(x, y, z)
+    S = 24
+    n = x.shape[0]
+    res = {}
+    for flag in ("1", "0"):
+        monkeypatch.setenv("AFMM_TREE_GRAPH", flag)
+        t = afmm.GpuTree(0)
+        bufs = [torch.empty((3, n), device="cuda") for _ in range(2)]
+        t.build(_dev(x), _dev(y), _dev(z), S, domain=dom)
+        To = oracle.Tree(x, y, z, S, domain=dom, ulist=False)
+        px, py, pz, qx, qy, qz = (a[To.perm] for a in (x, y, z, vx, vy, vz))
+        out = []
+        for step in range(7):
+            px, py, pz = oracle.drift(px, py, pz, qx, qy, qz, 0.3)
+            b = bufs[step % 2]
+            b.copy_(torch.from_numpy(np.stack([px, py, pz])))
+            t.enforce(b[0], b[1], b[2], S)
+            G = _tree_and_nodes(t, n)
+            To2 = To.enforce(px, py, pz, S)
+            for k in ("perm", "leaf_start", "leaf_count", "leaf_level", "leaf_prefix", "u_off", "u_idx"):
+                assert np.array_equal(G[k], getattr(To2, k)), (flag, step, k)
+            out.append(G)
+            px, py, pz, qx, qy, qz = (a[To2.perm] for a in (px, py, pz, qx, qy, qz))
+            To = To2
+        res[flag] = (out, t.counters())
+        t.close()
+    assert res["1"][1]["graph_launches"] >= 6 and res["0"][1]["graph_launches"] == 0
+    for step, (a, b) in enumerate(zip(res["1"][0], res["0"][0])):
+        for k in a:
+            assert np.array_equal(np.asarray(a[k]), np.asarray(b[k])), (step, k)
