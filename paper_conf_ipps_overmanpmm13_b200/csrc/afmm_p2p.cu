@@ -1446,7 +1446,10 @@ static afmm_status resolve_stream_ops(afmm_p2p *h) {
 using WriteValueFn = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
 
 static constexpr int kMaxPieces = 64;
-static constexpr int kInChunks = 8;                 // input chunks of the streamed H2D
+// input chunks of the streamed H2D: 8 up to 8 Mi bodies, then one per Mi bodies up to 16 (the first chunk's
+// PCIe time is what the kernel's early tasks wait for; A/B on C2: 8 best, on C4 (16 Mi): 16 best, +2 %,
+// profiles/r1_ab_input_chunks.txt, profiles/r2_ab_input_chunks_C4.txt)
+static int in_chunks(long long n) { return (int)std::min<long long>(16, std::max<long long>(8, n >> 20)); }
 static constexpr int kMaxChunks = 16;               // chunk masks ride in the high 16 bits of Task.piece
 
 // Regroup this rank's tasks into P pieces of consecutive targets (equal modelled
@@ -1514,7 +1517,7 @@ static afmm_status build_pipe(afmm_p2p *h, int P) {
     // first chunk and stays behind the copies, and every output piece's stragglers (leaves
     // whose U-lists reach far in Morton order) run as soon as the last chunk lands.
     const char *kenv = getenv("AFMM_E2E_CHUNKS");             // measurements only
-    const int kin = kenv ? std::max(1, std::min(kMaxChunks, atoi(kenv))) : kInChunks;
+    const int kin = kenv ? std::max(1, std::min(kMaxChunks, atoi(kenv))) : in_chunks(h->n);
     const int K = (int)std::min<long long>(kin, std::max<long long>(1, h->n / 4096));
     const long long chunk = (h->n + K - 1) / K;
     std::vector<int> need_chunk(nt, 0);
