@@ -164,7 +164,7 @@ afmm_status fail(afmm_p2p *h, afmm_status st, const char *fmt, ...) {
         vsnprintf(buf, sizeof(buf), fmt, ap);
         va_end(ap);
         h->err = buf;
-        if (st == AFMM_ECUDA || st == AFMM_ENOMEM) h->poisoned = true;
+        if (st == AFMM_ECUDA || st == AFMM_ENOMEM || st == AFMM_ENCCL) h->poisoned = true;   // (header: poisoned)
     }
     return st;
 }
@@ -452,6 +452,12 @@ extern "C" afmm_status afmm_p2p_create(const afmm_p2p_config *cfg, afmm_p2p **ou
 extern "C" void afmm_p2p_destroy(afmm_p2p *h) {
     if (!h) return;
     cudaSetDevice(h->cfg.device);
+    // a poisoned handle's communicator is aborted first (ncclCommAbort on fatal errors), so
+    // outstanding NCCL work waiting on a failed peer does not block the stream synchronises below
+    if (h->comm && h->poisoned && afmm::nccl_api().CommAbort) {
+        afmm::nccl_api().CommAbort(h->comm);
+        h->comm = nullptr;
+    }
     if (h->stream) cudaStreamSynchronize(h->stream);
     cudaFree(h->d_bodies);
     cudaFree(h->d_soa);
