@@ -1457,6 +1457,16 @@ static constexpr int kMaxPieces = 64;
 // profiles/r1_ab_input_chunks.txt, profiles/r2_ab_input_chunks_C4.txt)
 static int in_chunks(long long n) { return (int)std::min<long long>(16, std::max<long long>(8, n >> 20)); }
 static constexpr int kMaxChunks = 16;               // chunk masks ride in the high 16 bits of Task.piece
+// First body of input chunk k of K (k = K: n).  Equal chunks up to 8 Mi bodies; above, quadratic boundaries
+// n (k/K)^2 (small chunks first, large ones late: C4 host-to-host +0.9 %, C2 -2 %; a small first chunk followed
+// by equal ones gains nothing; AFMM_E2E_UNIFORM=1 / 2 forces equal / quadratic; profiles/r2_ab_input_chunks_C4.txt)
+static long long chunk_bound(int k, int K, long long n) {
+    static const int force = [] { const char *e = getenv("AFMM_E2E_UNIFORM"); return e ? atoi(e) : 0; }();
+    if (k >= K) return n;
+    const bool quad = force == 2 || (force == 0 && n >= (8LL << 20));
+    const long long b = quad ? n * k * k / ((long long)K * K) : (long long)k * ((n + K - 1) / K);
+    return std::min<long long>(n, b & ~3LL);                    // multiples of 4: the packs' float4 path stays aligned
+}
 
 // Regroup this rank's tasks into P pieces of consecutive targets (equal modelled
 // cost tgt_count * nsrc, cut in tgt_start order); inside a piece the tasks keep
@@ -1517,7 +1527,7 @@ static afmm_status build_pipe(afmm_p2p *h, int P) {
         if (q > 0) h->pipe_need[q] = std::max(h->pipe_need[q], h->pipe_need[q - 1]);
         if (h->pipe_lo[q] > h->pipe_hi[q]) h->pipe_lo[q] = h->pipe_hi[q] = 0;   // empty piece
     }
-    // Input chunks: the bodies in K equal Morton ranges, copied and packed in order while
+    // Input chunks: the bodies in K Morton ranges (chunk_bound), copied and packed in order while
     // the kernel runs.  Task order: by the last input chunk the task needs (its sources
     // and targets), then by output piece, LPT kept inside -- so the kernel starts on the
     // first chunk and stays behind the copies, and every output piece's stragglers (leaves
@@ -1525,7 +1535,6 @@ static afmm_status build_pipe(afmm_p2p *h, int P) {
     const char *kenv = getenv("AFMM_E2E_CHUNKS");             // measurements only
     const int kin = kenv ? std::max(1, std::min(kMaxChunks, atoi(kenv))) : in_chunks(h->n);
     const int K = (int)std::min<long long>(kin, std::max<long long>(1, h->n / 4096));
-    const long long chunk = (h->n + K - 1) / K;
     std::vector<int> need_chunk(nt, 0);
     for (int i = 0; i < nt; ++i) {
         long long need = (long long)t[i].tgt_start + t[i].tgt_count;
@@ -1533,7 +1542,9 @@ static afmm_status build_pipe(afmm_p2p *h, int P) {
             const afmm::Seg &z = sg[t[i].seg_begin + j];
             need = std::max(need, (long long)z.gstart + z.len);
         }
-        need_chunk[i] = (int)std::min<long long>(K - 1, (need - 1) / chunk);
+        int c = 0;                                              // the chunk holding body need - 1
+        while (c < K - 1 && chunk_bound(c + 1, K, h->n) < need) ++c;
+        need_chunk[i] = c;
     }
     std::vector<int> ord2(nt);
     for (int i = 0; i < nt; ++i) ord2[i] = i;
@@ -1703,7 +1714,6 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
         return AFMM_OK;
     };
     const int K = h->pipe_K;
-    const long long chunk = (n + K - 1) / K;
     // Without room for a pack block beside a P2P CTA (co_resident_pack) the chain
     // could not progress under the persistent kernel: pack every chunk first, then
     // launch (the kernel's chunk waits then pass at once).
@@ -1712,7 +1722,7 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
     // Enqueue the input chain: pack chunk k, then publish k + 1 (stream write).
     auto enqueue_inputs = [&](bool capturing) -> afmm_status {
         for (int k = 0; k < K; ++k) {
-            const long long lo = k * chunk, hi = std::min<long long>(n, lo + chunk);
+            const long long lo = chunk_bound(k, K, n), hi = chunk_bound(k + 1, K, n);
             if (hi > lo) {
                 const float *src[4];
                 for (int a = 0; a < 4; ++a) {
