@@ -13,6 +13,6 @@ timeout 900 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/b
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv \
     --log-file gpurun_out/launches_$TAG.csv python bench.py --steps 3 --warmup 3 --no-sweep --no-cpu-baseline \
     --no-stokeslet --no-proxy > /dev/null 2>&1
-timeout 900 ncu --set full --import-source on --clock-control none -k regex:p2p_kernel -s 1 -c 1 \
+[ -n "$NO_FULL" ] || timeout 900 ncu --set full --import-source on --clock-control none -k regex:p2p_kernel -s 1 -c 1 \
     -o gpurun_out/p2p_full_C4_$TAG python tools/prof_p2p.py --config C4 --S 256 --evals 2 > /dev/null 2>&1
 ls -la gpurun_out | tail -12
