@@ -696,54 +696,91 @@ __device__ __forceinline__ bool dir_bad(const DirCtl *c) {
     return c->sort_overflow | c->cap_overflow | c->ulist_overflow | c->nnz_overflow;
 }
 
+// Range maxima over the window arrays: per 32-position block a prefix and a suffix
+// maximum (warp scans) and a sparse table over the block maxima, so a window is
+// max(suffix of its first block, prefix of its last, table lookup of the full
+// blocks between) -- 2 warp scans per array instead of log2(S) doubling passes.
+constexpr int kDirLen = kDirTile + kDirMaxS, kDirNB = kDirLen / 32, kDirST = 7;   // 2^6 = 64 < 96 blocks
+static_assert(kDirLen % 32 == 0 && (1 << (kDirST - 1)) * 2 > kDirNB, "window table sizes");
+__device__ __forceinline__ int dir_rmq(const signed char *X, const signed char *P, const signed char *Q,
+                                       const signed char (*ST)[kDirNB], int lo, int hi) {
+    const int bl = lo >> 5, bh = hi >> 5;
+    if (bl == bh) {
+        int m = -1;
+        for (int a = lo; a <= hi; ++a) m = max(m, (int)X[a]);
+        return m;
+    }
+    int m = max((int)Q[lo], (int)P[hi]);
+    const int nbt = bh - bl - 1;
+    if (nbt > 0) {
+        const int k = 31 - __clz(nbt);
+        m = max(m, max((int)ST[k][bl + 1], (int)ST[k][bh - (1 << k)]));
+    }
+    return m;
+}
+
 __global__ void __launch_bounds__(kDirThreads) leaf_level_kernel(long long n, const unsigned long long *__restrict__ keys,
                                                                  int S, int mode, PrevTree pv,
                                                                  const int *__restrict__ pv_levels,
                                                                  unsigned char *__restrict__ lvl, int *__restrict__ flag) {
     if (pv_levels) pv.levels = mode == kModeEnforce ? *pv_levels : 0;   // the previous build's (device word)
-    // [buffer][array][pos]: array 0 = windows of S + 1 (w), 1 = windows of S (v);
-    // position a <-> window start j = t0 - S + a; -1 = no such window
-    __shared__ signed char win[2][2][kDirTile + kDirMaxS];
+    // array 0 = windows of S + 1 (w), 1 = windows of S (v, Enforce_S only); position a <->
+    // window start j = t0 - S + a; -1 = no such window
+    __shared__ signed char X[2][kDirLen], P[2][kDirLen], Q[2][kDirLen];
+    __shared__ signed char ST[2][kDirST][kDirNB];
+    const bool enf = mode == kModeEnforce && pv.levels > 0;
+    const int na = enf ? 2 : 1;
     const long long t0 = (long long)blockIdx.x * kDirTile;
-    const int len = kDirTile + S;
-    for (int a = threadIdx.x; a < len; a += blockDim.x) {
+    const int len = kDirTile + S, nb = (len + 31) >> 5;
+    for (int a = threadIdx.x; a < nb * 32; a += blockDim.x) {
         const long long j = t0 - S + a;
         signed char w = -1, v = -1;
-        if (j >= 0) {
+        if (a < len && j >= 0) {
             const unsigned long long kj = j < n ? keys[j] : 0ull;
             if (j + S < n) w = (signed char)lcp_digits(kj, keys[j + S]);
-            if (j + S - 1 < n) v = (signed char)lcp_digits(kj, keys[j + S - 1]);
+            if (enf && j + S - 1 < n) v = (signed char)lcp_digits(kj, keys[j + S - 1]);
         }
-        win[0][0][a] = w;
-        win[0][1][a] = v;
+        X[0][a] = w;
+        X[1][a] = v;
     }
-    // doubling: after the pass of step h, X[a] = max over [a, a + 2h)
-    int HA = 1, HB = 1;                      // largest powers of two <= S + 1 and <= S
-    while (2 * HA <= S + 1) HA *= 2;
-    while (2 * HB <= S) HB *= 2;
-    int cur = 0;
-    for (int h = 1; h < HA; h *= 2) {
-        __syncthreads();
-        for (int a = threadIdx.x; a < len; a += blockDim.x) {
-            const signed char x = win[cur][0][a], y = a + h < len ? win[cur][0][a + h] : (signed char)-1;
-            win[cur ^ 1][0][a] = x > y ? x : y;
-            const signed char p = win[cur][1][a], q = a + h < len ? win[cur][1][a + h] : (signed char)-1;
-            win[cur ^ 1][1][a] = h < HB ? (p > q ? p : q) : p;
+    __syncthreads();
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    for (int bk = wid; bk < nb; bk += kDirThreads / 32)
+        for (int ar = 0; ar < na; ++ar) {
+            const int x = X[ar][32 * bk + lane];
+            int pre = x, suf = x;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int u = __shfl_up_sync(0xffffffffu, pre, o), d = __shfl_down_sync(0xffffffffu, suf, o);
+                if (lane >= o) pre = max(pre, u);
+                if (lane + o < 32) suf = max(suf, d);
+            }
+            P[ar][32 * bk + lane] = (signed char)pre;
+            Q[ar][32 * bk + lane] = (signed char)suf;
+            if (lane == 31) ST[ar][0][bk] = (signed char)pre;
         }
-        cur ^= 1;
+    const int kmax = 31 - __clz(max(1, (S >> 5) + 2));          // full blocks inside a window: < S / 32 + 2
+    for (int k = 1; k <= kmax && k < kDirST; ++k) {
+        __syncthreads();
+        for (int t = threadIdx.x; t < na * nb; t += blockDim.x) {
+            const int ar = t / nb, bk = t - ar * nb, o = 1 << (k - 1);
+            const signed char x = ST[ar][k - 1][bk], y = bk + o < nb ? ST[ar][k - 1][bk + o] : (signed char)-1;
+            ST[ar][k][bk] = x > y ? x : y;
+        }
     }
     __syncthreads();
     for (int a0 = threadIdx.x; a0 < kDirTile; a0 += blockDim.x) {
         const long long i = t0 + a0;
         if (i >= n) break;
         // windows of S + 1 containing i: j in [i - S, i] -> a in [a0, a0 + S]
-        const int m1 = max((int)win[cur][0][a0], (int)win[cur][0][a0 + S + 1 - HA]);
-        // windows of S containing i: j in [i - S + 1, i] -> a in [a0 + 1, a0 + S]
-        const int m2 = max((int)win[cur][1][a0 + 1], (int)win[cur][1][a0 + 1 + S - HB]);
+        const int m1 = dir_rmq(X[0], P[0], Q[0], ST[0], a0, a0 + S);
         const unsigned long long ki = keys[i];
         int l = m1 < 0 ? 0 : min(m1 + 1, kMaxLevel);
-        if (mode == kModeEnforce && pv.levels > 0)
+        if (enf && l < kMaxLevel) {
+            // windows of S containing i: j in [i - S + 1, i] -> a in [a0 + 1, a0 + S]
+            const int m2 = dir_rmq(X[1], P[1], Q[1], ST[1], a0 + 1, a0 + S);
             while (l < kMaxLevel && l <= m2 && prev_internal(pv, l, ki >> (3 * (kMaxLevel - l)))) ++l;
+        }
         lvl[i] = (unsigned char)l;
         flag[i] = (i == 0 || lcp_digits(keys[i - 1], ki) < l) ? 1 : 0;
     }
