@@ -33,3 +33,32 @@ def test_bench_two_ranks_same_gpu_gloo():
     assert d["config"]["name"] == "C1" and d["config"]["parallelism"].endswith("x2 (cost model, PAPER L16)")
     assert d["gpu_launches"] >= 2 * 3                  # at least a P2P launch per rank per timed step
     assert d["e2e"]["value"] > 0
+
+
+def test_bench_n1_contract_fields():
+    """bench.py at N = 1 on the small C1 workload prints one JSON line with every
+    key the driver contract names: metric/value/unit, timing, roofline (bound,
+    achieved, peak, frac, traffic), cpu_baseline (oracle, cores, sample), e2e with
+    the copied bytes, clocks sampled during the timed region, gpu_launches."""
+    cmd = [sys.executable, os.path.join(ROOT, "bench.py"), "--config", "C1", "--steps", "3", "--warmup", "3",
+           "--no-sweep", "--no-stokeslet", "--no-proxy", "--cpu-seconds", "0.5", "--cpu-seconds-1core", "0.3"]
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, r.stdout[-2000:]
+    d = json.loads(lines[0])
+    for k in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better", "scaling",
+              "vs_baseline", "dtype", "data", "config", "roofline", "cpu_baseline", "e2e", "clocks", "gpu_launches"):
+        assert k in d, k
+    assert d["n_gpus"] == 1 and d["steps"] == 3 and d["warmup"] >= 3 and d["value"] > 0
+    assert d["unit"] == "interactions/s" and d["higher_is_better"] is True and d["dtype"] == "f32"
+    rf = d["roofline"]
+    assert rf["bound"] == "alu" and rf["unit"] == "TFLOP/s" and 0 < rf["frac"] < 1
+    assert abs(rf["frac"] - rf["achieved"] / rf["peak"]) < 1e-9
+    cb = d["cpu_baseline"]
+    assert cb["kind"] == "oracle" and cb["cores"] >= 1 and cb["value"] > 0 and cb["sample"]
+    e = d["e2e"]
+    assert e["value"] > 0 and e["h2d_bytes_per_step"] > 0 and e["d2h_bytes_per_step"] > 0
+    assert d["gpu_launches"] >= 3
+    assert "sm_mhz" in d["clocks"] and "reasons" in d["clocks"]
+    assert d["config"]["name"] == "C1" and d["config"]["workload"]
