@@ -1986,11 +1986,15 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
         t->pv_prefix = nullptr;
         t->pv_nchild = nullptr;
         t->pv_cap = 0;
+        ++t->ws_gen;                               // a captured direct build referenced the old arrays
         TCU(t, cudaMalloc(&t->pv_prefix, (size_t)nn * sizeof(unsigned long long)));
         TCU(t, cudaMalloc(&t->pv_nchild, (size_t)nn * sizeof(int)));
         t->pv_cap = (size_t)nn;
     }
-    if (!t->pv_base) TCU(t, cudaMalloc(&t->pv_base, (kMaxLevel + 2) * sizeof(long long)));
+    if (!t->pv_base) {
+        TCU(t, cudaMalloc(&t->pv_base, (kMaxLevel + 2) * sizeof(long long)));
+        ++t->ws_gen;
+    }
     TCU(t, cudaMemcpyAsync(t->pv_prefix, nd.prefix, nn * sizeof(unsigned long long), cudaMemcpyDeviceToDevice, st));
     TCU(t, cudaMemcpyAsync(t->pv_nchild, nd.nchild, nn * sizeof(int), cudaMemcpyDeviceToDevice, st));
     TCU(t, cudaMemcpyAsync(t->pv_base, lvl_base.data(), lvl_base.size() * sizeof(long long),
