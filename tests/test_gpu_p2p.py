@@ -578,3 +578,36 @@ def test_unequal_masses_general_path_and_equal_mass_path():
     g8, _ = gpu_eval(xs, ys, zs, (ms * 8).astype(np.float32), d, 1e-6)
     for a, b in zip(g_eq, g8):
         assert np.array_equal(a * 8, b)
+
+
+def test_eval_host_pipelined_large_quadratic_chunks(monkeypatch):
+    """Above 8 Mi bodies the streamed host-to-host evaluation cuts its input into
+    one chunk per Mi bodies with quadratic boundaries n (k/K)^2 (afmm_p2p.cu
+    chunk_bound): on 9 Mi Plummer bodies (K = 9, an odd n) its outputs are
+    bit-identical to afmm_p2p_eval on device buffers, zero-copy in and out."""
+    monkeypatch.setenv("AFMM_E2E_ZEROCOPY", "1")
+    afmm = _afmm()
+    n = 9 * (1 << 20) + 3
+    x, y, z, m = synth.make("plummer", n, 29)
+    tree = afmm.GpuTree(0)
+    X, Y, Z, M = (torch.from_numpy(v).cuda() for v in (x, y, z, m))
+    info = tree.build(X, Y, Z, 256)
+    d = tree.device_arrays()
+    bod = torch.empty((4, n), device="cuda")
+    for a, src in enumerate((X, Y, Z, M)):
+        tree.gather(src, bod[a])
+    hb = [bod[a].cpu().pin_memory() for a in range(4)]
+    got = [torch.full((n,), float("nan")).pin_memory() for _ in range(4)]
+    ref = torch.full((4, n), float("nan"), device="cuda")
+    h = afmm.P2P(eps2=1e-6)
+    h.set_bodies(bod[0], bod[1], bod[2], bod[3])
+    h.set_tree_device(info["n_leaves"], d["leaf_start"], d["leaf_count"], d["u_off"], d["u_idx"])
+    h.eval(ref[0], ref[1], ref[2], ref[3])
+    st = h.eval_host_pipelined(*hb, *got, pieces=1)
+    assert st["zero_copy"] == 1
+    r_ = ref.cpu().numpy()
+    assert np.isfinite(r_).all()
+    for a in range(4):
+        assert np.array_equal(got[a].numpy(), r_[a])
+    h.close()
+    tree.close()
