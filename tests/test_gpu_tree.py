@@ -275,3 +275,39 @@ def test_enforce_graph_replay_matches_direct_launches(monkeypatch):
     for step, (a, b) in enumerate(zip(res["1"][0], res["0"][0])):
         for k in a:
             assert np.array_equal(np.asarray(a[k]), np.asarray(b[k])), (step, k)
+
+
+def test_randomised_builds_and_enforce_chains_bit_exact():
+    """30 seeded random cases: n in [1, 30000], S in [1, 2100] (around the direct
+    construction's tile and window limits: S = 2048 is its largest, 2049+ takes the
+    level loop), uniform / Plummer / colliding / clustered duplicates, fresh builds
+    and short Enforce_S chains with a changing S on one handle -- every tree and
+    U-list bit-exact with the oracle."""
+    afmm = _afmm()
+    rng = np.random.default_rng(2026)
+    dists = ("uniform", "plummer", "colliding")
+    t = afmm.GpuTree(0)
+    for case in range(30):
+        n = int(rng.choice([1, 2, 3, 17, 63, 64, 65, 1000, 4096, 9999, 30000]))
+        S = int(rng.choice([1, 2, 7, 31, 32, 33, 64, 100, 255, 1024, 2047, 2048, 2049, 2100]))
+        x, y, z, m = synth.make(dists[case % 3], n, 100 + case)
+        if case % 5 == 4:                                    # clustered duplicates
+            idx = rng.integers(0, max(1, n // 7), n)
+            x, y, z = x[idx], y[idx], z[idx]
+        dom = (np.array([-16.0, -16.0, -16.0]), 5)
+        t.build(_dev(x), _dev(y), _dev(z), S, domain=dom)
+        To = oracle.Tree(x, y, z, S, domain=dom)
+        assert_same_tree(t.copy_out(n), To)
+        px, py, pz = x[To.perm], y[To.perm], z[To.perm]
+        for step in range(2):
+            S2 = max(1, int(S * rng.choice([0.5, 1.0, 1.5])))
+            d = rng.standard_normal((3, n)).astype(np.float32) * np.float32(0.01)
+            px, py, pz = (px + d[0]).astype(np.float32), (py + d[1]).astype(np.float32), (pz + d[2]).astype(np.float32)
+            t.enforce(_dev(px), _dev(py), _dev(pz), S2)
+            To2 = To.enforce(px, py, pz, S2)
+            G = t.copy_out(n)
+            for k in ("perm", "leaf_start", "leaf_count", "leaf_level", "leaf_prefix", "u_off", "u_idx"):
+                assert np.array_equal(G[k], getattr(To2, k)), (case, n, S, S2, step, k)
+            px, py, pz = px[To2.perm], py[To2.perm], pz[To2.perm]
+            To = To2
+    t.close()
