@@ -611,3 +611,26 @@ def test_eval_host_pipelined_large_quadratic_chunks(monkeypatch):
         assert np.array_equal(got[a].numpy(), r_[a])
     h.close()
     tree.close()
+
+
+def test_randomised_parity():
+    """24 seeded random cases against the fp64 oracle (reading R16): n in [2, 20000],
+    S in [1, 300], uniform / Plummer / colliding positions, equal or random masses
+    (the equal-mass and general pair loops), eps^2 in {0 (distinct points only),
+    1e-8, 1e-6, 1e-3}, G != 1, worlds 1..3 merged -- plus the interaction count."""
+    rng = np.random.default_rng(77)
+    dists = ("uniform", "plummer", "colliding")
+    for case in range(24):
+        n = int(rng.choice([2, 5, 33, 500, 2048, 7777, 20000]))
+        S = int(rng.choice([1, 3, 8, 17, 64, 128, 200, 300]))
+        eps2 = float(rng.choice([0.0, 1e-8, 1e-6, 1e-3]))
+        x, y, z, m = synth.make(dists[case % 3], n, 500 + case)
+        if case % 2:
+            m = rng.uniform(0.5, 2.0, n).astype(np.float32) / np.float32(n)
+        if eps2 == 0.0:                                   # R21: coincident bodies need a softening
+            keys = np.stack([x, y, z], 1)
+            if np.unique(keys, axis=0).shape[0] < n:
+                eps2 = 1e-8
+        G = float(rng.choice([1.0, 0.5, 6.674e-11]))
+        world = int(rng.choice([1, 2, 3]))
+        _parity(x, y, z, m, S, eps2, G=G, world=world)
