@@ -721,7 +721,7 @@ __device__ __forceinline__ void load_targets(Targets &T, const float4 *__restric
 // back to packing every chunk before the launch when it does not hold.
 constexpr int kMaxRegs = kThreads <= 384 ? 160 : ((65536 - 4096) / kThreads) / 8 * 8;   // (tuning builds: more warps)
 static_assert(kMinBlocksPerSM == 1 && kMaxRegs * kThreads <= 65536, "register budget: one CTA per SM");
-// (The device-path kernel keeps __launch_bounds__: the same 158 registers, but
+// (The device-path kernel keeps __launch_bounds__: about the same register count, but
 // its code under __maxnreg__ measured 1.2 % slower, profiles/r2_ab_regs.txt.)
 template <class Law, bool kStream>
 __device__ __forceinline__ void p2p_body(const P2PParams &p) {
