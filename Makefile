@@ -21,10 +21,17 @@ $(LIB): $(CU_SRCS) $(CU_HDRS)
 $(ORACLE): oracle/oracle.c
 	gcc -O2 -fopenmp -ffp-contract=off -fno-fast-math -fPIC -shared -std=c11 -o $@ $< -lm
 
+# plain-C caller of the C ABI (no Python): examples/c_abi_demo.c
+DEMO      := examples/c_abi_demo
+$(DEMO): examples/c_abi_demo.c $(LIB) include/afmm_p2p.h include/afmm_tree.h
+	gcc -O2 -std=c11 -Wall -Iinclude -I/usr/local/cuda/include -o $@ $< -L$(PKG) -lafmm_p2p \
+	    -L/usr/local/cuda/lib64 -lcudart -lm -Wl,-rpath,'$$ORIGIN/../$(PKG)' -Wl,-rpath,/usr/local/cuda/lib64
+demo: $(DEMO)
+
 sass: $(LIB)
 	cuobjdump -sass $(LIB) > $(PKG)/sass.txt
 
 clean:
-	rm -f $(LIB) $(ORACLE) $(PKG)/ptxas.log
+	rm -f $(LIB) $(ORACLE) $(PKG)/ptxas.log $(DEMO)
 
-.PHONY: all clean sass
+.PHONY: all clean sass demo

@@ -99,3 +99,13 @@ def test_ctypes_structs_match_the_c_headers(tmp_path):
         assert got[(cname, "size")] == ctypes.sizeof(py), cname
         for f, _ in py._fields_:
             assert got[(cname, f)] == getattr(py, f).offset, (cname, f)
+
+
+def test_plain_c_caller_builds():
+    """examples/c_abi_demo.c -- a C program using only include/*.h and the .so
+    (tree builder + host-pointer P2P entry points + stats) -- compiles and links
+    with gcc (`make demo`); it runs on the GPU in tests/test_gpu_c_demo.py."""
+    import subprocess
+    r = subprocess.run(["make", "-C", ROOT, "demo"], capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
+    assert os.path.exists(os.path.join(ROOT, "examples", "c_abi_demo"))
