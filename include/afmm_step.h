@@ -27,6 +27,13 @@ afmm_status afmm_kick(long long n, float *vx, float *vy, float *vz, const float 
 afmm_status afmm_drift(long long n, float *x, float *y, float *z, const float *vx, const float *vy,
                        const float *vz, float dt, void *stream);
 
+/* kick then drift in one pass (the first two updates of a KDK step):
+ * v <- v + h * a, then x <- x + dt * v with the kicked v -- the same two
+ * roundings per component as afmm_kick followed by afmm_drift (bit-identical),
+ * one read of a, v, x and one write of v, x instead of two launches. */
+afmm_status afmm_kick_drift(long long n, float *x, float *y, float *z, float *vx, float *vy, float *vz,
+                            const float *ax, const float *ay, const float *az, float h, float dt, void *stream);
+
 #ifdef __cplusplus
 }
 #endif

@@ -117,6 +117,7 @@ _sig("afmm_cost_fit", _i, _i, _p, _p, _p)
 _sig("afmm_p2p_set_cost_coef", _i, _p, _p)
 _sig("afmm_kick", _i, _ll, _p, _p, _p, _p, _p, _p, C.c_float, _p)
 _sig("afmm_drift", _i, _ll, _p, _p, _p, _p, _p, _p, C.c_float, _p)
+_sig("afmm_kick_drift", _i, _ll, _p, _p, _p, _p, _p, _p, _p, _p, _p, C.c_float, C.c_float, _p)
 _sig("afmm_fp32_peak", _i, _i, C.POINTER(_d), C.POINTER(_d), C.POINTER(_d))
 _sig("afmm_version", C.c_char_p)
 _sig("afmm_launch_count", C.c_longlong)
@@ -172,7 +173,7 @@ EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
             "afmm_p2p_kernel_times",
             "afmm_p2p_destroy", "afmm_p2p_last_error", "afmm_interactions",
             "afmm_partition_literal", "afmm_partition_weighted", "afmm_partition_rebalance",
-            "afmm_cost_fit", "afmm_p2p_set_cost_coef", "afmm_kick", "afmm_drift",
+            "afmm_cost_fit", "afmm_p2p_set_cost_coef", "afmm_kick", "afmm_drift", "afmm_kick_drift",
             "afmm_fp32_peak", "afmm_version",
             "afmm_tree_create", "afmm_tree_build", "afmm_tree_enforce", "afmm_tree_info", "afmm_tree_counters",
             "afmm_tree_farfield_counts", "afmm_lb_config_init", "afmm_lb_create", "afmm_lb_step",
@@ -322,6 +323,14 @@ def drift(x, y, z, vx, vy, vz, dt, stream=None):
                          float(dt), stream)
     if st:
         raise AfmmError(st, "afmm_drift")
+
+
+def kick_drift(x, y, z, vx, vy, vz, ax, ay, az, h, dt, stream=None):
+    """Kick then drift in one kernel (afmm_kick_drift; bit-identical to kick + drift)."""
+    st = _lib.afmm_kick_drift(int(x.shape[0]), _ptr(x), _ptr(y), _ptr(z), _ptr(vx), _ptr(vy), _ptr(vz), _ptr(ax),
+                              _ptr(ay), _ptr(az), float(h), float(dt), stream)
+    if st:
+        raise AfmmError(st, "afmm_kick_drift")
 
 
 def fp32_peak(device: int = 0):

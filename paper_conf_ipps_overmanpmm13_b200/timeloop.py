@@ -6,8 +6,8 @@ arithmetic step runs in libafmm_p2p.so kernels).
 Per time step (PAPER L16 SIII.D "the particle positions are updated ... and
 then any tree optimizations are done to improve the run on the next time step";
 L20 SVI.A Enforce_S; L18 SIV.D observational coefficients):
-  1. kick(dt/2) with the current accelerations      (afmm_kick, own slice)
-  2. drift(dt)                                        (afmm_drift, own slice)
+  1. kick(dt/2) with the current accelerations      (afmm_kick_drift: 1 and 2 in one kernel,
+  2. drift(dt)                                         own slice; the same roundings as afmm_kick + afmm_drift)
   3. N > 1: replicate positions and velocities        (allgatherv of slices)
   4. Enforce_S on the moved bodies (fixed domain)     (afmm_tree_enforce)
   5. carry the state into the new tree order          (afmm_tree_gather)
@@ -40,7 +40,7 @@ import numpy as np
 import torch
 
 from . import (LB_ENFORCE, LB_FINE, LB_KEEP, LB_REBUILD, TREE_KEEP, GpuTree, P2P, cost_fit, drift,
-               kick, lb_predict)
+               kick, kick_drift, lb_predict)
 
 # Default modelled far-field costs (seconds per operation: P2M, M2M, M2L, L2L,
 # L2P), reading R29: translation operators of an order-p expansion cost
@@ -114,6 +114,13 @@ class TimeLoop:
         s = self.state
         drift(s[0, lo:hi], s[1, lo:hi], s[2, lo:hi], s[4, lo:hi], s[5, lo:hi], s[6, lo:hi], self.dt,
               self.stream.cuda_stream)
+
+    def _kick_drift(self):
+        """kick(dt/2) then drift(dt) in one kernel (afmm_kick_drift: the same two roundings)."""
+        lo, hi = self._slice()
+        s, a = self.state, self.acc
+        kick_drift(s[0, lo:hi], s[1, lo:hi], s[2, lo:hi], s[4, lo:hi], s[5, lo:hi], s[6, lo:hi], a[0, lo:hi],
+                   a[1, lo:hi], a[2, lo:hi], 0.5 * self.dt, self.dt, self.stream.cuda_stream)
 
     def _refit(self):
         """N > 1: per-bucket coefficients from this step's kernel times (L18 SIV.D)."""
@@ -193,8 +200,7 @@ class TimeLoop:
         t0 = time.perf_counter()
         ev[0].record(self.stream)
         self._refit()
-        self._kick()
-        self._drift()
+        self._kick_drift()
         if self.world > 1:
             from . import dist as pdist
             pdist.gather_slices([self.state[a] for a in (0, 1, 2, 4, 5, 6)], self.body_split)

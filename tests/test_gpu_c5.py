@@ -48,6 +48,13 @@ def test_leapfrog_kernels_vs_oracle():
         assert _ulp_close(g.cpu().numpy(), r)
     for g, r in zip(dx, rx):
         assert _ulp_close(g.cpu().numpy(), r)
+    # the fused kick + drift (afmm_kick_drift, used by the C5 loop) is bit-identical to the two kernels
+    fv = [torch.from_numpy(t).cuda() for t in v]
+    fx = [torch.from_numpy(t).cuda() for t in x]
+    afmm.kick_drift(*fx, *fv, *da, h, np.float32(0.05))
+    torch.cuda.synchronize()
+    for f, g in zip(fv + fx, dv + dx):
+        assert torch.equal(f, g)
 
 
 def test_gpu_enforce_bit_exact_along_trajectory():
