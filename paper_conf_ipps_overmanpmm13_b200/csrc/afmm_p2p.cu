@@ -110,6 +110,7 @@ struct afmm_p2p {
     std::vector<int> pipe_off;                       // P + 1 offsets into d_ptasks
     std::vector<long long> pipe_need, pipe_lo, pipe_hi;   // bodies needed (prefix), output range per piece
     int pipe_K = 0;                                   // input chunks (streamed H2D)
+    int last_tail_ctas = 0;                           // chunked eval: CTAs of the tail grid on the comm SMs
     afmm::Task *d_ptasks = nullptr;
     size_t ptasks_cap = 0;
     int *d_pqueue = nullptr;                         // kMaxPieces counters
@@ -1926,24 +1927,7 @@ static afmm_status launch_chunked(afmm_p2p *h, float *ax, float *ay, float *az, 
     const unsigned tag = h->epoch << 16;
     CUDA_TRY(h, cudaMemsetAsync(w_err(h), 0, sizeof(int), h->stream));
     CUDA_TRY(h, cudaMemsetAsync(h->d_queue, 0, sizeof(int), h->stream));
-    if (deliver) {
-        const afmm::NcclApi &nc = afmm::nccl_api();
-        CUDA_TRY(h, cudaEventRecord(h->ev_c0, h->stream));    // the root's pack, earlier readers of the bodies
-        CUDA_TRY(h, cudaStreamWaitEvent(h->s_comm, h->ev_c0, 0));
-        NCCL_TRY(h, nc.Broadcast(mass_flag(h), mass_flag(h), sizeof(float4), ncclChar, 0, h->comm, h->s_comm));
-        unsigned cum = 0;
-        for (int j = 0; j < h->chunk_K; ++j) {
-            const int c = h->chunk_order[j];
-            const long long lo = h->chunk_bounds[c], cnt = h->chunk_bounds[c + 1] - lo;
-            if (cnt > 0)
-                NCCL_TRY(h, nc.Broadcast(h->d_bodies + lo, h->d_bodies + lo, (size_t)cnt * sizeof(float4), ncclChar, 0,
-                                         h->comm, h->s_comm));
-            cum |= 1u << c;
-            const CUresult r = write32((CUstream)h->s_comm, (CUdeviceptr)w_ready(h), (cuuint32_t)(tag | cum), 0);
-            if (r != CUDA_SUCCESS) return fail(h, AFMM_ECUDA, "chunked eval: cuStreamWriteValue32 failed (%d)", (int)r);
-        }
-        CUDA_TRY(h, cudaEventRecord(h->ev_c1, h->s_comm));
-    }
+    if (h->comm && (st = reset_tspan(h))) return st;          // before the communication stream may start a kernel
     afmm::P2PParams p;
     p.bodies = h->d_bodies;
     p.tasks = h->d_ctasks;
@@ -1965,7 +1949,36 @@ static afmm_status launch_chunked(afmm_p2p *h, float *ax, float *ay, float *az, 
     p.m0_ptr = reinterpret_cast<const float *>(mass_flag(h) + 1);                            // trailer word 1
     p.out_coalesce = 0;
     p.tspan = h->comm ? w_tspan(h) : nullptr;
-    if (h->comm && (st = reset_tspan(h))) return st;
+    h->last_tail_ctas = 0;
+    if (deliver) {
+        const afmm::NcclApi &nc = afmm::nccl_api();
+        CUDA_TRY(h, cudaEventRecord(h->ev_c0, h->stream));    // the root's pack, earlier readers of the bodies
+        CUDA_TRY(h, cudaStreamWaitEvent(h->s_comm, h->ev_c0, 0));
+        NCCL_TRY(h, nc.Broadcast(mass_flag(h), mass_flag(h), sizeof(float4), ncclChar, 0, h->comm, h->s_comm));
+        unsigned cum = 0;
+        for (int j = 0; j < h->chunk_K; ++j) {
+            const int c = h->chunk_order[j];
+            const long long lo = h->chunk_bounds[c], cnt = h->chunk_bounds[c + 1] - lo;
+            if (cnt > 0)
+                NCCL_TRY(h, nc.Broadcast(h->d_bodies + lo, h->d_bodies + lo, (size_t)cnt * sizeof(float4), ncclChar, 0,
+                                         h->comm, h->s_comm));
+            cum |= 1u << c;
+            const CUresult r = write32((CUstream)h->s_comm, (CUdeviceptr)w_ready(h), (cuuint32_t)(tag | cum), 0);
+            if (r != CUDA_SUCCESS) return fail(h, AFMM_ECUDA, "chunked eval: cuStreamWriteValue32 failed (%d)", (int)r);
+        }
+        // The SMs kept free for NCCL idle once the last chunk is out: a second, small grid of the same
+        // kernel on the communication stream takes tasks from the same queue until it is empty (every
+        // result is the same whichever CTA computes it).  AFMM_TAIL_KERNEL=0 disables it.
+        const char *tenv = getenv("AFMM_TAIL_KERNEL");
+        const int tail = std::min(comm_sms(h), (p.n_tasks + afmm::kWarps - 1) / afmm::kWarps);
+        if (p.n_tasks > 0 && tail > 0 && !(tenv && tenv[0] == '0')) {
+            afmm::p2p_stream_kernel_t<afmm::Gravity><<<tail, afmm::kThreads, afmm::kDynSmem, h->s_comm>>>(p);
+            COUNT_LAUNCH(1);
+            CUDA_TRY(h, cudaGetLastError());
+            h->last_tail_ctas = tail;
+        }
+        CUDA_TRY(h, cudaEventRecord(h->ev_c1, h->s_comm));
+    }
     h->last_zero_copy = false;
     h->last_input_graph = false;
     h->last_streamed = false;
@@ -1980,7 +1993,7 @@ static afmm_status launch_chunked(afmm_p2p *h, float *ax, float *ay, float *az, 
         afmm::p2p_stream_kernel_t<afmm::Gravity><<<grid, afmm::kThreads, afmm::kDynSmem, h->stream>>>(p);
         COUNT_LAUNCH(1);
         CUDA_TRY(h, cudaGetLastError());
-        nlaunch = 1;
+        nlaunch = 1 + (h->last_tail_ctas > 0);
     }
     CUDA_TRY(h, cudaEventRecord(h->ev1, h->stream));
     *h->h_cerr = 0;

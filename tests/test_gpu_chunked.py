@@ -58,9 +58,10 @@ def _plain(bod, T, world=1, rank=0, slice_world=0):
 def test_library_communicator_one_rank(unequal):
     """A 1-rank library communicator through the C ABI: the eval after
     set_bodies runs the chunked path (NCCL broadcast of the trailer + chunks on
-    the communication stream, kernel waiting per task), the next eval the plain
-    one; both bit-identical to a handle without communicator; kernel_ms_max is
-    the all-reduced device-timer span (one rank: its own)."""
+    the communication stream, kernel waiting per task, then a tail grid of the same
+    kernel on the communication SMs draining the same task queue), the next eval
+    the plain one; both bit-identical to a handle without communicator;
+    kernel_ms_max is the all-reduced device-timer span (one rank: its own)."""
     afmm = _afmm()
     bod, T = _setup(unequal=unequal)
     ref, _, _ = _plain(bod, T)
@@ -72,6 +73,8 @@ def test_library_communicator_one_rank(unequal):
         out = torch.full((4, n), float("nan"), device="cuda")
         st = h.eval(out[0], out[1], out[2], out[3], stats=True)
         assert st["chunked_bodies"] == (1 if it == 0 else 0)
+        # the chunked eval also runs the tail grid on the communication SMs after the broadcast (2 launches)
+        assert st["n_launches"] == (2 if it == 0 else 1), st
         assert 0.3 * st["kernel_ms"] <= st["kernel_ms_max"] <= 3.0 * st["kernel_ms"] + 0.05, st
         assert np.array_equal(out.cpu().numpy(), ref)
     K, order = h.chunks()[0].shape[0] - 1, h.chunks()[1]
