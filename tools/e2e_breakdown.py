@@ -19,6 +19,8 @@ import synth  # noqa: E402
 ap = argparse.ArgumentParser()
 ap.add_argument("--reps", type=int, default=20)
 ap.add_argument("--config", default="C2")
+ap.add_argument("--pieces", type=int, default=1, help="output pieces (staged-output modes copy each back as it completes)")
+ap.add_argument("--modes", default="1,i,o,0")
 a = ap.parse_args()
 c = synth.CONFIGS[a.config]
 x, y, z, m = synth.make(a.config)
@@ -40,17 +42,17 @@ h.set_tree(T["leaf_start"], T["leaf_count"], T["u_off"], T["u_idx"])
 d = [torch.empty(n, device="cuda") for _ in range(4)]
 inter = h.eval(*d, stats=True)["interactions_total"]
 res = {"interactions": inter}
-for mode in ("1", "i", "o", "0"):
+for mode in a.modes.split(","):
     os.environ["AFMM_E2E_ZEROCOPY"] = mode
     for _ in range(3):
-        h.eval_host_pipelined(*hx, *ho, pieces=1)
+        h.eval_host_pipelined(*hx, *ho, pieces=a.pieces)
     torch.cuda.synchronize()
     wall, span, kern = [], [], []
     for _ in range(a.reps):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(st)
         t0 = time.perf_counter()
-        h.eval_host_pipelined(*hx, *ho, pieces=1)
+        h.eval_host_pipelined(*hx, *ho, pieces=a.pieces)
         wall.append((time.perf_counter() - t0) * 1e3)
         e1.record(st)
         e1.synchronize()
