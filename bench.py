@@ -12,7 +12,8 @@ largest one that fits one GPU, so N = 1 and N > 1 measure the same workload
 One step = one pass of the whole hot path over the workload with inputs
 resident in HBM: body ingest (pack on rank 0) and the P2P evaluation.
   N = 1: pack + P2P kernel.
-  N > 1: the library communicator (afmm_p2p_config.nccl_id): rank 0 packs, the
+  N > 1: the library communicator (afmm_p2p_config.nccl_id): rank 0 packs each
+         chunk right before its broadcast (afmm_p2p_set_bodies_deferred), the
          eval broadcasts the packed bodies in chunks on a communication stream
          WHILE the P2P kernel runs (each warp waits only for the chunks its task
          needs), the kernel stores every result into every rank's output array
@@ -500,7 +501,9 @@ def main():
     packed = pdist.packed_bodies(h, dev) if world > 1 and comm_mode != "library" else None
 
     def step():
-        if world == 1 or rank == 0:
+        if world > 1 and rank == 0 and comm_mode == "library":
+            h.set_bodies_deferred(bod[0], bod[1], bod[2], bod[3])   # a1: packed chunk by chunk inside the eval
+        elif world == 1 or rank == 0:
             h.set_bodies(bod[0], bod[1], bod[2], bod[3])      # a1: pack (1 kernel; the root only at N > 1)
         elif comm_mode == "library":
             h.set_bodies(None, None, None, None, n=n)         # a4: to be received in the next eval
@@ -634,8 +637,9 @@ def main():
             "config": config_dict(args.config, S, n, info["n_leaves"], info["nnz"], inter, world),
             "step": {
                 "what": ("pack + P2P kernel" if world == 1 else
-                         ("rank 0 packs; eval: chunked NCCL broadcast of the packed bodies overlapped with the "
-                          "P2P kernel (library communicator), kernel stores every result into all ranks' outputs "
+                         ("eval: rank 0 packs each chunk right before its NCCL broadcast, the broadcasts overlapped with the "
+                          "P2P kernel (library communicator) and followed by a tail grid of it on the NCCL SMs, kernel stores every "
+                          "result into all ranks' outputs "
                           "over CUDA-IPC peer windows (fused gather), 8-byte in-stream all-reduce of the kernel "
                           "time = completion" if comm_mode == "library" else
                           "rank 0 packs + one NCCL broadcast of the packed bodies + P2P kernel storing into peer "

@@ -77,6 +77,7 @@ def _sig(name, res, *args):
 _sig("afmm_p2p_config_init", _i, C.POINTER(Config))
 _sig("afmm_p2p_create", _i, C.POINTER(Config), C.POINTER(_p))
 _sig("afmm_p2p_set_bodies", _i, _p, _ll, _p, _p, _p, _p)
+_sig("afmm_p2p_set_bodies_deferred", _i, _p, _ll, _p, _p, _p, _p)
 _sig("afmm_p2p_set_bodies_host", _i, _p, _ll, _p, _p, _p, _p)
 _sig("afmm_p2p_bodies_buffer", _i, _p, C.POINTER(_p), C.POINTER(_ll))
 _sig("afmm_p2p_set_bodies_stokeslet", _i, _p, _ll, _p, _p, _p, _p, _p, _p)
@@ -169,7 +170,7 @@ EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
             "afmm_p2p_set_bodies_stokeslet",
             "afmm_p2p_set_partition", "afmm_p2p_get_partition", "afmm_p2p_rebalance",
             "afmm_p2p_set_tree_device", "afmm_tree_device_arrays",
-            "afmm_p2p_eval", "afmm_p2p_eval_host", "afmm_p2p_stats_get", "afmm_p2p_stream",
+            "afmm_p2p_eval", "afmm_p2p_eval_host", "afmm_p2p_stats_get", "afmm_p2p_stream", "afmm_p2p_set_bodies_deferred",
             "afmm_p2p_kernel_times",
             "afmm_p2p_destroy", "afmm_p2p_last_error", "afmm_interactions",
             "afmm_partition_literal", "afmm_partition_weighted", "afmm_partition_rebalance",
@@ -407,6 +408,15 @@ class P2P:
             x, y, z, m = (_np(v, np.float32) for v in (x, y, z, m))
             self._check(_lib.afmm_p2p_set_bodies_host(self._h, n, _ptr(x), _ptr(y), _ptr(z), _ptr(m)),
                         "afmm_p2p_set_bodies_host")
+
+    def set_bodies_deferred(self, x, y, z, m):
+        """afmm_p2p_set_bodies_deferred (torch CUDA tensors, root of a library
+        communicator): packed chunk by chunk inside the next eval; the tensors must
+        stay alive and unchanged until that eval's stream work completes."""
+        if not _is_device(x):
+            raise ValueError("set_bodies_deferred takes CUDA tensors")
+        self._check(_lib.afmm_p2p_set_bodies_deferred(self._h, int(x.shape[0]), _ptr(x), _ptr(y), _ptr(z), _ptr(m)),
+                    "afmm_p2p_set_bodies_deferred")
 
     def set_bodies_stokeslet(self, x, y, z, fx, fy, fz):
         """Stokeslet bodies: torch CUDA tensors (device pointers), tree order."""

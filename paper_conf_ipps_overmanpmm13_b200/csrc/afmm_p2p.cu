@@ -140,6 +140,8 @@ struct afmm_p2p {
     cudaStream_t s_comm = nullptr;                   // NCCL work + chunk publication
     cudaEvent_t ev_c0 = nullptr, ev_c1 = nullptr, ev_c2 = nullptr, ev_c3 = nullptr;
     bool bodies_pending = false;                     // set_bodies since the last eval: replicate in the next
+    const float *def_soa[4] = {nullptr, nullptr, nullptr, nullptr};   // set_bodies_deferred: the root's SoA,
+    bool deferred = false;                           // packed chunk by chunk inside the next chunked eval
     bool last_chunked = false;
     // device words: [0] chunk mask (epoch << 16 | mask), [1] wait-timeout flag, then
     // tspan[2] (u64, %globaltimer), kernel_ms[2] (double: own span, max over ranks)
@@ -542,6 +544,54 @@ static afmm_status pack(afmm_p2p *h, const float *x, const float *y, const float
     return AFMM_OK;
 }
 
+// set_bodies_deferred (library communicator, root): the trailer -- "some mass differs
+// from m_0" and m_0 -- from the caller's SoA before any chunk is broadcast, then each
+// chunk packed right before its broadcast (pack_range_kernel), so the root's pack
+// overlaps the replication instead of preceding it.
+__global__ void mass_trailer_kernel(long long n, const float *__restrict__ m, int *__restrict__ trailer) {
+    const float m0 = m[0];
+    if (blockIdx.x == 0 && threadIdx.x == 0) trailer[1] = __float_as_int(m0);
+    bool diff = false;
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+        diff |= m[i] != m0;
+    if (__any_sync(0xffffffffu, diff) && (threadIdx.x & 31) == 0) atomicOr(trailer, -1);
+}
+__global__ void pack_range_kernel(long long n, const float *__restrict__ x, const float *__restrict__ y,
+                                  const float *__restrict__ z, const float *__restrict__ m, float4 *__restrict__ out) {
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+        out[i] = make_float4(x[i], y[i], z[i], m[i]);
+}
+// a deferred pack that something other than the chunked eval needs now: pack in full
+static afmm_status flush_deferred(afmm_p2p *h) {
+    if (!h->deferred) return AFMM_OK;
+    h->deferred = false;
+    return pack(h, h->def_soa[0], h->def_soa[1], h->def_soa[2], h->def_soa[3]);
+}
+
+extern "C" afmm_status afmm_p2p_set_bodies_deferred(afmm_p2p *h, long long n, const float *x, const float *y,
+                                                    const float *z, const float *m) {
+    NvtxScope nvtx_("afmm.set_bodies_deferred");
+    CHECK_HANDLE(h);
+    if (h->cfg.law != AFMM_LAW_GRAVITY) return fail(h, AFMM_EINVAL, "set_bodies_deferred: handle law is not gravity");
+    if (n < 1 || n >= (1LL << 31)) return fail(h, AFMM_EINVAL, "set_bodies_deferred: n=%lld out of [1, 2^31)", n);
+    if (!x || !y || !z || !m) return fail(h, AFMM_EINVAL, "set_bodies_deferred: null pointer");
+    afmm_status st = set_device(h);
+    if (st) return st;
+    if ((st = alloc_bodies(h, n))) return st;
+    if (!h->comm || h->cfg.rank != 0) {                     // nothing to overlap: pack now
+        h->deferred = false;
+        h->bodies_pending = h->comm != nullptr;
+        return pack(h, x, y, z, m);
+    }
+    h->def_soa[0] = x;
+    h->def_soa[1] = y;
+    h->def_soa[2] = z;
+    h->def_soa[3] = m;
+    h->deferred = true;
+    h->bodies_pending = true;
+    return AFMM_OK;
+}
+
 extern "C" afmm_status afmm_p2p_set_bodies(afmm_p2p *h, long long n, const float *x,
                                            const float *y, const float *z, const float *m) {
     NvtxScope nvtx_("afmm.set_bodies");
@@ -554,6 +604,7 @@ extern "C" afmm_status afmm_p2p_set_bodies(afmm_p2p *h, long long n, const float
     if (st) return st;
     if ((st = alloc_bodies(h, n))) return st;
     h->bodies_pending = h->comm != nullptr;          // the next eval replicates them (library communicator)
+    h->deferred = false;
     if (nn == 4) return pack(h, x, y, z, m);
     // allocate only: the equal-mass flag reads "unequal" until a full-buffer
     // broadcast (afmm_p2p_bodies_buffer, trailer included) brings the root's
@@ -572,6 +623,7 @@ extern "C" afmm_status afmm_p2p_set_bodies_host(afmm_p2p *h, long long n, const 
     if (st) return st;
     if ((st = alloc_bodies(h, n))) return st;
     h->bodies_pending = h->comm != nullptr;
+    h->deferred = false;
     if (4 * n > h->soa_cap) {
         cudaFree(h->d_soa);
         h->d_soa = nullptr;
@@ -612,6 +664,7 @@ extern "C" afmm_status afmm_p2p_set_bodies_stokeslet(afmm_p2p *h, long long n, c
 
 extern "C" afmm_status afmm_p2p_bodies_buffer(afmm_p2p *h, void **dev_ptr, long long *bytes) {
     CHECK_HANDLE(h);
+    if (afmm_status st0 = flush_deferred(h)) return st0;
     if (!h->d_bodies || h->n < 1) return fail(h, AFMM_ESTATE, "bodies_buffer: no bodies set");
     if (dev_ptr) *dev_ptr = h->d_bodies;
     if (bytes) *bytes = (h->n * words_of(h) + 1) * (long long)sizeof(float4);   // + the flag trailer
@@ -1657,6 +1710,7 @@ extern "C" afmm_status afmm_p2p_eval_host_pipelined(afmm_p2p *h, long long n, co
     h->last_zero_copy = zc;
     const float m0 = m[0];                          // equal-mass test of the streamed chunks
     h->bodies_pending = false;                      // every body comes from this call's host arrays
+    h->deferred = false;
     h->last_chunked = false;
     CUDA_TRY(h, cudaMemsetAsync(mass_flag(h), 0xff, sizeof(int), h->stream));   // bodies replaced: flag "unequal"
     CUDA_TRY(h, cudaEventRecord(h->ev_start, h->stream));      // earlier readers of the bodies / outputs
@@ -1954,11 +2008,27 @@ static afmm_status launch_chunked(afmm_p2p *h, float *ax, float *ay, float *az, 
         const afmm::NcclApi &nc = afmm::nccl_api();
         CUDA_TRY(h, cudaEventRecord(h->ev_c0, h->stream));    // the root's pack, earlier readers of the bodies
         CUDA_TRY(h, cudaStreamWaitEvent(h->s_comm, h->ev_c0, 0));
+        const bool defer = h->deferred;                        // root of set_bodies_deferred: pack per chunk here
+        h->deferred = false;
+        const int TH = 256;
+        if (defer) {
+            CUDA_TRY(h, cudaMemsetAsync(mass_flag(h), 0, sizeof(int), h->s_comm));
+            mass_trailer_kernel<<<h->num_sms * 2, TH, 0, h->s_comm>>>(h->n, h->def_soa[3], mass_flag(h));
+            COUNT_LAUNCH(1);
+            CUDA_TRY(h, cudaGetLastError());
+        }
         NCCL_TRY(h, nc.Broadcast(mass_flag(h), mass_flag(h), sizeof(float4), ncclChar, 0, h->comm, h->s_comm));
         unsigned cum = 0;
         for (int j = 0; j < h->chunk_K; ++j) {
             const int c = h->chunk_order[j];
             const long long lo = h->chunk_bounds[c], cnt = h->chunk_bounds[c + 1] - lo;
+            if (defer && cnt > 0) {
+                const int blocks = (int)std::min<long long>((cnt + TH - 1) / TH, (long long)h->num_sms * 4);
+                pack_range_kernel<<<blocks, TH, 0, h->s_comm>>>(cnt, h->def_soa[0] + lo, h->def_soa[1] + lo,
+                                                                h->def_soa[2] + lo, h->def_soa[3] + lo, h->d_bodies + lo);
+                COUNT_LAUNCH(1);
+                CUDA_TRY(h, cudaGetLastError());
+            }
             if (cnt > 0)
                 NCCL_TRY(h, nc.Broadcast(h->d_bodies + lo, h->d_bodies + lo, (size_t)cnt * sizeof(float4), ncclChar, 0,
                                          h->comm, h->s_comm));
@@ -2058,6 +2128,7 @@ extern "C" afmm_status afmm_p2p_worklist(afmm_p2p *h, int *tasks, long long cap_
 extern "C" afmm_status afmm_p2p_eval_chunked(afmm_p2p *h, float *ax, float *ay, float *az, float *phi) {
     NvtxScope nvtx_("afmm.eval_chunked");
     CHECK_HANDLE(h);
+    if (afmm_status st0 = flush_deferred(h)) return st0;
     if (!h->d_bodies || !h->have_tree) return fail(h, AFMM_ESTATE, "eval_chunked: set_bodies and set_tree first");
     if (!ax || !ay || !az || !phi) return fail(h, AFMM_EINVAL, "eval_chunked: null output pointer");
     afmm_status st = set_device(h);

@@ -79,6 +79,20 @@ def test_library_communicator_one_rank(unequal):
         assert np.array_equal(out.cpu().numpy(), ref)
     K, order = h.chunks()[0].shape[0] - 1, h.chunks()[1]
     assert sorted(order.tolist()) == list(range(K))
+    # the root's deferred pack: every chunk packed right before its broadcast, inside the eval
+    h.set_bodies_deferred(bod[0], bod[1], bod[2], bod[3])
+    out = torch.full((4, n), float("nan"), device="cuda")
+    st = h.eval(out[0], out[1], out[2], out[3], stats=True)
+    assert st["chunked_bodies"] == 1
+    assert np.array_equal(out.cpu().numpy(), ref)
+    # a deferred pack that afmm_p2p_bodies_buffer needs first is packed in full
+    h.set_bodies_deferred(bod[0], bod[1], bod[2], bod[3])
+    ptr, nbytes = h.bodies_buffer()
+    assert nbytes == 16 * (n + 1)
+    out.fill_(float("nan"))
+    h.eval(out[0], out[1], out[2], out[3])
+    torch.cuda.synchronize()
+    assert np.array_equal(out.cpu().numpy(), ref)
     # host outputs (afmm_p2p_eval_host) through the same communicator, after a new set_bodies
     h.set_bodies(bod[0], bod[1], bod[2], bod[3])
     ho = [np.full(n, np.nan, np.float32) for _ in range(4)]
