@@ -77,6 +77,7 @@ def _sig(name, res, *args):
 _sig("afmm_p2p_config_init", _i, C.POINTER(Config))
 _sig("afmm_p2p_create", _i, C.POINTER(Config), C.POINTER(_p))
 _sig("afmm_p2p_set_bodies", _i, _p, _ll, _p, _p, _p, _p)
+_sig("afmm_p2p_interactions", _i, _p, C.POINTER(_ll), C.POINTER(_ll))
 _sig("afmm_p2p_set_bodies_deferred", _i, _p, _ll, _p, _p, _p, _p)
 _sig("afmm_p2p_set_bodies_host", _i, _p, _ll, _p, _p, _p, _p)
 _sig("afmm_p2p_bodies_buffer", _i, _p, C.POINTER(_p), C.POINTER(_ll))
@@ -170,7 +171,7 @@ EXPORTED = ["afmm_p2p_config_init", "afmm_p2p_create", "afmm_p2p_set_bodies",
             "afmm_p2p_set_bodies_stokeslet",
             "afmm_p2p_set_partition", "afmm_p2p_get_partition", "afmm_p2p_rebalance",
             "afmm_p2p_set_tree_device", "afmm_tree_device_arrays",
-            "afmm_p2p_eval", "afmm_p2p_eval_host", "afmm_p2p_stats_get", "afmm_p2p_stream", "afmm_p2p_set_bodies_deferred",
+            "afmm_p2p_eval", "afmm_p2p_eval_host", "afmm_p2p_stats_get", "afmm_p2p_stream", "afmm_p2p_set_bodies_deferred", "afmm_p2p_interactions",
             "afmm_p2p_kernel_times",
             "afmm_p2p_destroy", "afmm_p2p_last_error", "afmm_interactions",
             "afmm_partition_literal", "afmm_partition_weighted", "afmm_partition_rebalance",
@@ -549,6 +550,12 @@ class P2P:
         if cnt < 0:
             self._check(cnt, "afmm_p2p_kernel_times")
         return buf[:cnt].copy()
+
+    def interactions(self):
+        """(total, this rank's) interactions of the current tree (afmm_p2p_interactions; no sync)."""
+        t, r = _ll(), _ll()
+        self._check(_lib.afmm_p2p_interactions(self._h, C.byref(t), C.byref(r)), "afmm_p2p_interactions")
+        return t.value, r.value
 
     def stats(self):
         s = Stats()

@@ -1436,6 +1436,14 @@ static afmm_status launch_any(afmm_p2p *h, float *ax, float *ay, float *az, floa
     return h->comm ? comm_finish(h) : AFMM_OK;
 }
 
+extern "C" afmm_status afmm_p2p_interactions(const afmm_p2p *h, long long *total, long long *rank) {
+    if (!h) return AFMM_EINVAL;
+    if (!h->have_tree) return AFMM_ESTATE;
+    if (total) *total = h->I_total;
+    if (rank) *rank = h->rank_interactions;
+    return AFMM_OK;
+}
+
 extern "C" afmm_status afmm_p2p_eval(afmm_p2p *h, float *ax, float *ay, float *az, float *phi,
                                      afmm_p2p_stats *stats) {
     NvtxScope nvtx_("afmm.eval");

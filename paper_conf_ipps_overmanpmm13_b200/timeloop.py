@@ -191,11 +191,17 @@ class TimeLoop:
                     "S_next": S, "next": ("keep", "rebuild", "enforce", "fine")[a]})
 
     # ------------------------------------------------------------------ one step
-    def step(self, hooks=None):
+    def step(self, hooks=None, sync=True):
         """One KDK step.  hooks (optional dict of callables) receive the state
         for verification: 'pre_enforce'(x, y, z) with positions in the old tree
         order, 'post_maintain'(loop, rec) after the tree maintenance (loop.tree
-        holds the new tree), 'post_eval'(loop) after the new accelerations."""
+        holds the new tree), 'post_eval'(loop) after the new accelerations.
+        sync=False (no load balancer, no hooks): the step is only enqueued past
+        the library's own readbacks -- no synchronise at its end, so the next
+        step's host work overlaps this step's P2P kernel; the record's timings
+        are filled in later by finish(records) after one synchronise."""
+        if not sync and (self.lb is not None or hooks):
+            raise ValueError("sync=False needs lb=None and no hooks")
         ev = [torch.cuda.Event(enable_timing=True) for _ in range(6)]
         t0 = time.perf_counter()
         ev[0].record(self.stream)
@@ -221,6 +227,12 @@ class TimeLoop:
         ev[4].record(self.stream)
         self._kick()
         ev[5].record(self.stream)
+        if not sync:
+            rec = {"step": self.step_no, "n_leaves": self.T["n_leaves"], "interactions": self.h.interactions()[0],
+                   "S": self.S, "_events": ev}
+            self.log.append(rec)
+            self.step_no += 1
+            return rec
         torch.cuda.synchronize()
         st = self.h.stats()
         rec = {"step": self.step_no, "n_leaves": self.T["n_leaves"], "interactions": st["interactions_total"],
@@ -238,6 +250,19 @@ class TimeLoop:
         if hooks and "post_eval" in hooks:
             hooks["post_eval"](self)
         return rec
+
+    def finish(self, recs):
+        """After steps taken with sync=False: synchronise once and fill each record's
+        timings from its events and the library's kernel-time ring (last <= 64 evals)."""
+        torch.cuda.synchronize()
+        kt = self.h.kernel_times(len(recs)) if recs else []
+        kt = list(kt)[-len(recs):] if recs else []
+        for r, k in zip(recs, [None] * (len(recs) - len(kt)) + kt):
+            ev = r.pop("_events")
+            r.update({"kernel_ms": k, "kick_drift_ms": ev[0].elapsed_time(ev[1]),
+                      "enforce_ms": ev[1].elapsed_time(ev[2]), "set_tree_ms": ev[2].elapsed_time(ev[3]),
+                      "eval_ms": ev[3].elapsed_time(ev[4]), "gpu_step_ms": ev[0].elapsed_time(ev[5])})
+        return recs
 
     def close(self):
         self.h.close()

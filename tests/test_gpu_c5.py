@@ -129,3 +129,26 @@ def test_c5_timeloop_per_step_parity():
     p0 = (m.astype(float)[None, :] * np.stack([vx, vy, vz]).astype(float)).sum(1)
     assert np.abs(p - p0).max() < 1e-4
     loop.close()
+
+
+def test_c5_async_steps_bit_identical():
+    """TimeLoop.step(sync=False) (steps enqueued back to back, one synchronise in
+    finish) gives a trajectory bit-identical to synchronised steps, and finish()
+    fills every record's timings (the bench's C5 line runs this way)."""
+    from paper_conf_ipps_overmanpmm13_b200.timeloop import TimeLoop
+    n, S, eps2, dt = 1 << 16, 64, 1e-4, 0.05
+    x, y, z, m, vx, vy, vz = synth.colliding_with_velocities(n, 8)
+    dom = synth.c5_domain(x, y, z)
+    a = TimeLoop(x, y, z, m, vx, vy, vz, S, eps2, dt, dom)
+    for _ in range(8):
+        a.step()
+    sa = a.state.cpu().numpy().copy()
+    a.close()
+    b = TimeLoop(x, y, z, m, vx, vy, vz, S, eps2, dt, dom)
+    recs = [b.step(sync=False) for _ in range(8)]
+    b.finish(recs)
+    sb = b.state.cpu().numpy().copy()
+    b.close()
+    assert np.array_equal(sa, sb)
+    for r in recs:
+        assert r["kernel_ms"] > 0 and r["enforce_ms"] > 0 and r["interactions"] > 0 and "_events" not in r
