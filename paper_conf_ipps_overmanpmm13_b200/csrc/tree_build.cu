@@ -113,8 +113,12 @@ struct Nodes {
 // bucket by (key, input index) and concatenating them in bucket order IS the
 // stable sort by (key, index) (round 1: CUB's 8-pass 63-bit radix sort).  Most
 // bodies stay in their leaf's cell between steps (≈ 74 % on C5), the buckets hold
-// about a leaf each, and a warp sorts one (bitonic, <= kBucketCap keys).
+// about a leaf each, and a warp sorts one (bitonic, <= kBucketCap keys); the few
+// larger buckets (a KEEP rebuild lets leaves grow past S) go to a list that one CTA
+// each sorts in shared memory (<= kBigCap keys); beyond that a full sort.
 constexpr int kBucketCap = 512;
+constexpr int kBigCap = 8192, kBigList = 128, kBigThreads = 1024;
+constexpr size_t kBigSmem = (size_t)kBigCap * (sizeof(unsigned long long) + sizeof(int));
 __global__ void cell_range_kernel(const int *__restrict__ Ldev, const int *__restrict__ ll,
                                   const unsigned long long *__restrict__ lp, unsigned long long *__restrict__ clo,
                                   unsigned long long *__restrict__ chi) {
@@ -254,7 +258,8 @@ __global__ void __launch_bounds__(32 * kBucketWarps) bucket_sort_kernel(const in
                                                                         const int *__restrict__ bidx,
                                                                         unsigned long long *__restrict__ okeys,
                                                                         int *__restrict__ oidx,
-                                                                        int *__restrict__ overflow) {
+                                                                        int *__restrict__ overflow,
+                                                                        int *__restrict__ big) {
     const int lane = threadIdx.x & 31;
     const int nb = 2 * *Ldev + 1;
     const int b = blockIdx.x * kBucketWarps + (threadIdx.x >> 5);
@@ -267,8 +272,12 @@ __global__ void __launch_bounds__(32 * kBucketWarps) bucket_sort_kernel(const in
         }
         return;
     }
-    if (cnt > kBucketCap) {                                   // rare: the caller falls back to a full sort
-        if (lane == 0) atomicExch(overflow, 1);
+    if (cnt > kBucketCap) {                                   // to the CTA sort; rarer still: a full sort
+        if (lane == 0) {
+            const int q = atomicAdd(big, 1);
+            if (q < kBigList && cnt <= kBigCap) big[1 + q] = b;
+            else atomicExch(overflow, 1);
+        }
         return;
     }
     if (cnt <= 32) warp_bitonic<1>(o, cnt, bkeys, bidx, okeys, oidx, lane);
@@ -276,6 +285,55 @@ __global__ void __launch_bounds__(32 * kBucketWarps) bucket_sort_kernel(const in
     else if (cnt <= 128) warp_bitonic<4>(o, cnt, bkeys, bidx, okeys, oidx, lane);
     else if (cnt <= 256) warp_bitonic<8>(o, cnt, bkeys, bidx, okeys, oidx, lane);
     else warp_bitonic<16>(o, cnt, bkeys, bidx, okeys, oidx, lane);
+}
+
+// The listed buckets of kBucketCap < count <= kBigCap keys: one CTA per bucket, a
+// bitonic network over (key, input index) in shared memory, padded to a power of
+// two with keys above every 63-bit key.  A fixed grid that reads the list length
+// on the device (graph-stable).
+__global__ void __launch_bounds__(kBigThreads) bucket_big_kernel(const int *__restrict__ big,
+                                                                 const int *__restrict__ boff,
+                                                                 const unsigned long long *__restrict__ bkeys,
+                                                                 const int *__restrict__ bidx,
+                                                                 unsigned long long *__restrict__ okeys,
+                                                                 int *__restrict__ oidx) {
+    extern __shared__ unsigned long long sk[];
+    int *si = reinterpret_cast<int *>(sk + kBigCap);
+    const int nbig = min(big[0], kBigList);
+    for (int q = blockIdx.x; q < nbig; q += gridDim.x) {
+        const int b = big[1 + q], o = boff[b], cnt = boff[b + 1] - o;
+        if (cnt > kBigCap) continue;                          // flagged: the caller sorts in full
+        int P = 1;
+        while (P < cnt) P <<= 1;
+        for (int e = threadIdx.x; e < P; e += blockDim.x) {
+            sk[e] = e < cnt ? bkeys[o + e] : ~0ull;
+            si[e] = e < cnt ? bidx[o + e] : 0x7fffffff;
+        }
+        __syncthreads();
+        for (int k = 2; k <= P; k <<= 1)
+            for (int j = k >> 1; j > 0; j >>= 1) {
+                for (int e = threadIdx.x; e < P; e += blockDim.x) {
+                    const int pe = e ^ j;
+                    if (pe > e) {
+                        const bool up = (e & k) == 0;
+                        const unsigned long long ka = sk[e], kb = sk[pe];
+                        const int ia = si[e], ib = si[pe];
+                        if (pair_gt(ka, ia, kb, ib) == up) {
+                            sk[e] = kb;
+                            sk[pe] = ka;
+                            si[e] = ib;
+                            si[pe] = ia;
+                        }
+                    }
+                }
+                __syncthreads();
+            }
+        for (int e = threadIdx.x; e < cnt; e += blockDim.x) {
+            okeys[o + e] = sk[e];
+            oidx[o + e] = si[e];
+        }
+        __syncthreads();
+    }
 }
 
 // Internal nodes of the previous build, for Enforce_S: per level, node prefixes
@@ -721,17 +779,21 @@ __device__ __forceinline__ int dir_rmq(const signed char *X, const signed char *
 
 __global__ void __launch_bounds__(kDirThreads) leaf_level_kernel(long long n, const unsigned long long *__restrict__ keys,
                                                                  int S, int mode, PrevTree pv,
-                                                                 const int *__restrict__ pv_levels,
+                                                                 const int *__restrict__ pv_levels, Edits ed,
+                                                                 const int *__restrict__ hint_bucket,
+                                                                 const int *__restrict__ hint_perm,
+                                                                 const int *__restrict__ hint_ll,
                                                                  unsigned char *__restrict__ lvl, int *__restrict__ flag) {
-    if (pv_levels) pv.levels = mode == kModeEnforce ? *pv_levels : 0;   // the previous build's (device word)
+    if (pv_levels) pv.levels = mode != kModeFresh ? *pv_levels : 0;    // the previous build's (device word)
     // array 0 = windows of S + 1 (w), 1 = windows of S (v, Enforce_S only); position a <->
-    // window start j = t0 - S + a; -1 = no such window
+    // window start j = t0 - S + a; -1 = no such window.  KEEP needs no counts: no windows.
     __shared__ signed char X[2][kDirLen], P[2][kDirLen], Q[2][kDirLen];
     __shared__ signed char ST[2][kDirST][kDirNB];
+    const bool keep = mode == kModeKeep;
     const bool enf = mode == kModeEnforce && pv.levels > 0;
-    const int na = enf ? 2 : 1;
+    const int na = keep ? 0 : enf ? 2 : 1;
     const long long t0 = (long long)blockIdx.x * kDirTile;
-    const int len = kDirTile + S, nb = (len + 31) >> 5;
+    const int len = keep ? 0 : kDirTile + S, nb = (len + 31) >> 5;
     for (int a = threadIdx.x; a < nb * 32; a += blockDim.x) {
         const long long j = t0 - S + a;
         signed char w = -1, v = -1;
@@ -773,13 +835,40 @@ __global__ void __launch_bounds__(kDirThreads) leaf_level_kernel(long long n, co
         const long long i = t0 + a0;
         if (i >= n) break;
         // windows of S + 1 containing i: j in [i - S, i] -> a in [a0, a0 + S]
-        const int m1 = dir_rmq(X[0], P[0], Q[0], ST[0], a0, a0 + S);
         const unsigned long long ki = keys[i];
-        int l = m1 < 0 ? 0 : min(m1 + 1, kMaxLevel);
-        if (enf && l < kMaxLevel) {
-            // windows of S containing i: j in [i - S + 1, i] -> a in [a0 + 1, a0 + S]
-            const int m2 = dir_rmq(X[1], P[1], Q[1], ST[1], a0 + 1, a0 + S);
-            while (l < kMaxLevel && l <= m2 && prev_internal(pv, l, ki >> (3 * (kMaxLevel - l)))) ++l;
+        int l;
+        if (keep && hint_bucket && (hint_bucket[hint_perm[i]] & 1)) {
+            // KEEP, body still inside previous leaf j's cell (bucket 2j + 1 of the sort):
+            // its path's nodes above that leaf were parents, the leaf was not
+            l = hint_ll[hint_bucket[hint_perm[i]] >> 1];
+        } else if (keep) {
+            // KEEP: the node on i's path at level l splits iff it was a parent before -- true
+            // down to some level and false below (a parent's parent is a parent): bisect for
+            // the first level that was not
+            int lo = 0, hi = min(pv.levels, kMaxLevel);
+            while (lo < hi) {
+                const int mid = (lo + hi) >> 1;
+                if (prev_internal(pv, mid, ki >> (3 * (kMaxLevel - mid)))) lo = mid + 1;
+                else hi = mid;
+            }
+            l = lo;
+        } else {
+            const int m1 = dir_rmq(X[0], P[0], Q[0], ST[0], a0, a0 + S);
+            l = m1 < 0 ? 0 : min(m1 + 1, kMaxLevel);
+            if (enf && l < kMaxLevel) {
+                // windows of S containing i: j in [i - S + 1, i] -> a in [a0 + 1, a0 + S]
+                const int m2 = dir_rmq(X[1], P[1], Q[1], ST[1], a0 + 1, a0 + S);
+                while (l < kMaxLevel && l <= m2 && prev_internal(pv, l, ki >> (3 * (kMaxLevel - l)))) ++l;
+            }
+        }
+        if (ed.n > 0) {
+            // FineGrainedOptimize's edits on top (node_splits' override): above the rule's
+            // leaf level l0 a Collapse stops the path, from l0 on a PushDown continues it
+            const int l0 = l;
+            for (l = 0; l < kMaxLevel; ++l) {
+                const int a = edit_of(ed, l, ki >> (3 * (kMaxLevel - l)));
+                if (a == 1 || (l >= l0 && a != 2)) break;
+            }
         }
         lvl[i] = (unsigned char)l;
         flag[i] = (i == 0 || lcp_digits(keys[i - 1], ki) < l) ? 1 : 0;
@@ -1364,9 +1453,13 @@ struct afmm_tree {
     int *d_state = nullptr;
     DirCtl *h_ctl = nullptr;         // pinned readback of the direct build
     unsigned long long ws_gen = 0;   // bumped whenever a workspace buffer is reallocated (graph key)
-    cudaGraphExec_t tg_exec[2] = {nullptr, nullptr};   // captured direct builds (two alternating input sets)
-    GraphKey tg_key[2] = {};
-    int tg_next = 0;
+    static constexpr int kSlots = 4;                   // captured direct builds (the C5 loop alternates two input
+    cudaGraphExec_t tg_exec[kSlots] = {};              // sets; the LB loop also alternates modes)
+    GraphKey tg_key[kSlots] = {};
+    long long tg_used[kSlots] = {};                    // last use (LRU replacement)
+    GraphKey tg_seen[kSlots] = {};                     // keys of recent uncaptured builds: capture on a key's 2nd use
+    int tg_seen_next = 0;
+    long long tg_clock = 0;
     bool graph_broken = false;
     long long graph_launches = 0;
     long long dir_leaf_cap = 0;      // direct build: leaf / U-list entry capacities (grow-only, checked on the
@@ -1435,7 +1528,7 @@ enum Slot {
     kScanTmp, kFlag, kLeafAt, kNodeLeaf, kScan2, kLs, kLc, kLl, kLp, kLeafNode, kCounts, kUoff, kScan3, kUidx,
     kFarfield, kEditPrefix, kEditAction, kEditBase, kURows, kUOvf, kLvlCtl, kTsum, kAnc,
     kCellLo, kCellHi, kBucket, kSlot, kBCount, kBOff, kBKeys, kBIdx, kBScan, kBOvf,
-    kDirLvl, kDirFk, kDirLlo, kDirChunkCnt, kDirChunkBase, kDirLevelCnt, kDirCtl, kDirRank
+    kDirLvl, kDirFk, kDirLlo, kDirChunkCnt, kDirChunkBase, kDirLevelCnt, kDirCtl, kDirRank, kBBig
 };
 
 __global__ void root_kernel(Nodes nd, int n) {
@@ -1573,7 +1666,7 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     const char *lv_env = getenv("AFMM_TREE_LEVELS");                 // tests / A-B: force the level loop
     const char *dfs_env = getenv("AFMM_ULIST_DFS");                  // tests: force the DFS U-list fallback
     const char *gr_env = getenv("AFMM_TREE_GRAPH");                  // 0: no CUDA graph for the direct build
-    const bool direct = mode != kModeKeep && ed.n == 0 && S <= kDirMaxS && !(lv_env && lv_env[0] == '1');
+    const bool direct = (mode == kModeKeep || S <= kDirMaxS) && !(lv_env && lv_env[0] == '1');
     if (direct) {
         const char *small_env = getenv("AFMM_TREE_SMALL_CAPS");        // tests: start every capacity tiny
         const bool small = small_env && small_env[0] == '1';
@@ -1587,6 +1680,7 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     int *bovf = nullptr;
     unsigned long long *b_clo = nullptr, *b_chi = nullptr, *b_keys = nullptr;
     int *b_bucket = nullptr, *b_slot = nullptr, *b_count = nullptr, *b_off = nullptr, *b_idx = nullptr;
+    int *b_big = nullptr;
     char *b_sbuf = nullptr;
     size_t b_sb = 0;
     int kb_grid = 0;
@@ -1601,6 +1695,8 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
         if (afmm_status s = wsalloc(t, kBKeys, &b_keys, n)) return s;
         if (afmm_status s = wsalloc(t, kBIdx, &b_idx, n)) return s;
         if (afmm_status s = wsalloc(t, kBOvf, &bovf, 1)) return s;
+        if (afmm_status s = wsalloc(t, kBBig, &b_big, 1 + kBigList)) return s;
+        TCU(t, cudaFuncSetAttribute(bucket_big_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBigSmem));
         TCU(t, cub::DeviceScan::ExclusiveSum(nullptr, b_sb, b_count, b_off, (int)(nbcap + 1), st));
         if (afmm_status s = wsalloc(t, kBScan, &b_sbuf, b_sb)) return s;
         int dev_sms = 0;
@@ -1611,6 +1707,7 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     auto enq_buckets = [&]() -> afmm_status {
         TCU(t, cudaMemsetAsync(b_count, 0, ((size_t)nbcap + 1) * sizeof(int), st));
         TCU(t, cudaMemsetAsync(bovf, 0, sizeof(int), st));
+        TCU(t, cudaMemsetAsync(b_big, 0, sizeof(int), st));
         cell_range_kernel<<<grid_for(bcap, TH), TH, 0, st>>>(t->d_state, t->ll, t->lp, b_clo, b_chi);
         keys_bucket_kernel<<<kb_grid, kKeysThreads, 0, st>>>(n, x, y, z, t->lo[0], t->lo[1], t->lo[2], scale, keys,
                                                              t->d_state, b_clo, b_chi, b_bucket, b_slot, b_count);
@@ -1618,7 +1715,9 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
         TCU(t, cub::DeviceScan::ExclusiveSum(b_sbuf, sb, b_count, b_off, (int)(nbcap + 1), st));
         bucket_scatter_kernel<<<grid_for(n, TH), TH, 0, st>>>(n, keys, b_bucket, b_slot, b_off, b_keys, b_idx);
         bucket_sort_kernel<<<(int)((nbcap + kBucketWarps - 1) / kBucketWarps), 32 * kBucketWarps, 0, st>>>(
-            t->d_state, b_off, b_keys, b_idx, t->keys_sorted, t->perm, bovf);
+            t->d_state, b_off, b_keys, b_idx, t->keys_sorted, t->perm, bovf, b_big);
+        bucket_big_kernel<<<kBigList / 2, kBigThreads, kBigSmem, st>>>(b_big, b_off, b_keys, b_idx, t->keys_sorted,
+                                                                      t->perm);
         TCU(t, cudaGetLastError());
         return AFMM_OK;
     };
@@ -1731,11 +1830,15 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
             TCU(t, cudaMalloc(&t->pv_base, (kMaxLevel + 2) * sizeof(long long)));
             ++t->ws_gen;
         }
+        // KEEP after the bucket sort: a body's bucket names the previous leaf it stayed in, whose
+        // level (t->ll, still the previous build's on a first attempt only) is its leaf level
+        const bool hints = mode == kModeKeep && use_buckets && attempt == 0;
         auto enq_direct = [&]() -> afmm_status {
             TCU(t, cudaMemsetAsync(dctl, 0, sizeof(DirCtl), st));
             if (use_buckets) TCU(t, cudaMemcpyAsync(&dctl->sort_overflow, bovf, sizeof(int), cudaMemcpyDeviceToDevice, st));
             leaf_level_kernel<<<(int)((n + kDirTile - 1) / kDirTile), kDirThreads, 0, st>>>(
-                n, t->keys_sorted, S, mode, pv, t->d_state + 1, lvl, flag);
+                n, t->keys_sorted, S, mode, pv, t->d_state + 1, ed, hints ? b_bucket : nullptr, t->perm, t->ll,
+                lvl, flag);
             TCU(t, cudaGetLastError());
             size_t sb = sb2;
             TCU(t, cub::DeviceScan::ExclusiveSum(sbuf2, sb, flag, leaf_at, (int)(n + 1), st));
@@ -1763,16 +1866,21 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
             TCU(t, cudaMemcpyAsync(t->h_ctl, dctl, sizeof(DirCtl), cudaMemcpyDeviceToHost, st));
             return AFMM_OK;
         };
-        const bool graph = use_buckets && !(gr_env && gr_env[0] == '0') && !t->graph_broken;
+        // not with edits: FineGrainedOptimize's trial rebuilds are one-offs (a capture each would cost more)
+        const bool graph = use_buckets && ed.n == 0 && !(gr_env && gr_env[0] == '0') && !t->graph_broken;
         if (graph) {
             const GraphKey key{x, y, z, n, S, mode, t->ws_gen, cap, (long long)lcap, t->dir_nnz_cap,
                                {t->lo[0], t->lo[1], t->lo[2]}, t->k};
             int slot = -1;
-            for (int g = 0; g < 2; ++g)
+            for (int g = 0; g < afmm_tree::kSlots; ++g)
                 if (t->tg_exec[g] && t->tg_key[g] == key) slot = g;
-            if (slot < 0) {                           // capture (the C5 loop alternates two state buffers: 2 slots)
-                slot = t->tg_next;
-                t->tg_next ^= 1;
+            bool seen = false;                        // a key used once (a Search step's S) is not worth a capture
+            for (int g = 0; g < afmm_tree::kSlots; ++g) seen |= t->tg_seen[g] == key;
+            if (slot < 0 && !seen) t->tg_seen[t->tg_seen_next++ % afmm_tree::kSlots] = key;
+            if (slot < 0 && seen) {                   // capture into the least recently used slot
+                slot = 0;
+                for (int g = 1; g < afmm_tree::kSlots; ++g)
+                    if (t->tg_used[g] < t->tg_used[slot]) slot = g;
                 if (t->tg_exec[slot]) cudaGraphExecDestroy(t->tg_exec[slot]);
                 t->tg_exec[slot] = nullptr;
                 cudaGraph_t gph = nullptr;
@@ -1794,7 +1902,8 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
                     t->tg_key[slot] = key;
                 }
             }
-            if (t->tg_exec[slot]) {
+            if (slot >= 0 && t->tg_exec[slot]) {
+                t->tg_used[slot] = ++t->tg_clock;
                 TCU(t, cudaGraphLaunch(t->tg_exec[slot], st));
                 ++t->graph_launches;
             } else {

@@ -271,10 +271,92 @@ def test_enforce_graph_replay_matches_direct_launches(monkeypatch):
             To = To2
         res[flag] = (out, t.counters())
         t.close()
-    assert res["1"][1]["graph_launches"] >= 6 and res["0"][1]["graph_launches"] == 0
+    # a key is captured on its second use (steps 0, 1 launch directly; 2..6 replay or capture + replay)
+    assert res["1"][1]["graph_launches"] >= 5 and res["0"][1]["graph_launches"] == 0
     for step, (a, b) in enumerate(zip(res["1"][0], res["0"][0])):
         for k in a:
             assert np.array_equal(np.asarray(a[k]), np.asarray(b[k])), (step, k)
+
+
+def _edits_for(t, rng, frac=0.1):
+    """A seeded set of FineGrainedOptimize edits on the handle's current nodes:
+    Collapse on some parents, PushDown on some leaves (incl. a level-21 cap case)."""
+    nd = t.nodes()
+    lev, pre, nch = nd["level"], nd["prefix"], nd["nchild"]
+    pick = rng.random(lev.shape[0]) < frac
+    return [(int(l), int(p), 1 if c > 0 else 2) for l, p, c, k in zip(lev, pre, nch, pick) if k]
+
+
+def test_direct_keep_and_edits_match_level_loop(monkeypatch):
+    """afmm_tree_rebuild (KEEP structure, or Enforce_S, with FineGrainedOptimize's
+    Collapse / PushDown edits) through the direct construction -- per-body leaf level
+    by bisection over the previous parents, edits applied along the path -- equals the
+    level loop (AFMM_TREE_LEVELS=1) tree and node arrays, with and without CUDA graph
+    replay, and the oracle's rebuild."""
+    afmm = _afmm()
+    x, y, z, m, vx, vy, vz = synth.colliding_with_velocities(30000, 8)
+    dom = synth.c5_domain(x, y, z)
+    n = x.shape[0]
+    plan = [(2, 0.0), (2, 0.0), (2, 0.1), (1, 0.05), (2, 0.0), (1, 0.0), (2, 0.2), (2, 0.2), (1, 0.1)]
+    res = {}
+    for levels, graph in (("0", "1"), ("0", "0"), ("1", "0")):
+        monkeypatch.setenv("AFMM_TREE_LEVELS", levels)
+        monkeypatch.setenv("AFMM_TREE_GRAPH", graph)
+        rng = np.random.default_rng(11)
+        t = afmm.GpuTree(0)
+        bufs = [torch.empty((3, n), device="cuda") for _ in range(2)]
+        S = 20
+        t.build(_dev(x), _dev(y), _dev(z), S, domain=dom)
+        To = oracle.Tree(x, y, z, S, domain=dom, ulist=False)
+        px, py, pz, qx, qy, qz = (a[To.perm] for a in (x, y, z, vx, vy, vz))
+        out = []
+        for step, (mode, frac) in enumerate(plan):
+            px, py, pz = oracle.drift(px, py, pz, qx, qy, qz, 0.2)
+            ed = _edits_for(t, rng, frac) if frac > 0 else []
+            b = bufs[step % 2]
+            b.copy_(torch.from_numpy(np.stack([px, py, pz])))
+            t.rebuild(b[0], b[1], b[2], S, mode=mode, edits=ed)
+            G = _tree_and_nodes(t, n)
+            To2 = To.rebuild(px, py, pz, S=S, mode=mode, edits=ed, ulist=False)
+            for k in ("perm", "leaf_start", "leaf_count", "leaf_level", "leaf_prefix"):
+                assert np.array_equal(G[k], getattr(To2, k)), (levels, graph, step, k)
+            out.append(G)
+            px, py, pz, qx, qy, qz = (a[To2.perm] for a in (px, py, pz, qx, qy, qz))
+            To = To2
+        res[levels + graph] = out
+        t.close()
+    for other in ("00", "10"):
+        for step, (a, b) in enumerate(zip(res["01"], res[other])):
+            for k in a:
+                assert np.array_equal(np.asarray(a[k]), np.asarray(b[k])), (other, step, k)
+
+
+@pytest.mark.parametrize("S,fallback", [(600, False), (3000, False), (20000, True)])
+def test_large_buckets_cta_sort(S, fallback):
+    """Rebuilds whose previous leaves hold more than the warp sort's 512 keys: buckets
+    of up to 8192 keys are sorted by one CTA each in shared memory (no full-sort
+    fallback), larger ones fall back to the full sort -- the tree bit-exact with the
+    oracle's Enforce_S chain either way."""
+    afmm = _afmm()
+    x, y, z, m, vx, vy, vz = synth.colliding_with_velocities(60000, 4)
+    dom = synth.c5_domain(x, y, z)
+    n = x.shape[0]
+    t = afmm.GpuTree(0)
+    t.build(_dev(x), _dev(y), _dev(z), S, domain=dom)
+    To = oracle.Tree(x, y, z, S, domain=dom, ulist=False)
+    assert To.leaf_count.max() > 512
+    px, py, pz, qx, qy, qz = (a[To.perm] for a in (x, y, z, vx, vy, vz))
+    for step in range(3):
+        px, py, pz = oracle.drift(px, py, pz, qx, qy, qz, 0.2)
+        t.enforce(_dev(px), _dev(py), _dev(pz), S)
+        To2 = To.enforce(px, py, pz, S, ulist=False)
+        G = t.copy_out(n)
+        for k in ("perm", "leaf_start", "leaf_count", "leaf_level", "leaf_prefix"):
+            assert np.array_equal(G[k], getattr(To2, k)), (S, step, k)
+        px, py, pz, qx, qy, qz = (a[To2.perm] for a in (px, py, pz, qx, qy, qz))
+        To = To2
+    assert (t.counters()["sort_fallbacks"] > 0) == fallback
+    t.close()
 
 
 def test_randomised_builds_and_enforce_chains_bit_exact():

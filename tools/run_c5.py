@@ -97,7 +97,7 @@ print(json.dumps({
     **({"lb": {"cpu_coef": list(map(float, loop.cpu_coef)),
                "trajectory": [{k: (round(v, 7) if isinstance(v, float) else v) for k, v in r.items()
                                if k in ("step", "S", "action", "lb_state", "t_cpu_model", "t_gpu", "compute",
-                                        "n_leaves", "lb_ms", "step_ms")} for r in L],
+                                        "n_leaves", "lb_ms", "step_ms", "enforce_ms")} for r in L],
                "fine": [dict(step=r["step"], **r["fine"]) for r in L if "fine" in r],
                "compute_ms_by_quarter": [round(1e3 * float(np.mean([r["compute"] for r in
                                                                     L[q * len(L) // 4:(q + 1) * len(L) // 4]])), 4)
