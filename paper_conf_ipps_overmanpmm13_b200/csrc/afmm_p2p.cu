@@ -816,10 +816,20 @@ __global__ void collect_kernel(int L, int W, int r, const long long *__restrict_
     }
     *nt_eff = (e || ov) ? 0 : (int)nt;                      // gates write_kernel and the sort
 }
-// the U-list indices into the handle's own buffer (capacity cap; nnz = uo[L] on the device)
+// the tree into the handle's own buffers: leaf arrays, and the U-list indices (capacity
+// cap; nnz = uo[L] on the device)
 __global__ void copy_ui_kernel(int L, const long long *__restrict__ uo, const int *__restrict__ src,
                                int *__restrict__ dst, long long cap, const int *__restrict__ err,
-                               long long *__restrict__ rb) {
+                               long long *__restrict__ rb, const int *__restrict__ ls, const int *__restrict__ lc,
+                               int *__restrict__ ols, int *__restrict__ olc, long long *__restrict__ ouo) {
+    const long long g0 = blockIdx.x * (long long)blockDim.x + threadIdx.x, gs = (long long)gridDim.x * blockDim.x;
+    for (long long i = g0; i <= L; i += gs) {               // the leaf arrays too (one kernel, not three copies)
+        if (i < L) {
+            ols[i] = ls[i];
+            olc[i] = lc[i];
+        }
+        ouo[i] = uo[i];
+    }
     if (*err) return;
     const long long nnz = uo[L];
     if (nnz > cap) {
@@ -962,22 +972,19 @@ static afmm_status ingest(afmm_p2p *h, int n_leaves, const int *leaf_start, cons
     };
     if ((st = write_lists())) return st;
     // 5. the handle's own copy of the tree (set_partition / rebalance re-ingest it)
-    int *oui = nullptr;
+    int *oui = nullptr, *ols = nullptr, *olc = nullptr;
+    long long *ouo = nullptr;
     auto copy_ui = [&](size_t cap) -> afmm_status {
         if (afmm_status s2 = dws(h, sOwnUI, &oui, cap)) return s2;
-        dev_ingest::copy_ui_kernel<<<h->num_sms * 4, TH, 0, s>>>(L, u_off, u_idx, oui, (long long)cap, err, rb);
+        dev_ingest::copy_ui_kernel<<<h->num_sms * 4, TH, 0, s>>>(L, u_off, u_idx, oui, (long long)cap, err, rb,
+                                                                 leaf_start, leaf_count, ols, olc, ouo);
         COUNT_LAUNCH(1);
         CUDA_TRY(h, cudaGetLastError());
         return AFMM_OK;
     };
     if (keep) {
-        int *ols, *olc;
-        long long *ouo;
         if ((st = dws(h, sOwnLS, &ols, L)) || (st = dws(h, sOwnLC, &olc, L)) || (st = dws(h, sOwnUO, &ouo, L + 1)))
             return st;
-        CUDA_TRY(h, cudaMemcpyAsync(ols, leaf_start, L * sizeof(int), cudaMemcpyDeviceToDevice, s));
-        CUDA_TRY(h, cudaMemcpyAsync(olc, leaf_count, L * sizeof(int), cudaMemcpyDeviceToDevice, s));
-        CUDA_TRY(h, cudaMemcpyAsync(ouo, u_off, (L + 1) * sizeof(long long), cudaMemcpyDeviceToDevice, s));
         const size_t have = slot_capacity(h, sOwnUI) / sizeof(int);
         if ((st = copy_ui(std::max<size_t>(have, (size_t)32 * L)))) return st;
     }
