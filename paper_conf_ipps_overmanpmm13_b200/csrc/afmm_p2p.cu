@@ -772,7 +772,7 @@ __global__ void body_split_kernel(int G, int L, long long n, const long long *__
     if (r <= G) bsplit[r] = split[r] >= L ? n : ls[split[r]];
 }
 
-enum DwsSlot { sI, sP, sW, sPW, sSplit, sErr, sNseg, sNtask, sNsrc, sSegOff, sTaskOff, sStats, sKeys, sVals, sKeys2,
+enum DwsSlot { sI, sP, sW, sPW, sSplit, sErr, sNseg, sNsrc, sSegOff, sStats, sKeys, sVals, sKeys2,
                sVals2, sTasksU, sCoef, sTmp, sBsplit, sPlan, sPlanHdr, sNnz,
                sOwnLS, sOwnLC, sOwnUO, sOwnUI,               // the handle's own copy of the tree (re-ingest)
                sSortStat, sSortCtl, sNsegAll, sNsrcAll, sRb, sNtEff };              // task_sort_kernel's digit totals, status words, barrier
@@ -794,14 +794,14 @@ enum : long long { kOvSegs = 1, kOvTasks = 2, kOvOwnUI = 4 };
 namespace dev_ingest {
 __global__ void collect_kernel(int L, int W, int r, const long long *__restrict__ split,
                                const long long *__restrict__ bsplit, const long long *__restrict__ P,
-                               const long long *__restrict__ uo, const int *__restrict__ seg_off,
-                               const int *__restrict__ task_off, const unsigned long long *__restrict__ stats,
+                               const long long *__restrict__ uo, const unsigned long long *__restrict__ off2,
+                               const unsigned long long *__restrict__ stats,
                                const int *__restrict__ err, long long segs_cap, long long tasks_cap,
                                long long *__restrict__ rb, int *__restrict__ nt_eff) {
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
     const int e = *err;
     const long long m = split[r + 1] - split[r];
-    const long long nsegs = e ? 0 : seg_off[m], nt = e ? 0 : task_off[m];
+    const long long nsegs = e ? 0 : (long long)(unsigned)off2[m], nt = e ? 0 : (long long)(off2[m] >> 32);
     const long long ov = (nsegs > segs_cap ? kOvSegs : 0) | (nt > tasks_cap ? kOvTasks : 0);
     rb[rbErr] = e;
     rb[rbOverflow] = ov;
@@ -851,15 +851,15 @@ static afmm_status ingest(afmm_p2p *h, int n_leaves, const int *leaf_start, cons
     long long *I, *P, *split, *nsrc, *bsplit, *nsrc_all, *rb;
     unsigned short *plan;
     int4 *plan_hdr;
-    int *err, *nseg, *ntask, *seg_off, *task_off, *nseg_all, *nt_eff;
+    int *err, *nseg_all, *nt_eff;
+    unsigned long long *nst, *off2;
     unsigned long long *stats;
     const size_t rb_len = (size_t)rbSplit + 2 * (W + 1);
     if ((st = dws(h, sI, &I, L)) || (st = dws(h, sP, &P, L)) || (st = dws(h, sSplit, &split, W + 1)) ||
         (st = dws(h, sErr, &err, 1)) || (st = dws(h, sBsplit, &bsplit, W + 1)) ||
         (st = dws(h, sNsegAll, &nseg_all, L)) || (st = dws(h, sNsrcAll, &nsrc_all, L)) ||
-        (st = dws(h, sNseg, &nseg, (size_t)L + 1)) || (st = dws(h, sNtask, &ntask, (size_t)L + 1)) ||
-        (st = dws(h, sNsrc, &nsrc, (size_t)L + 1)) || (st = dws(h, sSegOff, &seg_off, (size_t)L + 1)) ||
-        (st = dws(h, sTaskOff, &task_off, (size_t)L + 1)) || (st = dws(h, sStats, &stats, 10)) ||
+        (st = dws(h, sNseg, &nst, (size_t)L + 1)) || (st = dws(h, sNsrc, &nsrc, (size_t)L + 1)) ||
+        (st = dws(h, sSegOff, &off2, (size_t)L + 1)) || (st = dws(h, sStats, &stats, 10)) ||
         (st = dws(h, sPlan, &plan, (size_t)(L + 1) * afmm::kMaxDpSlices)) ||
         (st = dws(h, sPlanHdr, &plan_hdr, (size_t)L + 1)) || (st = dws(h, sRb, &rb, rb_len)) ||
         (st = dws(h, sNtEff, &nt_eff, 1)))
@@ -916,17 +916,16 @@ static afmm_status ingest(afmm_p2p *h, int n_leaves, const int *leaf_start, cons
     // 3. this rank's segment / slice counts (leaves split[r] .. split[r+1], read on the device)
     dev::count_kernel<<<grid((long long)L + 1), TH, 0, s>>>(L, r, split, P, slice_world(h),
                                                            (long long)h->num_sms * h->blocks_per_sm * afmm::kWarps,
-                                                           err, leaf_count, nseg_all, nsrc_all, I, nseg, ntask, nsrc,
+                                                           err, leaf_count, nseg_all, nsrc_all, I, nst, nsrc,
                                                            stats, plan, plan_hdr);
     COUNT_LAUNCH(1);
     CUDA_TRY(h, cudaGetLastError());
     {
         size_t tb = 0;
-        CUDA_TRY(h, cub::DeviceScan::ExclusiveSum(nullptr, tb, nseg, seg_off, L + 1, s));
+        CUDA_TRY(h, cub::DeviceScan::ExclusiveSum(nullptr, tb, nst, off2, L + 1, s));
         char *tmp;
         if ((st = dws(h, sTmp, &tmp, tb))) return st;
-        CUDA_TRY(h, cub::DeviceScan::ExclusiveSum(tmp, tb, nseg, seg_off, L + 1, s));
-        CUDA_TRY(h, cub::DeviceScan::ExclusiveSum(tmp, tb, ntask, task_off, L + 1, s));
+        CUDA_TRY(h, cub::DeviceScan::ExclusiveSum(tmp, tb, nst, off2, L + 1, s));   // segment | task offsets
     }
     // 4. the lists, into the current capacities (a first guess from L when there are none)
     if ((st = ensure_device(h, &h->d_segs, h->segs_cap, std::max<size_t>(h->segs_cap, (size_t)12 * L))) ||
@@ -942,11 +941,11 @@ static afmm_status ingest(afmm_p2p *h, int n_leaves, const int *leaf_start, cons
             (s2 = dws(h, sVals, &vals, tcap)) || (s2 = dws(h, sKeys2, &keys2, tcap)) ||
             (s2 = dws(h, sVals2, &vals2, tcap)))
             return s2;
-        dev_ingest::collect_kernel<<<1, 1, 0, s>>>(L, W, r, split, bsplit, P, u_off, seg_off, task_off, stats, err,
+        dev_ingest::collect_kernel<<<1, 1, 0, s>>>(L, W, r, split, bsplit, P, u_off, off2, stats, err,
                                                    (long long)h->segs_cap, (long long)tcap, rb, nt_eff);
         COUNT_LAUNCH(1);
         dev::write_kernel<<<grid(32LL * L), TH, 0, s>>>(r, split, nt_eff, leaf_start, leaf_count, u_off, u_idx,
-                                                       seg_off, task_off, nsrc, h->d_segs, tasks_u, keys, vals, plan,
+                                                       off2, nsrc, h->d_segs, tasks_u, keys, vals, plan,
                                                        plan_hdr, stats + 9);
         COUNT_LAUNCH(1);
         CUDA_TRY(h, cudaGetLastError());

@@ -145,29 +145,26 @@ __global__ void weighted_cut_kernel(int L, int G, const double *__restrict__ P, 
 __global__ void count_kernel(int L, int r, const long long *__restrict__ split, const long long *__restrict__ P,
                              int sw, long long warps, const int *__restrict__ err, const int *__restrict__ lc,
                              const int *__restrict__ nseg_all, const long long *__restrict__ nsrc_all,
-                             const long long *__restrict__ I, int *__restrict__ nseg, int *__restrict__ ntask,
+                             const long long *__restrict__ I, unsigned long long *__restrict__ nst,
                              long long *__restrict__ nsrc, unsigned long long *__restrict__ stats,
                              unsigned short *__restrict__ plan, int4 *__restrict__ plan_hdr) {
     if (*err) return;
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     const int lo = (int)split[r], m = (int)(split[r + 1] - split[r]);
     const long long cap = task_cap(P[L - 1] / sw, warps);
-    if (i >= m && i <= L) {
-        nseg[i] = 0;
-        ntask[i] = 0;
-    }
+    if (i >= m && i <= L) nst[i] = 0;
     const bool live = i < m;
     unsigned long long inter = 0, cm = 0;
     int bk = -1;
     if (live) {
         const int t = lo + i;
         const long long src = nsrc_all[t];
-        nseg[i] = nseg_all[t];
         nsrc[i] = src;
         int n_full = 0, full_m = 0, max_m = 0;
         const int k = plan_slices(lc[t], src, cap, &n_full, &full_m, plan + (size_t)i * kMaxDpSlices, &max_m);
         plan_hdr[i] = make_int4(n_full, full_m, k, 0);
-        ntask[i] = n_full + k;
+        // segment and task counts packed (tasks << 32 | segments): one scan gives both offsets
+        nst[i] = (unsigned long long)(n_full + k) << 32 | (unsigned)nseg_all[t];
         inter = (unsigned long long)I[t];
         bk = bucket_of_d(lc[t]);
         cm = (unsigned long long)slice_iters(src, max_m);    // the largest slice has the largest cost
@@ -197,7 +194,7 @@ __global__ void count_kernel(int L, int r, const long long *__restrict__ split, 
 __global__ void write_kernel(int r, const long long *__restrict__ split, const int *__restrict__ gate,
                              const int *__restrict__ ls, const int *__restrict__ lc,
                              const long long *__restrict__ uo, const int *__restrict__ ui,
-                             const int *__restrict__ seg_off, const int *__restrict__ task_off,
+                             const unsigned long long *__restrict__ off2,
                              const long long *__restrict__ nsrc, Seg *__restrict__ segs, Task *__restrict__ tasks,
                              unsigned long long *__restrict__ keys, int *__restrict__ vals,
                              const unsigned short *__restrict__ plan, const int4 *__restrict__ plan_hdr,
@@ -208,7 +205,7 @@ __global__ void write_kernel(int r, const long long *__restrict__ split, const i
     if (gw >= m || *gate == 0) return;                        // whole warps; gate: valid and fits
     const int i = (int)gw, t = lo + i;
     const int ts = ls[t], tn = lc[t];
-    const int seg_begin = seg_off[i];
+    const int seg_begin = (int)(unsigned)off2[i], task_begin = (int)(off2[i] >> 32);
     const long long b = uo[t], en = uo[t + 1];
     bool self = false;
     for (long long u = b + lane; u < en; u += 32) self |= ui[u] == t;
@@ -260,7 +257,7 @@ __global__ void write_kernel(int r, const long long *__restrict__ split, const i
             if (lane >= o) inc += v;
         }
         if (j < total) {
-            const int q = task_off[i] + j;
+            const int q = task_begin + j;
             tasks[q] = Task{ts + carry + inc - cnt, cnt, ts, self ? tn : 0, seg_begin, seg_count, (int)src, 0};
             keys[q] = cmax - (unsigned long long)slice_iters(src, cnt);   // ascending = largest cost first
             vals[q] = q;
