@@ -772,7 +772,7 @@ __global__ void body_split_kernel(int G, int L, long long n, const long long *__
     if (r <= G) bsplit[r] = split[r] >= L ? n : ls[split[r]];
 }
 
-enum DwsSlot { sI, sP, sW, sPW, sSplit, sErr, sNseg, sNsrc, sSegOff, sStats, sKeys, sVals, sKeys2,
+enum DwsSlot { sI, sP, sW, sPW, sSplit, sNseg, sNsrc, sSegOff, sStats, sKeys, sVals, sKeys2,
                sVals2, sTasksU, sCoef, sTmp, sBsplit, sPlan, sPlanHdr, sNnz,
                sOwnLS, sOwnLC, sOwnUO, sOwnUI,               // the handle's own copy of the tree (re-ingest)
                sSortStat, sSortCtl, sNsegAll, sNsrcAll, sRb, sNtEff };              // task_sort_kernel's digit totals, status words, barrier
@@ -856,10 +856,10 @@ static afmm_status ingest(afmm_p2p *h, int n_leaves, const int *leaf_start, cons
     unsigned long long *stats;
     const size_t rb_len = (size_t)rbSplit + 2 * (W + 1);
     if ((st = dws(h, sI, &I, L)) || (st = dws(h, sP, &P, L)) || (st = dws(h, sSplit, &split, W + 1)) ||
-        (st = dws(h, sErr, &err, 1)) || (st = dws(h, sBsplit, &bsplit, W + 1)) ||
+        (st = dws(h, sBsplit, &bsplit, W + 1)) ||
         (st = dws(h, sNsegAll, &nseg_all, L)) || (st = dws(h, sNsrcAll, &nsrc_all, L)) ||
         (st = dws(h, sNseg, &nst, (size_t)L + 1)) || (st = dws(h, sNsrc, &nsrc, (size_t)L + 1)) ||
-        (st = dws(h, sSegOff, &off2, (size_t)L + 1)) || (st = dws(h, sStats, &stats, 10)) ||
+        (st = dws(h, sSegOff, &off2, (size_t)L + 1)) || (st = dws(h, sStats, &stats, 11)) ||
         (st = dws(h, sPlan, &plan, (size_t)(L + 1) * afmm::kMaxDpSlices)) ||
         (st = dws(h, sPlanHdr, &plan_hdr, (size_t)L + 1)) || (st = dws(h, sRb, &rb, rb_len)) ||
         (st = dws(h, sNtEff, &nt_eff, 1)))
@@ -872,8 +872,8 @@ static afmm_status ingest(afmm_p2p *h, int n_leaves, const int *leaf_start, cons
         h->h_rb_len = rb_len;
     }
     // 1. validation + Interactions(t) + per-leaf segment counts and source totals
-    CUDA_TRY(h, cudaMemsetAsync(err, 0, sizeof(int), s));
-    CUDA_TRY(h, cudaMemsetAsync(stats, 0, 10 * sizeof(unsigned long long), s));
+    err = reinterpret_cast<int *>(stats + 10);     // the error flags share the stats' reset
+    CUDA_TRY(h, cudaMemsetAsync(stats, 0, 11 * sizeof(unsigned long long), s));
     dev::validate_interactions_kernel<<<grid(32LL * L), TH, 0, s>>>(L, h->n, h->cfg.max_leaf, leaf_start,
                                                                    leaf_count, u_off, u_idx, I, nseg_all, nsrc_all,
                                                                    err);
@@ -888,6 +888,7 @@ static afmm_status ingest(afmm_p2p *h, int n_leaves, const int *leaf_start, cons
         if ((st = dws(h, sTmp, &tmp, tb))) return st;
         CUDA_TRY(h, cub::DeviceScan::InclusiveSum(tmp, tb, I, P, L, s));
     }
+    bool literal = false;
     if (h->user_partition && (long long)h->leaf_split.size() == W + 1 && h->leaf_split[W] == L) {
         CUDA_TRY(h, cudaMemcpyAsync(split, h->leaf_split.data(), (W + 1) * sizeof(long long),
                                     cudaMemcpyHostToDevice, s));
@@ -906,13 +907,16 @@ static afmm_status ingest(afmm_p2p *h, int n_leaves, const int *leaf_start, cons
         COUNT_LAUNCH(1);
         clear_user = true;
     } else {
-        dev::literal_cut_kernel<<<1, 1, 0, s>>>(L, W, P, split);
+        literal = true;
+        dev::literal_cut_kernel<<<1, 1, 0, s>>>(L, W, P, split, h->n, leaf_start, bsplit);   // + the body split
         COUNT_LAUNCH(1);
         clear_user = true;
     }
     CUDA_TRY(h, cudaGetLastError());
-    body_split_kernel<<<(W + 1 + 63) / 64, 64, 0, s>>>(W, L, h->n, split, leaf_start, bsplit);
-    COUNT_LAUNCH(1);
+    if (!literal) {
+        body_split_kernel<<<(W + 1 + 63) / 64, 64, 0, s>>>(W, L, h->n, split, leaf_start, bsplit);
+        COUNT_LAUNCH(1);
+    }
     // 3. this rank's segment / slice counts (leaves split[r] .. split[r+1], read on the device)
     dev::count_kernel<<<grid((long long)L + 1), TH, 0, s>>>(L, r, split, P, slice_world(h),
                                                            (long long)h->num_sms * h->blocks_per_sm * afmm::kWarps,

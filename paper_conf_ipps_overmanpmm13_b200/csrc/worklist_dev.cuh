@@ -88,7 +88,9 @@ __global__ void validate_interactions_kernel(int L, long long n, int max_leaf, c
 // Literal greedy cut (PAPER L16 SIII.C) from the inclusive prefix sums P[t] =
 // sum_{u <= t} I(u): cut r+1 = 1 + first t >= cut_r whose running count
 // P[t] - P[cut_r - 1] satisfies count * G >= total.  Single thread, G <= 64 binary searches.
-__global__ void literal_cut_kernel(int L, int G, const long long *__restrict__ P, long long *__restrict__ split) {
+// (+ the body range of every slice, bsplit[g] = first body of leaf split[g], n past the end)
+__global__ void literal_cut_kernel(int L, int G, const long long *__restrict__ P, long long *__restrict__ split,
+                                   long long n, const int *__restrict__ ls, long long *__restrict__ bsplit) {
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
     const long long total = P[L - 1];
     long long start = 0;
@@ -107,6 +109,7 @@ __global__ void literal_cut_kernel(int L, int G, const long long *__restrict__ P
         split[g + 1] = start;
     }
     for (int r = g + 1; r <= G; ++r) split[r] = L;
+    for (int r = 0; r <= G; ++r) bsplit[r] = split[r] >= L ? n : ls[split[r]];
 }
 
 // The same rule on weights w(t) = I(t) * coef[bucket(n_t)] (prefix sums in fp64).
