@@ -38,7 +38,12 @@ def timed(name, fn):
     t0 = time.perf_counter()
     info = fn()
     torch.cuda.synchronize()
-    print(f"{name:28s} {1e3 * (time.perf_counter() - t0):8.3f} ms  L={info['n_leaves']}  {t.counters()}", flush=True)
+    dt = 1e3 * (time.perf_counter() - t0)
+    t1 = time.perf_counter()
+    c = t.farfield_counts()
+    dc = 1e3 * (time.perf_counter() - t1)
+    print(f"{name:28s} {dt:8.3f} ms  L={info['n_leaves']}  {t.counters()}  farfield_counts {dc:.3f} ms {c.tolist()}",
+          flush=True)
 
 
 timed("build S=128", lambda: t.build(P[0], P[1], P[2], 128, domain=dom))
