@@ -1757,7 +1757,7 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     int level = 0;
     int *cb = nullptr, *nc = nullptr, *off = nullptr;
     bool done_levels = false;
-    // 4d. direct construction from the sorted keys (fresh / Enforce_S, no edits, S <= kDirMaxS):
+    // 4d. direct construction from the sorted keys (fresh / Enforce_S with S <= kDirMaxS; KEEP; edits on either):
     //     leaves, nodes and U-lists by flat kernels that read their sizes on the device,
     //     into grow-only capacities checked on the device; ONE host readback at the end
     //     (sizes + overflow flags; an overflow grows the capacities and reruns, a warp
