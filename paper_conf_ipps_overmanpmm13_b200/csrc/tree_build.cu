@@ -259,7 +259,10 @@ __global__ void __launch_bounds__(32 * kBucketWarps) bucket_sort_kernel(const in
                                                                         unsigned long long *__restrict__ okeys,
                                                                         int *__restrict__ oidx,
                                                                         int *__restrict__ overflow,
-                                                                        int *__restrict__ big) {
+                                                                        int *__restrict__ big,
+                                                                        int *__restrict__ mid) {
+    // buckets of <= 64 keys here (register-light: full occupancy), 65..512 keys listed
+    // for bucket_mid_kernel, larger ones for bucket_big_kernel
     const int lane = threadIdx.x & 31;
     const int nb = 2 * *Ldev + 1;
     const int b = blockIdx.x * kBucketWarps + (threadIdx.x >> 5);
@@ -282,9 +285,23 @@ __global__ void __launch_bounds__(32 * kBucketWarps) bucket_sort_kernel(const in
     }
     if (cnt <= 32) warp_bitonic<1>(o, cnt, bkeys, bidx, okeys, oidx, lane);
     else if (cnt <= 64) warp_bitonic<2>(o, cnt, bkeys, bidx, okeys, oidx, lane);
-    else if (cnt <= 128) warp_bitonic<4>(o, cnt, bkeys, bidx, okeys, oidx, lane);
-    else if (cnt <= 256) warp_bitonic<8>(o, cnt, bkeys, bidx, okeys, oidx, lane);
-    else warp_bitonic<16>(o, cnt, bkeys, bidx, okeys, oidx, lane);
+    else if (lane == 0) mid[1 + atomicAdd(mid, 1)] = b;       // the list holds every bucket if need be
+}
+// The listed buckets of 65..kBucketCap keys, a warp each (a fixed grid striding
+// over the list, its length read on the device).
+__global__ void __launch_bounds__(32 * kBucketWarps) bucket_mid_kernel(const int *__restrict__ mid,
+                                                                       const int *__restrict__ boff,
+                                                                       const unsigned long long *__restrict__ bkeys,
+                                                                       const int *__restrict__ bidx,
+                                                                       unsigned long long *__restrict__ okeys,
+                                                                       int *__restrict__ oidx) {
+    const int lane = threadIdx.x & 31, nmid = *mid;
+    for (int q = blockIdx.x * kBucketWarps + (threadIdx.x >> 5); q < nmid; q += gridDim.x * kBucketWarps) {
+        const int b = mid[1 + q], o = boff[b], cnt = boff[b + 1] - o;
+        if (cnt <= 128) warp_bitonic<4>(o, cnt, bkeys, bidx, okeys, oidx, lane);
+        else if (cnt <= 256) warp_bitonic<8>(o, cnt, bkeys, bidx, okeys, oidx, lane);
+        else warp_bitonic<16>(o, cnt, bkeys, bidx, okeys, oidx, lane);
+    }
 }
 
 // The listed buckets of kBucketCap < count <= kBigCap keys: one CTA per bucket, a
@@ -1532,7 +1549,7 @@ enum Slot {
     kScanTmp, kFlag, kLeafAt, kNodeLeaf, kScan2, kLs, kLc, kLl, kLp, kLeafNode, kCounts, kUoff, kScan3, kUidx,
     kFarfield, kEditPrefix, kEditAction, kEditBase, kURows, kUOvf, kLvlCtl, kTsum, kAnc,
     kCellLo, kCellHi, kBucket, kSlot, kBCount, kBOff, kBKeys, kBIdx, kBScan, kBOvf,
-    kDirLvl, kDirFk, kDirLlo, kDirChunkCnt, kDirChunkBase, kDirLevelCnt, kDirCtl, kDirRank, kBBig
+    kDirLvl, kDirFk, kDirLlo, kDirChunkCnt, kDirChunkBase, kDirLevelCnt, kDirCtl, kDirRank, kBBig, kBMid
 };
 
 __global__ void root_kernel(Nodes nd, int n) {
@@ -1684,7 +1701,7 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
     int *bovf = nullptr;
     unsigned long long *b_clo = nullptr, *b_chi = nullptr, *b_keys = nullptr;
     int *b_bucket = nullptr, *b_slot = nullptr, *b_count = nullptr, *b_off = nullptr, *b_idx = nullptr;
-    int *b_big = nullptr;
+    int *b_big = nullptr, *b_mid = nullptr;
     char *b_sbuf = nullptr;
     size_t b_sb = 0;
     int kb_grid = 0;
@@ -1700,6 +1717,7 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
         if (afmm_status s = wsalloc(t, kBIdx, &b_idx, n)) return s;
         if (afmm_status s = wsalloc(t, kBOvf, &bovf, 1)) return s;
         if (afmm_status s = wsalloc(t, kBBig, &b_big, 1 + kBigList)) return s;
+        if (afmm_status s = wsalloc(t, kBMid, &b_mid, (size_t)nbcap + 1)) return s;
         TCU(t, cudaFuncSetAttribute(bucket_big_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBigSmem));
         TCU(t, cub::DeviceScan::ExclusiveSum(nullptr, b_sb, b_count, b_off, (int)(nbcap + 1), st));
         if (afmm_status s = wsalloc(t, kBScan, &b_sbuf, b_sb)) return s;
@@ -1712,6 +1730,7 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
         TCU(t, cudaMemsetAsync(b_count, 0, ((size_t)nbcap + 1) * sizeof(int), st));
         TCU(t, cudaMemsetAsync(bovf, 0, sizeof(int), st));
         TCU(t, cudaMemsetAsync(b_big, 0, sizeof(int), st));
+        TCU(t, cudaMemsetAsync(b_mid, 0, sizeof(int), st));
         cell_range_kernel<<<grid_for(bcap, TH), TH, 0, st>>>(t->d_state, t->ll, t->lp, b_clo, b_chi);
         keys_bucket_kernel<<<kb_grid, kKeysThreads, 0, st>>>(n, x, y, z, t->lo[0], t->lo[1], t->lo[2], scale, keys,
                                                              t->d_state, b_clo, b_chi, b_bucket, b_slot, b_count);
@@ -1719,7 +1738,8 @@ static afmm_status build_impl(afmm_tree *t, long long n, const float *x, const f
         TCU(t, cub::DeviceScan::ExclusiveSum(b_sbuf, sb, b_count, b_off, (int)(nbcap + 1), st));
         bucket_scatter_kernel<<<grid_for(n, TH), TH, 0, st>>>(n, keys, b_bucket, b_slot, b_off, b_keys, b_idx);
         bucket_sort_kernel<<<(int)((nbcap + kBucketWarps - 1) / kBucketWarps), 32 * kBucketWarps, 0, st>>>(
-            t->d_state, b_off, b_keys, b_idx, t->keys_sorted, t->perm, bovf, b_big);
+            t->d_state, b_off, b_keys, b_idx, t->keys_sorted, t->perm, bovf, b_big, b_mid);
+        bucket_mid_kernel<<<148 * 8, 32 * kBucketWarps, 0, st>>>(b_mid, b_off, b_keys, b_idx, t->keys_sorted, t->perm);
         bucket_big_kernel<<<kBigList / 2, kBigThreads, kBigSmem, st>>>(b_big, b_off, b_keys, b_idx, t->keys_sorted,
                                                                       t->perm);
         TCU(t, cudaGetLastError());
